@@ -1,0 +1,347 @@
+"""bench.py — CA-GMRES(s, m) time-to-solution on B200 (BASELINE.json metric), one JSON line.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config C2]
+
+A step = one full cagmres_solve (all SURVEY §8(a) rows: MPK, BOrth, TSQR, small factor,
+Hessenberg update, LS, x update, explicit residual; the first Newton cycle is GMRES(m))
+from x0 = 0 to ||r|| <= 1e-8 ||r0|| on the N=1 workload, config C2 (BASELINE.json
+configs[1]: 3D convection-diffusion 7-point 128^3, s=10, m=30, Newton, CholQR).
+Inputs are resident in HBM before timing (A 175 MB + V 520 MB, larger than the 126 MB L2;
+an L2 flush buffer is also written between steps).  value = mean device time per solve (ms,
+lower is better); e2e = the same solve through the C ABI with b copied from pinned host
+memory and x copied back inside the timed region.
+
+Multi-GPU (torchrun, one process per GPU): the rows of the same matrix are partitioned in
+contiguous blocks and solved with NCCL halo exchange + allreduces (strong scaling);
+the time is the max over ranks.  --impl reference times the CPU oracle (oracle/) on a
+bounded sample (rank 0 only).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from synth import generators as G  # noqa: E402
+
+CFG = {"C2": dict(build=lambda rows=None: G.convection_diffusion(128, 3, 7, rows=rows), n=128 ** 3,
+                  s=10, m=30, basis="newton", tsqr="cholqr", reorth=False,
+                  workload="C2: 3D convection-diffusion 7-pt 128^3 (n=2,097,152), s=10, m=30, Newton, CholQR"),
+       "C3": dict(build=lambda rows=None: G.g3_shaped(rows=rows), n=1585478, s=5, m=60, basis="newton",
+                  tsqr="cholqr", reorth=False,
+                  workload="C3: G3_circuit-shaped (n=1,585,478), s=5, m=60, Newton, CholQR"),
+       "C1": dict(build=lambda rows=None: G.convection_diffusion(32, 2, 5, rows=rows), n=1024, s=5, m=30,
+                  basis="newton", tsqr="cholqr", reorth=False,
+                  workload="C1: 2D convection-diffusion 5-pt 32^2 (n=1024), s=5, m=30, Newton, CholQR")}
+TOL = 1e-8
+METRIC = "CA-GMRES time-to-solution (rel. residual 1e-8)"
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+class Clocks:
+    """nvidia-smi sampler running during the timed region."""
+
+    def __init__(self, idx):
+        self.idx = idx
+        self.path = os.path.join("/tmp", f"clocks_{os.getpid()}.csv")
+        self.p = None
+
+    def __enter__(self):
+        try:
+            self.f = open(self.path, "w")
+            self.p = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.idx),
+                 "--query-gpu=clocks.sm,clocks.max.sm,clocks_event_reasons.active,"
+                 "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
+                 "--format=csv,noheader,nounits", "-lms", "100"], stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+        return self
+
+    def __exit__(self, *a):
+        if self.p is not None:
+            self.p.terminate()
+            try:
+                self.p.wait(timeout=5)
+            except Exception:
+                self.p.kill()
+            self.f.close()
+
+    def summary(self):
+        if self.p is None or not os.path.exists(self.path):
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in open(self.path):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0])); mx.append(float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": float(max(mx)), "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    lrank = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, lrank
+
+
+def ghost_rows(cfg, row_starts, rank, s):
+    """Rows this rank needs: owned rows plus every row within s-1 hops.  For the
+    naturally ordered configs a contiguous band suffices; found by BFS on generated rows."""
+    n = cfg["n"]
+    lo, hi = int(row_starts[rank]), int(row_starts[rank + 1])
+    A = cfg["build"]((lo, hi))
+    rows = np.repeat(np.arange(lo, hi), np.diff(A.rowptr))
+    bw = int(np.abs(A.colind.astype(np.int64) - rows).max()) if A.nnz else 0
+    clo, chi = max(0, lo - (s - 1) * bw), min(n, hi + (s - 1) * bw)
+    return cfg["build"]((clo, chi))
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_yamazakiathd14_b200 import _lib as L
+    from paper_conf_ipps_yamazakiathd14_b200.solver import Solver
+
+    ws, rank, lrank = dist_env()
+    torch.cuda.set_device(lrank)
+    group = None
+    cfg = CFG[args.config]
+    if ws > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", lrank))
+        group = dist.group.WORLD
+    t0 = time.time()
+    if ws == 1:
+        A = cfg["build"]()
+        S = Solver(A, cfg["s"], cfg["m"], basis=cfg["basis"], tsqr=cfg["tsqr"], reorth=cfg["reorth"])
+        b_host = G.rhs(cfg["n"])
+    else:
+        rs = np.array([(p * cfg["n"]) // ws for p in range(ws + 1)], dtype=np.int64)
+        A = ghost_rows(cfg, rs, rank, cfg["s"])
+        S = Solver(A, cfg["s"], cfg["m"], basis=cfg["basis"], tsqr=cfg["tsqr"], reorth=cfg["reorth"],
+                   group=group, row_starts=rs)
+        b_host = G.rhs(cfg["n"], rows=(rs[rank], rs[rank + 1]))
+    setup_s = time.time() - t0
+    stream = torch.cuda.current_stream()
+    b = torch.tensor(b_host, device="cuda")
+    x = torch.zeros_like(b)
+    flush = torch.empty(64 * 1024 * 1024, dtype=torch.float32, device="cuda")   # 256 MB > L2
+
+    def one(timing):
+        x.zero_()
+        return S.solve(b, x, tol=TOL, maxit=200, timing=timing)
+
+    for _ in range(args.warmup):
+        one(False)
+    # ---- timed region: device events on the solver's stream, barrier + sync both sides ----
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    stats = []
+    l0 = None
+    with Clocks(lrank) as clk:
+        for k in range(args.steps):
+            flush.fill_(float(k))
+            if group is not None:
+                dist.barrier()
+            torch.cuda.synchronize()
+            if l0 is None:
+                l0 = L.load().cagmres_kernel_launches()
+            ev[k][0].record(stream)
+            _, st = one(True)
+            ev[k][1].record(stream)
+            torch.cuda.synchronize()
+            if k == 0:
+                l1 = L.load().cagmres_kernel_launches()
+            stats.append(st)
+    launches_first = l1 - l0
+    ms = np.array([e[0].elapsed_time(e[1]) for e in ev])
+    ms_step = float(ms.mean())
+    if group is not None:
+        t = torch.tensor([ms_step], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_step = float(t.item())
+    st0 = stats[-1]
+    # ---- dominant kernel (MPK SpMV) roofline, measured live inside the timed region ----
+    spmv_ms = np.mean([s.ms["spmv"] / max(s.spmv_launches, 1) for s in stats])
+    spmv_bytes = st0.bytes["spmv"] / max(st0.spmv_launches, 1)
+    peak, peak_kind = peaks()
+    achieved = spmv_bytes / (spmv_ms * 1e-3) / 1e9
+    phase = {k: float(np.mean([s.ms[k] for s in stats])) for k in ("mpk", "borth", "tsqr", "other", "total")}
+    phase_gbs = {k: (st0.bytes[k] / (phase[k] * 1e-3) / 1e9 if phase[k] > 0 else None)
+                 for k in ("mpk", "borth", "tsqr", "other")}
+    traffic = None
+    tf = os.path.join(ROOT, "profiles", "spmv_traffic.json")
+    if os.path.exists(tf):
+        with open(tf) as f:
+            traffic = json.load(f).get(args.config)
+    # ---- e2e: host b (pinned) -> device, solve via the C ABI, x -> host, all timed ----
+    b_pin = torch.tensor(b_host).pin_memory()
+    x_pin = torch.empty_like(b_pin).pin_memory()
+    e2e_ms = []
+    for k in range(args.steps):
+        flush.fill_(float(k))
+        if group is not None:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        bd = b_pin.to("cuda", non_blocking=True)
+        xd = torch.zeros_like(bd)
+        S.solve(bd, xd, tol=TOL, maxit=200)
+        x_pin.copy_(xd, non_blocking=True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        e2e_ms.append(e0.elapsed_time(e1))
+    e2e = float(np.mean(e2e_ms))
+    if group is not None:
+        t = torch.tensor([e2e], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e = float(t.item())
+    clocks = clk.summary()
+    out = None
+    if rank == 0:
+        cpu = cpu_baseline(cfg, st0.cycles, ws) if (ws == 1 and not args.no_cpu) else None
+        out = {
+            "metric": METRIC, "value": round(ms_step, 4), "unit": "ms", "n_gpus": ws,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 4),
+            "higher_is_better": False, "scaling": "strong" if ws > 1 else "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": cfg["workload"], "n": cfg["n"], "s": cfg["s"], "m": cfg["m"],
+                       "tol": TOL, "cycles": st0.cycles, "parallelism": f"rows{ws}",
+                       "l2": "inputs larger than L2 (A 175 MB, V 520 MB) + 256 MB flush between steps",
+                       "setup_s": round(setup_s, 2)},
+            "e2e": {"value": round(e2e, 4), "unit": "ms", "h2d_bytes_per_step": 8 * len(b_host),
+                    "d2h_bytes_per_step": 8 * len(b_host)},
+            "gpu_launches": int(launches_first),
+            "roofline": {"bound": "hbm", "kernel": "k_spmv_sell32 (MPK SpMV step)",
+                         "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                         "frac": round(achieved / peak, 4), "traffic": traffic,
+                         "peak_source": peak_kind, "bytes_per_launch": spmv_bytes,
+                         "avg_launch_us": round(spmv_ms * 1e3, 2), "launches_per_step": st0.spmv_launches},
+            "phases_ms": {k: round(v, 3) for k, v in phase.items()},
+            "phases_gbs": {k: (round(v, 1) if v else None) for k, v in phase_gbs.items()},
+            "clocks": clocks,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(out), flush=True)
+    S.close()
+    if group is not None:
+        dist.barrier()
+        dist.destroy_process_group()
+    return out
+
+
+def _cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count()
+
+
+def cpu_baseline(cfg, gpu_cycles, ws):
+    """The oracle as it stands, on this host's cores, on a bounded sample: 2 restart cycles of
+    the same workload (cycle 1 = GMRES(m) shift cycle, cycle 2 = CA), time per cycle
+    extrapolated to the GPU-measured cycle count."""
+    from oracle import cagmres_oracle as O
+    A = cfg["build"]().to_scipy()
+    b = G.rhs(cfg["n"])
+    t0 = time.perf_counter()
+    O.cagmres(A, b, cfg["s"], cfg["m"], basis=cfg["basis"], tsqr=cfg["tsqr"], reorth=cfg["reorth"],
+              tol=TOL, maxcyc=2)
+    dt = time.perf_counter() - t0
+    threads = _cores()
+    try:
+        from threadpoolctl import threadpool_info
+        threads = max([i.get("num_threads", 1) for i in threadpool_info()] + [1])
+    except Exception:
+        pass
+    return {"value": round(dt / 2 * gpu_cycles * 1e3, 1), "unit": "ms", "cores": threads,
+            "kind": "oracle",
+            "sample": f"2 restart cycles of {cfg['workload']} on the host (NumPy/SciPy fp64, "
+                      f"{dt:.1f} s), per-cycle time x {gpu_cycles} cycles (GPU cycle count), extrapolated"}
+
+
+def run_reference(args):
+    ws, rank, _ = dist_env()
+    if rank != 0:
+        return None
+    from oracle import cagmres_oracle as O
+    cfg = CFG[args.config]
+    A = cfg["build"]().to_scipy()
+    b = G.rhs(cfg["n"])
+    # warm-up steps also establish the oracle's own cycle count to tolerance (one full solve)
+    t0 = time.perf_counter()
+    full = O.cagmres(A, b, cfg["s"], cfg["m"], basis=cfg["basis"], tsqr=cfg["tsqr"], reorth=cfg["reorth"],
+                     tol=TOL, maxcyc=200)
+    t_full = time.perf_counter() - t0
+    cycles = full["cycles"]
+    re, im = full["shifts"]
+    times = []
+    for k in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        O.cagmres(A, b, cfg["s"], cfg["m"], basis=cfg["basis"], tsqr=cfg["tsqr"], reorth=cfg["reorth"],
+                  tol=0.0, maxcyc=1, shifts=(re, im))
+        if k >= args.warmup:
+            times.append(time.perf_counter() - t0)
+    per = float(np.mean(times))
+    val = per * cycles * 1e3
+    cores = _cores()
+    out = {"metric": METRIC, "value": round(val, 1), "unit": "ms", "n_gpus": ws, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": round(per * 1e3, 1), "higher_is_better": False,
+           "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
+           "config": {"workload": cfg["workload"], "n": cfg["n"], "s": cfg["s"], "m": cfg["m"], "tol": TOL,
+                      "cycles": cycles, "full_oracle_solve_s": round(t_full, 2)},
+           "cpu_baseline": {"value": round(val, 1), "unit": "ms", "cores": cores, "kind": "oracle",
+                            "sample": f"each step = 1 CA restart cycle (shifts from the oracle's own "
+                                      f"first cycle); value = mean cycle time x {cycles} cycles"},
+           "e2e": {"value": round(val, 1), "unit": "ms", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+    return out
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C2", choices=sorted(CFG))
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

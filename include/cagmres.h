@@ -1,0 +1,212 @@
+/*
+ * cagmres.h — C ABI of the B200-native CA-GMRES(s, m) hot path.
+ *
+ * Method: Yamazaki, Anzt, Tomov, Hoemmen, Dongarra, "Improving the Performance of CA-GMRES
+ * on Multicores with Multiple GPUs", IPDPS 2014.  "P:n" cites /root/reference/PAPER.md line n.
+ * One restart cycle = MPK (Fig. 4) -> BOrth (CGS) -> TSQR (CholQR P:162-166 /
+ * SVQR P:172; MGS/CGS comparators, Fig. 9) -> Hessenberg update per block of
+ * s_b = min(s, m - j) basis vectors, then the least-squares solve on the host and
+ * x := x + V_{1:m} y.
+ *
+ * Conventions (all functions):
+ *   - return int status: 0 = CAGMRES_OK, > 0 warning, < 0 error.  Never abort, never print.
+ *   - every double is IEEE fp64; matrices are COLUMN-MAJOR with explicit leading dimension.
+ *   - "dev" pointers are CUDA device pointers on the handle's device (e.g. a torch tensor's
+ *     data_ptr()); "host" pointers are ordinary CPU memory.  The caller owns every pointer it
+ *     passes; the library never frees or retains them beyond the call.
+ *   - all device work is enqueued on the handle's stream (cagmres_set_stream; default: a
+ *     stream created by the handle).  Functions that return a value the host needs
+ *     (tsqr breakdown, solve) synchronise that stream before returning.
+ *   - multi-GPU: one process per GPU; collectives are NCCL over NVLink (P:45 block rows).
+ *     A distributed function must be called by every rank with the same scalar arguments.
+ *   - vectors and panels passed to mpk/borth/tsqr/solve hold this rank's OWNED rows only
+ *     (n_loc = own_end - own_begin rows); ghost rows are managed inside the handle.
+ */
+#ifndef CAGMRES_H
+#define CAGMRES_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---- status codes ------------------------------------------------------------------ */
+#define CAGMRES_OK              0
+#define CAGMRES_NOT_CONVERGED   1   /* solve: maxit cycles done, x holds the last iterate     */
+#define CAGMRES_EINVAL         -1   /* bad argument, shape, leading dimension or alignment    */
+#define CAGMRES_ECUDA          -2   /* a CUDA runtime call failed (no device, launch error)   */
+#define CAGMRES_ENCCL          -3   /* an NCCL call failed                                    */
+#define CAGMRES_EBREAKDOWN     -4   /* Cholesky pivot <= 0, zero norm, singular T     */
+#define CAGMRES_ENOMEM         -5   /* device or host allocation failed                       */
+#define CAGMRES_EGHOST         -6   /* supplied rows do not cover the (s-1)-hop ghost rows    */
+#define CAGMRES_ENOTSUP        -7   /* option not supported by this build                     */
+
+/* ---- options ----------------------------------------------------------------------- */
+enum { CAGMRES_MONOMIAL = 0, CAGMRES_NEWTON = 1 };               /* MPK basis      */
+enum { CAGMRES_CHOLQR = 0, CAGMRES_SVQR = 1, CAGMRES_CGS = 2,     /* TSQR, Fig. 9/10     */
+       CAGMRES_MGS = 3, CAGMRES_CAQR = 4 };
+#define CAGMRES_TSQR_MASK   0xff
+#define CAGMRES_REORTH      0x100   /* "2x": BOrth+TSQR twice (Fig. 14)       */
+#define CAGMRES_BORTH_MGS   0x200   /* BOrth by MGS instead of CGS      */
+
+typedef struct cagmres* cagmres_t;
+
+/* Sparse matrix rows handed to create (host CSR, copied to the device by create).
+ *   n                : global dimension (A is n x n, nonsymmetric allowed)
+ *   row_begin/row_end: global ids of the rows described by rowptr (nrows = row_end-row_begin)
+ *   rowptr           : host, nrows+1 entries, rowptr[0] == 0, int64
+ *   colind           : host, global column ids in [0, n), int32
+ *   val              : host, fp64 values
+ *   own_begin/own_end: the rows this rank owns (block-row distribution);
+ *                      must satisfy row_begin <= own_begin <= own_end <= row_end.
+ * For the distributed handle the described rows must contain every row within graph
+ * distance s-1 of the owned rows (the boundary sets delta^(d,k)); else EGHOST. */
+typedef struct {
+    int64_t n, nnz;
+    const int64_t* rowptr;
+    const int32_t* colind;
+    const double*  val;
+    int64_t row_begin, row_end;
+    int64_t own_begin, own_end;
+} cagmres_csr;
+
+/* Statistics of a solve (Fig. 14 columns).  hist is caller-owned (host). */
+typedef struct {
+    int    cycles;          /* restart cycles executed                                      */
+    int    iters;           /* basis vectors generated (cycles * m)                          */
+    int    hist_cap;        /* capacity of rel_resid_hist                                    */
+    int    hist_len;        /* entries written                                               */
+    double* rel_resid_hist; /* ||b - A x_c|| / ||b - A x_0|| after each cycle (host)         */
+    int    collect_timing;  /* in: 1 = time phases with CUDA events (adds event records)     */
+    double ms_mpk, ms_borth, ms_tsqr, ms_other, ms_total;   /* device time per phase (ms)   */
+    double bytes_mpk, bytes_borth, bytes_tsqr, bytes_other; /* algorithmic bytes */
+    int    spmv_launches;   /* SpMV launches timed in ms_spmv                                */
+    double ms_spmv;         /* device time of the SpMV launches alone                        */
+    double bytes_spmv;      /* algorithmic bytes of those launches                           */
+} cagmres_stats;
+
+/* ---- lifetime ---------------------------------------------------------------------- */
+/* Single-GPU handle on the current CUDA device.  A: all n rows (row_begin=own_begin=0,
+ * row_end=own_end=n).  s >= 1 block size, m >= 1 restart length, s <= m; basis
+ * CAGMRES_MONOMIAL|NEWTON; orth = TSQR kind | flags.  Copies A to the device (sliced-ELL
+ * layout) and allocates the basis V (n x (m+1)) and all workspace.
+ * Errors: EINVAL, ECUDA, ENOMEM. */
+int cagmres_create(cagmres_t* h, const cagmres_csr* A, int s, int m, int basis, int orth);
+
+/* Distributed handle: one per rank, NCCL communicator built from nccl_unique_id (128-byte
+ * ncclUniqueId created by rank 0 and broadcast by the caller).  row_starts (host, nranks+1)
+ * is the global block-row partition: rank p owns [row_starts[p], row_starts[p+1]), and
+ * A->own_begin/own_end must equal this rank's range.  Computes the boundary sets
+ * delta^(d,k) and the halo schedule (exchanging request lists over NCCL).
+ * Errors: EINVAL, EGHOST, ECUDA, ENCCL, ENOMEM. */
+int cagmres_create_dist(cagmres_t* h, const cagmres_csr* A, const int64_t* row_starts,
+                        int s, int m, int basis, int orth,
+                        const void* nccl_unique_id, int rank, int nranks, int cuda_device);
+
+int cagmres_destroy(cagmres_t h);                 /* frees everything create allocated */
+const char* cagmres_strerror(int status);         /* static string, never NULL         */
+
+/* cudaStream_t to enqueue on (NULL = the handle's own stream).  Not owned. */
+int cagmres_set_stream(cagmres_t h, void* cuda_stream);
+
+/* Sizes: n_loc owned rows, n_ext owned+ghost rows (P:60 i^(d,1)), ldv = leading dim of V. */
+int cagmres_sizes(cagmres_t h, int64_t* n_loc, int64_t* n_ext, int64_t* ldv);
+
+/* ---- shifts ------------------------------------------------------------------ */
+/* Newton shifts theta_k = re[k] + i im[k], k < count, in application order, conjugate pairs
+ * adjacent with +im first.  Replaces any shifts the first GMRES cycle would compute.
+ * count >= 1 (extra entries beyond s are ignored).  Errors: EINVAL (pair not adjacent). */
+int cagmres_set_shifts(cagmres_t h, const double* re, const double* im, int count);
+/* Copies the current shifts (after a Newton solve: the Leja-ordered Ritz values) to host
+ * arrays of capacity cap; *count = number available (0 if none). */
+int cagmres_get_shifts(cagmres_t h, double* re, double* im, int cap, int* count);
+
+/* ---- hot-path kernels (callable individually; "MPK, BOrth, and TSQR") ---------- */
+/* MPK(s_b, q) of Fig. 4: W[:,0] = q, W[:,k] = (A - theta_k I) W[:,k-1] for
+ * k = 1..sb (theta = 0 for the monomial basis; complex pairs in real arithmetic).
+ * One halo exchange of q's ghost rows (distributed), then sb local SpMVs on shrinking row
+ * sets i^(d,k+1) with no further communication.  Uses the handle's first sb shifts.
+ *   q : dev, n_loc           W : dev, ldw x (sb+1), ldw >= n_loc, owned rows written
+ * Errors: EINVAL (sb < 1 or sb > s, ldw < n_loc, Newton without shifts). */
+int cagmres_mpk(cagmres_t h, const double* q, double* W, int64_t ldw, int sb);
+
+/* BOrth by CGS: C = Q^T P (global sum over ranks), P := P - Q C.
+ *   Q : dev, ldq x j (orthonormal columns)   P : dev, ldp x w, updated in place
+ *   C : dev, j x w, leading dimension j (output)
+ * j == 0 is a no-op.  Errors: EINVAL. */
+int cagmres_borth(cagmres_t h, const double* Q, int64_t ldq, int j,
+                  double* P, int64_t ldp, int w, double* C);
+
+/* TSQR of the tall-skinny panel P (Fig. 9): P := Q with Q^T Q = I and P_in = Q R.
+ *   P : dev, ldp x w (w <= 32), in place      R : dev, w x w col-major, upper, diag > 0
+ *   orth: CAGMRES_CHOLQR | SVQR | CGS | MGS (| CAGMRES_REORTH for the "2x" variant).
+ * Synchronises the stream.  Errors: EINVAL, EBREAKDOWN (CholQR pivot <= 0). */
+int cagmres_tsqr(cagmres_t h, double* P, int64_t ldp, int w, double* R, int orth);
+
+/* ---- solver -------------------------------------------------------------- */
+/* Solves A x = b with CA-GMRES(s, m) restarted until ||b - A x|| <= tol ||b - A x0||
+ * (explicit residual at each restart) or maxit cycles.  Newton basis without
+ * preset shifts: the first cycle is GMRES(m) and its Ritz values, Leja-ordered, become the
+ * shifts.
+ *   b : dev, n_loc (owned rows)    x : dev, n_loc, in: x0, out: solution
+ *   st: optional (may be NULL), host struct filled on return.
+ * Returns OK, NOT_CONVERGED, or an error (EBREAKDOWN, ECUDA, ENCCL, EINVAL). */
+int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit,
+                  cagmres_stats* st);
+
+/* Process-wide number of CUDA kernel launches this library has issued (all handles).  Lets a
+ * caller count the kernels inside a timed region (bench.py "gpu_launches"). */
+int64_t cagmres_kernel_launches(void);
+
+/* ---- host-only setup plan, exported for tests of the multi-GPU setup ------- */
+/* Pure host functions (no CUDA, no NCCL): boundary sets, extended-row numbering
+ * [owned | delta^(s) | ... | delta^(1)] (distance 1 first), halo request / send lists. */
+typedef struct cagmres_plan* cagmres_plan_t;
+int cagmres_plan_create(cagmres_plan_t* p, const cagmres_csr* A, const int64_t* row_starts,
+                        int nranks, int rank, int s);
+int cagmres_plan_destroy(cagmres_plan_t p);
+/* n_loc, n_ext, n_mat (rows stored = distance <= s-1), level_len[h] (h = 0..s): number of
+ * extended rows at distance <= h; nnz_mat: nonzeros of the stored extended rows. */
+int cagmres_plan_info(cagmres_plan_t p, int64_t* n_loc, int64_t* n_ext, int64_t* n_mat,
+                      int64_t* nnz_mat, int64_t* level_len);
+/* global id of each extended row (host, n_ext). */
+int cagmres_plan_ext_rows(cagmres_plan_t p, int64_t* gids);
+/* extended local CSR of the n_mat stored rows (host; rowptr n_mat+1, colind/val nnz_mat). */
+int cagmres_plan_ext_csr(cagmres_plan_t p, int64_t* rowptr, int32_t* colind, double* val);
+/* Requests this rank makes: counts[nranks]; gids / levels concatenated by owner rank, each
+ * owner's list sorted by (level, gid).  Pass NULL gids to query counts only. */
+int cagmres_plan_requests(cagmres_plan_t p, int64_t* counts, int64_t* gids, int32_t* levels);
+/* Receive position (extended row id) of each requested gid, same order as requests. */
+int cagmres_plan_recv_index(cagmres_plan_t p, int64_t* ext_ids);
+/* Install the requests other ranks made of this rank (counts[nranks], concatenated by
+ * requester).  Errors: EINVAL (a gid not owned here). */
+int cagmres_plan_set_sends(cagmres_plan_t p, const int64_t* counts, const int64_t* gids,
+                           const int32_t* levels);
+/* Send lists: owned local indices in request order (host, total = sum counts). */
+int cagmres_plan_send_index(cagmres_plan_t p, int64_t* local_idx);
+
+/* ---- host-only small dense algorithms of the cycle (exported for tests) -------------- */
+/* Eigenvalues (Ritz values) of the upper Hessenberg H (m x m, ld ldh), Francis
+ * double-shift QR; conjugate pairs returned adjacent (+im first).  EBREAKDOWN if the QR
+ * iteration does not converge. */
+int cagmres_host_eigvals(const double* H, int ldh, int m, double* wr, double* wi);
+/* Modified Leja ordering (reading G10) of cnt Ritz values; writes up to cap
+ * shifts, *nout = number produced (>= s when cnt allows). */
+int cagmres_host_leja(const double* wr, const double* wi, int cnt, int s, double* ore,
+                      double* oim, int cap, int* nout);
+/* Change-of-basis B ((sb+1) x sb, ld sb+1) of the Newton/monomial MPK: A W[:,0:sb] = W B. */
+int cagmres_host_change_of_basis(const double* re, const double* im, int sb, double* B);
+/* Hessenberg update of a block:
+ * H[0:j+sb+1, j:j+sb] = (Rt B - [H[0:j+1,0:j] Rt[0:j,0:sb]; 0]) T^{-1}, T = Rt[j:j+sb,0:sb]. */
+int cagmres_host_hessenberg_update(double* H, int ldh, int j, int sb, const double* Rt,
+                                   int ldr, const double* B);
+/* y = argmin ||beta e1 - H y|| (H (k+1) x k upper Hessenberg, Givens QR); res[i] =
+ * residual estimate after i+1 columns (may be NULL). */
+int cagmres_host_givens_ls(const double* H, int ldh, int k, double beta, double* y,
+                           double* res);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CAGMRES_H */

@@ -1,0 +1,66 @@
+// kernels.h — launchers of the sm_100a FP64 kernels of the CA-GMRES hot path.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace kern {
+
+// Process-wide count of kernel launches issued by this library (bench.py gpu_launches).
+extern long long g_launches;
+
+// Device properties used for grid sizing (filled once per handle).
+struct Dev {
+    int sms = 148;
+    int device = 0;
+};
+
+// Sliced ELLPACK, slice height 32 (one warp), column-major inside a slice.
+struct Sell {
+    int64_t nrows = 0;          // stored rows (extended rows at distance <= s-1)
+    int64_t nslices = 0;
+    int64_t nstored = 0;        // stored entries incl. padding
+    int64_t nnz = 0;            // true nonzeros
+    int64_t* sptr = nullptr;    // nslices+1 offsets (elements)
+    int32_t* col = nullptr;     // local (extended) column ids
+    double* val = nullptr;
+};
+
+// Status bits written by device kernels into the handle's status word.
+enum : int { ST_CHOL = 1, ST_SVQR = 2, ST_NORM = 4 };
+
+// y[0:nrows) = A x + bu*u + bw*w  (u, w may be null).  Newton step: u = x, bu = -theta;
+// second step of a complex pair: w = x_prev, bw = b^2.
+void spmv(const Dev& d, const Sell& A, int64_t nrows, const double* x, double* y,
+          const double* u, double bu, const double* w, double bw, cudaStream_t st);
+// r[0:nrows) = b - A x
+void residual(const Dev& d, const Sell& A, int64_t nrows, const double* x, const double* b,
+              double* r, cudaStream_t st);
+
+// Partial + deterministic total of C = X^T Y (X: n x jx, ld ldx; Y: n x w, ld ldy), written
+// to out (jx x w, ld jx).  fin_chol: out is the Gram (X == Y, jx == w) and R = chol(out)
+// (upper, ld w) is computed in the same launch; breakdown sets ST_CHOL in *status.
+// ws: workspace of at least xty_ws_doubles() doubles; counter: a zeroed device uint.
+struct XtyWs { double* part = nullptr; size_t cap = 0; unsigned int* counter = nullptr; };
+size_t xty_ws_doubles(const Dev& d, int jx, int w);
+int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const double* Y,
+        int64_t ldy, int w, double* out, bool fin_chol, double* R, int* status,
+        const XtyWs& ws, cudaStream_t st);
+
+// R = chol(G) (upper, ld w), one tiny launch (used after a cross-rank allreduce of G).
+void chol(const double* G, int w, double* R, int* status, cudaStream_t st);
+// SVQR small factor: R from the Gram G (w x w), one CTA.
+void svqr_factor(const double* G, int w, double* R, int* status, cudaStream_t st);
+
+// P[:, 0:w] -= X C  (C: jx x w, ld jx)      (BOrth pass 2)
+void update(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, double* P,
+            int64_t ldp, int w, const double* C, cudaStream_t st);
+// P[:, c0:w] = (P R^{-1})[:, c0:w]   (R upper w x w, ld w)
+void trsm(const Dev& d, int64_t n, double* P, int64_t ldp, int w, const double* R, int c0,
+          cudaStream_t st);
+// dst[k] = src[idx[k]]  /  dst[idx[k]] = src[k]
+void gather(const double* src, const int64_t* idx, int64_t cnt, double* dst, cudaStream_t st);
+void scatter(const double* src, const int64_t* idx, int64_t cnt, double* dst, cudaStream_t st);
+// small device helpers
+void add_small(const double* a, const double* b, double* c, int cnt, cudaStream_t st);
+
+}  // namespace kern

@@ -1,0 +1,806 @@
+// solver.cu — the CA-GMRES(s, m) handle: setup, MPK / BOrth / TSQR drivers, NCCL halo and
+// allreduces, and the restart loop of cagmres_solve (§III-§V).
+//
+// Data layout in HBM:
+//   V   : ldv x (m+1) column-major, ldv = round_up(n_ext, 32).  Rows [0, n_loc) of column k
+//         hold the k-th basis vector's owned rows; rows [n_loc, n_ext) are the MPK ghost
+//         scratch of that column (P:66 z^(d,k)), so the matrix powers kernel writes its
+//         outputs straight into the basis — no expand/copy step (P:66, P:132 fn 4).
+//   A   : extended rows in SELL-32 (kern::Sell), columns in extended local ids.
+//   tab : per-cycle device table of the BOrth coefficients C and TSQR factors R of every
+//         block (and of the reorthogonalisation pass); copied to the host once per cycle
+//         for the Hessenberg update and the least-squares solve.
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include "internal.h"
+#include "kernels.h"
+
+#define CU(x)                                                       \
+    do {                                                            \
+        cudaError_t e_ = (x);                                       \
+        if (e_ != cudaSuccess) { return CAGMRES_ECUDA; }            \
+    } while (0)
+#define NC(x)                                                       \
+    do {                                                            \
+        ncclResult_t r_ = (x);                                      \
+        if (r_ != ncclSuccess) { return CAGMRES_ENCCL; }            \
+    } while (0)
+#define TRY(x)                                                      \
+    do {                                                            \
+        int s_ = (x);                                               \
+        if (s_ < 0) return s_;                                      \
+    } while (0)
+
+namespace {
+
+enum Phase { PH_MPK = 0, PH_BORTH = 1, PH_TSQR = 2, PH_OTHER = 3, PH_SPMV = 4, PH_N = 5 };
+
+struct Timer {
+    bool on = false;
+    std::vector<cudaEvent_t> pool;
+    size_t used = 0;
+    std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> rec;
+    cudaEvent_t get() {
+        if (used == pool.size()) {
+            cudaEvent_t e;
+            cudaEventCreate(&e);
+            pool.push_back(e);
+        }
+        return pool[used++];
+    }
+    void reset() { used = 0; rec.clear(); }
+    ~Timer() { for (auto e : pool) cudaEventDestroy(e); }
+};
+
+struct Block { int j, sb; size_t c1, r1, c2, r2; };
+
+}  // namespace
+
+struct cagmres {
+    int s = 1, m = 1, basis = CAGMRES_NEWTON, orth = CAGMRES_CHOLQR;
+    int64_t n = 0, n_loc = 0, n_ext = 0, ldv = 0;
+    int rank = 0, nranks = 1;
+    ncclComm_t comm = nullptr;
+    kern::Dev dev;
+    cudaStream_t stream = nullptr, own_stream = nullptr;
+    kern::Sell A;
+    std::vector<int64_t> level_len;        // ext rows with distance <= h
+    std::vector<int64_t> nnz_prefix;       // nnz of stored rows with distance <= h (h <= s-1)
+    double* V = nullptr;
+    double* xe = nullptr;                  // ext scratch for the residual (distributed)
+    double* tab = nullptr; size_t tab_cap = 0;
+    double* gbuf = nullptr;                // Gram / small scratch
+    double* ybuf = nullptr;                // LS solution (m)
+    kern::XtyWs ws;
+    int* status = nullptr;
+    // halo (distributed)
+    std::vector<int64_t> send_off, recv_off;
+    std::vector<std::vector<int64_t>> send_pre, recv_pre;   // [rank][depth]
+    int64_t nsend = 0, nrecv = 0;
+    int64_t* d_send_idx = nullptr;
+    int64_t* d_recv_ext = nullptr;
+    double* d_sendbuf = nullptr;
+    double* d_recvbuf = nullptr;
+    // shifts
+    std::vector<double> sh_re, sh_im;
+    bool have_shifts = false;
+    Timer timer;
+    double bytes[PH_N] = {0, 0, 0, 0, 0};
+    int spmv_launches = 0;
+
+    ~cagmres() {
+        cudaFree(A.sptr); cudaFree(A.col); cudaFree(A.val);
+        cudaFree(V); cudaFree(xe); cudaFree(tab); cudaFree(gbuf); cudaFree(ybuf);
+        cudaFree(ws.part); cudaFree(ws.counter); cudaFree(status);
+        cudaFree(d_send_idx); cudaFree(d_recv_ext); cudaFree(d_sendbuf); cudaFree(d_recvbuf);
+        if (comm) ncclCommDestroy(comm);
+        if (own_stream) cudaStreamDestroy(own_stream);
+    }
+};
+
+namespace {
+
+// ---- timing helpers --------------------------------------------------------------------
+struct Scope {
+    cagmres* h; int ph; cudaEvent_t e0 = nullptr;
+    Scope(cagmres* hh, int p) : h(hh), ph(p) {
+        if (h->timer.on) { e0 = h->timer.get(); cudaEventRecord(e0, h->stream); }
+    }
+    ~Scope() {
+        if (h->timer.on) {
+            cudaEvent_t e1 = h->timer.get();
+            cudaEventRecord(e1, h->stream);
+            h->timer.rec.push_back({ph, {e0, e1}});
+        }
+    }
+};
+
+int64_t round_up(int64_t a, int64_t b) { return (a + b - 1) / b * b; }
+
+// ---- SELL-32 build (host) + upload ------------------------------------------------------
+int build_sell(cagmres* h, const cagmres_plan& p) {
+    const int64_t nr = p.n_mat;
+    const int64_t ns = (nr + 31) / 32;
+    std::vector<int64_t> sptr(size_t(ns) + 1, 0);
+    for (int64_t sl = 0; sl < ns; ++sl) {
+        int64_t wmax = 0;
+        for (int64_t r = sl * 32; r < std::min(nr, sl * 32 + 32); ++r)
+            wmax = std::max(wmax, p.rowptr[size_t(r) + 1] - p.rowptr[size_t(r)]);
+        sptr[size_t(sl) + 1] = sptr[size_t(sl)] + 32 * wmax;
+    }
+    const int64_t tot = sptr[size_t(ns)];
+    std::vector<int32_t> col(static_cast<size_t>(tot));
+    std::vector<double> val(static_cast<size_t>(tot));
+    for (int64_t sl = 0; sl < ns; ++sl) {
+        const int64_t wdt = (sptr[size_t(sl) + 1] - sptr[size_t(sl)]) / 32;
+        for (int lane = 0; lane < 32; ++lane) {
+            const int64_t r = sl * 32 + lane;
+            const int64_t b = r < nr ? p.rowptr[size_t(r)] : 0, e = r < nr ? p.rowptr[size_t(r) + 1] : 0;
+            for (int64_t t = 0; t < wdt; ++t) {
+                const int64_t o = sptr[size_t(sl)] + 32 * t + lane;
+                if (b + t < e) {
+                    col[size_t(o)] = p.colind[size_t(b + t)];
+                    val[size_t(o)] = p.val[size_t(b + t)];
+                } else {
+                    col[size_t(o)] = int32_t(r < nr ? r : 0);
+                    val[size_t(o)] = 0.0;
+                }
+            }
+        }
+    }
+    h->A.nrows = nr; h->A.nslices = ns; h->A.nstored = tot; h->A.nnz = p.nnz_mat;
+    CU(cudaMalloc(&h->A.sptr, sizeof(int64_t) * size_t(ns + 1)));
+    CU(cudaMalloc(&h->A.col, sizeof(int32_t) * size_t(std::max<int64_t>(tot, 1))));
+    CU(cudaMalloc(&h->A.val, sizeof(double) * size_t(std::max<int64_t>(tot, 1))));
+    CU(cudaMemcpy(h->A.sptr, sptr.data(), sizeof(int64_t) * size_t(ns + 1), cudaMemcpyHostToDevice));
+    if (tot) {
+        CU(cudaMemcpy(h->A.col, col.data(), sizeof(int32_t) * size_t(tot), cudaMemcpyHostToDevice));
+        CU(cudaMemcpy(h->A.val, val.data(), sizeof(double) * size_t(tot), cudaMemcpyHostToDevice));
+    }
+    // nnz of the first level_len[h] rows (algorithmic byte model of a prefix SpMV)
+    h->nnz_prefix.assign(size_t(h->s) + 1, 0);
+    for (int hh = 0; hh <= h->s; ++hh) {
+        const int64_t rows = std::min(nr, p.level_len[size_t(hh)]);
+        h->nnz_prefix[size_t(hh)] = p.rowptr[size_t(rows)];
+    }
+    return CAGMRES_OK;
+}
+
+size_t tab_doubles(int s, int m) {
+    const size_t M = size_t(m) + 2, W = size_t(s) + 2;
+    return 4 * M * M + 4 * M * W * W + 64;
+}
+
+int common_alloc(cagmres* h) {
+    h->ldv = round_up(std::max<int64_t>(h->n_ext, 1), 32);
+    const size_t vbytes = sizeof(double) * size_t(h->ldv) * size_t(h->m + 1);
+    if (cudaMalloc(&h->V, vbytes) != cudaSuccess) return CAGMRES_ENOMEM;
+    CU(cudaMemset(h->V, 0, vbytes));
+    if (h->nranks > 1) {
+        if (cudaMalloc(&h->xe, sizeof(double) * size_t(h->ldv)) != cudaSuccess) return CAGMRES_ENOMEM;
+        CU(cudaMemset(h->xe, 0, sizeof(double) * size_t(h->ldv)));
+    }
+    h->tab_cap = tab_doubles(h->s, h->m);
+    CU(cudaMalloc(&h->tab, sizeof(double) * h->tab_cap));
+    CU(cudaMemset(h->tab, 0, sizeof(double) * h->tab_cap));
+    CU(cudaMalloc(&h->gbuf, sizeof(double) * size_t(h->m + 2) * size_t(std::max(h->m, 32) + 2)));
+    CU(cudaMalloc(&h->ybuf, sizeof(double) * size_t(h->m + 2)));
+    size_t cap = 0;
+    for (int w = 1; w <= 32; ++w) cap = std::max(cap, kern::xty_ws_doubles(h->dev, h->m + 1, w));
+    h->ws.cap = cap;
+    CU(cudaMalloc(&h->ws.part, sizeof(double) * cap));
+    CU(cudaMalloc(&h->ws.counter, sizeof(unsigned int)));
+    CU(cudaMemset(h->ws.counter, 0, sizeof(unsigned int)));
+    CU(cudaMalloc(&h->status, sizeof(int)));
+    CU(cudaMemset(h->status, 0, sizeof(int)));
+    return CAGMRES_OK;
+}
+
+int init_common(cagmres* h, const cagmres_csr* A, const int64_t* row_starts, int s, int m,
+                int basis, int orth) {
+    if (s < 1 || m < 1 || s > m || s > 31 || (basis != CAGMRES_MONOMIAL && basis != CAGMRES_NEWTON))
+        return CAGMRES_EINVAL;
+    const int kind = orth & CAGMRES_TSQR_MASK;
+    if (kind > CAGMRES_MGS) return kind == CAGMRES_CAQR ? CAGMRES_ENOTSUP : CAGMRES_EINVAL;
+    h->s = s; h->m = m; h->basis = basis; h->orth = orth;
+    int dv = 0;
+    CU(cudaGetDevice(&dv));
+    h->dev.device = dv;
+    CU(cudaDeviceGetAttribute(&h->dev.sms, cudaDevAttrMultiProcessorCount, dv));
+    CU(cudaStreamCreateWithFlags(&h->own_stream, cudaStreamNonBlocking));
+    h->stream = h->own_stream;
+    cagmres_plan plan;
+    try {
+        TRY(plan_build(&plan, A, row_starts, h->nranks, h->rank, s));
+    } catch (...) {
+        return CAGMRES_ENOMEM;
+    }
+    h->n = A->n; h->n_loc = plan.n_loc; h->n_ext = plan.n_ext;
+    h->level_len = plan.level_len;
+    TRY(build_sell(h, plan));
+    TRY(common_alloc(h));
+    if (h->nranks > 1) {
+        // ---- exchange request lists (setup, "compress ... needed by other GPUs") ----
+        const int P = h->nranks;
+        std::vector<int64_t> myc(plan.req_counts);
+        int64_t *d_cnt = nullptr, *d_all = nullptr;
+        CU(cudaMalloc(&d_cnt, sizeof(int64_t) * size_t(P)));
+        CU(cudaMalloc(&d_all, sizeof(int64_t) * size_t(P) * size_t(P)));
+        CU(cudaMemcpy(d_cnt, myc.data(), sizeof(int64_t) * size_t(P), cudaMemcpyHostToDevice));
+        NC(ncclAllGather(d_cnt, d_all, size_t(P), ncclInt64, h->comm, h->stream));
+        std::vector<int64_t> all(size_t(P) * size_t(P));
+        CU(cudaMemcpyAsync(all.data(), d_all, sizeof(int64_t) * all.size(), cudaMemcpyDeviceToHost, h->stream));
+        CU(cudaStreamSynchronize(h->stream));
+        cudaFree(d_cnt); cudaFree(d_all);
+        std::vector<int64_t> inc(static_cast<size_t>(P));                // what q requests of me
+        int64_t tin = 0, tout = int64_t(plan.req_gid.size());
+        for (int q = 0; q < P; ++q) { inc[size_t(q)] = all[size_t(q) * P + size_t(h->rank)]; tin += inc[size_t(q)]; }
+        int64_t *d_og = nullptr, *d_ig = nullptr;
+        int32_t *d_ol = nullptr, *d_il = nullptr;
+        CU(cudaMalloc(&d_og, sizeof(int64_t) * size_t(std::max<int64_t>(tout, 1))));
+        CU(cudaMalloc(&d_ol, sizeof(int32_t) * size_t(std::max<int64_t>(tout, 1))));
+        CU(cudaMalloc(&d_ig, sizeof(int64_t) * size_t(std::max<int64_t>(tin, 1))));
+        CU(cudaMalloc(&d_il, sizeof(int32_t) * size_t(std::max<int64_t>(tin, 1))));
+        if (tout) {
+            CU(cudaMemcpy(d_og, plan.req_gid.data(), sizeof(int64_t) * size_t(tout), cudaMemcpyHostToDevice));
+            CU(cudaMemcpy(d_ol, plan.req_level.data(), sizeof(int32_t) * size_t(tout), cudaMemcpyHostToDevice));
+        }
+        NC(ncclGroupStart());
+        int64_t oo = 0, io = 0;
+        for (int q = 0; q < P; ++q) {
+            const int64_t so = plan.req_counts[size_t(q)], si = inc[size_t(q)];
+            if (so) { NC(ncclSend(d_og + oo, size_t(so), ncclInt64, q, h->comm, h->stream));
+                      NC(ncclSend(d_ol + oo, size_t(so), ncclInt32, q, h->comm, h->stream)); }
+            if (si) { NC(ncclRecv(d_ig + io, size_t(si), ncclInt64, q, h->comm, h->stream));
+                      NC(ncclRecv(d_il + io, size_t(si), ncclInt32, q, h->comm, h->stream)); }
+            oo += so; io += si;
+        }
+        NC(ncclGroupEnd());
+        std::vector<int64_t> ig(static_cast<size_t>(tin));
+        std::vector<int32_t> il(static_cast<size_t>(tin));
+        if (tin) {
+            CU(cudaMemcpyAsync(ig.data(), d_ig, sizeof(int64_t) * size_t(tin), cudaMemcpyDeviceToHost, h->stream));
+            CU(cudaMemcpyAsync(il.data(), d_il, sizeof(int32_t) * size_t(tin), cudaMemcpyDeviceToHost, h->stream));
+        }
+        CU(cudaStreamSynchronize(h->stream));
+        cudaFree(d_og); cudaFree(d_ol); cudaFree(d_ig); cudaFree(d_il);
+        TRY(cagmres_plan_set_sends(&plan, inc.data(), ig.data(), il.data()));
+        // ---- device halo tables -------------------------------------------------------
+        h->nsend = tin; h->nrecv = tout;
+        h->send_off.assign(size_t(P) + 1, 0); h->recv_off.assign(size_t(P) + 1, 0);
+        h->send_pre.assign(size_t(P), std::vector<int64_t>(size_t(s) + 1, 0));
+        h->recv_pre.assign(size_t(P), std::vector<int64_t>(size_t(s) + 1, 0));
+        for (int q = 0; q < P; ++q) {
+            h->send_off[size_t(q) + 1] = h->send_off[size_t(q)] + inc[size_t(q)];
+            h->recv_off[size_t(q) + 1] = h->recv_off[size_t(q)] + plan.req_counts[size_t(q)];
+            for (int d = 0; d <= s; ++d) {
+                h->send_pre[size_t(q)][size_t(d)] = plan_prefix_count(plan.send_counts, plan.send_level, q, d);
+                h->recv_pre[size_t(q)][size_t(d)] = plan_prefix_count(plan.req_counts, plan.req_level, q, d);
+            }
+        }
+        CU(cudaMalloc(&h->d_send_idx, sizeof(int64_t) * size_t(std::max<int64_t>(tin, 1))));
+        CU(cudaMalloc(&h->d_recv_ext, sizeof(int64_t) * size_t(std::max<int64_t>(tout, 1))));
+        CU(cudaMalloc(&h->d_sendbuf, sizeof(double) * size_t(std::max<int64_t>(tin, 1))));
+        CU(cudaMalloc(&h->d_recvbuf, sizeof(double) * size_t(std::max<int64_t>(tout, 1))));
+        if (tin) CU(cudaMemcpy(h->d_send_idx, plan.send_idx.data(), sizeof(int64_t) * size_t(tin), cudaMemcpyHostToDevice));
+        if (tout) CU(cudaMemcpy(h->d_recv_ext, plan.req_ext.data(), sizeof(int64_t) * size_t(tout), cudaMemcpyHostToDevice));
+    }
+    return CAGMRES_OK;
+}
+
+// ---- collectives ---------------------------------------------------------------------
+int allreduce(cagmres* h, double* buf, size_t cnt) {
+    if (h->nranks == 1 || cnt == 0) return CAGMRES_OK;
+    NC(ncclAllReduce(buf, buf, cnt, ncclDouble, ncclSum, h->comm, h->stream));
+    return CAGMRES_OK;
+}
+
+// Halo exchange of the ghost rows (distance <= depth) of an extended vector (Fig. 4 setup,
+// P:66): pack owned values other ranks need, NCCL send/recv over NVLink, unpack.
+int halo(cagmres* h, double* vec, int depth) {
+    if (h->nranks == 1 || depth <= 0) return CAGMRES_OK;
+    kern::gather(vec, h->d_send_idx, h->nsend, h->d_sendbuf, h->stream);
+    NC(ncclGroupStart());
+    for (int q = 0; q < h->nranks; ++q) {
+        const int64_t sc = h->send_pre[size_t(q)][size_t(depth)], rc = h->recv_pre[size_t(q)][size_t(depth)];
+        if (sc) NC(ncclSend(h->d_sendbuf + h->send_off[size_t(q)], size_t(sc), ncclDouble, q, h->comm, h->stream));
+        if (rc) NC(ncclRecv(h->d_recvbuf + h->recv_off[size_t(q)], size_t(rc), ncclDouble, q, h->comm, h->stream));
+    }
+    NC(ncclGroupEnd());
+    kern::scatter(h->d_recvbuf, h->d_recv_ext, h->nrecv, vec, h->stream);
+    return CAGMRES_OK;
+}
+
+// ---- building blocks ------------------------------------------------------------------
+// C = X^T Y summed over ranks (out ld ldo); optional R = chol(C) (CholQR Gram)
+int xty_global(cagmres* h, const double* X, int64_t ldx, int jx, const double* Y, int64_t ldy,
+               int w, double* out, bool chol, double* R) {
+    if (h->nranks == 1) {
+        if (kern::xty(h->dev, h->n_loc, X, ldx, jx, Y, ldy, w, out, chol, R, h->status, h->ws, h->stream))
+            return CAGMRES_EINVAL;
+        return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
+    }
+    if (kern::xty(h->dev, h->n_loc, X, ldx, jx, Y, ldy, w, out, false, nullptr, h->status, h->ws, h->stream))
+        return CAGMRES_EINVAL;
+    TRY(allreduce(h, out, size_t(jx) * size_t(w)));
+    if (chol) kern::chol(out, w, R, h->status, h->stream);
+    return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
+}
+
+double spmv_bytes(cagmres* h, int64_t rows_out, int depth_in, bool pair2) {
+    // 12 nnz + 4 (r+1) + 8 r' + 8 r (+ 8 r for the pair's second step)
+    const int64_t r = rows_out;
+    int hh = 0;
+    while (hh < h->s && h->level_len[size_t(hh)] < r) ++hh;
+    const double nnz = double(h->nnz_prefix[size_t(std::min(hh, h->s))]);
+    const double rin = double(h->level_len[size_t(std::min(depth_in, h->s))]);
+    return 12.0 * nnz + 4.0 * double(r + 1) + 8.0 * rin + 8.0 * double(r) + (pair2 ? 8.0 * double(r) : 0.0);
+}
+
+// MPK of one block (Fig. 4): V[:, j+1 .. j+sb] from V[:, j].  Step k computes the rows at
+// distance <= sb-k (a prefix of the extended numbering) from the rows at distance <= sb-k+1.
+int mpk_block(cagmres* h, int j, int sb, const std::vector<host::Step>& steps) {
+    Scope sc(h, PH_MPK);
+    TRY(halo(h, h->V + size_t(h->ldv) * j, sb));
+    for (int k = 1; k <= sb; ++k) {
+        const host::Step& stp = steps[size_t(k - 1)];
+        const double* x = h->V + size_t(h->ldv) * (j + k - 1);
+        double* y = h->V + size_t(h->ldv) * (j + k);
+        const int64_t rows = h->level_len[size_t(sb - k)];
+        const bool pair2 = stp.kind == 2;
+        {
+            Scope sv(h, PH_SPMV);
+            kern::spmv(h->dev, h->A, rows, x, y, stp.a != 0.0 ? x : nullptr, -stp.a,
+                       pair2 ? h->V + size_t(h->ldv) * (j + k - 2) : nullptr, stp.b2, h->stream);
+        }
+        const double by = spmv_bytes(h, rows, sb - k + 1, pair2);
+        h->bytes[PH_MPK] += by;
+        h->bytes[PH_SPMV] += by;
+        h->spmv_launches++;
+    }
+    return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
+}
+
+// BOrth of the panel columns P (n_loc x w, ld ldp) against Q (n_loc x j): CGS or MGS
+// (P:144).  C: device j x w, ld j.
+int borth_panel(cagmres* h, const double* Q, int64_t ldq, int j, double* P, int64_t ldp, int w,
+                double* C, bool mgs) {
+    if (j <= 0) return CAGMRES_OK;
+    Scope sc(h, PH_BORTH);
+    if (!mgs) {
+        TRY(xty_global(h, Q, ldq, j, P, ldp, w, C, false, nullptr));
+        // C is jx x w with ld jx = j: xty writes ld jx
+        kern::update(h->dev, h->n_loc, Q, ldq, j, P, ldp, w, C, h->stream);
+        h->bytes[PH_BORTH] += 8.0 * double(h->n_loc) * (2.0 * j + 3.0 * w);
+    } else {
+        // row l of C (1 x w, ld j) via a scratch row then copied with ld j on the host view:
+        for (int l = 0; l < j; ++l) {
+            double* row = h->gbuf;
+            TRY(xty_global(h, Q + size_t(ldq) * l, ldq, 1, P, ldp, w, row, false, nullptr));
+            kern::update(h->dev, h->n_loc, Q + size_t(ldq) * l, ldq, 1, P, ldp, w, row, h->stream);
+            CU(cudaMemcpy2DAsync(C + l, sizeof(double) * size_t(j), row, sizeof(double), sizeof(double),
+                                 size_t(w), cudaMemcpyDeviceToDevice, h->stream));
+            h->bytes[PH_BORTH] += 8.0 * double(h->n_loc) * (2.0 + 3.0 * w);
+        }
+    }
+    return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
+}
+
+// TSQR of the panel P (n_loc x w, ld ldp), R (device w x w, ld w).  c0 = 1 leaves column 0
+// unwritten (the block's start vector q_j is kept, reading G2).
+int tsqr_panel(cagmres* h, double* P, int64_t ldp, int w, double* R, int kind, int c0) {
+    Scope sc(h, PH_TSQR);
+    const double nl = double(h->n_loc);
+    if (kind == CAGMRES_CHOLQR || kind == CAGMRES_SVQR) {
+        if (kind == CAGMRES_CHOLQR) {
+            TRY(xty_global(h, P, ldp, w, P, ldp, w, h->gbuf, true, R));     // B = V^T V ; R = chol(B)
+        } else {
+            TRY(xty_global(h, P, ldp, w, P, ldp, w, h->gbuf, false, nullptr));
+            kern::svqr_factor(h->gbuf, w, R, h->status, h->stream);
+        }
+        kern::trsm(h->dev, h->n_loc, P, ldp, w, R, c0, h->stream);          // V := V R^{-1}
+        h->bytes[PH_TSQR] += 8.0 * nl * (2.0 * w + double(w - c0));
+    } else {
+        CU(cudaMemsetAsync(R, 0, sizeof(double) * size_t(w) * size_t(w), h->stream));
+        for (int k = 0; k < w; ++k) {
+            double* pk = P + size_t(ldp) * k;
+            if (k > 0) {
+                if (kind == CAGMRES_CGS) {          // Fig. 9 right: r = V_{1:k-1}^T v_k
+                    TRY(xty_global(h, P, ldp, k, pk, ldp, 1, R + size_t(w) * k, false, nullptr));
+                    kern::update(h->dev, h->n_loc, P, ldp, k, pk, ldp, 1, R + size_t(w) * k, h->stream);
+                    h->bytes[PH_TSQR] += 8.0 * nl * (2.0 * k + 3.0);
+                } else {                             // Fig. 9 left: one dot at a time
+                    for (int l = 0; l < k; ++l) {
+                        double* rl = R + l + size_t(w) * k;
+                        TRY(xty_global(h, P + size_t(ldp) * l, ldp, 1, pk, ldp, 1, rl, false, nullptr));
+                        kern::update(h->dev, h->n_loc, P + size_t(ldp) * l, ldp, 1, pk, ldp, 1, rl, h->stream);
+                        h->bytes[PH_TSQR] += 8.0 * nl * 5.0;
+                    }
+                }
+            }
+            double* rkk = R + k + size_t(w) * k;
+            TRY(xty_global(h, pk, ldp, 1, pk, ldp, 1, h->gbuf, true, rkk));   // r_kk = ||v_k||
+            if (k >= c0) kern::trsm(h->dev, h->n_loc, pk, ldp, 1, rkk, 0, h->stream);
+            h->bytes[PH_TSQR] += 8.0 * nl * (k >= c0 ? 3.0 : 1.0);
+        }
+    }
+    return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
+}
+
+std::vector<Block> schedule(int s, int m) {
+    std::vector<Block> bl;
+    size_t off = 0;
+    for (int j = 0; j < m;) {
+        const int sb = std::min(s, m - j), w = sb + 1;
+        Block b{j, sb, 0, 0, 0, 0};
+        b.c1 = off; off += size_t(j) * size_t(sb);
+        b.r1 = off; off += size_t(w) * size_t(w);
+        b.c2 = off; off += size_t(j) * size_t(sb);
+        b.r2 = off; off += size_t(w) * size_t(w);
+        bl.push_back(b);
+        j += sb;
+    }
+    return bl;
+}
+
+// One CA cycle's GPU work: per block MPK -> BOrth -> TSQR [-> BOrth -> TSQR].
+int ca_cycle(cagmres* h, const std::vector<Block>& bl) {
+    const int kind = h->orth & CAGMRES_TSQR_MASK;
+    const bool re2 = (h->orth & CAGMRES_REORTH) != 0, mgs = (h->orth & CAGMRES_BORTH_MGS) != 0;
+    for (const Block& b : bl) {
+        const int j = b.j, sb = b.sb, w = sb + 1;
+        const std::vector<host::Step> steps = h->basis == CAGMRES_MONOMIAL
+            ? host::block_steps({}, {}, sb) : host::block_steps(h->sh_re, h->sh_im, sb);
+        TRY(mpk_block(h, j, sb, steps));
+        double* Pj = h->V + size_t(h->ldv) * j;                 // panel [q_j | W_1 .. W_sb]
+        for (int pass = 0; pass < (re2 ? 2 : 1); ++pass) {
+            double* C = h->tab + (pass ? b.c2 : b.c1);
+            double* R = h->tab + (pass ? b.r2 : b.r1);
+            TRY(borth_panel(h, h->V, h->ldv, j, Pj + h->ldv, h->ldv, sb, C, mgs));
+            TRY(tsqr_panel(h, Pj, h->ldv, w, R, kind, 1));
+        }
+    }
+    return CAGMRES_OK;
+}
+
+// First Newton cycle = GMRES(m) with CGS2 Arnoldi (reading G12), on the
+// same kernels with panel width 1.  tab layout: per k: c1 (m+1), c2 (m+1), r (1).
+int arnoldi_cycle(cagmres* h) {
+    const int m = h->m;
+    const size_t stride = 2 * size_t(m + 1) + 1;
+    for (int k = 0; k < m; ++k) {
+        double* vk = h->V + size_t(h->ldv) * k;
+        double* v = h->V + size_t(h->ldv) * (k + 1);
+        double* c1 = h->tab + stride * k;
+        double* c2 = c1 + (m + 1);
+        double* r = c2 + (m + 1);
+        {
+            Scope sc(h, PH_MPK);
+            TRY(halo(h, vk, 1));
+            Scope sv(h, PH_SPMV);
+            kern::spmv(h->dev, h->A, h->n_loc, vk, v, nullptr, 0.0, nullptr, 0.0, h->stream);
+            const double by = spmv_bytes(h, h->n_loc, 1, false);
+            h->bytes[PH_MPK] += by; h->bytes[PH_SPMV] += by; h->spmv_launches++;
+        }
+        TRY(borth_panel(h, h->V, h->ldv, k + 1, v, h->ldv, 1, c1, false));
+        TRY(borth_panel(h, h->V, h->ldv, k + 1, v, h->ldv, 1, c2, false));
+        TRY(tsqr_panel(h, v, h->ldv, 1, r, CAGMRES_CHOLQR, 0));
+    }
+    return CAGMRES_OK;
+}
+
+// residual r = b - A x into V[:,0]; returns ||r|| (host) and leaves r/||r|| in V[:,0].
+int residual_norm(cagmres* h, const double* b, const double* x, double* beta, bool scale) {
+    Scope sc(h, PH_OTHER);
+    const double* xx = x;
+    if (h->nranks > 1) {
+        CU(cudaMemcpyAsync(h->xe, x, sizeof(double) * size_t(h->n_loc), cudaMemcpyDeviceToDevice, h->stream));
+        TRY(halo(h, h->xe, 1));
+        xx = h->xe;
+    }
+    kern::residual(h->dev, h->A, h->n_loc, xx, b, h->V, h->stream);
+    double* rr = h->gbuf + 8;
+    TRY(xty_global(h, h->V, h->ldv, 1, h->V, h->ldv, 1, h->gbuf, true, rr));
+    CU(cudaMemcpyAsync(beta, rr, sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+    CU(cudaStreamSynchronize(h->stream));
+    if (scale && *beta > 0.0) kern::trsm(h->dev, h->n_loc, h->V, h->ldv, 1, rr, 0, h->stream);
+    h->bytes[PH_OTHER] += spmv_bytes(h, h->n_loc, 1, false) + 8.0 * double(h->n_loc) * (1.0 + (scale ? 2.0 : 0.0));
+    return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
+}
+
+void collect_timing(cagmres* h, cagmres_stats* st) {
+    double ms[PH_N] = {0, 0, 0, 0, 0};
+    for (auto& r : h->timer.rec) {
+        float t = 0.f;
+        cudaEventElapsedTime(&t, r.second.first, r.second.second);
+        ms[r.first] += double(t);
+    }
+    st->ms_mpk = ms[PH_MPK]; st->ms_borth = ms[PH_BORTH]; st->ms_tsqr = ms[PH_TSQR];
+    st->ms_other = ms[PH_OTHER]; st->ms_spmv = ms[PH_SPMV];
+    h->timer.reset();
+}
+
+}  // namespace
+
+// =======================================================================================
+// C ABI
+// =======================================================================================
+extern "C" {
+
+const char* cagmres_strerror(int s) {
+    switch (s) {
+        case CAGMRES_OK: return "ok";
+        case CAGMRES_NOT_CONVERGED: return "not converged within maxit restart cycles";
+        case CAGMRES_EINVAL: return "invalid argument";
+        case CAGMRES_ECUDA: return "CUDA error";
+        case CAGMRES_ENCCL: return "NCCL error";
+        case CAGMRES_EBREAKDOWN: return "numerical breakdown (Cholesky pivot <= 0 / zero norm)";
+        case CAGMRES_ENOMEM: return "out of memory";
+        case CAGMRES_EGHOST: return "supplied rows do not cover the ghost rows";
+        case CAGMRES_ENOTSUP: return "option not supported by this build";
+        default: return "unknown status";
+    }
+}
+
+int64_t cagmres_kernel_launches(void) { return int64_t(kern::g_launches); }
+
+int cagmres_create(cagmres_t* out, const cagmres_csr* A, int s, int m, int basis, int orth) {
+    if (!out || !A) return CAGMRES_EINVAL;
+    *out = nullptr;
+    if (A->row_begin != 0 || A->row_end != A->n || A->own_begin != 0 || A->own_end != A->n)
+        return CAGMRES_EINVAL;
+    cagmres* h = new (std::nothrow) cagmres();
+    if (!h) return CAGMRES_ENOMEM;
+    const int64_t rs[2] = {0, A->n};
+    const int st = init_common(h, A, rs, s, m, basis, orth);
+    if (st != CAGMRES_OK) { delete h; return st; }
+    *out = h;
+    return CAGMRES_OK;
+}
+
+int cagmres_create_dist(cagmres_t* out, const cagmres_csr* A, const int64_t* row_starts,
+                        int s, int m, int basis, int orth, const void* nccl_unique_id,
+                        int rank, int nranks, int cuda_device) {
+    if (!out || !A || !row_starts || !nccl_unique_id || nranks < 1 || rank < 0 || rank >= nranks)
+        return CAGMRES_EINVAL;
+    *out = nullptr;
+    if (cudaSetDevice(cuda_device) != cudaSuccess) return CAGMRES_ECUDA;
+    cagmres* h = new (std::nothrow) cagmres();
+    if (!h) return CAGMRES_ENOMEM;
+    h->rank = rank; h->nranks = nranks;
+    if (nranks > 1) {
+        ncclUniqueId id;
+        std::memcpy(&id, nccl_unique_id, sizeof(id));
+        if (ncclCommInitRank(&h->comm, nranks, id, rank) != ncclSuccess) { delete h; return CAGMRES_ENCCL; }
+    }
+    const int st = init_common(h, A, row_starts, s, m, basis, orth);
+    if (st != CAGMRES_OK) { delete h; return st; }
+    *out = h;
+    return CAGMRES_OK;
+}
+
+int cagmres_destroy(cagmres_t h) {
+    if (!h) return CAGMRES_OK;
+    cudaStreamSynchronize(h->stream);
+    delete h;
+    return CAGMRES_OK;
+}
+
+int cagmres_set_stream(cagmres_t h, void* s) {
+    if (!h) return CAGMRES_EINVAL;
+    h->stream = s ? static_cast<cudaStream_t>(s) : h->own_stream;
+    return CAGMRES_OK;
+}
+
+int cagmres_sizes(cagmres_t h, int64_t* n_loc, int64_t* n_ext, int64_t* ldv) {
+    if (!h) return CAGMRES_EINVAL;
+    if (n_loc) *n_loc = h->n_loc;
+    if (n_ext) *n_ext = h->n_ext;
+    if (ldv) *ldv = h->ldv;
+    return CAGMRES_OK;
+}
+
+int cagmres_set_shifts(cagmres_t h, const double* re, const double* im, int count) {
+    if (!h || !re || !im || count < 1) return CAGMRES_EINVAL;
+    for (int k = 0; k < count; ++k) {
+        if (im[k] > 0.0 && k + 1 < count && !(re[k + 1] == re[k] && im[k + 1] == -im[k])) return CAGMRES_EINVAL;
+        if (im[k] < 0.0 && (k == 0 || !(re[k - 1] == re[k] && im[k - 1] == -im[k]))) return CAGMRES_EINVAL;
+    }
+    h->sh_re.assign(re, re + count);
+    h->sh_im.assign(im, im + count);
+    h->have_shifts = true;
+    return CAGMRES_OK;
+}
+
+int cagmres_get_shifts(cagmres_t h, double* re, double* im, int cap, int* count) {
+    if (!h || !count) return CAGMRES_EINVAL;
+    *count = h->have_shifts ? int(h->sh_re.size()) : 0;
+    for (int k = 0; k < std::min(cap, *count); ++k) { re[k] = h->sh_re[size_t(k)]; im[k] = h->sh_im[size_t(k)]; }
+    return CAGMRES_OK;
+}
+
+int cagmres_mpk(cagmres_t h, const double* q, double* W, int64_t ldw, int sb) {
+    if (!h || !q || !W || sb < 1 || sb > h->s || ldw < h->n_loc || sb > h->m) return CAGMRES_EINVAL;
+    if (h->basis == CAGMRES_NEWTON && !h->have_shifts) return CAGMRES_EINVAL;
+    CU(cudaMemcpyAsync(h->V, q, sizeof(double) * size_t(h->n_loc), cudaMemcpyDeviceToDevice, h->stream));
+    const std::vector<host::Step> steps = h->basis == CAGMRES_MONOMIAL
+        ? host::block_steps({}, {}, sb) : host::block_steps(h->sh_re, h->sh_im, sb);
+    TRY(mpk_block(h, 0, sb, steps));
+    CU(cudaMemcpy2DAsync(W, sizeof(double) * size_t(ldw), h->V, sizeof(double) * size_t(h->ldv),
+                         sizeof(double) * size_t(h->n_loc), size_t(sb) + 1, cudaMemcpyDeviceToDevice, h->stream));
+    CU(cudaStreamSynchronize(h->stream));
+    h->timer.reset();
+    return CAGMRES_OK;
+}
+
+int cagmres_borth(cagmres_t h, const double* Q, int64_t ldq, int j, double* P, int64_t ldp,
+                  int w, double* C) {
+    if (!h || j < 0 || w < 1 || w > 32 || ldq < h->n_loc || ldp < h->n_loc) return CAGMRES_EINVAL;
+    if (j == 0) return CAGMRES_OK;
+    if (!Q || !P || !C || j > int(h->tab_cap)) return CAGMRES_EINVAL;
+    TRY(borth_panel(h, Q, ldq, j, P, ldp, w, C, (h->orth & CAGMRES_BORTH_MGS) != 0));
+    CU(cudaStreamSynchronize(h->stream));
+    h->timer.reset();
+    return CAGMRES_OK;
+}
+
+int cagmres_tsqr(cagmres_t h, double* P, int64_t ldp, int w, double* R, int orth) {
+    if (!h || !P || !R || w < 1 || w > 32 || ldp < h->n_loc) return CAGMRES_EINVAL;
+    const int kind = orth & CAGMRES_TSQR_MASK;
+    if (kind > CAGMRES_MGS) return kind == CAGMRES_CAQR ? CAGMRES_ENOTSUP : CAGMRES_EINVAL;
+    CU(cudaMemsetAsync(h->status, 0, sizeof(int), h->stream));
+    TRY(tsqr_panel(h, P, ldp, w, R, kind, 0));
+    if (orth & CAGMRES_REORTH) {
+        double* R2 = h->tab;                        // scratch
+        TRY(tsqr_panel(h, P, ldp, w, R2, kind, 0));
+        std::vector<double> r1(size_t(w) * w), r2(size_t(w) * w), rr(size_t(w) * w, 0.0);
+        CU(cudaMemcpyAsync(r1.data(), R, sizeof(double) * r1.size(), cudaMemcpyDeviceToHost, h->stream));
+        CU(cudaMemcpyAsync(r2.data(), R2, sizeof(double) * r2.size(), cudaMemcpyDeviceToHost, h->stream));
+        CU(cudaStreamSynchronize(h->stream));
+        for (int c = 0; c < w; ++c)
+            for (int i = 0; i <= c; ++i) {
+                double a = 0.0;
+                for (int k = i; k <= c; ++k) a += r2[size_t(i) + size_t(w) * k] * r1[size_t(k) + size_t(w) * c];
+                rr[size_t(i) + size_t(w) * c] = a;
+            }
+        CU(cudaMemcpyAsync(R, rr.data(), sizeof(double) * rr.size(), cudaMemcpyHostToDevice, h->stream));
+    }
+    int stat = 0;
+    CU(cudaMemcpyAsync(&stat, h->status, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+    CU(cudaStreamSynchronize(h->stream));
+    h->timer.reset();
+    return stat ? CAGMRES_EBREAKDOWN : CAGMRES_OK;
+}
+
+int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit, cagmres_stats* st) {
+    if (!h || !b || !x || maxit < 0 || !(tol >= 0.0)) return CAGMRES_EINVAL;
+    const int m = h->m;
+    h->timer.reset();
+    h->timer.on = st && st->collect_timing;
+    for (double& v : h->bytes) v = 0.0;
+    h->spmv_launches = 0;
+    if (st) { st->cycles = 0; st->iters = 0; st->hist_len = 0; }
+    cudaEvent_t t0 = nullptr, t1 = nullptr;
+    if (h->timer.on) { t0 = h->timer.get(); cudaEventRecord(t0, h->stream); }
+    CU(cudaMemsetAsync(h->status, 0, sizeof(int), h->stream));
+    double rho0 = 0.0, beta = 0.0;
+    TRY(residual_norm(h, b, x, &rho0, true));
+    beta = rho0;
+    int rc = CAGMRES_NOT_CONVERGED;
+    if (rho0 == 0.0) rc = CAGMRES_OK;
+    std::vector<double> H(static_cast<size_t>(m + 1) * static_cast<size_t>(m)), y(static_cast<size_t>(m)), htab(h->tab_cap);
+    const std::vector<Block> bl = schedule(h->s, m);
+    int cyc = 0;
+    for (; cyc < maxit && rc != CAGMRES_OK; ++cyc) {
+        const bool first_newton = h->basis == CAGMRES_NEWTON && !h->have_shifts;
+        std::fill(H.begin(), H.end(), 0.0);
+        if (first_newton) {
+            TRY(arnoldi_cycle(h));
+        } else {
+            TRY(ca_cycle(h, bl));
+        }
+        int stat = 0;
+        CU(cudaMemcpyAsync(htab.data(), h->tab, sizeof(double) * htab.size(), cudaMemcpyDeviceToHost, h->stream));
+        CU(cudaMemcpyAsync(&stat, h->status, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+        CU(cudaStreamSynchronize(h->stream));
+        if (stat) { rc = CAGMRES_EBREAKDOWN; break; }
+        // ---- Hessenberg matrix (host) ----
+        if (first_newton) {
+            const size_t stride = 2 * size_t(m + 1) + 1;
+            for (int k = 0; k < m; ++k) {
+                const double* c1 = htab.data() + stride * k;
+                for (int i = 0; i <= k; ++i) H[size_t(i) + size_t(m + 1) * k] = c1[i] + c1[i + m + 1];
+                H[size_t(k + 1) + size_t(m + 1) * k] = c1[2 * (m + 1)];
+            }
+        } else {
+            const bool re2 = (h->orth & CAGMRES_REORTH) != 0;
+            for (const Block& b0 : bl) {
+                const int j = b0.j, sb = b0.sb, w = sb + 1, nr = j + sb + 1;
+                std::vector<double> Rt(size_t(nr) * size_t(w), 0.0);
+                const double* C1 = htab.data() + b0.c1;
+                const double* R1 = htab.data() + b0.r1;
+                for (int c = 0; c < w; ++c) {
+                    for (int i = 0; i < j; ++i) Rt[size_t(i) + size_t(nr) * c] = c == 0 ? 0.0 : C1[size_t(i) + size_t(j) * (c - 1)];
+                    for (int i = 0; i <= c; ++i) Rt[size_t(j + i) + size_t(nr) * c] = R1[size_t(i) + size_t(w) * c];
+                }
+                if (re2) {   // C = C1 + C2 R1, R = R2 R1 (reading G16)
+                    const double* C2 = htab.data() + b0.c2;
+                    const double* R2 = htab.data() + b0.r2;
+                    std::vector<double> Rn(size_t(nr) * size_t(w), 0.0);
+                    for (int c = 0; c < w; ++c) {
+                        for (int i = 0; i < j; ++i) {
+                            double a = Rt[size_t(i) + size_t(nr) * c];
+                            for (int k = 1; k <= c; ++k) a += C2[size_t(i) + size_t(j) * (k - 1)] * R1[size_t(k) + size_t(w) * c];
+                            Rn[size_t(i) + size_t(nr) * c] = a;
+                        }
+                        for (int i = 0; i <= c; ++i) {
+                            double a = 0.0;
+                            for (int k = i; k <= c; ++k) a += R2[size_t(i) + size_t(w) * k] * R1[size_t(k) + size_t(w) * c];
+                            Rn[size_t(j + i) + size_t(nr) * c] = a;
+                        }
+                    }
+                    Rt.swap(Rn);
+                }
+                const std::vector<host::Step> steps = h->basis == CAGMRES_MONOMIAL
+                    ? host::block_steps({}, {}, sb) : host::block_steps(h->sh_re, h->sh_im, sb);
+                std::vector<double> B(size_t(w) * size_t(sb));
+                host::change_of_basis(steps, sb, B.data());
+                if (host::hessenberg_update(H.data(), m + 1, j, sb, Rt.data(), nr, B.data()) != CAGMRES_OK) {
+                    rc = CAGMRES_EBREAKDOWN;
+                    break;
+                }
+            }
+            if (rc == CAGMRES_EBREAKDOWN) break;
+        }
+        // ---- least squares + solution update ----
+        if (host::givens_ls(H.data(), m + 1, m, beta, y.data(), nullptr) != CAGMRES_OK) { rc = CAGMRES_EBREAKDOWN; break; }
+        for (double& v : y) v = -v;                              // update() subtracts X C
+        {
+            Scope sc(h, PH_OTHER);
+            CU(cudaMemcpyAsync(h->ybuf, y.data(), sizeof(double) * size_t(m), cudaMemcpyHostToDevice, h->stream));
+            kern::update(h->dev, h->n_loc, h->V, h->ldv, m, x, h->n_loc, 1, h->ybuf, h->stream);
+            h->bytes[PH_OTHER] += 8.0 * double(h->n_loc) * (m + 2.0);
+        }
+        if (first_newton) {                                      // Ritz values -> Leja shifts
+            std::vector<double> wr(static_cast<size_t>(m)), wi(static_cast<size_t>(m));
+            if (host::hessenberg_eigvals(H.data(), m + 1, m, wr.data(), wi.data()) != CAGMRES_OK) { rc = CAGMRES_EBREAKDOWN; break; }
+            host::modified_leja(wr.data(), wi.data(), m, h->s, h->sh_re, h->sh_im);
+            h->have_shifts = true;
+        }
+        double rho = 0.0;
+        TRY(residual_norm(h, b, x, &rho, true));
+        beta = rho;
+        if (st && st->rel_resid_hist && st->hist_len < st->hist_cap)
+            st->rel_resid_hist[st->hist_len++] = rho0 > 0.0 ? rho / rho0 : 0.0;
+        if (rho <= tol * rho0) rc = CAGMRES_OK;
+    }
+    if (h->timer.on) { t1 = h->timer.get(); cudaEventRecord(t1, h->stream); }
+    CU(cudaStreamSynchronize(h->stream));
+    if (st) {
+        st->cycles = cyc;
+        st->iters = cyc * m;
+        st->bytes_mpk = h->bytes[PH_MPK]; st->bytes_borth = h->bytes[PH_BORTH];
+        st->bytes_tsqr = h->bytes[PH_TSQR]; st->bytes_other = h->bytes[PH_OTHER];
+        st->bytes_spmv = h->bytes[PH_SPMV]; st->spmv_launches = h->spmv_launches;
+        st->ms_mpk = st->ms_borth = st->ms_tsqr = st->ms_other = st->ms_total = st->ms_spmv = 0.0;
+        if (h->timer.on) {
+            float tt = 0.f;
+            cudaEventElapsedTime(&tt, t0, t1);
+            st->ms_total = double(tt);
+            collect_timing(h, st);
+        }
+    }
+    h->timer.reset();
+    h->timer.on = false;
+    return rc;
+}
+
+}  // extern "C"

@@ -1,0 +1,160 @@
+"""CPU tests of the C-ABI library: every declared symbol is exported, and the host-only
+parts (setup plan, Ritz values, Leja order, change of basis, Hessenberg update, Givens LS)
+agree with the oracle / with dense linear algebra.  No compute call needs a GPU here."""
+import os
+import re
+
+import numpy as np
+import pytest
+
+from oracle import cagmres_oracle as O
+from synth import generators as G
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def lib():
+    from paper_conf_ipps_yamazakiathd14_b200 import _lib
+    return _lib.load()
+
+
+def declared_symbols():
+    src = open(os.path.join(ROOT, "include", "cagmres.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(cagmres_\w+)\s*\(", src)))
+
+
+def test_library_exports_every_declared_symbol(lib):
+    syms = declared_symbols()
+    assert len(syms) >= 25
+    for s in syms:
+        assert hasattr(lib, s), s
+
+
+def test_strerror_covers_codes(lib):
+    for code in (0, 1, -1, -2, -3, -4, -5, -6, -7):
+        assert lib.cagmres_strerror(code) not in (None, b"unknown status")
+
+
+def test_create_rejects_bad_arguments(lib):
+    import ctypes as C
+    from paper_conf_ipps_yamazakiathd14_b200 import _lib as L
+    from paper_conf_ipps_yamazakiathd14_b200.solver import _csr_struct
+    A = G.convection_diffusion(8, 2, 5)
+    st, keep = _csr_struct(A)
+    h = C.c_void_p()
+    assert lib.cagmres_create(C.byref(h), C.byref(st), 0, 10, L.NEWTON, L.CHOLQR) == L.EINVAL
+    assert lib.cagmres_create(C.byref(h), C.byref(st), 5, 4, L.NEWTON, L.CHOLQR) == L.EINVAL
+    assert lib.cagmres_create(C.byref(h), C.byref(st), 2, 4, 7, L.CHOLQR) == L.EINVAL
+    assert lib.cagmres_create(None, C.byref(st), 2, 4, L.NEWTON, L.CHOLQR) == L.EINVAL
+
+
+def test_host_eigvals_match_numpy():
+    from paper_conf_ipps_yamazakiathd14_b200 import host
+    A = G.convection_diffusion(16, 2, 5).to_scipy()
+    b = G.rhs(A.shape[0])
+    for m in (5, 12, 30):
+        _, H, _ = O.arnoldi_cgs2(A, b, m)
+        ev = np.sort_complex(host.eigvals(H[:m + 1, :m], m))
+        ref = np.sort_complex(np.linalg.eigvals(H[:m, :m]))
+        assert np.allclose(ev, ref, rtol=1e-10, atol=1e-10 * abs(ref).max())
+    # random Hessenberg with complex pairs
+    Hr = np.triu(G.random_panel(21, 20, 9), -1)
+    ev = np.sort_complex(host.eigvals(Hr, 20))
+    ref = np.sort_complex(np.linalg.eigvals(Hr[:20, :20]))
+    assert np.allclose(ev, ref, rtol=1e-9, atol=1e-9)
+    # conjugate pairs exact
+    assert np.all(np.isin(ev[ev.imag != 0], np.conj(ev[ev.imag != 0])))
+
+
+def test_host_leja_matches_oracle():
+    from paper_conf_ipps_yamazakiathd14_b200 import host
+    pts = np.array([3.0, -1.0 + 2.0j, -1.0 - 2.0j, 0.5, 2.0 + 0.5j, 2.0 - 0.5j, -2.5, 1.25])
+    for s in (1, 2, 3, 5, 8):
+        r1, i1 = host.leja(pts, s)
+        r2, i2 = O.modified_leja(pts, s)
+        assert np.array_equal(r1, r2) and np.array_equal(i1, i2)
+    A = G.convection_diffusion(32, 2, 5).to_scipy()
+    _, H, _ = O.arnoldi_cgs2(A, G.rhs(1024), 30)
+    th = np.linalg.eigvals(H[:30, :30])
+    r1, i1 = host.leja(th, 10)
+    r2, i2 = O.modified_leja(th, 10)
+    assert np.allclose(r1, r2) and np.allclose(i1, i2)
+
+
+@pytest.mark.parametrize("shifts", [([0.0] * 5, [0.0] * 5), ([1.0, 2.0, 2.0, 0.5, 4.0], [0.0, 1.0, -1.0, 0.0, 0.0]),
+                                    ([1.0, 2.0, 2.0, 3.0, 3.0], [0.0, 0.0, 0.0, 0.5, -0.5])])
+def test_host_change_of_basis_matches_oracle(shifts):
+    from paper_conf_ipps_yamazakiathd14_b200 import host
+    re_, im_ = map(np.array, shifts)
+    for sb in (1, 2, 4, 5):
+        assert np.array_equal(host.change_of_basis(re_, im_, sb), O.change_of_basis(sb, re_, im_))
+
+
+def test_host_hessenberg_update_and_ls_match_oracle():
+    from paper_conf_ipps_yamazakiathd14_b200 import host
+    A = G.convection_diffusion(32, 2, 5).to_scipy()
+    n, m, s = 1024, 12, 4
+    b = G.rhs(n)
+    Q = np.zeros((n, m + 1), order="F"); Q[:, 0] = b / np.linalg.norm(b)
+    H = np.zeros((m + 1, m))
+    Hc = np.zeros((m + 1, m), order="F")
+    re_, im_ = np.array([4.0, 1.0, 1.0, 6.0]), np.array([0.0, 0.5, -0.5, 0.0])
+    j = 0
+    while j < m:
+        sb = min(s, m - j)
+        W = O.mpk(A, Q[:, j], sb, re_, im_)
+        B = O.change_of_basis(sb, re_, im_)
+        C = np.zeros((j, sb + 1)); P = W.copy()
+        if j:
+            Cp, P[:, 1:] = O.borth_cgs(Q[:, :j], W[:, 1:]); C[:, 1:] = Cp
+        Qh, R = O.tsqr_cholqr(P)
+        Q[:, j + 1:j + sb + 1] = Qh[:, 1:]
+        Rt = np.vstack([C, R])
+        O.hessenberg_update(H, j, sb, Rt, B)
+        Hc = host.hessenberg_update(Hc, j, sb, Rt, B)
+        j += sb
+    assert np.allclose(Hc, H, rtol=1e-13, atol=1e-14)
+    y1, r1 = host.givens_ls(H, 3.0)
+    y2, r2 = O.givens_ls(H, 3.0)
+    assert np.allclose(y1, y2, rtol=1e-12) and np.allclose(r1, r2, rtol=1e-12)
+
+
+@pytest.mark.parametrize("gen,nr,s", [("cd5", 3, 3), ("g3", 4, 3), ("band", 2, 2), ("cd27", 3, 2)])
+def test_plan_levels_match_oracle_boundary_sets(gen, nr, s):
+    from paper_conf_ipps_yamazakiathd14_b200.host import Plan
+    A = {"cd5": lambda: G.convection_diffusion(20, 2, 5),
+         "g3": lambda: G.g3_shaped(n=3000, width=60),
+         "band": lambda: G.banded(n=2000),
+         "cd27": lambda: G.convection_diffusion(10, 3, 27)}[gen]()
+    As = A.to_scipy()
+    rs = O.block_rows(A.n, nr)
+    for r in range(nr):
+        p = Plan(A, rs, r, s)
+        lv = O.boundary_sets(As, rs[r], rs[r + 1], s)
+        ext = p.ext_rows()
+        assert np.array_equal(ext[:p.n_loc], np.arange(rs[r], rs[r + 1]))
+        for h in range(1, s + 1):
+            seg = ext[p.level_len[h - 1]:p.level_len[h]]
+            assert np.array_equal(seg, lv[h - 1])
+        # extended CSR rows = global rows with global-order columns mapped to extended ids
+        rp, ci, va = p.ext_csr()
+        assert p.n_mat == p.level_len[s - 1]
+        for e in np.linspace(0, p.n_mat - 1, 25).astype(int):
+            g = ext[e]
+            lo, hi = As.indptr[g], As.indptr[g + 1]
+            assert np.array_equal(ext[ci[rp[e]:rp[e + 1]]], As.indices[lo:hi])
+            assert np.array_equal(va[rp[e]:rp[e + 1]], As.data[lo:hi])
+
+
+def test_plan_reports_missing_ghost_rows():
+    from paper_conf_ipps_yamazakiathd14_b200 import _lib as L
+    from paper_conf_ipps_yamazakiathd14_b200.host import Plan
+    full = G.convection_diffusion(16, 2, 5)
+    rs = O.block_rows(full.n, 2)
+    part = G.convection_diffusion(16, 2, 5, rows=(0, rs[1] + 16))   # only 1 ghost row-plane
+    Plan(part, rs, 0, 2)                                            # s=2 needs 1 hop: fine
+    with pytest.raises(L.CagmresError) as e:
+        Plan(part, rs, 0, 3)                                        # s=3 needs 2 hops
+    assert e.value.status == L.EGHOST

@@ -1,0 +1,220 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the oracle on identical seeded inputs.
+
+Tolerances (from BASELINE.json north_star + SURVEY §8(c)):
+  MPK columns: |W_gpu - W_orc| <= 1e-12 * max|W_orc[:,k]| (FMA contraction / order only)
+  R, C (well conditioned): relative 1e-10
+  per-cycle rho: |rho_gpu - rho_orc| <= 1e-10 * rho_orc + 1e-15 (units of ||r0||)
+  restart cycles to 1e-8: +-1
+"""
+import numpy as np
+import pytest
+
+from oracle import cagmres_oracle as O
+from synth import generators as G
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _cuda():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_ipps_yamazakiathd14_b200 import _lib
+    _lib.load()
+    torch.cuda.set_device(0)
+
+
+def Solver(*a, **k):
+    from paper_conf_ipps_yamazakiathd14_b200.solver import Solver as S
+    return S(*a, **k)
+
+
+def dev(x):
+    return torch.tensor(np.ascontiguousarray(x), dtype=torch.float64, device="cuda")
+
+
+def colmajor(M):
+    """device column-major copy of a 2-D numpy array (stride(0) == 1)."""
+    return dev(np.asarray(M).T).t()
+
+
+def hist_close(h, ref, rtol=1e-10, atol=1e-15):
+    k = min(len(h), len(ref))
+    return np.all(np.abs(h[:k] - ref[:k]) <= rtol * ref[:k] + atol)
+
+
+SHIFTS = (np.array([7.9, 7.9, 0.09, 0.09, 3.8, 5.5, 1.2, 6.6, 2.5, 4.4]),
+          np.array([0.02, -0.02, 0.03, -0.03, 0.0, 0.0, 0.0, 0.0, 0.0, 0.0]))
+
+
+# ----------------------------------------------------------------------------- MPK
+@pytest.mark.parametrize("basis", ["monomial", "newton"])
+@pytest.mark.parametrize("gen", ["C1", "cd27_ragged", "g3_small"])
+def test_mpk_parity(basis, gen):
+    A = {"C1": lambda: G.convection_diffusion(32, 2, 5),
+         "cd27_ragged": lambda: G.convection_diffusion(13, 3, 27),       # n = 2197, ragged tail
+         "g3_small": lambda: G.g3_shaped(n=50001, width=250)}[gen]()
+    As = A.to_scipy()
+    s = 6
+    S = Solver(A, s=s, m=12, basis=basis)
+    re, im = (None, None)
+    if basis == "newton":
+        re, im = SHIFTS[0][:s], SHIFTS[1][:s]
+        S.set_shifts(re, im)
+    q = G.u(11, np.arange(A.n))
+    for sb in (1, 3, s):
+        W = S.mpk(dev(q), sb).cpu().numpy()
+        Wo = O.mpk(As, q, sb, re, im)
+        for k in range(sb + 1):
+            assert np.max(np.abs(W[:, k] - Wo[:, k])) <= 1e-12 * np.max(np.abs(Wo[:, k])), (sb, k)
+
+
+def test_mpk_newton_zero_shifts_bitwise_equals_monomial():
+    A = G.convection_diffusion(20, 3, 7)
+    q = dev(G.u(3, np.arange(A.n)))
+    S1 = Solver(A, s=5, m=10, basis="monomial")
+    S2 = Solver(A, s=5, m=10, basis="newton")
+    S2.set_shifts(np.zeros(5))
+    assert torch.equal(S1.mpk(q, 5), S2.mpk(q, 5))
+
+
+def test_mpk_full_size_C2():
+    """Config C2 at full size (n = 2,097,152) in the launch configuration bench.py times."""
+    A = G.convection_diffusion(128, 3, 7)
+    As = A.to_scipy()
+    S = Solver(A, s=10, m=30, basis="newton")
+    S.set_shifts(*SHIFTS)
+    q = G.rhs(A.n)
+    q /= np.linalg.norm(q)
+    W = S.mpk(dev(q), 10).cpu().numpy()
+    Wo = O.mpk(As, q, 10, *SHIFTS)
+    for k in range(11):
+        assert np.max(np.abs(W[:, k] - Wo[:, k])) <= 1e-12 * np.max(np.abs(Wo[:, k]))
+
+
+# ----------------------------------------------------------------------------- BOrth / TSQR
+@pytest.mark.parametrize("n,j,w", [(5000, 12, 6), (70001, 55, 5), (3000, 1, 1), (40000, 30, 11),
+                                   (1000, 70, 3)])
+def test_borth_parity(n, j, w):
+    A = G.convection_diffusion(10, 2, 5)                         # any handle works; rows = n
+    A = G.banded(n=n)
+    S = Solver(A, s=1, m=max(j, 1), basis="monomial")
+    Q, _ = np.linalg.qr(G.random_panel(n, j, 21))
+    P = G.random_panel(n, w, 22)
+    Qd, Pd = colmajor(Q), colmajor(P)
+    C = S.borth(Qd, j, Pd, w).cpu().numpy()
+    Co, Po = O.borth_cgs(Q, P)
+    assert np.allclose(C, Co, rtol=1e-10, atol=1e-12)
+    assert np.allclose(Pd.cpu().numpy(), Po, rtol=1e-10, atol=1e-12)
+
+
+@pytest.mark.parametrize("kind,reorth", [("cholqr", False), ("cholqr", True), ("svqr", False),
+                                         ("cgs", False), ("mgs", False)])
+@pytest.mark.parametrize("n,w", [(100003, 11), (777, 6), (4096, 1), (20000, 16)])
+def test_tsqr_parity(kind, reorth, n, w):
+    A = G.banded(n=n)
+    S = Solver(A, s=1, m=2, basis="monomial")
+    P = G.random_panel(n, w, 31)
+    if w > 2:
+        P[:, 2] += 0.3 * P[:, 1]
+    Pd = colmajor(P)
+    R = S.tsqr(Pd, w, kind, reorth).cpu().numpy()
+    Q = Pd.cpu().numpy()
+    _, Rr = np.linalg.qr(P)
+    Rr = np.sign(np.diag(Rr))[:, None] * Rr
+    assert np.allclose(R, Rr, rtol=1e-10, atol=1e-10 * np.abs(Rr).max())
+    assert O.orth_error(Q) < 1e-12
+    assert O.fact_error(P, Q, R) < 1e-13
+
+
+def test_tsqr_cholqr_breakdown_reported():
+    from paper_conf_ipps_yamazakiathd14_b200 import _lib as L
+    n = 5000
+    S = Solver(G.banded(n=n), s=1, m=2, basis="monomial")
+    P = G.random_panel(n, 4, 5)
+    P[:, 3] = P[:, 0] + P[:, 1]
+    with pytest.raises(L.CagmresError) as e:
+        S.tsqr(colmajor(P), 4, "cholqr")
+    assert e.value.status == L.EBREAKDOWN
+
+
+# ----------------------------------------------------------------------------- solve
+@pytest.mark.parametrize("basis,tsqr,reorth,borth", [
+    ("newton", "cholqr", False, "cgs"), ("monomial", "cholqr", False, "cgs"),
+    ("newton", "cholqr", True, "cgs"), ("newton", "svqr", False, "cgs"),
+    ("newton", "cgs", True, "cgs"), ("newton", "mgs", False, "mgs")])
+def test_solve_C1_injected_shifts(basis, tsqr, reorth, borth):
+    A = G.convection_diffusion(32, 2, 5)
+    As = A.to_scipy()
+    b = G.rhs(A.n)
+    S = Solver(A, s=5, m=30, basis=basis, tsqr=tsqr, reorth=reorth, borth=borth)
+    sh = None
+    if basis == "newton":
+        sh = O.modified_leja(O.ritz_values(O.arnoldi_cgs2(As, b, 30)[1], 30), 5)
+        S.set_shifts(*sh)
+    x, st = S.solve(dev(b), tol=1e-8, maxit=40)
+    ref = O.cagmres(As, b, 5, 30, basis=basis, tsqr=tsqr, reorth=reorth, borth=borth,
+                    tol=1e-8, shifts=sh)
+    assert st.status == 0
+    assert abs(st.cycles - ref["cycles"]) <= 1
+    assert hist_close(st.hist, ref["hist"])
+    xs = np.linalg.solve(As.toarray(), b)
+    assert np.linalg.norm(x.cpu().numpy() - xs) <= 1e-6 * np.linalg.norm(xs)
+
+
+def test_solve_C1_newton_first_cycle_gmres():
+    """Newton without preset shifts: cycle 1 is GMRES(m) on the GPU, its Ritz values (host
+    Francis QR) in Leja order become the shifts."""
+    A = G.convection_diffusion(32, 2, 5)
+    As = A.to_scipy()
+    b = G.rhs(A.n)
+    S = Solver(A, s=5, m=30, basis="newton")
+    x, st = S.solve(dev(b), tol=1e-8, maxit=40)
+    ref = O.cagmres(As, b, 5, 30, basis="newton", tol=1e-8)
+    re, im = S.get_shifts()
+    assert np.allclose(re[:5], ref["shifts"][0][:5], rtol=1e-8)
+    assert np.allclose(im[:5], ref["shifts"][1][:5], rtol=1e-8, atol=1e-12)
+    assert abs(st.cycles - ref["cycles"]) <= 1
+    assert hist_close(st.hist, ref["hist"])
+    g = O.gmres(As, b, 30, tol=1e-8)
+    assert abs(st.cycles - g["cycles"]) <= 1
+    assert np.all(np.diff(st.hist) <= 0)
+
+
+def test_solve_partial_last_block_and_ragged_n():
+    """(s, m) = (7, 30) -> blocks 7,7,7,7,2 (P:273 'generates 20 and then 10'); n = 2197."""
+    A = G.convection_diffusion(13, 3, 27)
+    As = A.to_scipy()
+    b = G.rhs(A.n)
+    S = Solver(A, s=7, m=30, basis="monomial", reorth=True)
+    x, st = S.solve(dev(b), tol=1e-10, maxit=20)
+    ref = O.cagmres(As, b, 7, 30, basis="monomial", reorth=True, tol=1e-10)
+    assert abs(st.cycles - ref["cycles"]) <= 1 and hist_close(st.hist, ref["hist"])
+
+
+def test_solve_g3_shaped_small():
+    A = G.g3_shaped(n=40000, width=200)
+    As = A.to_scipy()
+    b = G.rhs(A.n)
+    S = Solver(A, s=5, m=60, basis="newton")
+    x, st = S.solve(dev(b), tol=1e-8, maxit=200)
+    ref = O.cagmres(As, b, 5, 60, basis="newton", tol=1e-8, maxcyc=200)
+    assert abs(st.cycles - ref["cycles"]) <= 1
+    assert hist_close(st.hist, ref["hist"], rtol=1e-8)
+
+
+def test_solve_full_size_C2():
+    """Config C2 (bench workload) at full size: per-cycle residuals vs the oracle."""
+    A = G.convection_diffusion(128, 3, 7)
+    As = A.to_scipy()
+    b = G.rhs(A.n)
+    S = Solver(A, s=10, m=30, basis="newton")
+    x, st = S.solve(dev(b), tol=1e-8, maxit=60)
+    ref = O.cagmres(As, b, 10, 30, basis="newton", tol=1e-8, maxcyc=60)
+    assert st.status == 0
+    assert abs(st.cycles - ref["cycles"]) <= 1
+    assert hist_close(st.hist, ref["hist"], rtol=1e-8)
+    r = b - As @ x.cpu().numpy()
+    assert np.linalg.norm(r) <= 1.01e-8 * np.linalg.norm(b)
