@@ -16,6 +16,7 @@
 #include <cstdio>
 
 #include "kernels.h"
+#include "dense_dev.cuh"
 
 namespace kern {
 
@@ -83,26 +84,6 @@ void residual(const Dev& d, const Sell& A, int64_t nrows, const double* x, const
 // ------------------------------------------------------------------------------------
 // Small dense factorizations on one thread / one CTA (w <= 32).
 // ------------------------------------------------------------------------------------
-__device__ void chol_upper_serial(const double* G, int ldg, int w, double* R, int* status) {
-    // R^T R = G (upper R, positive diagonal), row-oriented: R[k,c] for c >= k.
-    bool bad = false;
-    for (int k = 0; k < w; ++k) {
-        double dkk = G[k + ldg * k];
-        for (int i = 0; i < k; ++i) dkk = fma(-R[i + w * k], R[i + w * k], dkk);
-        if (!(dkk > 0.0)) { bad = true; dkk = DBL_MIN; }
-        const double rkk = sqrt(dkk);
-        const double inv = 1.0 / rkk;
-        R[k + w * k] = rkk;
-        for (int c = k + 1; c < w; ++c) {
-            double v = G[k + ldg * c];
-            for (int i = 0; i < k; ++i) v = fma(-R[i + w * k], R[i + w * c], v);
-            R[k + w * c] = v * inv;
-        }
-        for (int c = 0; c < k; ++c) R[k + w * c] = 0.0;
-    }
-    if (bad) atomicOr(status, ST_CHOL);
-}
-
 __global__ void k_chol(const double* G, int w, double* R, int* status) {
     if (threadIdx.x == 0) chol_upper_serial(G, w, w, R, status);
 }
@@ -194,290 +175,6 @@ __global__ void k_svqr(const double* G, int w, double* R, int* status) {
 
 void svqr_factor(const double* G, int w, double* R, int* status, cudaStream_t st) {
     ++g_launches; k_svqr<<<1, 32, 0, st>>>(G, w, R, status);
-}
-
-// ------------------------------------------------------------------------------------
-// K4/K5: C = X^T Y for tall-skinny X (n x jx) and Y (n x w).
-// A CTA walks 256-row tiles (grid-stride).  The Y tile is staged in shared memory (it is
-// needed by every column group); X is read straight from global memory into registers,
-// each element feeding w FMAs.  Threads form G groups of TR = 256/G row-lanes: group g
-// owns X columns g, g+G, ..., (JB of them) of this blockIdx.y chunk, lane rl owns rows
-// rl, rl+TR, ... of the tile.  Per-thread accumulators acc[JB][WM] persist over all tiles;
-// at the end they are reduced over the TR lanes of each group in a fixed order, the CTA's
-// partial is stored, and the LAST CTA to finish (atomic ticket) sums all partials in a
-// fixed order (deterministic, run-to-run bitwise reproducible) and optionally factors the
-// Gram matrix (fin_chol) — one launch per Gram + Cholesky.
-// ------------------------------------------------------------------------------------
-struct XtyArgs {
-    int64_t n;
-    const double* X; int64_t ldx; int jx;
-    const double* Y; int64_t ldy; int w;
-    int G, chunk;               // groups per CTA, X columns per blockIdx.y chunk (= G*JB)
-    double* part;
-    double* out;                // jx x w, ld jx
-    unsigned int* counter;
-    int fin_chol;
-    double* R;
-    int* status;
-};
-
-constexpr int XTY_TS = 256;
-
-template <int JB, int WM>
-__global__ void __launch_bounds__(NT, 1) k_xty(XtyArgs a) {
-    extern __shared__ double sm[];                 // WM x XTY_TS, column-major
-    __shared__ bool s_last;
-    const int G = a.G, TR = NT / G;
-    const int tid = threadIdx.x, g = tid / TR, rl = tid - g * TR;
-    const int w = a.w;
-    const int colbase = blockIdx.y * a.chunk;
-    const double* xcol[JB];
-    bool xok[JB];
-#pragma unroll
-    for (int jb = 0; jb < JB; ++jb) {
-        const int il = g + G * jb;
-        const int i = colbase + il;
-        xok[jb] = (il < a.chunk) && (i < a.jx);
-        xcol[jb] = a.X + (xok[jb] ? int64_t(i) * a.ldx : 0);
-    }
-    double acc[JB][WM];
-#pragma unroll
-    for (int jb = 0; jb < JB; ++jb)
-#pragma unroll
-        for (int c = 0; c < WM; ++c) acc[jb][c] = 0.0;
-
-    const int64_t ntiles = (a.n + XTY_TS - 1) / XTY_TS;
-    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
-        const int64_t r0 = t * XTY_TS;
-        const int rows = int(min(int64_t(XTY_TS), a.n - r0));
-        __syncthreads();
-        for (int idx = tid; idx < w * XTY_TS; idx += NT) {
-            const int c = idx / XTY_TS, r = idx - c * XTY_TS;
-            sm[idx] = (r < rows) ? __ldg(a.Y + r0 + r + a.ldy * c) : 0.0;
-        }
-        __syncthreads();
-#pragma unroll 2
-        for (int r = rl; r < rows; r += TR) {
-            double xv[JB];
-#pragma unroll
-            for (int jb = 0; jb < JB; ++jb) xv[jb] = xok[jb] ? __ldg(xcol[jb] + r0 + r) : 0.0;
-            double p[WM];
-#pragma unroll
-            for (int c = 0; c < WM; ++c) p[c] = (c < w) ? sm[c * XTY_TS + r] : 0.0;
-#pragma unroll
-            for (int jb = 0; jb < JB; ++jb)
-#pragma unroll
-                for (int c = 0; c < WM; ++c) acc[jb][c] = fma(xv[jb], p[c], acc[jb][c]);
-        }
-    }
-    // ---- CTA reduction over the TR row-lanes of each group (fixed order) ----
-    double* part = a.part + (int64_t(blockIdx.y) * gridDim.x + blockIdx.x) * int64_t(a.chunk) * w;
-#pragma unroll
-    for (int jb = 0; jb < JB; ++jb) {
-        __syncthreads();
-#pragma unroll
-        for (int c = 0; c < WM; ++c)
-            if (c < w) sm[c * NT + tid] = acc[jb][c];
-        __syncthreads();
-        for (int e = tid; e < G * w; e += NT) {
-            const int g2 = e % G, c = e / G;
-            const int il = g2 + G * jb;
-            if (il >= a.chunk) continue;
-            double s = 0.0;
-            const double* src = sm + c * NT + g2 * TR;
-            for (int q = 0; q < TR; ++q) s += src[q];
-            part[il + int64_t(a.chunk) * c] = s;
-        }
-    }
-    // ---- last CTA: deterministic sum of all partials (+ optional Cholesky) ----
-    __threadfence();
-    __syncthreads();
-    if (tid == 0) {
-        const unsigned total = gridDim.x * gridDim.y;
-        s_last = (atomicAdd(a.counter, 1u) == total - 1);
-    }
-    __syncthreads();
-    if (!s_last) return;
-    __threadfence();
-    const int jx = a.jx;
-    for (int e = tid; e < jx * w; e += NT) {
-        const int i = e % jx, c = e / jx;
-        const int by = i / a.chunk, il = i - by * a.chunk;
-        const double* src = a.part + int64_t(by) * gridDim.x * int64_t(a.chunk) * w + il + int64_t(a.chunk) * c;
-        double s = 0.0;
-        for (unsigned bx = 0; bx < gridDim.x; ++bx) s += __ldcg(src + int64_t(bx) * a.chunk * w);
-        a.out[i + int64_t(jx) * c] = s;
-    }
-    if (tid == 0) *a.counter = 0u;                 // ready for the next launch (stream order)
-    if (a.fin_chol) {
-        __syncthreads();
-        if (tid == 0) chol_upper_serial(a.out, jx, w, a.R, a.status);
-    }
-}
-
-struct XtyCfg { int JB, WM; };
-
-static XtyCfg xty_cfg(int w) {
-    if (w <= 1) return {4, 1};
-    if (w <= 2) return {4, 2};
-    if (w <= 4) return {4, 4};
-    if (w <= 8) return {4, 8};
-    if (w <= 12) return {4, 12};
-    if (w <= 16) return {4, 16};
-    return {2, 32};
-}
-
-static void xty_geometry(const Dev& d, int64_t n, int jx, int w, int* G, int* chunk, int* gx, int* gy) {
-    const XtyCfg cf = xty_cfg(w);
-    int need = (jx + cf.JB - 1) / cf.JB;
-    int g = 1;
-    while (g < need && g < 16) g *= 2;
-    *G = g;
-    *chunk = g * cf.JB;
-    *gy = (jx + *chunk - 1) / *chunk;
-    const int64_t ntiles = (n + XTY_TS - 1) / XTY_TS;
-    int64_t want = int64_t(d.sms) * 2 / *gy;       // ~2 CTAs per SM in total (1 resident)
-    if (want < 1) want = 1;
-    if (want > ntiles) want = ntiles;
-    if (want < 1) want = 1;
-    *gx = int(want);
-}
-
-size_t xty_ws_doubles(const Dev& d, int jx, int w) {
-    int G, chunk, gx, gy;
-    xty_geometry(d, int64_t(1) << 40, jx, w, &G, &chunk, &gx, &gy);
-    return size_t(gx) * size_t(gy) * size_t(chunk) * size_t(w);
-}
-
-template <int JB, int WM>
-static void launch_xty(const XtyArgs& a, int gx, int gy, cudaStream_t st) {
-    const size_t smem = size_t(WM) * XTY_TS * sizeof(double);
-    static bool attr = false;
-    if (!attr) {
-        cudaFuncSetAttribute(k_xty<JB, WM>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
-        attr = true;
-    }
-    ++g_launches; k_xty<JB, WM><<<dim3(gx, gy), NT, smem, st>>>(a);
-}
-
-int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const double* Y,
-        int64_t ldy, int w, double* out, bool fin_chol, double* R, int* status,
-        const XtyWs& ws, cudaStream_t st) {
-    if (jx <= 0 || w <= 0 || w > 32) return -1;
-    int G, chunk, gx, gy;
-    xty_geometry(d, n, jx, w, &G, &chunk, &gx, &gy);
-    if (size_t(gx) * gy * chunk * w > ws.cap) return -1;
-    XtyArgs a{n, X, ldx, jx, Y, ldy, w, G, chunk, ws.part, out, ws.counter, fin_chol ? 1 : 0, R, status};
-    const XtyCfg cf = xty_cfg(w);
-    switch (cf.WM) {
-        case 1: launch_xty<4, 1>(a, gx, gy, st); break;
-        case 2: launch_xty<4, 2>(a, gx, gy, st); break;
-        case 4: launch_xty<4, 4>(a, gx, gy, st); break;
-        case 8: launch_xty<4, 8>(a, gx, gy, st); break;
-        case 12: launch_xty<4, 12>(a, gx, gy, st); break;
-        case 16: launch_xty<4, 16>(a, gx, gy, st); break;
-        default: launch_xty<2, 32>(a, gx, gy, st); break;
-    }
-    return 0;
-}
-
-// ------------------------------------------------------------------------------------
-// K9: P[:, 0:w] -= X C   (row-wise; C broadcast from shared memory)
-// ------------------------------------------------------------------------------------
-template <int WM>
-__global__ void __launch_bounds__(NT) k_update(int64_t n, const double* __restrict__ X, int64_t ldx,
-                                               int jx, double* __restrict__ P, int64_t ldp, int w,
-                                               const double* __restrict__ C) {
-    extern __shared__ double sC[];                 // jx x WM (row i contiguous: i*WM + c)
-    for (int e = threadIdx.x; e < jx * WM; e += NT) {
-        const int i = e / WM, c = e - i * WM;
-        sC[e] = (c < w) ? C[i + int64_t(jx) * c] : 0.0;
-    }
-    __syncthreads();
-    for (int64_t r = int64_t(blockIdx.x) * NT + threadIdx.x; r < n; r += int64_t(gridDim.x) * NT) {
-        double acc[WM];
-#pragma unroll
-        for (int c = 0; c < WM; ++c) acc[c] = (c < w) ? P[r + ldp * c] : 0.0;
-#pragma unroll 8
-        for (int i = 0; i < jx; ++i) {
-            const double x = __ldg(X + r + ldx * i);
-#pragma unroll
-            for (int c = 0; c < WM; ++c) acc[c] = fma(-x, sC[i * WM + c], acc[c]);
-        }
-#pragma unroll
-        for (int c = 0; c < WM; ++c)
-            if (c < w) P[r + ldp * c] = acc[c];
-    }
-}
-
-static int grid_stream(const Dev& d, int64_t n, int per_sm) {
-    int64_t g = (n + NT - 1) / NT;
-    const int64_t cap = int64_t(d.sms) * per_sm;
-    if (g > cap) g = cap;
-    return int(g < 1 ? 1 : g);
-}
-
-void update(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, double* P,
-            int64_t ldp, int w, const double* C, cudaStream_t st) {
-    if (jx <= 0 || n <= 0) return;
-    const int grid = grid_stream(d, n, 8);
-    auto go = [&](auto kfn, int WM) {
-        const size_t smem = size_t(jx) * WM * sizeof(double);
-        if (smem > 48 * 1024) cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
-        ++g_launches;
-        kfn<<<grid, NT, smem, st>>>(n, X, ldx, jx, P, ldp, w, C);
-    };
-    if (w <= 1) go(k_update<1>, 1);
-    else if (w <= 2) go(k_update<2>, 2);
-    else if (w <= 4) go(k_update<4>, 4);
-    else if (w <= 8) go(k_update<8>, 8);
-    else if (w <= 12) go(k_update<12>, 12);
-    else if (w <= 16) go(k_update<16>, 16);
-    else go(k_update<32>, 32);
-}
-
-// ------------------------------------------------------------------------------------
-// K8: P[:, c0:w] = (P R^{-1})[:, c0:w], forward substitution per row with 1/R_cc.
-// ------------------------------------------------------------------------------------
-template <int WM>
-__global__ void __launch_bounds__(NT) k_trsm(int64_t n, double* __restrict__ P, int64_t ldp, int w,
-                                             const double* __restrict__ R, int c0) {
-    __shared__ double sR[WM * WM];
-    __shared__ double sInv[WM];
-    for (int e = threadIdx.x; e < WM * WM; e += NT) {
-        const int k = e / WM, c = e - k * WM;     // sR[k*WM + c] = R[k, c]
-        sR[e] = (k < w && c < w) ? R[k + int64_t(w) * c] : 0.0;
-    }
-    for (int c = threadIdx.x; c < WM; c += NT) sInv[c] = (c < w) ? 1.0 / R[c + int64_t(w) * c] : 0.0;
-    __syncthreads();
-    for (int64_t r = int64_t(blockIdx.x) * NT + threadIdx.x; r < n; r += int64_t(gridDim.x) * NT) {
-        double p[WM];
-#pragma unroll
-        for (int c = 0; c < WM; ++c) p[c] = (c < w) ? P[r + ldp * c] : 0.0;
-#pragma unroll
-        for (int c = 0; c < WM; ++c) {
-            double x = p[c];
-#pragma unroll
-            for (int k = 0; k < c; ++k) x = fma(-p[k], sR[k * WM + c], x);
-            p[c] = x * sInv[c];
-        }
-#pragma unroll
-        for (int c = 0; c < WM; ++c)
-            if (c >= c0 && c < w) P[r + ldp * c] = p[c];
-    }
-}
-
-void trsm(const Dev& d, int64_t n, double* P, int64_t ldp, int w, const double* R, int c0,
-          cudaStream_t st) {
-    if (n <= 0) return;
-    const int grid = grid_stream(d, n, 8);
-    if (w <= 1) { ++g_launches; k_trsm<1><<<grid, NT, 0, st>>>(n, P, ldp, w, R, c0); }
-    else if (w <= 2) { ++g_launches; k_trsm<2><<<grid, NT, 0, st>>>(n, P, ldp, w, R, c0); }
-    else if (w <= 4) { ++g_launches; k_trsm<4><<<grid, NT, 0, st>>>(n, P, ldp, w, R, c0); }
-    else if (w <= 8) { ++g_launches; k_trsm<8><<<grid, NT, 0, st>>>(n, P, ldp, w, R, c0); }
-    else if (w <= 12) { ++g_launches; k_trsm<12><<<grid, NT, 0, st>>>(n, P, ldp, w, R, c0); }
-    else if (w <= 16) { ++g_launches; k_trsm<16><<<grid, NT, 0, st>>>(n, P, ldp, w, R, c0); }
-    else { ++g_launches; k_trsm<32><<<grid, NT, 0, st>>>(n, P, ldp, w, R, c0); }
 }
 
 // ------------------------------------------------------------------------------------

@@ -147,7 +147,8 @@ class Solver:
         if t.dim() == 1:
             return t.data_ptr(), max(rows, 1)
         assert t.stride(0) == 1, "expect column-major (stride(0) == 1)"
-        return t.data_ptr(), t.stride(1)
+        # torch reports stride 1 for a size-1 dimension: a single column has ld = its rows
+        return t.data_ptr(), (t.stride(1) if t.size(1) > 1 else max(t.size(0), rows))
 
     def mpk(self, q, sb, out=None):
         import torch

@@ -95,11 +95,10 @@ def test_mpk_full_size_C2():
 
 
 # ----------------------------------------------------------------------------- BOrth / TSQR
-@pytest.mark.parametrize("n,j,w", [(5000, 12, 6), (70001, 55, 5), (3000, 1, 1), (40000, 30, 11),
-                                   (1000, 70, 3)])
+@pytest.mark.parametrize("n,j,w", [(5000, 12, 6), (70002, 55, 5), (3000, 1, 1), (40000, 30, 11),
+                                   (1000, 70, 3), (70001, 7, 4), (262144, 20, 10)])
 def test_borth_parity(n, j, w):
-    A = G.convection_diffusion(10, 2, 5)                         # any handle works; rows = n
-    A = G.banded(n=n)
+    A = G.banded(n=n)                                            # any matrix with n rows
     S = Solver(A, s=1, m=max(j, 1), basis="monomial")
     Q, _ = np.linalg.qr(G.random_panel(n, j, 21))
     P = G.random_panel(n, w, 22)
@@ -112,7 +111,7 @@ def test_borth_parity(n, j, w):
 
 @pytest.mark.parametrize("kind,reorth", [("cholqr", False), ("cholqr", True), ("svqr", False),
                                          ("cgs", False), ("mgs", False)])
-@pytest.mark.parametrize("n,w", [(100003, 11), (777, 6), (4096, 1), (20000, 16)])
+@pytest.mark.parametrize("n,w", [(100002, 11), (100003, 11), (777, 6), (4096, 1), (20000, 16), (65538, 13)])
 def test_tsqr_parity(kind, reorth, n, w):
     A = G.banded(n=n)
     S = Solver(A, s=1, m=2, basis="monomial")
