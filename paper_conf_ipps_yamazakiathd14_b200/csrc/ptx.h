@@ -1,5 +1,6 @@
 // ptx.h — sm_100a inline-PTX helpers: mbarrier + 1-D bulk async copies (TMA engine,
-// SASS UBLKCP) used to stream tall-skinny panel tiles into shared memory.
+// SASS UBLKCP) used to stream tall-skinny panel tiles into shared memory, and the FP64
+// tensor-core MMA (DMMA, mma.sync m8n8k4 f64).
 #pragma once
 #include <cstdint>
 
@@ -46,6 +47,14 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         "}\n" ::"r"(smem_u32(bar)),
         "r"(parity)
         : "memory");
+}
+
+// D(8x8) += A(8x4) B(4x8) in FP64 on the tensor core.  Fragments (lane = 4*gid + tig):
+//   a = A[gid][tig], b = B[tig][gid], d0 = D[gid][2*tig], d1 = D[gid][2*tig+1].
+__device__ __forceinline__ void dmma(double& d0, double& d1, double a, double b) {
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+                 : "+d"(d0), "+d"(d1)
+                 : "d"(a), "d"(b));
 }
 
 }  // namespace ptx

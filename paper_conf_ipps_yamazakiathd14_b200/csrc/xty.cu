@@ -2,19 +2,21 @@
 //   * BOrth pass 1: C = Q[:,0:j]^T P            ("MAGMA tall-skinny DGEMV")
 //   * CholQR Gram:  B = V^T V, then R = chol(B)  ("batched DGEMM")
 //
-// Main path (k_xty_tma): a persistent CTA per SM streams full row tiles of every needed
-// column into a 4-stage shared-memory ring with 1-D bulk async copies (the TMA engine,
-// cp.async.bulk + mbarrier complete_tx), so ~100 KB per SM is in flight without holding
-// registers — the tall-skinny panel is read from HBM exactly once.  Threads then compute
-// from shared memory with per-thread register accumulators that persist over all tiles:
-//   SYM  (Gram, w <= 12): every thread owns whole rows and accumulates the full upper
-//        triangle w(w+1)/2 in registers (one smem load per operand, ~w/2 FMAs per load);
-//   general: G groups x TR row-lanes; group g owns X columns g, g+G, .. (JB of them),
-//        loads its rows' w Y-values once and feeds JB*w FMAs.
-// At the end a fixed-order warp-butterfly + smem reduction produces the CTA partial, and
-// the LAST CTA (atomic ticket) sums all partials in a fixed order (run-to-run bitwise
-// reproducible) and, for CholQR on one GPU, factors the Gram in the same launch.
-// Fallback (k_xty_ldg): register loads, used only when a user panel is not 16-B aligned.
+// Main path (k_xty_mma): a persistent CTA per SM streams full row tiles of every needed
+// column into a 4-stage shared-memory ring with 1-D bulk async copies (TMA engine,
+// cp.async.bulk + mbarrier complete_tx): ~100 KB per SM in flight without holding
+// registers, so the panel is read from HBM exactly once at full rate.  The contraction over
+// rows runs on the FP64 tensor core: each warp owns a slice of the tile's rows and issues
+// mma.sync.m8n8k4.f64 (256 FMAs per warp instruction) for all 8x8 output tiles of its CTA's
+// column chunk — with scalar DFMA the kernel was issue-bound at 8 warps/SM (ncu: 107 M
+// instructions, 0.7 IPC); DMMA cuts the instruction count ~15x at the same FLOP rate.
+// Column stride in shared memory is TS+4 doubles (== 4 mod 16) so the 8-column x 4-row
+// fragment loads are bank-conflict free.  Gram (X == Y): A and B fragments coincide and
+// only the upper block triangle is multiplied.
+// At the end a fixed-order smem reduction over warps produces the CTA partial, and the LAST
+// CTA (atomic ticket) sums all partials in a fixed order (run-to-run bitwise reproducible)
+// and, for CholQR on one GPU, factors the Gram in the same launch.
+// Fallback (k_xty_ldg): register loads, used when a user panel is not 16-B aligned.
 #include <cstdint>
 
 #include "dense_dev.cuh"
@@ -25,6 +27,7 @@ namespace kern {
 
 namespace {
 constexpr int NT = 256;
+constexpr int NWARP = NT / 32;
 constexpr int XTY_STAGES = 4;
 constexpr int XTY_STAGE_BYTES = 32 * 1024;
 }
@@ -34,9 +37,9 @@ struct XtyArgs {
     const double* X; int64_t ldx; int jx;
     const double* Y; int64_t ldy; int w;
     int same;                   // X == Y (and jx == w): X columns come from the Y tile
-    int G, chunk;               // groups per CTA, X columns per blockIdx.y chunk (= G*JB)
+    int G, chunk;               // fallback: groups per CTA; X columns per blockIdx.y chunk
     int TS;                     // rows per tile (TMA path)
-    double* part;               // per-CTA partials
+    double* part;               // per-CTA partials (chunk x w each)
     double* out;                // jx x w, ld jx
     unsigned int* counter;
     int fin_chol;
@@ -73,70 +76,56 @@ __device__ __forceinline__ void xty_finish(const XtyArgs& a, int nent_cta) {
 }
 
 // ======================================================================================
-// TMA-pipelined kernel
+// TMA ring + DMMA kernel.  MT = 8-column tiles of X per chunk (chunk = 8*MT), NTN = 8-col
+// tiles of Y.  SYM: X == Y, MT == NTN, upper block triangle only.
 // ======================================================================================
-template <int JB, int WM, bool SYM>
-__device__ __forceinline__ void xty_rows(const XtyArgs& a, double (&acc)[SYM ? WM * (WM + 1) / 2 : JB * WM],
-                                         const double* Yb, int64_t ldY, const double* Xb, int64_t ldX,
-                                         int rows, int g, int rl, int TR, const bool (&xok)[JB],
-                                         const int (&xoff)[JB]) {
-    const int w = a.w;
+template <int MT, int NTN, bool SYM>
+__device__ __forceinline__ void xty_kstep(double (&acc)[MT][NTN][2], const double* Ys, int64_t ldY,
+                                          const double* Xs, int64_t ldX, int64_t row, int lane, int w,
+                                          int nxc, bool valid) {
+    const int gid = lane >> 2;
+    double bn[NTN];
+#pragma unroll
+    for (int nt = 0; nt < NTN; ++nt) {
+        const int c = min(8 * nt + gid, w - 1);
+        bn[nt] = valid ? Ys[row + ldY * c] : 0.0;
+    }
     if constexpr (SYM) {
-        for (int r = threadIdx.x; r < rows; r += NT) {
-            double p[WM];
 #pragma unroll
-            for (int c = 0; c < WM; ++c) p[c] = (c < w) ? Yb[r + ldY * c] : 0.0;
-            int idx = 0;
+        for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
-            for (int i = 0; i < WM; ++i)
-#pragma unroll
-                for (int c = i; c < WM; ++c) { acc[idx] = fma(p[i], p[c], acc[idx]); ++idx; }
-        }
+            for (int nt = mt; nt < NTN; ++nt) ptx::dmma(acc[mt][nt][0], acc[mt][nt][1], bn[mt], bn[nt]);
     } else {
-        for (int r = rl; r < rows; r += TR) {
-            double p[WM];
 #pragma unroll
-            for (int c = 0; c < WM; ++c) p[c] = (c < w) ? Yb[r + ldY * c] : 0.0;
-            double xv[JB];
+        for (int mt = 0; mt < MT; ++mt) {
+            const int c = min(8 * mt + gid, nxc - 1);
+            const double am = valid ? Xs[row + ldX * c] : 0.0;
 #pragma unroll
-            for (int jb = 0; jb < JB; ++jb) xv[jb] = xok[jb] ? Xb[r + ldX * xoff[jb]] : 0.0;
-#pragma unroll
-            for (int jb = 0; jb < JB; ++jb)
-#pragma unroll
-                for (int c = 0; c < WM; ++c) acc[jb * WM + c] = fma(xv[jb], p[c], acc[jb * WM + c]);
+            for (int nt = 0; nt < NTN; ++nt) ptx::dmma(acc[mt][nt][0], acc[mt][nt][1], am, bn[nt]);
         }
     }
-    (void)g;
 }
 
-template <int JB, int WM, bool SYM>
-__global__ void __launch_bounds__(NT, 1) k_xty_tma(XtyArgs a) {
-    constexpr int NACC = SYM ? WM * (WM + 1) / 2 : JB * WM;
+template <int MT, int NTN, bool SYM>
+__global__ void __launch_bounds__(NT, 1) k_xty_mma(XtyArgs a) {
     extern __shared__ __align__(128) unsigned char smraw[];
     uint64_t* bars = reinterpret_cast<uint64_t*>(smraw);
     double* slots = reinterpret_cast<double*>(smraw + 128);
-    const int tid = threadIdx.x;
-    const int TS = a.TS, w = a.w;
-    const int G = SYM ? 1 : a.G, TR = NT / G;
-    const int g = tid / TR, rl = tid - g * TR;
+    const int tid = threadIdx.x, lane = tid & 31, wp = tid >> 5;
+    const int TS = a.TS, SP = TS + 4, w = a.w;
     const int colbase = blockIdx.y * a.chunk;
-    const int nx = (SYM || a.same) ? 0 : min(a.chunk, a.jx - colbase);   // X columns loaded
+    const int nxc = SYM ? w : min(a.chunk, a.jx - colbase);          // X columns of this chunk
+    const int nx = (SYM || a.same) ? 0 : nxc;                         // X columns loaded
     const int ncol = w + nx;
-    const int64_t slot_d = int64_t(ncol) * TS;
+    const int64_t slot_d = int64_t(ncol) * SP;
     const int64_t ntiles = a.n / TS;
     const int64_t my_tiles = ntiles > int64_t(blockIdx.x) ? (ntiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
 
-    bool xok[JB];
-    int xoff[JB];
+    double acc[MT][NTN][2];
 #pragma unroll
-    for (int jb = 0; jb < JB; ++jb) {
-        const int il = g + G * jb;
-        xok[jb] = !SYM && (il < a.chunk) && (colbase + il < a.jx);
-        xoff[jb] = a.same ? (colbase + il) : il;      // column inside the X source
-    }
-    double acc[NACC];
+    for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
-    for (int e = 0; e < NACC; ++e) acc[e] = 0.0;
+        for (int nt = 0; nt < NTN; ++nt) acc[mt][nt][0] = acc[mt][nt][1] = 0.0;
 
     if (tid == 0) {
         for (int s = 0; s < XTY_STAGES; ++s) ptx::mbar_init(&bars[s], 1);
@@ -150,65 +139,57 @@ __global__ void __launch_bounds__(NT, 1) k_xty_tma(XtyArgs a) {
         double* dst = slots + s * slot_d;
         ptx::fence_proxy_async();                      // generic reads of the slot precede the async writes
         ptx::mbar_arrive_expect_tx(&bars[s], colbytes * uint32_t(ncol));
-        for (int c = 0; c < w; ++c) ptx::bulk_g2s(dst + int64_t(c) * TS, a.Y + a.ldy * c + r0, colbytes, &bars[s]);
+        for (int c = 0; c < w; ++c) ptx::bulk_g2s(dst + int64_t(c) * SP, a.Y + a.ldy * c + r0, colbytes, &bars[s]);
         for (int c = 0; c < nx; ++c)
-            ptx::bulk_g2s(dst + int64_t(w + c) * TS, a.X + a.ldx * (colbase + c) + r0, colbytes, &bars[s]);
+            ptx::bulk_g2s(dst + int64_t(w + c) * SP, a.X + a.ldx * (colbase + c) + r0, colbytes, &bars[s]);
     };
     if (tid == 0)
         for (int64_t k = 0; k < my_tiles && k < XTY_STAGES; ++k) issue(k);
+    const int rw = TS / NWARP;                                        // rows per warp per tile (mult. of 4)
     for (int64_t k = 0; k < my_tiles; ++k) {
         const int s = int(k % XTY_STAGES);
         ptx::mbar_wait(&bars[s], uint32_t((k / XTY_STAGES) & 1));
         const double* Ys = slots + s * slot_d;
-        const double* Xs = a.same ? Ys : Ys + int64_t(w) * TS;
-        xty_rows<JB, WM, SYM>(a, acc, Ys, TS, Xs, TS, TS, g, rl, TR, xok, xoff);
-        __syncthreads();                               // every thread is done with slot s
+        const double* Xs = a.same ? Ys + int64_t(SP) * colbase : Ys + int64_t(SP) * w;
+#pragma unroll 2
+        for (int kr = wp * rw; kr < (wp + 1) * rw; kr += 4)
+            xty_kstep<MT, NTN, SYM>(acc, Ys, SP, Xs, SP, kr + (lane & 3), lane, w, nxc, true);
+        __syncthreads();                               // every warp is done with slot s
         if (tid == 0 && k + XTY_STAGES < my_tiles) issue(k + XTY_STAGES);
     }
-    // ragged tail [ntiles*TS, n): CTA x = 0 reads it straight from global memory
+    // ragged tail [ntiles*TS, n): CTA x = 0, k-steps of 4 rows from global, zero padded
     if (blockIdx.x == 0 && ntiles * TS < a.n) {
         const int64_t r0 = ntiles * TS;
-        const int rows = int(a.n - r0);
-        const double* Xb = a.same ? a.Y + r0 : a.X + a.ldx * colbase + r0;
-        xty_rows<JB, WM, SYM>(a, acc, a.Y + r0, a.ldy, Xb, a.same ? a.ldy : a.ldx, rows, g, rl, TR, xok, xoff);
+        const double* Xb = a.same ? a.Y + a.ldy * colbase : a.X + a.ldx * colbase;
+        const int64_t ldX = a.same ? a.ldy : a.ldx;
+        for (int64_t kr = r0 + 4 * wp; kr < a.n; kr += 4 * NWARP) {
+            const int64_t row = kr + (lane & 3);
+            xty_kstep<MT, NTN, SYM>(acc, a.Y, a.ldy, Xb, ldX, row, lane, w, nxc, row < a.n);
+        }
     }
-    // ---- CTA reduction (fixed order): butterfly over row-lanes, then smem over warps ----
+    // ---- CTA reduction over warps (fixed order) ----
     __syncthreads();
-    double* red = slots;                                    // reuse the ring
-    const int lanes = SYM ? 32 : min(TR, 32);               // lanes of one group in a warp
-    const int warp = tid >> 5, lane = tid & 31;
+    double* red = slots;                                    // reuse the ring: NWARP x MT x NTN x 64
+    constexpr int FR = MT * NTN * 64;
 #pragma unroll
-    for (int e = 0; e < NACC; ++e) {
-        double v = acc[e];
-        for (int off = lanes >> 1; off > 0; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
-        acc[e] = v;
-    }
-    const int npg = SYM ? NT / 32 : max(1, TR / 32);        // partials per group
-    if ((lane % lanes) == 0) {
-        const int k = SYM ? warp : (rl / 32);
+    for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
-        for (int e = 0; e < NACC; ++e) red[(int64_t(g) * npg + k) * NACC + e] = acc[e];
-    }
+        for (int nt = 0; nt < NTN; ++nt) {
+            red[wp * FR + (mt * NTN + nt) * 64 + lane * 2 + 0] = acc[mt][nt][0];
+            red[wp * FR + (mt * NTN + nt) * 64 + lane * 2 + 1] = acc[mt][nt][1];
+        }
     __syncthreads();
     const int nent = a.chunk * w;                           // entries of this CTA's partial
     double* part = a.part + (int64_t(blockIdx.y) * gridDim.x + blockIdx.x) * nent;
-    if constexpr (SYM) {
-        for (int e = tid; e < w * w; e += NT) {
-            const int i = e % w, c = e / w;
-            const int lo = min(i, c), hi = max(i, c);
-            const int idx = lo * WM - lo * (lo - 1) / 2 + (hi - lo);
-            double s = 0.0;
-            for (int k = 0; k < npg; ++k) s += red[int64_t(k) * NACC + idx];
-            part[i + int64_t(a.chunk) * c] = s;
-        }
-    } else {
-        for (int e = tid; e < a.chunk * w; e += NT) {
-            const int il = e % a.chunk, c = e / a.chunk;
-            const int g2 = il % G, jb = il / G;
-            double s = 0.0;
-            for (int k = 0; k < npg; ++k) s += red[(int64_t(g2) * npg + k) * NACC + jb * WM + c];
-            part[il + int64_t(a.chunk) * c] = s;
-        }
+    for (int e = tid; e < a.chunk * w; e += NT) {
+        const int il = e % a.chunk, c = e / a.chunk;
+        int mt = il >> 3, nt = c >> 3, ml = il & 7, nl = c & 7;
+        if (SYM && mt > nt) { const int t = mt; mt = nt; nt = t; const int u = ml; ml = nl; nl = u; }
+        const int ln = ml * 4 + (nl >> 1), h = nl & 1;
+        double sum = 0.0;
+        if (mt < MT && nt < NTN)
+            for (int q = 0; q < NWARP; ++q) sum += red[q * FR + (mt * NTN + nt) * 64 + ln * 2 + h];
+        part[il + int64_t(a.chunk) * c] = sum;
     }
     xty_finish(a, nent);
 }
@@ -286,68 +267,62 @@ __global__ void __launch_bounds__(NT, 1) k_xty_ldg(XtyArgs a) {
 // host side
 // ======================================================================================
 namespace {
-struct Cfg { int JB, WM; bool sym; };
+struct Geo { int G, chunk, gx, gy, TS, MT, NTN; bool tma, sym; size_t smem; int JB, WM; };
 
-Cfg cfg_for(int jx, int w, bool same) {
-    if (same && w <= 12) {
-        if (w <= 1) return {1, 1, true};
-        if (w <= 2) return {1, 2, true};
-        if (w <= 4) return {1, 4, true};
-        if (w <= 8) return {1, 8, true};
-        return {1, 12, true};
-    }
-    (void)jx;
-    if (w <= 1) return {8, 1, false};
-    if (w <= 2) return {8, 2, false};
-    if (w <= 4) return {4, 4, false};
-    if (w <= 8) return {4, 8, false};
-    if (w <= 12) return {4, 12, false};
-    if (w <= 16) return {4, 16, false};
-    return {2, 32, false};
-}
-
-struct Geo { int G, chunk, gx, gy, TS; bool tma; Cfg cf; };
+int ceil8(int x) { return (x + 7) / 8; }
 
 Geo geometry(const Dev& d, int64_t n, int jx, int w, bool same, bool aligned) {
-    Geo o;
-    o.cf = cfg_for(jx, w, same);
-    if (o.cf.sym) {
-        o.G = 1; o.chunk = w; o.gy = 1;
+    Geo o{};
+    o.tma = aligned;
+    if (o.tma) {
+        o.NTN = w <= 8 ? 1 : (w <= 16 ? 2 : 4);
+        o.sym = same;
+        if (same) {
+            o.MT = o.NTN; o.chunk = 8 * o.MT; o.gy = 1;
+        } else {
+            const int mt = ceil8(jx);
+            o.MT = mt <= 1 ? 1 : (mt <= 2 ? 2 : (mt <= 4 ? 4 : 8));
+            if (o.NTN == 4 && o.MT > 4) o.MT = 4;                    // register budget
+            o.chunk = 8 * o.MT;
+            o.gy = (jx + o.chunk - 1) / o.chunk;
+        }
+        const int ncol = w + ((same) ? 0 : std::min(o.chunk, jx));
+        int TS = 4096;
+        while (TS > 64 && int64_t(TS + 4) * ncol * 8 > XTY_STAGE_BYTES) TS /= 2;
+        o.TS = TS;
+        const size_t ring = size_t(XTY_STAGES) * size_t(ncol) * size_t(TS + 4) * sizeof(double);
+        const size_t red = size_t(NWARP) * o.MT * o.NTN * 64 * sizeof(double);
+        o.smem = 128 + (ring > red ? ring : red);
+        const int64_t tiles = n / TS;
+        int64_t want = int64_t(d.sms) / o.gy;
+        if (want > tiles) want = tiles;
+        if (want < 1) want = 1;
+        o.gx = int(want);
     } else {
-        const int need = (jx + o.cf.JB - 1) / o.cf.JB;
+        if (w <= 1) { o.JB = 8; o.WM = 1; } else if (w <= 2) { o.JB = 8; o.WM = 2; }
+        else if (w <= 4) { o.JB = 4; o.WM = 4; } else if (w <= 8) { o.JB = 4; o.WM = 8; }
+        else if (w <= 12) { o.JB = 4; o.WM = 12; } else if (w <= 16) { o.JB = 4; o.WM = 16; }
+        else { o.JB = 2; o.WM = 32; }
+        const int need = (jx + o.JB - 1) / o.JB;
         int g = 1;
         while (g < need && g < 16) g *= 2;
-        o.G = g; o.chunk = g * o.cf.JB;
-        if (same) o.chunk = o.chunk < w ? w : o.chunk;
-        o.gy = same ? 1 : (jx + o.chunk - 1) / o.chunk;
+        o.G = g; o.chunk = g * o.JB;
+        o.gy = (jx + o.chunk - 1) / o.chunk;
+        o.smem = size_t(o.WM) * 256 * sizeof(double);
+        const int64_t tiles = (n + 255) / 256;
+        int64_t want = int64_t(d.sms) * 2 / o.gy;
+        if (want > tiles) want = tiles;
+        if (want < 1) want = 1;
+        o.gx = int(want);
     }
-    o.tma = aligned;
-    const int ncol = w + ((o.cf.sym || same) ? 0 : o.chunk);
-    int TS = 4096;
-    while (TS > 32 && TS * ncol * 8 > XTY_STAGE_BYTES) TS /= 2;
-    o.TS = TS;
-    const int64_t tiles = o.tma ? (n / TS) : (n + 255) / 256;
-    int64_t want = o.tma ? int64_t(d.sms) / o.gy : int64_t(d.sms) * 2 / o.gy;
-    if (want > tiles) want = tiles;
-    if (want < 1) want = 1;
-    o.gx = int(want);
     return o;
 }
 
-size_t smem_bytes(const Geo& o, int w) {
-    if (!o.tma) return size_t(o.cf.WM) * 256 * sizeof(double);
-    const int ncol = w + (o.cf.sym ? 0 : o.chunk);
-    size_t ring = size_t(XTY_STAGES) * size_t(ncol) * size_t(o.TS) * sizeof(double);
-    const int nacc = o.cf.sym ? o.cf.WM * (o.cf.WM + 1) / 2 : o.cf.JB * o.cf.WM;
-    const size_t red = size_t(16) * size_t(nacc) * sizeof(double);   // G*npg <= 16 partial rows
-    return 128 + (ring > red ? ring : red);
-}
-
 template <typename K>
-void launch(K kfn, const Geo& o, size_t smem, const XtyArgs& a, cudaStream_t st) {
-    cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+void launch(K kfn, const Geo& o, const XtyArgs& a, cudaStream_t st) {
+    cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, int(o.smem));
     ++g_launches;
-    kfn<<<dim3(o.gx, o.gy), NT, smem, st>>>(a);
+    kfn<<<dim3(o.gx, o.gy), NT, o.smem, st>>>(a);
 }
 }  // namespace
 
@@ -373,46 +348,36 @@ int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const dou
     if (size_t(o.gx) * o.gy * o.chunk * w > ws.cap) return -1;
     XtyArgs a{n, X, ldx, jx, Y, ldy, w, same ? 1 : 0, o.G, o.chunk, o.TS, ws.part, out, ws.counter,
               fin_chol ? 1 : 0, R, status};
-    const size_t smem = smem_bytes(o, w);
-    const Cfg c = o.cf;
     if (o.tma) {
-        if (c.sym) {
-            switch (c.WM) {
-                case 1: launch(k_xty_tma<1, 1, true>, o, smem, a, st); break;
-                case 2: launch(k_xty_tma<1, 2, true>, o, smem, a, st); break;
-                case 4: launch(k_xty_tma<1, 4, true>, o, smem, a, st); break;
-                case 8: launch(k_xty_tma<1, 8, true>, o, smem, a, st); break;
-                default: launch(k_xty_tma<1, 12, true>, o, smem, a, st); break;
-            }
+        if (o.sym) {
+            if (o.NTN == 1) launch(k_xty_mma<1, 1, true>, o, a, st);
+            else if (o.NTN == 2) launch(k_xty_mma<2, 2, true>, o, a, st);
+            else launch(k_xty_mma<4, 4, true>, o, a, st);
         } else {
-            switch (c.WM) {
-                case 1: launch(k_xty_tma<8, 1, false>, o, smem, a, st); break;
-                case 2: launch(k_xty_tma<8, 2, false>, o, smem, a, st); break;
-                case 4: launch(k_xty_tma<4, 4, false>, o, smem, a, st); break;
-                case 8: launch(k_xty_tma<4, 8, false>, o, smem, a, st); break;
-                case 12: launch(k_xty_tma<4, 12, false>, o, smem, a, st); break;
-                case 16: launch(k_xty_tma<4, 16, false>, o, smem, a, st); break;
-                default: launch(k_xty_tma<2, 32, false>, o, smem, a, st); break;
+            const int key = o.MT * 10 + o.NTN;
+            switch (key) {
+                case 11: launch(k_xty_mma<1, 1, false>, o, a, st); break;
+                case 21: launch(k_xty_mma<2, 1, false>, o, a, st); break;
+                case 41: launch(k_xty_mma<4, 1, false>, o, a, st); break;
+                case 81: launch(k_xty_mma<8, 1, false>, o, a, st); break;
+                case 12: launch(k_xty_mma<1, 2, false>, o, a, st); break;
+                case 22: launch(k_xty_mma<2, 2, false>, o, a, st); break;
+                case 42: launch(k_xty_mma<4, 2, false>, o, a, st); break;
+                case 82: launch(k_xty_mma<8, 2, false>, o, a, st); break;
+                case 14: launch(k_xty_mma<1, 4, false>, o, a, st); break;
+                case 24: launch(k_xty_mma<2, 4, false>, o, a, st); break;
+                default: launch(k_xty_mma<4, 4, false>, o, a, st); break;
             }
         }
     } else {
-        // fallback never uses the symmetric layout
-        Geo g2 = o;
-        if (c.sym) {
-            g2 = geometry(d, n, jx, w, false, false);
-            a.G = g2.G; a.chunk = g2.chunk;
-            if (size_t(g2.gx) * g2.gy * g2.chunk * w > ws.cap) return -1;
-        }
-        const Cfg c2 = g2.cf;
-        const size_t sm2 = smem_bytes(g2, w);
-        switch (c2.WM) {
-            case 1: launch(k_xty_ldg<8, 1>, g2, sm2, a, st); break;
-            case 2: launch(k_xty_ldg<8, 2>, g2, sm2, a, st); break;
-            case 4: launch(k_xty_ldg<4, 4>, g2, sm2, a, st); break;
-            case 8: launch(k_xty_ldg<4, 8>, g2, sm2, a, st); break;
-            case 12: launch(k_xty_ldg<4, 12>, g2, sm2, a, st); break;
-            case 16: launch(k_xty_ldg<4, 16>, g2, sm2, a, st); break;
-            default: launch(k_xty_ldg<2, 32>, g2, sm2, a, st); break;
+        switch (o.WM) {
+            case 1: launch(k_xty_ldg<8, 1>, o, a, st); break;
+            case 2: launch(k_xty_ldg<8, 2>, o, a, st); break;
+            case 4: launch(k_xty_ldg<4, 4>, o, a, st); break;
+            case 8: launch(k_xty_ldg<4, 8>, o, a, st); break;
+            case 12: launch(k_xty_ldg<4, 12>, o, a, st); break;
+            case 16: launch(k_xty_ldg<4, 16>, o, a, st); break;
+            default: launch(k_xty_ldg<2, 32>, o, a, st); break;
         }
     }
     return 0;
