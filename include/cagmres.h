@@ -110,6 +110,15 @@ const char* cagmres_strerror(int status);         /* static string, never NULL  
 /* cudaStream_t to enqueue on (NULL = the handle's own stream).  Not owned. */
 int cagmres_set_stream(cagmres_t h, void* cuda_stream);
 
+/* Tuning options (value semantics per option); EINVAL for an unknown option.
+ *   CAGMRES_OPT_MPK_WAVE : 1 (default) = single-GPU temporally blocked MPK when A is banded
+ *                          enough ("reducing communication of MPK on a single GPU");
+ *                          0 = one SpMV launch per step.  Results are bitwise identical.
+ *   CAGMRES_OPT_GRAPH    : 1 (default) = replay each CA cycle's GPU work as a CUDA graph. */
+#define CAGMRES_OPT_MPK_WAVE 1
+#define CAGMRES_OPT_GRAPH    2
+int cagmres_set_option(cagmres_t h, int opt, int64_t value);
+
 /* Sizes: n_loc owned rows, n_ext owned+ghost rows (P:60 i^(d,1)), ldv = leading dim of V. */
 int cagmres_sizes(cagmres_t h, int64_t* n_loc, int64_t* n_ext, int64_t* ldv);
 

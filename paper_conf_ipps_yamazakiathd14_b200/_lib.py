@@ -17,6 +17,7 @@ EINVAL, ECUDA, ENCCL, EBREAKDOWN, ENOMEM, EGHOST, ENOTSUP = -1, -2, -3, -4, -5, 
 MONOMIAL, NEWTON = 0, 1
 CHOLQR, SVQR, CGS, MGS, CAQR = 0, 1, 2, 3, 4
 REORTH, BORTH_MGS = 0x100, 0x200
+OPT_MPK_WAVE, OPT_GRAPH = 1, 2
 
 
 class CSRStruct(C.Structure):
@@ -59,6 +60,7 @@ SIGNATURES = {
                              C.c_int, _P, C.c_int, C.c_int, C.c_int], C.c_int),
     "cagmres_destroy": ([_P], C.c_int),
     "cagmres_set_stream": ([_P, _P], C.c_int),
+    "cagmres_set_option": ([_P, C.c_int, C.c_int64], C.c_int),
     "cagmres_sizes": ([_P, _PI64, _PI64, _PI64], C.c_int),
     "cagmres_set_shifts": ([_P, _PD, _PD, C.c_int], C.c_int),
     "cagmres_get_shifts": ([_P, _PD, _PD, C.c_int, C.POINTER(C.c_int)], C.c_int),

@@ -65,6 +65,7 @@ void spmv(const Dev& d, const Sell& A, int64_t nrows, const double* x, double* y
     if (nrows <= 0) return;
     const unsigned grid = unsigned((nrows + NT - 1) / NT);
     ++g_launches;
+    if (w && !u) { u = x; bu = 0.0; }             // pair step with a == 0: keep MODE 2 well formed
     if (w)
         k_spmv_sell32<2><<<grid, NT, 0, st>>>(nrows, A.sptr, A.col, A.val, x, u, bu, w, bw, y);
     else if (u)

@@ -25,6 +25,19 @@ struct Sell {
     double* val = nullptr;
 };
 
+// Single-GPU temporally blocked MPK (mpk_wave.cu).
+struct WaveArgs {
+    const int64_t* sptr; const int32_t* col; const double* val;
+    double* V; int64_t ldv; int j;
+    int64_t n; int R, CH, nT, C;          // rows, tile rows, chunk rows, tiles, chunks/tile
+    const int2* pairs; int npairs;        // (tile, step) items in wavefront order
+    int* done;                            // (sb+1) x nT completion counters (zeroed)
+    const int* cnt;                       // chunks per tile
+    double theta[32], b2[32];
+    int kind[32];
+};
+void mpk_wave(const Dev& d, const WaveArgs& a, cudaStream_t st);
+
 // Status bits written by device kernels into the handle's status word.
 enum : int { ST_CHOL = 1, ST_SVQR = 2, ST_NORM = 4 };
 

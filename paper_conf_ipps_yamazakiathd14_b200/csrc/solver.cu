@@ -95,8 +95,18 @@ struct cagmres {
     Timer timer;
     double bytes[PH_N] = {0, 0, 0, 0, 0};
     int spmv_launches = 0;
+    // single-GPU temporally blocked MPK (mpk_wave.cu)
+    bool wave_ok = false, wave_on = true;
+    bool graph_on = true;
+    int wave_R = 0, wave_CH = 2048, wave_nT = 0, wave_C = 0;
+    int* d_done = nullptr;
+    int* d_cnt = nullptr;
+    std::vector<int2*> d_pairs;            // indexed by sb
+    std::vector<int> npairs;
 
     ~cagmres() {
+        cudaFree(d_done); cudaFree(d_cnt);
+        for (int2* p : d_pairs) cudaFree(p);
         cudaFree(A.sptr); cudaFree(A.col); cudaFree(A.val);
         cudaFree(V); cudaFree(xe); cudaFree(tab); cudaFree(gbuf); cudaFree(ybuf);
         cudaFree(ws.part); cudaFree(ws.counter); cudaFree(status);
@@ -204,6 +214,47 @@ int common_alloc(cagmres* h) {
     return CAGMRES_OK;
 }
 
+// Temporal blocking is used when the matrix is banded enough that the live window (~2 s
+// tiles of A plus their vector slices) fits comfortably in the 126 MB L2.
+int wave_setup(cagmres* h, const cagmres_plan& p) {
+    int64_t bw = 0;
+    for (int64_t r = 0; r < p.n_mat; ++r)
+        for (int64_t e = p.rowptr[size_t(r)]; e < p.rowptr[size_t(r) + 1]; ++e) {
+            const int64_t d = std::llabs(int64_t(p.colind[size_t(e)]) - r);
+            bw = std::max(bw, d);
+        }
+    const int CH = h->wave_CH;
+    const int64_t R = std::max<int64_t>(CH, (bw + CH - 1) / CH * CH);
+    const int64_t n = h->n_loc;
+    const int64_t nT = (n + R - 1) / R;
+    const double nnz_row = n > 0 ? double(p.nnz_mat) / double(n) : 0.0;
+    const double tile_bytes = double(R) * (12.0 * nnz_row + 16.0);
+    if (nT < 3 || 2.0 * h->s * tile_bytes > 64.0e6 || R > (int64_t(1) << 30)) return CAGMRES_OK;
+    h->wave_R = int(R); h->wave_nT = int(nT); h->wave_C = int(R / CH);
+    std::vector<int> cnt(size_t(nT), 0);
+    for (int64_t t = 0; t < nT; ++t)
+        for (int c = 0; c < h->wave_C; ++c)
+            if (t * R + int64_t(c) * CH < n) cnt[size_t(t)]++;
+    CU(cudaMalloc(&h->d_cnt, sizeof(int) * size_t(nT)));
+    CU(cudaMemcpy(h->d_cnt, cnt.data(), sizeof(int) * size_t(nT), cudaMemcpyHostToDevice));
+    CU(cudaMalloc(&h->d_done, sizeof(int) * size_t(nT) * size_t(h->s + 1)));
+    h->d_pairs.assign(size_t(h->s) + 1, nullptr);
+    h->npairs.assign(size_t(h->s) + 1, 0);
+    for (int sb = 1; sb <= h->s; ++sb) {
+        std::vector<int2> pr;
+        for (int64_t tau = 0; tau <= nT - 1 + 2 * sb; ++tau)
+            for (int k = 1; k <= sb; ++k) {
+                const int64_t t = tau - 2 * k;
+                if (t >= 0 && t < nT) pr.push_back(make_int2(int(t), k));
+            }
+        CU(cudaMalloc(&h->d_pairs[size_t(sb)], sizeof(int2) * pr.size()));
+        CU(cudaMemcpy(h->d_pairs[size_t(sb)], pr.data(), sizeof(int2) * pr.size(), cudaMemcpyHostToDevice));
+        h->npairs[size_t(sb)] = int(pr.size());
+    }
+    h->wave_ok = true;
+    return CAGMRES_OK;
+}
+
 int init_common(cagmres* h, const cagmres_csr* A, const int64_t* row_starts, int s, int m,
                 int basis, int orth) {
     if (s < 1 || m < 1 || s > m || s > 31 || (basis != CAGMRES_MONOMIAL && basis != CAGMRES_NEWTON))
@@ -227,6 +278,7 @@ int init_common(cagmres* h, const cagmres_csr* A, const int64_t* row_starts, int
     h->level_len = plan.level_len;
     TRY(build_sell(h, plan));
     TRY(common_alloc(h));
+    if (h->nranks == 1) TRY(wave_setup(h, plan));
     if (h->nranks > 1) {
         // ---- exchange request lists (setup, "compress ... needed by other GPUs") ----
         const int P = h->nranks;
@@ -349,6 +401,30 @@ double spmv_bytes(cagmres* h, int64_t rows_out, int depth_in, bool pair2) {
 // distance <= sb-k (a prefix of the extended numbering) from the rows at distance <= sb-k+1.
 int mpk_block(cagmres* h, int j, int sb, const std::vector<host::Step>& steps) {
     Scope sc(h, PH_MPK);
+    if (h->wave_ok && h->wave_on && h->nranks == 1 && sb >= 2) {
+        kern::WaveArgs a{};
+        a.sptr = h->A.sptr; a.col = h->A.col; a.val = h->A.val;
+        a.V = h->V; a.ldv = h->ldv; a.j = j;
+        a.n = h->n_loc; a.R = h->wave_R; a.CH = h->wave_CH; a.nT = h->wave_nT; a.C = h->wave_C;
+        a.pairs = h->d_pairs[size_t(sb)]; a.npairs = h->npairs[size_t(sb)];
+        a.done = h->d_done; a.cnt = h->d_cnt;
+        for (int k = 1; k <= sb; ++k) {
+            a.theta[k - 1] = steps[size_t(k - 1)].a;
+            a.b2[k - 1] = steps[size_t(k - 1)].b2;
+            a.kind[k - 1] = steps[size_t(k - 1)].kind;
+        }
+        CU(cudaMemsetAsync(h->d_done, 0, sizeof(int) * size_t(h->wave_nT) * size_t(sb + 1), h->stream));
+        {
+            Scope sv(h, PH_SPMV);
+            kern::mpk_wave(h->dev, a, h->stream);
+        }
+        double by = 0.0;
+        for (int k = 1; k <= sb; ++k) by += spmv_bytes(h, h->n_loc, 1, steps[size_t(k - 1)].kind == 2);
+        h->bytes[PH_MPK] += by;
+        h->bytes[PH_SPMV] += by;
+        h->spmv_launches++;
+        return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
+    }
     TRY(halo(h, h->V + size_t(h->ldv) * j, sb));
     for (int k = 1; k <= sb; ++k) {
         const host::Step& stp = steps[size_t(k - 1)];
@@ -358,7 +434,7 @@ int mpk_block(cagmres* h, int j, int sb, const std::vector<host::Step>& steps) {
         const bool pair2 = stp.kind == 2;
         {
             Scope sv(h, PH_SPMV);
-            kern::spmv(h->dev, h->A, rows, x, y, stp.a != 0.0 ? x : nullptr, -stp.a,
+            kern::spmv(h->dev, h->A, rows, x, y, (stp.a != 0.0 || pair2) ? x : nullptr, -stp.a,
                        pair2 ? h->V + size_t(h->ldv) * (j + k - 2) : nullptr, stp.b2, h->stream);
         }
         const double by = spmv_bytes(h, rows, sb - k + 1, pair2);
@@ -598,6 +674,15 @@ int cagmres_set_stream(cagmres_t h, void* s) {
     if (!h) return CAGMRES_EINVAL;
     h->stream = s ? static_cast<cudaStream_t>(s) : h->own_stream;
     return CAGMRES_OK;
+}
+
+int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
+    if (!h) return CAGMRES_EINVAL;
+    switch (opt) {
+        case CAGMRES_OPT_MPK_WAVE: h->wave_on = value != 0; return CAGMRES_OK;
+        case CAGMRES_OPT_GRAPH: h->graph_on = value != 0; return CAGMRES_OK;
+        default: return CAGMRES_EINVAL;
+    }
 }
 
 int cagmres_sizes(cagmres_t h, int64_t* n_loc, int64_t* n_ext, int64_t* ldv) {

