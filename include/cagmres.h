@@ -114,9 +114,15 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
  *   CAGMRES_OPT_MPK_WAVE : 1 (default) = single-GPU temporally blocked MPK when A is banded
  *                          enough ("reducing communication of MPK on a single GPU");
  *                          0 = one SpMV launch per step.  Results are bitwise identical.
- *   CAGMRES_OPT_GRAPH    : 1 (default) = replay each CA cycle's GPU work as a CUDA graph. */
-#define CAGMRES_OPT_MPK_WAVE 1
-#define CAGMRES_OPT_GRAPH    2
+ *   CAGMRES_OPT_GRAPH    : 1 (default) = replay each CA cycle's GPU work as a CUDA graph.
+ *   CAGMRES_OPT_WAVE_CHUNK / _WAVE_CTAS / _WAVE_LAG : temporal-blocking tuning (rows per
+ *                          chunk, multiple of 256; resident CTAs per SM; wavefront lag in
+ *                          chunks, 0 = automatic). */
+#define CAGMRES_OPT_MPK_WAVE   1
+#define CAGMRES_OPT_GRAPH      2
+#define CAGMRES_OPT_WAVE_CHUNK 3
+#define CAGMRES_OPT_WAVE_CTAS  4
+#define CAGMRES_OPT_WAVE_LAG   5
 int cagmres_set_option(cagmres_t h, int opt, int64_t value);
 
 /* Sizes: n_loc owned rows, n_ext owned+ghost rows (P:60 i^(d,1)), ldv = leading dim of V. */

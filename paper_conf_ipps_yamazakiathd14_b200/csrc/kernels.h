@@ -29,14 +29,14 @@ struct Sell {
 struct WaveArgs {
     const int64_t* sptr; const int32_t* col; const double* val;
     double* V; int64_t ldv; int j;
-    int64_t n; int R, CH, nT, C;          // rows, tile rows, chunk rows, tiles, chunks/tile
-    const int2* pairs; int npairs;        // (tile, step) items in wavefront order
-    int* done;                            // (sb+1) x nT completion counters (zeroed)
-    const int* cnt;                       // chunks per tile
+    int64_t n; int64_t bw; int CH, nC;    // rows, half-bandwidth, rows per chunk, chunks
+    const int2* pairs; int npairs;        // (chunk, step) items in wavefront order
+    int* done;                            // (s+1) x nC epoch-stamped completion flags
+    int epoch;
     double theta[32], b2[32];
     int kind[32];
 };
-void mpk_wave(const Dev& d, const WaveArgs& a, cudaStream_t st);
+void mpk_wave(const Dev& d, const WaveArgs& a, int ctas_per_sm, cudaStream_t st);
 
 // Status bits written by device kernels into the handle's status word.
 enum : int { ST_CHOL = 1, ST_SVQR = 2, ST_NORM = 4 };

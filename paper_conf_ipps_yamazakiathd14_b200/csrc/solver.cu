@@ -98,14 +98,14 @@ struct cagmres {
     // single-GPU temporally blocked MPK (mpk_wave.cu)
     bool wave_ok = false, wave_on = true;
     bool graph_on = true;
-    int wave_R = 0, wave_CH = 2048, wave_nT = 0, wave_C = 0;
+    int64_t wave_bw = 0;
+    int wave_CH = 1024, wave_ctas = 2, wave_lag = 0, wave_nC = 0, wave_epoch = 0;
     int* d_done = nullptr;
-    int* d_cnt = nullptr;
-    std::vector<int2*> d_pairs;            // indexed by sb
+    std::vector<int2*> d_pairs;            // indexed by sb (built lazily)
     std::vector<int> npairs;
 
     ~cagmres() {
-        cudaFree(d_done); cudaFree(d_cnt);
+        cudaFree(d_done);
         for (int2* p : d_pairs) cudaFree(p);
         cudaFree(A.sptr); cudaFree(A.col); cudaFree(A.val);
         cudaFree(V); cudaFree(xe); cudaFree(tab); cudaFree(gbuf); cudaFree(ybuf);
@@ -214,45 +214,66 @@ int common_alloc(cagmres* h) {
     return CAGMRES_OK;
 }
 
-// Temporal blocking is used when the matrix is banded enough that the live window (~2 s
-// tiles of A plus their vector slices) fits comfortably in the 126 MB L2.
+// Temporal blocking is used when the matrix is banded enough that the reuse window of a
+// chunk of A (s * L chunks) fits comfortably in the 126 MB L2.
 int wave_setup(cagmres* h, const cagmres_plan& p) {
     int64_t bw = 0;
     for (int64_t r = 0; r < p.n_mat; ++r)
-        for (int64_t e = p.rowptr[size_t(r)]; e < p.rowptr[size_t(r) + 1]; ++e) {
-            const int64_t d = std::llabs(int64_t(p.colind[size_t(e)]) - r);
-            bw = std::max(bw, d);
-        }
-    const int CH = h->wave_CH;
-    const int64_t R = std::max<int64_t>(CH, (bw + CH - 1) / CH * CH);
-    const int64_t n = h->n_loc;
-    const int64_t nT = (n + R - 1) / R;
-    const double nnz_row = n > 0 ? double(p.nnz_mat) / double(n) : 0.0;
-    const double tile_bytes = double(R) * (12.0 * nnz_row + 16.0);
-    if (nT < 3 || 2.0 * h->s * tile_bytes > 64.0e6 || R > (int64_t(1) << 30)) return CAGMRES_OK;
-    h->wave_R = int(R); h->wave_nT = int(nT); h->wave_C = int(R / CH);
-    std::vector<int> cnt(size_t(nT), 0);
-    for (int64_t t = 0; t < nT; ++t)
-        for (int c = 0; c < h->wave_C; ++c)
-            if (t * R + int64_t(c) * CH < n) cnt[size_t(t)]++;
-    CU(cudaMalloc(&h->d_cnt, sizeof(int) * size_t(nT)));
-    CU(cudaMemcpy(h->d_cnt, cnt.data(), sizeof(int) * size_t(nT), cudaMemcpyHostToDevice));
-    CU(cudaMalloc(&h->d_done, sizeof(int) * size_t(nT) * size_t(h->s + 1)));
-    h->d_pairs.assign(size_t(h->s) + 1, nullptr);
-    h->npairs.assign(size_t(h->s) + 1, 0);
-    for (int sb = 1; sb <= h->s; ++sb) {
-        std::vector<int2> pr;
-        for (int64_t tau = 0; tau <= nT - 1 + 2 * sb; ++tau)
-            for (int k = 1; k <= sb; ++k) {
-                const int64_t t = tau - 2 * k;
-                if (t >= 0 && t < nT) pr.push_back(make_int2(int(t), k));
-            }
-        CU(cudaMalloc(&h->d_pairs[size_t(sb)], sizeof(int2) * pr.size()));
-        CU(cudaMemcpy(h->d_pairs[size_t(sb)], pr.data(), sizeof(int2) * pr.size(), cudaMemcpyHostToDevice));
-        h->npairs[size_t(sb)] = int(pr.size());
-    }
-    h->wave_ok = true;
+        for (int64_t e = p.rowptr[size_t(r)]; e < p.rowptr[size_t(r) + 1]; ++e)
+            bw = std::max<int64_t>(bw, std::llabs(int64_t(p.colind[size_t(e)]) - r));
+    h->wave_bw = bw;
+    h->wave_ok = bw < h->n_loc / 4;                      // otherwise no reuse window exists
     return CAGMRES_OK;
+}
+
+int wave_lag(const cagmres* h) {
+    // L > ceil(b/CH) keeps the order topological; the extra ~2*G/s chunks of slack give
+    // every step enough runnable chunks for the G resident CTAs.
+    if (h->wave_lag > 0) return h->wave_lag;
+    const int G = h->dev.sms * std::max(1, h->wave_ctas);
+    return int((h->wave_bw + h->wave_CH - 1) / h->wave_CH) + 1 + (2 * G + h->s - 1) / h->s;
+}
+
+bool wave_fits(const cagmres* h) {
+    const double nnz_row = h->n_loc > 0 ? double(h->A.nnz) / double(h->n_loc) : 0.0;
+    const double chunk_bytes = double(h->wave_CH) * (12.0 * nnz_row + 16.0);
+    return h->wave_ok && double(h->s) * wave_lag(h) * chunk_bytes <= 80.0e6 &&
+           h->n_loc >= 8 * int64_t(h->wave_CH);
+}
+
+// (chunk, step) items of a block of sb steps in wavefront order tau = c + L*k
+int wave_pairs(cagmres* h, int sb) {
+    const int nC = int((h->n_loc + h->wave_CH - 1) / h->wave_CH);
+    if (h->wave_nC != nC || h->d_pairs.size() != size_t(h->s) + 1) {
+        for (int2* q : h->d_pairs) cudaFree(q);
+        h->d_pairs.assign(size_t(h->s) + 1, nullptr);
+        h->npairs.assign(size_t(h->s) + 1, 0);
+        cudaFree(h->d_done);
+        h->d_done = nullptr;
+        CU(cudaMalloc(&h->d_done, sizeof(int) * size_t(nC) * size_t(h->s + 1)));
+        CU(cudaMemset(h->d_done, 0, sizeof(int) * size_t(nC) * size_t(h->s + 1)));
+        h->wave_nC = nC;
+        h->wave_epoch = 0;
+    }
+    if (h->d_pairs[size_t(sb)]) return CAGMRES_OK;
+    const int64_t L = wave_lag(h);
+    std::vector<int2> pr;
+    pr.reserve(size_t(nC) * size_t(sb));
+    for (int64_t tau = 0; tau <= nC - 1 + L * sb; ++tau)
+        for (int k = 1; k <= sb; ++k) {
+            const int64_t c = tau - L * k;
+            if (c >= 0 && c < nC) pr.push_back(make_int2(int(c), k));
+        }
+    CU(cudaMalloc(&h->d_pairs[size_t(sb)], sizeof(int2) * pr.size()));
+    CU(cudaMemcpy(h->d_pairs[size_t(sb)], pr.data(), sizeof(int2) * pr.size(), cudaMemcpyHostToDevice));
+    h->npairs[size_t(sb)] = int(pr.size());
+    return CAGMRES_OK;
+}
+
+void wave_reset_pairs(cagmres* h) {
+    for (int2* q : h->d_pairs) cudaFree(q);
+    h->d_pairs.clear();
+    h->wave_nC = 0;
 }
 
 int init_common(cagmres* h, const cagmres_csr* A, const int64_t* row_starts, int s, int m,
@@ -401,22 +422,27 @@ double spmv_bytes(cagmres* h, int64_t rows_out, int depth_in, bool pair2) {
 // distance <= sb-k (a prefix of the extended numbering) from the rows at distance <= sb-k+1.
 int mpk_block(cagmres* h, int j, int sb, const std::vector<host::Step>& steps) {
     Scope sc(h, PH_MPK);
-    if (h->wave_ok && h->wave_on && h->nranks == 1 && sb >= 2) {
+    if (h->wave_on && h->nranks == 1 && sb >= 2 && wave_fits(h)) {
+        TRY(wave_pairs(h, sb));
         kern::WaveArgs a{};
         a.sptr = h->A.sptr; a.col = h->A.col; a.val = h->A.val;
         a.V = h->V; a.ldv = h->ldv; a.j = j;
-        a.n = h->n_loc; a.R = h->wave_R; a.CH = h->wave_CH; a.nT = h->wave_nT; a.C = h->wave_C;
+        a.n = h->n_loc; a.bw = h->wave_bw; a.CH = h->wave_CH; a.nC = h->wave_nC;
         a.pairs = h->d_pairs[size_t(sb)]; a.npairs = h->npairs[size_t(sb)];
-        a.done = h->d_done; a.cnt = h->d_cnt;
+        a.done = h->d_done;
+        if (++h->wave_epoch == 0x7fffffff) {                 // epoch wrap: clear the flags
+            CU(cudaMemsetAsync(h->d_done, 0, sizeof(int) * size_t(h->wave_nC) * size_t(h->s + 1), h->stream));
+            h->wave_epoch = 1;
+        }
+        a.epoch = h->wave_epoch;
         for (int k = 1; k <= sb; ++k) {
             a.theta[k - 1] = steps[size_t(k - 1)].a;
             a.b2[k - 1] = steps[size_t(k - 1)].b2;
             a.kind[k - 1] = steps[size_t(k - 1)].kind;
         }
-        CU(cudaMemsetAsync(h->d_done, 0, sizeof(int) * size_t(h->wave_nT) * size_t(sb + 1), h->stream));
         {
             Scope sv(h, PH_SPMV);
-            kern::mpk_wave(h->dev, a, h->stream);
+            kern::mpk_wave(h->dev, a, h->wave_ctas, h->stream);
         }
         double by = 0.0;
         for (int k = 1; k <= sb; ++k) by += spmv_bytes(h, h->n_loc, 1, steps[size_t(k - 1)].kind == 2);
@@ -680,6 +706,11 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
     if (!h) return CAGMRES_EINVAL;
     switch (opt) {
         case CAGMRES_OPT_MPK_WAVE: h->wave_on = value != 0; return CAGMRES_OK;
+        case CAGMRES_OPT_WAVE_CHUNK:
+            if (value < 256 || value % 256) return CAGMRES_EINVAL;
+            h->wave_CH = int(value); wave_reset_pairs(h); return CAGMRES_OK;
+        case CAGMRES_OPT_WAVE_CTAS: h->wave_ctas = int(value); wave_reset_pairs(h); return CAGMRES_OK;
+        case CAGMRES_OPT_WAVE_LAG: h->wave_lag = int(value); wave_reset_pairs(h); return CAGMRES_OK;
         case CAGMRES_OPT_GRAPH: h->graph_on = value != 0; return CAGMRES_OK;
         default: return CAGMRES_EINVAL;
     }

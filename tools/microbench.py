@@ -49,7 +49,7 @@ def main():
     V = V[:n]
     for (j, w) in [(1, 1), (10, 1), (30, 1), (10, 10), (20, 10), (55, 5), (30, 6)]:
         Q = V[:, :j]
-        P = V[:, 40:40 + w]
+        P = V[:, 66 - w:66]                      # disjoint from Q (j <= 55)
         t = timeit(lambda: S.borth(Q, j, P, w))
         by = 8.0 * n * (2 * j + 3 * w)
         out[f"borth j={j} w={w}"] = dict(ms=round(t, 4), gbs=round(by / t / 1e6, 1))

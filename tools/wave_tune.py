@@ -1,0 +1,39 @@
+"""Sweep the temporal-blocking MPK parameters (chunk rows, CTAs/SM, lag) on C2-like matrices
+and compare with one SpMV launch per step.  Device time of cagmres_mpk (sb = s = 10)."""
+import json
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+from paper_conf_ipps_yamazakiathd14_b200.solver import Solver  # noqa: E402
+from synth import generators as G  # noqa: E402
+from tools.microbench import timeit  # noqa: E402
+
+torch.cuda.set_device(0)
+res = {}
+for name, A in [("C2", G.convection_diffusion(128, 3, 7)), ("band27_4M", G.banded(n=4194304)),
+                ("cd27_160", G.convection_diffusion(160, 3, 27))]:
+    S = Solver(A, s=10, m=30, basis="newton")
+    S.set_shifts(np.array([7.9, 7.9, 0.09, 0.09, 3.8, 5.5, 1.2, 6.6, 2.5, 4.4]),
+                 np.array([0.02, -0.02, 0.03, -0.03, 0, 0, 0, 0, 0, 0]))
+    q = torch.tensor(G.rhs(A.n), device="cuda")
+    W = torch.empty(11, A.n, dtype=torch.float64, device="cuda").t()
+    S.set_option("mpk_wave", 0)
+    base = timeit(lambda: S.mpk(q, 10, out=W))
+    ref = W.clone()
+    r = {"stepwise_ms": round(base, 4)}
+    S.set_option("mpk_wave", 1)
+    for ch in (512, 1024, 2048):
+        for ctas in (1, 2, 4):
+            for lag in (0, 24, 48, 96):
+                S.set_option("wave_chunk", ch)
+                S.set_option("wave_ctas", ctas)
+                S.set_option("wave_lag", lag)
+                t = timeit(lambda: S.mpk(q, 10, out=W))
+                ok = bool(torch.equal(W, ref))
+                r[f"ch{ch}_c{ctas}_L{lag}"] = (round(t, 4), ok)
+    res[name] = r
+    print(name, json.dumps(r), flush=True)
