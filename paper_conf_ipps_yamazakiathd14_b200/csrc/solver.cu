@@ -229,9 +229,10 @@ int wave_setup(cagmres* h, const cagmres_plan& p) {
 int wave_lag(const cagmres* h) {
     // L > ceil(b/CH) keeps the order topological; the extra ~2*G/s chunks of slack give
     // every step enough runnable chunks for the G resident CTAs.
-    if (h->wave_lag > 0) return h->wave_lag;
+    const int minlag = int((h->wave_bw + h->wave_CH - 1) / h->wave_CH) + 1;   // topological order
+    if (h->wave_lag > 0) return std::max(h->wave_lag, minlag);
     const int G = h->dev.sms * std::max(1, h->wave_ctas);
-    return int((h->wave_bw + h->wave_CH - 1) / h->wave_CH) + 1 + (2 * G + h->s - 1) / h->s;
+    return minlag + (2 * G + h->s - 1) / h->s;
 }
 
 bool wave_fits(const cagmres* h) {
