@@ -38,6 +38,23 @@ struct WaveArgs {
 };
 void mpk_wave(const Dev& d, const WaveArgs& a, int ctas_per_sm, cudaStream_t st);
 
+// Fused Arnoldi passes of the first (GMRES) cycle (arnoldi.cu).  mode 1: v -= Q c_in and
+// c_out = Q^T v; mode 2: v -= Q c_in and c_out[0] = v^T v (sqrt if sqrt_out).  jx <= 32
+// (returns -1 otherwise).  part: >= arnoldi_ws_doubles() doubles; counter: zeroed uint.
+struct ArnoldiArgs {
+    int64_t n;
+    const double* Q; int64_t ldq; int jx;
+    double* v;
+    const double* c_in;
+    double* c_out;
+    double* part;
+    unsigned int* counter;
+    int* status;
+    int sqrt_out;
+};
+int arnoldi_fused(const Dev& d, const ArnoldiArgs& a, int mode, cudaStream_t st);
+size_t arnoldi_ws_doubles(const Dev& d);
+
 // Status bits written by device kernels into the handle's status word.
 enum : int { ST_CHOL = 1, ST_SVQR = 2, ST_NORM = 4 };
 

@@ -13,7 +13,9 @@
 //   * a chunk waits (one warp, acquire loads) on the epoch-stamped completion flags of the
 //     <= 2*ceil(b/CH)+1 step-(k-1) chunks it reads — no grid barrier, no memset.
 // Each row is computed with exactly the operations of k_spmv_sell32, so the basis is bitwise
-// identical to the step-by-step MPK (tests/test_gpu_parity.py).
+// identical to the step-by-step MPK (tests/test_gpu_parity.py).  x gathers use L1-cached
+// loads: L1 is invalidated at every launch, nothing is read before the chunk that wrote it is
+// complete, and the waited range is widened by one L1 line, so no stale line can be hit.
 #include <cstdint>
 
 #include "kernels.h"
@@ -41,8 +43,10 @@ __global__ void __launch_bounds__(NT) k_mpk_wave(WaveArgs a) {
         const int64_t r0 = int64_t(c) * a.CH;
         const int64_t r1 = min(a.n, r0 + a.CH);
         if (k > 1 && wp == 0) {
-            const int64_t lo_r = r0 - a.bw < 0 ? 0 : r0 - a.bw;
-            const int64_t hi_r = min(a.n - 1, r1 - 1 + a.bw);
+            // rows read: [r0 - bw, r1 - 1 + bw], widened by one 128-B line (16 rows) so no L1
+            // line this chunk caches can hold rows of a not-yet-complete chunk
+            const int64_t lo_r = r0 - a.bw - 16 < 0 ? 0 : r0 - a.bw - 16;
+            const int64_t hi_r = min(a.n - 1, r1 - 1 + a.bw + 16);
             const int clo = int(lo_r / a.CH), chi = int(hi_r / a.CH);
             const int* f = a.done + int64_t(k - 1) * a.nC;
             for (int base = clo; base <= chi; base += 32) {
@@ -69,10 +73,10 @@ __global__ void __launch_bounds__(NT) k_mpk_wave(WaveArgs a) {
             const int64_t e = __ldg(a.sptr + sl + 1);
             double acc = 0.0;
 #pragma unroll 4
-            for (; o < e; o += 32) acc = fma(__ldg(a.val + o), __ldcg(x + __ldg(a.col + o)), acc);
+            for (; o < e; o += 32) acc = fma(__ldg(a.val + o), __ldca(x + __ldg(a.col + o)), acc);
             double out = acc;
-            if (th != 0.0) out = fma(-th, __ldcg(x + r), out);
-            if (xp) out = fma(b2, __ldcg(xp + r), out);
+            if (th != 0.0) out = fma(-th, __ldca(x + r), out);
+            if (xp) out = fma(b2, __ldca(xp + r), out);
             __stcg(y + r, out);
         }
         __syncthreads();

@@ -80,6 +80,9 @@ struct cagmres {
     double* gbuf = nullptr;                // Gram / small scratch
     double* ybuf = nullptr;                // LS solution (m)
     kern::XtyWs ws;
+    double* arn_part = nullptr;            // fused Arnoldi partials
+    unsigned int* arn_counter = nullptr;
+    bool arnoldi_fuse = true;
     int* status = nullptr;
     // halo (distributed)
     std::vector<int64_t> send_off, recv_off;
@@ -96,8 +99,9 @@ struct cagmres {
     double bytes[PH_N] = {0, 0, 0, 0, 0};
     int spmv_launches = 0;
     // single-GPU temporally blocked MPK (mpk_wave.cu)
-    bool wave_ok = false, wave_on = true;
+    bool wave_ok = false, wave_on = false;   // off until it beats the stepwise MPK
     bool graph_on = true;
+    bool wave_force = false;               // option value 2: skip the L2-fit heuristic
     int64_t wave_bw = 0;
     int wave_CH = 1024, wave_ctas = 2, wave_lag = 0, wave_nC = 0, wave_epoch = 0;
     int* d_done = nullptr;
@@ -110,6 +114,7 @@ struct cagmres {
         cudaFree(A.sptr); cudaFree(A.col); cudaFree(A.val);
         cudaFree(V); cudaFree(xe); cudaFree(tab); cudaFree(gbuf); cudaFree(ybuf);
         cudaFree(ws.part); cudaFree(ws.counter); cudaFree(status);
+        cudaFree(arn_part); cudaFree(arn_counter);
         cudaFree(d_send_idx); cudaFree(d_recv_ext); cudaFree(d_sendbuf); cudaFree(d_recvbuf);
         if (comm) ncclCommDestroy(comm);
         if (own_stream) cudaStreamDestroy(own_stream);
@@ -209,6 +214,9 @@ int common_alloc(cagmres* h) {
     CU(cudaMalloc(&h->ws.part, sizeof(double) * cap));
     CU(cudaMalloc(&h->ws.counter, sizeof(unsigned int)));
     CU(cudaMemset(h->ws.counter, 0, sizeof(unsigned int)));
+    CU(cudaMalloc(&h->arn_part, sizeof(double) * kern::arnoldi_ws_doubles(h->dev)));
+    CU(cudaMalloc(&h->arn_counter, sizeof(unsigned int)));
+    CU(cudaMemset(h->arn_counter, 0, sizeof(unsigned int)));
     CU(cudaMalloc(&h->status, sizeof(int)));
     CU(cudaMemset(h->status, 0, sizeof(int)));
     return CAGMRES_OK;
@@ -238,6 +246,7 @@ int wave_lag(const cagmres* h) {
 bool wave_fits(const cagmres* h) {
     const double nnz_row = h->n_loc > 0 ? double(h->A.nnz) / double(h->n_loc) : 0.0;
     const double chunk_bytes = double(h->wave_CH) * (12.0 * nnz_row + 16.0);
+    if (h->wave_force) return h->wave_ok;
     return h->wave_ok && double(h->s) * wave_lag(h) * chunk_bytes <= 80.0e6 &&
            h->n_loc >= 8 * int64_t(h->wave_CH);
 }
@@ -593,6 +602,34 @@ int arnoldi_cycle(cagmres* h) {
             const double by = spmv_bytes(h, h->n_loc, 1, false);
             h->bytes[PH_MPK] += by; h->bytes[PH_SPMV] += by; h->spmv_launches++;
         }
+        if (h->arnoldi_fuse && k + 1 <= 32) {
+            // c1 = Q^T v ; [v -= Q c1, c2 = Q^T v] ; [v -= Q c2, r = ||v||] ; v /= r
+            const double nl = double(h->n_loc);
+            kern::ArnoldiArgs aa{h->n_loc, h->V, h->ldv, k + 1, v, nullptr, nullptr, h->arn_part,
+                                 h->arn_counter, h->status, h->nranks == 1 ? 1 : 0};
+            {
+                Scope sc(h, PH_BORTH);
+                aa.c_out = c1;
+                if (kern::arnoldi_fused(h->dev, aa, 0, h->stream)) return CAGMRES_EINVAL;
+                TRY(allreduce(h, c1, size_t(k + 1)));
+                aa.c_in = c1; aa.c_out = c2;
+                if (kern::arnoldi_fused(h->dev, aa, 1, h->stream)) return CAGMRES_EINVAL;
+                TRY(allreduce(h, c2, size_t(k + 1)));
+                h->bytes[PH_BORTH] += 8.0 * nl * (3.0 * (k + 1) + 4.0);
+            }
+            {
+                Scope sc(h, PH_TSQR);
+                aa.c_in = c2; aa.c_out = r;
+                if (kern::arnoldi_fused(h->dev, aa, 2, h->stream)) return CAGMRES_EINVAL;
+                if (h->nranks > 1) {
+                    TRY(allreduce(h, r, 1));
+                    kern::chol(r, 1, r, h->status, h->stream);     // r = sqrt(r)
+                }
+                kern::trsm(h->dev, h->n_loc, v, h->ldv, 1, r, 0, h->stream);
+                h->bytes[PH_TSQR] += 8.0 * nl * ((k + 1) + 2.0 + 2.0);
+            }
+            continue;
+        }
         TRY(borth_panel(h, h->V, h->ldv, k + 1, v, h->ldv, 1, c1, false));
         TRY(borth_panel(h, h->V, h->ldv, k + 1, v, h->ldv, 1, c2, false));
         TRY(tsqr_panel(h, v, h->ldv, 1, r, CAGMRES_CHOLQR, 0));
@@ -611,7 +648,15 @@ int residual_norm(cagmres* h, const double* b, const double* x, double* beta, bo
     }
     kern::residual(h->dev, h->A, h->n_loc, xx, b, h->V, h->stream);
     double* rr = h->gbuf + 8;
-    TRY(xty_global(h, h->V, h->ldv, 1, h->V, h->ldv, 1, h->gbuf, true, rr));
+    {   // ||r|| by the scalar reduction kernel (mode 2 with no Q columns)
+        kern::ArnoldiArgs aa{h->n_loc, h->V, h->ldv, 0, h->V, nullptr, rr, h->arn_part, h->arn_counter,
+                             h->status, h->nranks == 1 ? 1 : 0};
+        if (kern::arnoldi_fused(h->dev, aa, 2, h->stream)) return CAGMRES_EINVAL;
+        if (h->nranks > 1) {
+            TRY(allreduce(h, rr, 1));
+            kern::chol(rr, 1, rr, h->status, h->stream);
+        }
+    }
     CU(cudaMemcpyAsync(beta, rr, sizeof(double), cudaMemcpyDeviceToHost, h->stream));
     CU(cudaStreamSynchronize(h->stream));
     if (scale && *beta > 0.0) kern::trsm(h->dev, h->n_loc, h->V, h->ldv, 1, rr, 0, h->stream);
@@ -706,7 +751,7 @@ int cagmres_set_stream(cagmres_t h, void* s) {
 int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
     if (!h) return CAGMRES_EINVAL;
     switch (opt) {
-        case CAGMRES_OPT_MPK_WAVE: h->wave_on = value != 0; return CAGMRES_OK;
+        case CAGMRES_OPT_MPK_WAVE: h->wave_on = value != 0; h->wave_force = value == 2; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK:
             if (value < 256 || value % 256) return CAGMRES_EINVAL;
             h->wave_CH = int(value); wave_reset_pairs(h); return CAGMRES_OK;

@@ -51,14 +51,19 @@ __device__ __forceinline__ void xty_finish(const XtyArgs& a, int nent_cta) {
     __syncthreads();
     if (!s_last) return;
     __threadfence();
+    // one warp per output entry: lane l sums the partials bx = l, l+32, ... (independent
+    // loads in flight), then a fixed xor butterfly -> deterministic, ~gx/32 L2 latencies
     const int jx = a.jx, w = a.w;
-    for (int e = threadIdx.x; e < jx * w; e += NT) {
+    const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5;
+    for (int e = wp; e < jx * w; e += NT / 32) {
         const int i = e % jx, c = e / jx;
         const int by = i / a.chunk, il = i - by * a.chunk;
         const double* src = a.part + int64_t(by) * gridDim.x * int64_t(nent_cta) + il + int64_t(a.chunk) * c;
         double s = 0.0;
-        for (unsigned bx = 0; bx < gridDim.x; ++bx) s += __ldcg(src + int64_t(bx) * nent_cta);
-        a.out[i + int64_t(jx) * c] = s;
+#pragma unroll 4
+        for (unsigned bx = lane; bx < gridDim.x; bx += 32) s += __ldcg(src + int64_t(bx) * nent_cta);
+        for (int off = 16; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
+        if (lane == 0) a.out[i + int64_t(jx) * c] = s;
     }
     if (threadIdx.x == 0) *a.counter = 0u;         // ready for the next launch (stream order)
     if (a.fin_chol) {
