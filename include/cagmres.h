@@ -78,7 +78,8 @@ typedef struct {
     int    hist_cap;        /* capacity of rel_resid_hist                                    */
     int    hist_len;        /* entries written                                               */
     double* rel_resid_hist; /* ||b - A x_c|| / ||b - A x_0|| after each cycle (host)         */
-    int    collect_timing;  /* in: 1 = time phases with CUDA events (adds event records)     */
+    int    collect_timing;  /* in: 1 = time every phase with CUDA events; 2 = only the MPK     *
+                             * kernel launches (ms_spmv) and ms_total; 0 = none               */
     double ms_mpk, ms_borth, ms_tsqr, ms_other, ms_total;   /* device time per phase (ms)   */
     double bytes_mpk, bytes_borth, bytes_tsqr, bytes_other; /* algorithmic bytes */
     int    spmv_launches;   /* SpMV launches timed in ms_spmv                                */
@@ -111,15 +112,14 @@ const char* cagmres_strerror(int status);         /* static string, never NULL  
 int cagmres_set_stream(cagmres_t h, void* cuda_stream);
 
 /* Tuning options (value semantics per option); EINVAL for an unknown option.
- *   CAGMRES_OPT_MPK_WAVE : 1 (default) = single-GPU temporally blocked MPK when A is banded
- *                          enough ("reducing communication of MPK on a single GPU");
- *                          0 = one SpMV launch per step.  Results are bitwise identical.
- *   CAGMRES_OPT_GRAPH    : 1 (default) = replay each CA cycle's GPU work as a CUDA graph.
+ *   CAGMRES_OPT_MPK_WAVE : 0 (default) = one SpMV launch per MPK step; 1 = single-GPU
+ *                          temporally blocked MPK when A is banded enough and the reuse
+ *                          window fits L2 ("reducing communication of MPK on a single
+ *                          GPU"); 2 = force it whenever A is banded.  Bitwise identical.
  *   CAGMRES_OPT_WAVE_CHUNK / _WAVE_CTAS / _WAVE_LAG : temporal-blocking tuning (rows per
  *                          chunk, multiple of 256; resident CTAs per SM; wavefront lag in
  *                          chunks, 0 = automatic). */
 #define CAGMRES_OPT_MPK_WAVE   1
-#define CAGMRES_OPT_GRAPH      2
 #define CAGMRES_OPT_WAVE_CHUNK 3
 #define CAGMRES_OPT_WAVE_CTAS  4
 #define CAGMRES_OPT_WAVE_LAG   5

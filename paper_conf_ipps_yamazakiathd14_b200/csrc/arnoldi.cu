@@ -13,6 +13,7 @@
 #include <cstdint>
 
 #include "kernels.h"
+#include "reduce.cuh"
 
 namespace kern {
 
@@ -72,19 +73,14 @@ __global__ void __launch_bounds__(NT) k_arnoldi_fused(ArnoldiArgs a) {
     if (!s_last) return;
     __threadfence();
     const int nout = MODE == 2 ? 1 : jx;
-    for (int i = wp; i < nout; i += NWARP) {                   // warp per entry, fixed order
-        double s = 0.0;
-#pragma unroll 4
-        for (unsigned b = lane; b < gridDim.x; b += 32) s += __ldcg(a.part + int64_t(b) * NA + i);
-        for (int off = 16; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
-        if (lane == 0) {
-            if (MODE == 2 && a.sqrt_out) {
-                if (!(s > 0.0)) atomicOr(a.status, ST_NORM);
-                s = sqrt(s);
-            }
-            a.c_out[i] = s;
+    __shared__ double sfin[NT];
+    final_reduce(a.part, int(gridDim.x), NA, nout, sfin, [&](int i, double s) {
+        if (MODE == 2 && a.sqrt_out) {
+            if (!(s > 0.0)) atomicOr(a.status, ST_NORM);
+            s = sqrt(s);
         }
-    }
+        a.c_out[i] = s;
+    });
     if (threadIdx.x == 0) *a.counter = 0u;
 }
 
@@ -94,7 +90,7 @@ int arnoldi_fused(const Dev& d, const ArnoldiArgs& a, int mode, cudaStream_t st)
     auto go = [&](auto kfn) {
         int occ = 0;
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kfn, NT, 0);
-        int64_t g = int64_t(d.sms) * (occ < 1 ? 1 : (occ > 2 ? 2 : occ));
+        int64_t g = int64_t(d.sms) * (occ < 1 ? 1 : (occ > 2 ? 2 : occ));   // <= 2 CTAs/SM: few partials
         if (g > blocks) g = blocks;
         if (g < 1) g = 1;
         ++g_launches;

@@ -55,6 +55,12 @@ struct ArnoldiArgs {
 int arnoldi_fused(const Dev& d, const ArnoldiArgs& a, int mode, cudaStream_t st);
 size_t arnoldi_ws_doubles(const Dev& d);
 
+// TSQR by CAQR (caqr.cu): P (n x w, w <= 32) := Q (columns >= c0 written), R (w x w, ld w,
+// diag > 0).  ws: caqr_ws_doubles(n, w) doubles.  Returns -1 on bad sizes (n < w).
+size_t caqr_ws_doubles(int64_t n, int w);
+int caqr(const Dev& d, int64_t n, double* P, int64_t ldp, int w, double* R, int c0, double* ws,
+         cudaStream_t st);
+
 // Status bits written by device kernels into the handle's status word.
 enum : int { ST_CHOL = 1, ST_SVQR = 2, ST_NORM = 4 };
 

@@ -45,6 +45,7 @@ enum Phase { PH_MPK = 0, PH_BORTH = 1, PH_TSQR = 2, PH_OTHER = 3, PH_SPMV = 4, P
 
 struct Timer {
     bool on = false;
+    bool light = false;                    // record only the dominant (MPK) kernel launches
     std::vector<cudaEvent_t> pool;
     size_t used = 0;
     std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> rec;
@@ -79,6 +80,8 @@ struct cagmres {
     double* tab = nullptr; size_t tab_cap = 0;
     double* gbuf = nullptr;                // Gram / small scratch
     double* ybuf = nullptr;                // LS solution (m)
+    double* caqr_ws = nullptr;             // CAQR tree workspace (lazy)
+    size_t caqr_cap = 0;
     kern::XtyWs ws;
     double* arn_part = nullptr;            // fused Arnoldi partials
     unsigned int* arn_counter = nullptr;
@@ -100,7 +103,6 @@ struct cagmres {
     int spmv_launches = 0;
     // single-GPU temporally blocked MPK (mpk_wave.cu)
     bool wave_ok = false, wave_on = false;   // off until it beats the stepwise MPK
-    bool graph_on = true;
     bool wave_force = false;               // option value 2: skip the L2-fit heuristic
     int64_t wave_bw = 0;
     int wave_CH = 1024, wave_ctas = 2, wave_lag = 0, wave_nC = 0, wave_epoch = 0;
@@ -112,7 +114,7 @@ struct cagmres {
         cudaFree(d_done);
         for (int2* p : d_pairs) cudaFree(p);
         cudaFree(A.sptr); cudaFree(A.col); cudaFree(A.val);
-        cudaFree(V); cudaFree(xe); cudaFree(tab); cudaFree(gbuf); cudaFree(ybuf);
+        cudaFree(V); cudaFree(xe); cudaFree(tab); cudaFree(gbuf); cudaFree(ybuf); cudaFree(caqr_ws);
         cudaFree(ws.part); cudaFree(ws.counter); cudaFree(status);
         cudaFree(arn_part); cudaFree(arn_counter);
         cudaFree(d_send_idx); cudaFree(d_recv_ext); cudaFree(d_sendbuf); cudaFree(d_recvbuf);
@@ -126,11 +128,12 @@ namespace {
 // ---- timing helpers --------------------------------------------------------------------
 struct Scope {
     cagmres* h; int ph; cudaEvent_t e0 = nullptr;
-    Scope(cagmres* hh, int p) : h(hh), ph(p) {
-        if (h->timer.on) { e0 = h->timer.get(); cudaEventRecord(e0, h->stream); }
+    bool act;
+    Scope(cagmres* hh, int p) : h(hh), ph(p), act(hh->timer.on && (!hh->timer.light || p == PH_SPMV)) {
+        if (act) { e0 = h->timer.get(); cudaEventRecord(e0, h->stream); }
     }
     ~Scope() {
-        if (h->timer.on) {
+        if (act) {
             cudaEvent_t e1 = h->timer.get();
             cudaEventRecord(e1, h->stream);
             h->timer.rec.push_back({ph, {e0, e1}});
@@ -291,7 +294,8 @@ int init_common(cagmres* h, const cagmres_csr* A, const int64_t* row_starts, int
     if (s < 1 || m < 1 || s > m || s > 31 || (basis != CAGMRES_MONOMIAL && basis != CAGMRES_NEWTON))
         return CAGMRES_EINVAL;
     const int kind = orth & CAGMRES_TSQR_MASK;
-    if (kind > CAGMRES_MGS) return kind == CAGMRES_CAQR ? CAGMRES_ENOTSUP : CAGMRES_EINVAL;
+    if (kind > CAGMRES_CAQR) return CAGMRES_EINVAL;
+    if (kind == CAGMRES_CAQR && h->nranks > 1) return CAGMRES_ENOTSUP;   // single-GPU tree only
     h->s = s; h->m = m; h->basis = basis; h->orth = orth;
     int dv = 0;
     CU(cudaGetDevice(&dv));
@@ -519,6 +523,17 @@ int tsqr_panel(cagmres* h, double* P, int64_t ldp, int w, double* R, int kind, i
             kern::svqr_factor(h->gbuf, w, R, h->status, h->stream);
         }
         kern::trsm(h->dev, h->n_loc, P, ldp, w, R, c0, h->stream);          // V := V R^{-1}
+        h->bytes[PH_TSQR] += 8.0 * nl * (2.0 * w + double(w - c0));
+    } else if (kind == CAGMRES_CAQR) {                       // Fig. 9 CAQR: TSQR tree
+        if (h->nranks > 1) return CAGMRES_ENOTSUP;
+        const size_t need = kern::caqr_ws_doubles(h->n_loc, w);
+        if (need > h->caqr_cap) {
+            cudaFree(h->caqr_ws);
+            h->caqr_ws = nullptr;
+            CU(cudaMalloc(&h->caqr_ws, sizeof(double) * need));
+            h->caqr_cap = need;
+        }
+        if (kern::caqr(h->dev, h->n_loc, P, ldp, w, R, c0, h->caqr_ws, h->stream)) return CAGMRES_EINVAL;
         h->bytes[PH_TSQR] += 8.0 * nl * (2.0 * w + double(w - c0));
     } else {
         CU(cudaMemsetAsync(R, 0, sizeof(double) * size_t(w) * size_t(w), h->stream));
@@ -757,7 +772,6 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
             h->wave_CH = int(value); wave_reset_pairs(h); return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CTAS: h->wave_ctas = int(value); wave_reset_pairs(h); return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_LAG: h->wave_lag = int(value); wave_reset_pairs(h); return CAGMRES_OK;
-        case CAGMRES_OPT_GRAPH: h->graph_on = value != 0; return CAGMRES_OK;
         default: return CAGMRES_EINVAL;
     }
 }
@@ -817,7 +831,7 @@ int cagmres_borth(cagmres_t h, const double* Q, int64_t ldq, int j, double* P, i
 int cagmres_tsqr(cagmres_t h, double* P, int64_t ldp, int w, double* R, int orth) {
     if (!h || !P || !R || w < 1 || w > 32 || ldp < h->n_loc) return CAGMRES_EINVAL;
     const int kind = orth & CAGMRES_TSQR_MASK;
-    if (kind > CAGMRES_MGS) return kind == CAGMRES_CAQR ? CAGMRES_ENOTSUP : CAGMRES_EINVAL;
+    if (kind > CAGMRES_CAQR) return CAGMRES_EINVAL;
     CU(cudaMemsetAsync(h->status, 0, sizeof(int), h->stream));
     TRY(tsqr_panel(h, P, ldp, w, R, kind, 0));
     if (orth & CAGMRES_REORTH) {
@@ -847,6 +861,7 @@ int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit
     const int m = h->m;
     h->timer.reset();
     h->timer.on = st && st->collect_timing;
+    h->timer.light = st && st->collect_timing == 2;
     for (double& v : h->bytes) v = 0.0;
     h->spmv_launches = 0;
     if (st) { st->cycles = 0; st->iters = 0; st->hist_len = 0; }

@@ -16,13 +16,14 @@
 #include <cstdint>
 
 #include "dense_dev.cuh"
+#include "reduce.cuh"
 #include "kernels.h"
 #include "ptx.h"
 
 namespace kern {
 
 namespace {
-constexpr int NT = 256;
+constexpr int NT = 512;                 // one CTA per SM: few partials for the final reduction
 constexpr int NWARP = NT / 32;
 }
 
@@ -51,19 +52,14 @@ __device__ __forceinline__ void xty_finish(const XtyArgs& a, int nent_cta) {
     __syncthreads();
     if (!s_last) return;
     __threadfence();
-    // one warp per output entry: lane l sums the partials bx = l, l+32, ... (independent
-    // loads in flight), then a fixed xor butterfly -> deterministic, ~gx/32 L2 latencies
     const int jx = a.jx, w = a.w;
-    const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5;
-    for (int e = wp; e < jx * w; e += NT / 32) {
-        const int i = e % jx, c = e / jx;
-        const int by = i / a.chunk, il = i - by * a.chunk;
-        const double* src = a.part + int64_t(by) * gridDim.x * int64_t(nent_cta) + il + int64_t(a.chunk) * c;
-        double s = 0.0;
-#pragma unroll 4
-        for (unsigned bx = lane; bx < gridDim.x; bx += 32) s += __ldcg(src + int64_t(bx) * nent_cta);
-        for (int off = 16; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
-        if (lane == 0) a.out[i + int64_t(jx) * c] = s;
+    extern __shared__ double red[];
+    for (int by = 0; by < int(gridDim.y); ++by) {
+        const double* pb = a.part + int64_t(by) * gridDim.x * int64_t(nent_cta);
+        final_reduce(pb, int(gridDim.x), nent_cta, a.chunk * w, red, [&](int e, double tot) {
+            const int il = e % a.chunk, c = e / a.chunk, i = by * a.chunk + il;
+            if (i < jx) a.out[i + int64_t(jx) * c] = tot;
+        });
     }
     if (threadIdx.x == 0) *a.counter = 0u;         // ready for the next launch (stream order)
     if (a.fin_chol) {
@@ -74,8 +70,8 @@ __device__ __forceinline__ void xty_finish(const XtyArgs& a, int nent_cta) {
 
 // MT = 8-column tiles of X per chunk, NTN = 8-column tiles of Y, U = k-steps in flight.
 template <int MT, int NTN, int U, bool SYM>
-__global__ void __launch_bounds__(NT) k_xty_mma(XtyArgs a) {
-    extern __shared__ double red[];                              // NWARP x MT x NTN x 64
+__global__ void __launch_bounds__(NT, 1) k_xty_mma(XtyArgs a) {
+    extern __shared__ double red[];                              // NWARP x MT x NTN x 64 (>= NT)
     const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5;
     const int gid = lane >> 2, tig = lane & 3;
     const int w = a.w;
@@ -185,10 +181,10 @@ Geo geometry(const Dev& d, int64_t n, int jx, int w, bool same) {
         o.gy = (jx + o.chunk - 1) / o.chunk;
     }
     const int per_ks = o.sym ? o.NTN : o.MT + o.NTN;               // loads per k-step per lane
-    o.U = per_ks <= 2 ? 8 : (per_ks <= 6 ? 4 : 2);
+    o.U = per_ks <= 1 ? 16 : (per_ks <= 2 ? 8 : (per_ks <= 6 ? 4 : (per_ks <= 9 ? 2 : 1)));
     const int64_t nss = (n + 4 * o.U - 1) / (4 * o.U);
-    const int ctas_per_sm = per_ks <= 4 ? 4 : 2;
-    int64_t want = int64_t(d.sms) * ctas_per_sm / o.gy;
+    int64_t want = int64_t(d.sms) / o.gy;
+    if (want < 1) want = 1;
     const int64_t cap = (nss + NWARP - 1) / NWARP;
     if (want > cap) want = cap;
     if (want < 1) want = 1;
@@ -198,7 +194,8 @@ Geo geometry(const Dev& d, int64_t n, int jx, int w, bool same) {
 
 template <typename K>
 void launch(K kfn, const Geo& o, const XtyArgs& a, cudaStream_t st) {
-    const size_t smem = size_t(NWARP) * o.MT * o.NTN * 64 * sizeof(double);
+    size_t smem = size_t(NWARP) * o.MT * o.NTN * 64 * sizeof(double);
+    if (smem < NT * sizeof(double)) smem = NT * sizeof(double);
     if (smem > 48 * 1024) cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
     ++g_launches;
     kfn<<<dim3(o.gx, o.gy), NT, smem, st>>>(a);
@@ -224,7 +221,7 @@ int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const dou
     if (size_t(o.gx) * o.gy * o.chunk * w > ws.cap) return -1;
     XtyArgs a{n, X, ldx, jx, Y, ldy, w, o.chunk, ws.part, out, ws.counter, fin_chol ? 1 : 0, R, status};
     if (o.sym) {
-        if (o.NTN == 1) launch(k_xty_mma<1, 1, 8, true>, o, a, st);
+        if (o.NTN == 1) launch(k_xty_mma<1, 1, 16, true>, o, a, st);
         else if (o.NTN == 2) launch(k_xty_mma<2, 2, 8, true>, o, a, st);
         else launch(k_xty_mma<4, 4, 4, true>, o, a, st);
         return 0;
@@ -237,7 +234,7 @@ int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const dou
         case 12: launch(k_xty_mma<1, 2, 4, false>, o, a, st); break;
         case 22: launch(k_xty_mma<2, 2, 4, false>, o, a, st); break;
         case 42: launch(k_xty_mma<4, 2, 4, false>, o, a, st); break;
-        case 82: launch(k_xty_mma<8, 2, 2, false>, o, a, st); break;
+        case 82: launch(k_xty_mma<8, 2, 1, false>, o, a, st); break;
         case 14: launch(k_xty_mma<1, 4, 4, false>, o, a, st); break;
         case 24: launch(k_xty_mma<2, 4, 4, false>, o, a, st); break;
         default: launch(k_xty_mma<4, 4, 2, false>, o, a, st); break;

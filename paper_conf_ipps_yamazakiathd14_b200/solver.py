@@ -116,8 +116,8 @@ class Solver:
         L.check(self._lib.cagmres_set_stream(self._h, C.c_void_p(s.cuda_stream)), "set_stream")
 
     def set_option(self, opt, value):
-        """opt: "mpk_wave", "graph", "wave_chunk", "wave_ctas", "wave_lag" (CAGMRES_OPT_*)."""
-        code = {"mpk_wave": 1, "graph": 2, "wave_chunk": 3, "wave_ctas": 4, "wave_lag": 5}[opt]
+        """opt: "mpk_wave", "wave_chunk", "wave_ctas", "wave_lag" (CAGMRES_OPT_*)."""
+        code = {"mpk_wave": 1, "wave_chunk": 3, "wave_ctas": 4, "wave_lag": 5}[opt]
         L.check(self._lib.cagmres_set_option(self._h, code, int(value)), "set_option")
 
     def close(self):
@@ -190,7 +190,7 @@ class Solver:
         st = L.StatsStruct()
         st.hist_cap = len(hist)
         st.rel_resid_hist = L.dptr(hist)
-        st.collect_timing = 1 if timing else 0
+        st.collect_timing = int(timing) if timing else 0       # True/1: all phases, 2: MPK kernel only
         status = self._lib.cagmres_solve(self._h, C.c_void_p(b.data_ptr()), C.c_void_p(x.data_ptr()),
                                          float(tol), int(maxit), C.byref(st))
         L.check(status, "solve")

@@ -151,7 +151,7 @@ def test_borth_parity(n, j, w):
 
 
 @pytest.mark.parametrize("kind,reorth", [("cholqr", False), ("cholqr", True), ("svqr", False),
-                                         ("cgs", False), ("mgs", False)])
+                                         ("cgs", False), ("mgs", False), ("caqr", False)])
 @pytest.mark.parametrize("n,w", [(100002, 11), (100003, 11), (777, 6), (4096, 1), (20000, 16), (65538, 13)])
 def test_tsqr_parity(kind, reorth, n, w):
     A = G.banded(n=n)
@@ -169,6 +169,21 @@ def test_tsqr_parity(kind, reorth, n, w):
     assert O.fact_error(P, Q, R) < 1e-13
 
 
+def test_caqr_is_unconditionally_orthogonal():
+    """Fig. 10: CAQR ||I - Q^T Q|| = O(eps) even where CholQR breaks down."""
+    n, w = 60000, 12
+    S = Solver(G.banded(n=n), s=1, m=2, basis="monomial")
+    U, _ = np.linalg.qr(G.random_panel(n, w, 41))
+    Vv, _ = np.linalg.qr(G.random_panel(w, w, 42))
+    P = U @ np.diag(np.logspace(0, -9, w)) @ Vv.T                # kappa = 1e9
+    Pd = colmajor(P)
+    R = S.tsqr(Pd, w, "caqr").cpu().numpy()
+    Q = Pd.cpu().numpy()
+    assert O.orth_error(Q) < 1e-13
+    assert O.fact_error(P, Q, R) < 1e-14
+    assert np.all(np.diag(R) > 0)
+
+
 def test_tsqr_cholqr_breakdown_reported():
     from paper_conf_ipps_yamazakiathd14_b200 import _lib as L
     n = 5000
@@ -184,7 +199,7 @@ def test_tsqr_cholqr_breakdown_reported():
 @pytest.mark.parametrize("basis,tsqr,reorth,borth", [
     ("newton", "cholqr", False, "cgs"), ("monomial", "cholqr", False, "cgs"),
     ("newton", "cholqr", True, "cgs"), ("newton", "svqr", False, "cgs"),
-    ("newton", "cgs", True, "cgs"), ("newton", "mgs", False, "mgs")])
+    ("newton", "cgs", True, "cgs"), ("newton", "mgs", False, "mgs"), ("newton", "caqr", False, "cgs")])
 def test_solve_C1_injected_shifts(basis, tsqr, reorth, borth):
     A = G.convection_diffusion(32, 2, 5)
     As = A.to_scipy()
