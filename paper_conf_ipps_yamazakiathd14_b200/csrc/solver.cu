@@ -81,6 +81,12 @@ struct cagmres {
     double* gbuf = nullptr;                // Gram / small scratch
     double* ybuf = nullptr;                // LS solution (m)
     double* caqr_ws = nullptr;             // CAQR tree workspace (lazy)
+    // pinned host mirrors + events of the per-cycle host <-> device exchange
+    double* h_tab = nullptr;
+    double* h_y = nullptr;
+    double* h_beta = nullptr;
+    int* h_stat = nullptr;
+    cudaEvent_t ev_tab = nullptr, ev_beta = nullptr;
     size_t caqr_cap = 0;
     kern::XtyWs ws;
     double* arn_part = nullptr;            // fused Arnoldi partials
@@ -115,6 +121,9 @@ struct cagmres {
         for (int2* p : d_pairs) cudaFree(p);
         cudaFree(A.sptr); cudaFree(A.col); cudaFree(A.val);
         cudaFree(V); cudaFree(xe); cudaFree(tab); cudaFree(gbuf); cudaFree(ybuf); cudaFree(caqr_ws);
+        cudaFreeHost(h_tab); cudaFreeHost(h_y); cudaFreeHost(h_beta); cudaFreeHost(h_stat);
+        if (ev_tab) cudaEventDestroy(ev_tab);
+        if (ev_beta) cudaEventDestroy(ev_beta);
         cudaFree(ws.part); cudaFree(ws.counter); cudaFree(status);
         cudaFree(arn_part); cudaFree(arn_counter);
         cudaFree(d_send_idx); cudaFree(d_recv_ext); cudaFree(d_sendbuf); cudaFree(d_recvbuf);
@@ -211,6 +220,12 @@ int common_alloc(cagmres* h) {
     CU(cudaMemset(h->tab, 0, sizeof(double) * h->tab_cap));
     CU(cudaMalloc(&h->gbuf, sizeof(double) * size_t(h->m + 2) * size_t(std::max(h->m, 32) + 2)));
     CU(cudaMalloc(&h->ybuf, sizeof(double) * size_t(h->m + 2)));
+    CU(cudaMallocHost(&h->h_tab, sizeof(double) * h->tab_cap));
+    CU(cudaMallocHost(&h->h_y, sizeof(double) * size_t(h->m + 2)));
+    CU(cudaMallocHost(&h->h_beta, sizeof(double) * 2));
+    CU(cudaMallocHost(&h->h_stat, sizeof(int) * 2));
+    CU(cudaEventCreateWithFlags(&h->ev_tab, cudaEventDisableTiming));
+    CU(cudaEventCreateWithFlags(&h->ev_beta, cudaEventDisableTiming));
     size_t cap = 0;
     for (int w = 1; w <= 32; ++w) cap = std::max(cap, kern::xty_ws_doubles(h->dev, h->m + 1, w));
     h->ws.cap = cap;
@@ -653,7 +668,9 @@ int arnoldi_cycle(cagmres* h) {
 }
 
 // residual r = b - A x into V[:,0]; returns ||r|| (host) and leaves r/||r|| in V[:,0].
-int residual_norm(cagmres* h, const double* b, const double* x, double* beta, bool scale) {
+// r = b - A x into V[:,0], beta = ||r|| (device), V[:,0] = r / beta, and an async copy of
+// beta to the pinned h_beta followed by ev_beta — the caller waits only when it needs beta.
+int residual_norm_async(cagmres* h, const double* b, const double* x) {
     Scope sc(h, PH_OTHER);
     const double* xx = x;
     if (h->nranks > 1) {
@@ -672,11 +689,24 @@ int residual_norm(cagmres* h, const double* b, const double* x, double* beta, bo
             kern::chol(rr, 1, rr, h->status, h->stream);
         }
     }
-    CU(cudaMemcpyAsync(beta, rr, sizeof(double), cudaMemcpyDeviceToHost, h->stream));
-    CU(cudaStreamSynchronize(h->stream));
-    if (scale && *beta > 0.0) kern::trsm(h->dev, h->n_loc, h->V, h->ldv, 1, rr, 0, h->stream);
-    h->bytes[PH_OTHER] += spmv_bytes(h, h->n_loc, 1, false) + 8.0 * double(h->n_loc) * (1.0 + (scale ? 2.0 : 0.0));
+    CU(cudaMemcpyAsync(h->h_beta, rr, sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+    CU(cudaEventRecord(h->ev_beta, h->stream));
+    kern::trsm(h->dev, h->n_loc, h->V, h->ldv, 1, rr, 0, h->stream);     // q_0 = r / beta
+    h->bytes[PH_OTHER] += spmv_bytes(h, h->n_loc, 1, false) + 8.0 * double(h->n_loc) * 3.0;
     return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
+}
+
+// One restart cycle's GPU work plus the async copy of its coefficient table and status.
+int enqueue_cycle(cagmres* h, bool first_newton, const std::vector<Block>& bl) {
+    if (first_newton) {
+        TRY(arnoldi_cycle(h));
+    } else {
+        TRY(ca_cycle(h, bl));
+    }
+    CU(cudaMemcpyAsync(h->h_tab, h->tab, sizeof(double) * h->tab_cap, cudaMemcpyDeviceToHost, h->stream));
+    CU(cudaMemcpyAsync(h->h_stat, h->status, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+    CU(cudaEventRecord(h->ev_tab, h->stream));
+    return CAGMRES_OK;
 }
 
 void collect_timing(cagmres* h, cagmres_stats* st) {
@@ -869,31 +899,30 @@ int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit
     if (h->timer.on) { t0 = h->timer.get(); cudaEventRecord(t0, h->stream); }
     CU(cudaMemsetAsync(h->status, 0, sizeof(int), h->stream));
     double rho0 = 0.0, beta = 0.0;
-    TRY(residual_norm(h, b, x, &rho0, true));
+    TRY(residual_norm_async(h, b, x));
+    CU(cudaEventSynchronize(h->ev_beta));
+    rho0 = *h->h_beta;
     beta = rho0;
     int rc = CAGMRES_NOT_CONVERGED;
     if (rho0 == 0.0) rc = CAGMRES_OK;
-    std::vector<double> H(static_cast<size_t>(m + 1) * static_cast<size_t>(m)), y(static_cast<size_t>(m)), htab(h->tab_cap);
+    std::vector<double> H(static_cast<size_t>(m + 1) * static_cast<size_t>(m)), y(static_cast<size_t>(m)),
+        res(static_cast<size_t>(m));
+    const double* htab = h->h_tab;
     const std::vector<Block> bl = schedule(h->s, m);
     int cyc = 0;
+    bool pending = false;                    // next cycle already enqueued (speculation)
     for (; cyc < maxit && rc != CAGMRES_OK; ++cyc) {
         const bool first_newton = h->basis == CAGMRES_NEWTON && !h->have_shifts;
         std::fill(H.begin(), H.end(), 0.0);
-        if (first_newton) {
-            TRY(arnoldi_cycle(h));
-        } else {
-            TRY(ca_cycle(h, bl));
-        }
-        int stat = 0;
-        CU(cudaMemcpyAsync(htab.data(), h->tab, sizeof(double) * htab.size(), cudaMemcpyDeviceToHost, h->stream));
-        CU(cudaMemcpyAsync(&stat, h->status, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
-        CU(cudaStreamSynchronize(h->stream));
-        if (stat) { rc = CAGMRES_EBREAKDOWN; break; }
+        if (!pending) TRY(enqueue_cycle(h, first_newton, bl));
+        pending = false;
+        CU(cudaEventSynchronize(h->ev_tab));
+        if (*h->h_stat) { rc = CAGMRES_EBREAKDOWN; break; }
         // ---- Hessenberg matrix (host) ----
         if (first_newton) {
             const size_t stride = 2 * size_t(m + 1) + 1;
             for (int k = 0; k < m; ++k) {
-                const double* c1 = htab.data() + stride * k;
+                const double* c1 = htab + stride * k;
                 for (int i = 0; i <= k; ++i) H[size_t(i) + size_t(m + 1) * k] = c1[i] + c1[i + m + 1];
                 H[size_t(k + 1) + size_t(m + 1) * k] = c1[2 * (m + 1)];
             }
@@ -902,15 +931,15 @@ int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit
             for (const Block& b0 : bl) {
                 const int j = b0.j, sb = b0.sb, w = sb + 1, nr = j + sb + 1;
                 std::vector<double> Rt(size_t(nr) * size_t(w), 0.0);
-                const double* C1 = htab.data() + b0.c1;
-                const double* R1 = htab.data() + b0.r1;
+                const double* C1 = htab + b0.c1;
+                const double* R1 = htab + b0.r1;
                 for (int c = 0; c < w; ++c) {
                     for (int i = 0; i < j; ++i) Rt[size_t(i) + size_t(nr) * c] = c == 0 ? 0.0 : C1[size_t(i) + size_t(j) * (c - 1)];
                     for (int i = 0; i <= c; ++i) Rt[size_t(j + i) + size_t(nr) * c] = R1[size_t(i) + size_t(w) * c];
                 }
                 if (re2) {   // C = C1 + C2 R1, R = R2 R1 (reading G16)
-                    const double* C2 = htab.data() + b0.c2;
-                    const double* R2 = htab.data() + b0.r2;
+                    const double* C2 = htab + b0.c2;
+                    const double* R2 = htab + b0.r2;
                     std::vector<double> Rn(size_t(nr) * size_t(w), 0.0);
                     for (int c = 0; c < w; ++c) {
                         for (int i = 0; i < j; ++i) {
@@ -938,22 +967,30 @@ int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit
             if (rc == CAGMRES_EBREAKDOWN) break;
         }
         // ---- least squares + solution update ----
-        if (host::givens_ls(H.data(), m + 1, m, beta, y.data(), nullptr) != CAGMRES_OK) { rc = CAGMRES_EBREAKDOWN; break; }
-        for (double& v : y) v = -v;                              // update() subtracts X C
+        if (host::givens_ls(H.data(), m + 1, m, beta, y.data(), res.data()) != CAGMRES_OK) { rc = CAGMRES_EBREAKDOWN; break; }
+        for (int i = 0; i < m; ++i) h->h_y[i] = -y[size_t(i)];    // update() subtracts X C
         {
             Scope sc(h, PH_OTHER);
-            CU(cudaMemcpyAsync(h->ybuf, y.data(), sizeof(double) * size_t(m), cudaMemcpyHostToDevice, h->stream));
+            CU(cudaMemcpyAsync(h->ybuf, h->h_y, sizeof(double) * size_t(m), cudaMemcpyHostToDevice, h->stream));
             kern::update(h->dev, h->n_loc, h->V, h->ldv, m, x, h->n_loc, 1, h->ybuf, h->stream);
             h->bytes[PH_OTHER] += 8.0 * double(h->n_loc) * (m + 2.0);
         }
+        TRY(residual_norm_async(h, b, x));                        // r, beta, q_0 for the next cycle
         if (first_newton) {                                      // Ritz values -> Leja shifts
             std::vector<double> wr(static_cast<size_t>(m)), wi(static_cast<size_t>(m));
             if (host::hessenberg_eigvals(H.data(), m + 1, m, wr.data(), wi.data()) != CAGMRES_OK) { rc = CAGMRES_EBREAKDOWN; break; }
             host::modified_leja(wr.data(), wi.data(), m, h->s, h->sh_re, h->sh_im);
             h->have_shifts = true;
         }
-        double rho = 0.0;
-        TRY(residual_norm(h, b, x, &rho, true));
+        // Speculate: the next cycle needs only the device-resident q_0, so enqueue it before
+        // waiting for beta unless the least-squares residual estimate says this cycle has
+        // (almost) converged — hides the host round trip of the convergence test.
+        if (cyc + 1 < maxit && res[size_t(m - 1)] > 2.0 * tol * rho0) {
+            TRY(enqueue_cycle(h, false, bl));
+            pending = true;
+        }
+        CU(cudaEventSynchronize(h->ev_beta));
+        const double rho = *h->h_beta;
         beta = rho;
         if (st && st->rel_resid_hist && st->hist_len < st->hist_cap)
             st->rel_resid_hist[st->hist_len++] = rho0 > 0.0 ? rho / rho0 : 0.0;
