@@ -49,6 +49,14 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         : "memory");
 }
 
+// 16-byte asynchronous global -> shared copy (LDGSTS), L2-only (.cg), commit / wait groups.
+__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
 // D(8x8) += A(8x4) B(4x8) in FP64 on the tensor core.  Fragments (lane = 4*gid + tig):
 //   a = A[gid][tig], b = B[tig][gid], d0 = D[gid][2*tig], d1 = D[gid][2*tig+1].
 __device__ __forceinline__ void dmma(double& d0, double& d1, double a, double b) {

@@ -125,8 +125,154 @@ __global__ void __launch_bounds__(NT) k_rows_mma(StreamArgs a) {
     }
 }
 
+// Per-warp cp.async pipeline (aligned panels): each warp streams contiguous TW-row tiles of
+// the input columns (X then P for the update, P for TRSM) through its own S-stage shared
+// ring; 8-row groups read A fragments (8 rows x 4 cols) from the ring with a column stride
+// of TW+8 doubles (== 8 mod 16: conflict free for that pattern) and store results directly.
+constexpr int RP_S = 3;
+
+template <int MODE, int KTM, int NTN, int TW>
+__global__ void __launch_bounds__(512, 1) k_rows_pipe(StreamArgs a) {
+    extern __shared__ __align__(16) double smp[];
+    constexpr int SP = TW + 8;
+    __shared__ double sB[32 * 32 + 32];
+    const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    const int gid = lane >> 2, tig = lane & 3;
+    const int w = a.w;
+    const int K = MODE == 0 ? a.jx : w;
+    if (MODE == 1) upper_inverse(a.M, w, sB, sB + 32 * 32);
+    double b[KTM][NTN];
+#pragma unroll
+    for (int kt = 0; kt < KTM; ++kt)
+#pragma unroll
+        for (int nt = 0; nt < NTN; ++nt) {
+            const int k = 4 * kt + tig, c = 8 * nt + gid;
+            double v = 0.0;
+            if (k < K && c < w) v = MODE == 0 ? a.M[k + a.ldm * c] : sB[k * 32 + c];
+            b[kt][nt] = v;
+        }
+    const int jxl = MODE == 0 ? a.jx : 0;
+    const int ncol = jxl + w;
+    const int64_t stage_d = int64_t(ncol) * SP;
+    double* ring = smp + int64_t(wp) * RP_S * stage_d;
+    const int64_t T = a.n / TW;
+    const int64_t W = int64_t(gridDim.x) * nw;
+    const int64_t g = int64_t(blockIdx.x) * nw + wp;
+    const int64_t t0 = g * T / W, t1 = (g + 1) * T / W;
+    auto colptr = [&](int c) -> const double* { return c < jxl ? a.X + a.ldx * c : a.P + a.ldp * (c - jxl); };
+    constexpr int CPC = TW * 8 / 16;
+    auto issue = [&](int64_t t, int stage) {
+        if (t < t1) {
+            double* dst = ring + stage * stage_d;
+            const int64_t r0 = t * TW;
+            for (int q = lane; q < ncol * CPC; q += 32) {
+                const int c = q / CPC, part = q - c * CPC;
+                ptx::cp_async16(dst + c * SP + part * 2, colptr(c) + r0 + part * 2);
+            }
+        }
+        ptx::cp_async_commit();
+    };
+    const int KT = (K + 3) / 4;
+    int acol[KTM];
+#pragma unroll
+    for (int kt = 0; kt < KTM; ++kt) acol[kt] = (MODE == 0 ? 0 : jxl) + min(4 * kt + tig, K - 1);
+    int pcol[NTN][2];
+    bool wcol[NTN][2];
+#pragma unroll
+    for (int nt = 0; nt < NTN; ++nt)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            const int c = 8 * nt + 2 * tig + h;
+            pcol[nt][h] = min(c, w - 1);
+            wcol[nt][h] = c < w && (MODE == 0 || c >= a.c0);
+        }
+#pragma unroll
+    for (int s = 0; s < RP_S - 1; ++s) issue(t0 + s, s);
+    int stage = 0;
+    for (int64_t t = t0; t < t1; ++t) {
+        issue(t + RP_S - 1, (stage + RP_S - 1) % RP_S);
+        ptx::cp_async_wait<RP_S - 1>();
+        __syncwarp();
+        const double* sl = ring + stage * stage_d;
+        double* outb = a.P + t * TW;
+#pragma unroll 1
+        for (int g8 = 0; g8 < TW / 8; ++g8) {
+            const int row = 8 * g8 + gid;
+            double d[NTN][2];
+#pragma unroll
+            for (int nt = 0; nt < NTN; ++nt)
+#pragma unroll
+                for (int h = 0; h < 2; ++h) d[nt][h] = MODE == 0 ? sl[(jxl + pcol[nt][h]) * SP + row] : 0.0;
+#pragma unroll
+            for (int kt = 0; kt < KTM; ++kt) {
+                if (kt < KT) {
+                    const double av = sl[acol[kt] * SP + row];
+                    const double am = MODE == 0 ? -av : av;
+#pragma unroll
+                    for (int nt = 0; nt < NTN; ++nt) ptx::dmma(d[nt][0], d[nt][1], am, b[kt][nt]);
+                }
+            }
+#pragma unroll
+            for (int nt = 0; nt < NTN; ++nt)
+#pragma unroll
+                for (int h = 0; h < 2; ++h)
+                    if (wcol[nt][h]) __stcs(outb + a.ldp * (8 * nt + 2 * tig + h) + row, d[nt][h]);
+        }
+        __syncwarp();
+        stage = (stage + 1) % RP_S;
+    }
+    ptx::cp_async_wait<0>();
+    // ragged tail rows [T*TW, n): warp 0 of CTA 0, direct zero-padded loads
+    if (blockIdx.x == 0 && wp == 0) {
+        for (int64_t r0 = T * TW; r0 < a.n; r0 += 8) {
+            const int64_t row = r0 + gid;
+            const bool ok = row < a.n;
+            double d[NTN][2];
+#pragma unroll
+            for (int nt = 0; nt < NTN; ++nt)
+#pragma unroll
+                for (int h = 0; h < 2; ++h) d[nt][h] = (MODE == 0 && ok) ? a.P[a.ldp * pcol[nt][h] + row] : 0.0;
+#pragma unroll
+            for (int kt = 0; kt < KTM; ++kt) {
+                if (kt < KT) {
+                    const double* src = acol[kt] < jxl ? a.X + a.ldx * acol[kt] : a.P + a.ldp * (acol[kt] - jxl);
+                    const double av = ok ? src[row] : 0.0;
+                    const double am = MODE == 0 ? -av : av;
+#pragma unroll
+                    for (int nt = 0; nt < NTN; ++nt) ptx::dmma(d[nt][0], d[nt][1], am, b[kt][nt]);
+                }
+            }
+            if (ok) {
+#pragma unroll
+                for (int nt = 0; nt < NTN; ++nt)
+#pragma unroll
+                    for (int h = 0; h < 2; ++h)
+                        if (wcol[nt][h]) a.P[a.ldp * (8 * nt + 2 * tig + h) + row] = d[nt][h];
+            }
+        }
+    }
+}
+
+template <int MODE, int KTM, int NTN>
+bool run_pipe(const Dev& d, const StreamArgs& a, cudaStream_t st) {
+    constexpr int TW = 32;
+    const bool aligned = ((reinterpret_cast<uintptr_t>(a.P) | reinterpret_cast<uintptr_t>(MODE == 0 ? a.X : a.P)) % 16 == 0) &&
+                         (a.ldp % 2 == 0) && (MODE == 1 || a.ldx % 2 == 0);
+    if (!aligned || a.n < 64 * TW) return false;
+    const int ncol = (MODE == 0 ? a.jx : 0) + a.w;
+    const size_t ring_w = size_t(RP_S) * ncol * (TW + 8) * sizeof(double);
+    int nw = int((200 * 1024) / ring_w);
+    nw = nw < 2 ? 2 : (nw > 16 ? 16 : nw);
+    const size_t smem = size_t(nw) * ring_w;
+    cudaFuncSetAttribute(k_rows_pipe<MODE, KTM, NTN, TW>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    ++g_launches;
+    k_rows_pipe<MODE, KTM, NTN, TW><<<unsigned(d.sms), 32 * nw, smem, st>>>(a);
+    return true;
+}
+
 template <int MODE, int KTM, int NTN, int U>
 void run(const Dev& d, const StreamArgs& a, cudaStream_t st) {
+    if (run_pipe<MODE, KTM, NTN>(d, a, st)) return;
     int occ = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_rows_mma<MODE, KTM, NTN, U>, NT, 0);
     if (occ < 1) occ = 1;

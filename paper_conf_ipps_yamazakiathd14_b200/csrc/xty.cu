@@ -13,6 +13,7 @@
 // Each CTA reduces its warps' 8x8 accumulators in a fixed order; the LAST CTA (atomic
 // ticket) sums all CTA partials in a fixed order (run-to-run bitwise reproducible) and, for
 // CholQR on one GPU, factors the Gram in the same launch.
+#include <algorithm>
 #include <cstdint>
 
 #include "dense_dev.cuh"
@@ -162,6 +163,146 @@ __global__ void __launch_bounds__(NT, 1) k_xty_mma(XtyArgs a) {
 }
 
 // ======================================================================================
+// Per-warp cp.async pipeline (aligned panels).  Each warp streams a contiguous range of
+// TW-row tiles of all ncol needed columns through its own S-stage shared-memory ring
+// (LDGSTS 16-B copies, commit/wait groups, __syncwarp only — no CTA barrier), so the bytes
+// in flight (~(S-1) stages per warp) live in shared memory instead of registers; the
+// register-load kernel above was latency-bound (ncu: long_scoreboard, 16 warps/SM).
+// Fragment reads use a column stride of TW+4 doubles (== 4 mod 16): conflict free.
+// ======================================================================================
+constexpr int PIPE_S = 3;
+
+template <int MT, int NTN, bool SYM, int TW>
+__global__ void __launch_bounds__(NT, 1) k_xty_pipe(XtyArgs a) {
+    extern __shared__ __align__(16) double smp[];
+    constexpr int SP = TW + 4;
+    const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    const int gid = lane >> 2, tig = lane & 3;
+    const int w = a.w;
+    const int colbase = SYM ? 0 : blockIdx.y * a.chunk;
+    const int nxc = SYM ? w : min(a.chunk, a.jx - colbase);
+    const int nx = (SYM || a.X == a.Y) ? 0 : nxc;                 // X columns streamed
+    const int ncol = w + nx;
+    const int64_t stage_d = int64_t(ncol) * SP;
+    double* ring = smp + int64_t(wp) * PIPE_S * stage_d;
+    const int64_t T = a.n / TW;                                    // full tiles
+    const int64_t W = int64_t(gridDim.x) * nw;
+    const int64_t g = int64_t(blockIdx.x) * nw + wp;
+    const int64_t t0 = g * T / W, t1 = (g + 1) * T / W;
+    // columns: Y cols 0..w-1 at slot cols 0..w-1; X cols (if streamed) at w..w+nx-1
+    const double* xbase = a.X == a.Y && !SYM ? a.Y + a.ldy * colbase : a.X + a.ldx * colbase;
+    auto colptr = [&](int c) -> const double* {
+        return c < w ? a.Y + a.ldy * c : xbase + a.ldx * (c - w);
+    };
+    constexpr int CPC = TW * 8 / 16;                               // 16-B chunks per column
+    auto issue = [&](int64_t t, int stage) {
+        if (t < t1) {
+            double* dst = ring + stage * stage_d;
+            const int64_t r0 = t * TW;
+            for (int q = lane; q < ncol * CPC; q += 32) {
+                const int c = q / CPC, part = q - c * CPC;
+                ptx::cp_async16(dst + c * SP + part * 2, colptr(c) + r0 + part * 2);
+            }
+        }
+        ptx::cp_async_commit();
+    };
+    double acc[MT][NTN][2];
+#pragma unroll
+    for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < NTN; ++nt) acc[mt][nt][0] = acc[mt][nt][1] = 0.0;
+    // slot column of each fragment lane (clamped: padded lanes feed discarded entries)
+    int ycol[NTN], xcol[SYM ? 1 : MT];
+#pragma unroll
+    for (int nt = 0; nt < NTN; ++nt) ycol[nt] = min(8 * nt + gid, w - 1);
+    if constexpr (!SYM) {
+#pragma unroll
+        for (int mt = 0; mt < MT; ++mt) xcol[mt] = (nx ? w : 0) + min(8 * mt + gid, nxc - 1);
+    }
+#pragma unroll
+    for (int s = 0; s < PIPE_S - 1; ++s) issue(t0 + s, s);
+    int stage = 0;
+    for (int64_t t = t0; t < t1; ++t) {
+        issue(t + PIPE_S - 1, (stage + PIPE_S - 1) % PIPE_S);
+        ptx::cp_async_wait<PIPE_S - 1>();
+        __syncwarp();
+        const double* sl = ring + stage * stage_d;
+#pragma unroll
+        for (int u = 0; u < TW / 4; ++u) {
+            const int row = 4 * u + tig;
+            double bn[NTN];
+#pragma unroll
+            for (int nt = 0; nt < NTN; ++nt) bn[nt] = sl[ycol[nt] * SP + row];
+            if constexpr (SYM) {
+#pragma unroll
+                for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+                    for (int nt = mt; nt < NTN; ++nt) ptx::dmma(acc[mt][nt][0], acc[mt][nt][1], bn[mt], bn[nt]);
+            } else {
+#pragma unroll
+                for (int mt = 0; mt < MT; ++mt) {
+                    const double am = sl[xcol[mt] * SP + row];
+#pragma unroll
+                    for (int nt = 0; nt < NTN; ++nt) ptx::dmma(acc[mt][nt][0], acc[mt][nt][1], am, bn[nt]);
+                }
+            }
+        }
+        __syncwarp();
+        stage = (stage + 1) % PIPE_S;
+    }
+    ptx::cp_async_wait<0>();
+    // ragged tail rows [T*TW, n): warp 0 of CTA 0, direct zero-padded loads
+    if (blockIdx.x == 0 && wp == 0) {
+        for (int64_t kr = T * TW; kr < a.n; kr += 4) {
+            const int64_t row = kr + tig;
+            const bool ok = row < a.n;
+            double bn[NTN];
+#pragma unroll
+            for (int nt = 0; nt < NTN; ++nt) bn[nt] = ok ? colptr(ycol[nt])[row] : 0.0;
+            if constexpr (SYM) {
+#pragma unroll
+                for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+                    for (int nt = mt; nt < NTN; ++nt) ptx::dmma(acc[mt][nt][0], acc[mt][nt][1], bn[mt], bn[nt]);
+            } else {
+#pragma unroll
+                for (int mt = 0; mt < MT; ++mt) {
+                    const double am = ok ? (xbase + a.ldx * min(8 * mt + gid, nxc - 1))[row] : 0.0;
+#pragma unroll
+                    for (int nt = 0; nt < NTN; ++nt) ptx::dmma(acc[mt][nt][0], acc[mt][nt][1], am, bn[nt]);
+                }
+            }
+        }
+    }
+    // ---- CTA reduction over warps (fixed order), reusing the ring ----
+    __syncthreads();
+    double* red = smp;
+    constexpr int FR = MT * NTN * 64;
+#pragma unroll
+    for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < NTN; ++nt) {
+            red[wp * FR + (mt * NTN + nt) * 64 + lane * 2 + 0] = acc[mt][nt][0];
+            red[wp * FR + (mt * NTN + nt) * 64 + lane * 2 + 1] = acc[mt][nt][1];
+        }
+    __syncthreads();
+    const int nent = a.chunk * w;
+    double* part = a.part + (int64_t(blockIdx.y) * gridDim.x + blockIdx.x) * nent;
+    for (int e = threadIdx.x; e < nent; e += blockDim.x) {
+        const int il = e % a.chunk, c = e / a.chunk;
+        int mt = il >> 3, nt = c >> 3, ml = il & 7, nl = c & 7;
+        if (SYM && mt > nt) { const int tt = mt; mt = nt; nt = tt; const int q = ml; ml = nl; nl = q; }
+        const int ln = ml * 4 + (nl >> 1), h = nl & 1;
+        double sum = 0.0;
+        if (mt < MT && nt < NTN)
+            for (int q = 0; q < nw; ++q) sum += red[q * FR + (mt * NTN + nt) * 64 + ln * 2 + h];
+        part[il + int64_t(a.chunk) * c] = sum;
+    }
+    __syncthreads();
+    xty_finish(a, nent);
+}
+
+// ======================================================================================
 // host side
 // ======================================================================================
 namespace {
@@ -212,14 +353,57 @@ size_t xty_ws_doubles(const Dev& d, int jx, int w) {
     return m;
 }
 
+template <typename K>
+void launch_pipe(K kfn, const Geo& o, int nw, size_t smem, const XtyArgs& a, cudaStream_t st) {
+    cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    ++g_launches;
+    kfn<<<dim3(o.gx, o.gy), 32 * nw, smem, st>>>(a);
+}
+
 int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const double* Y,
         int64_t ldy, int w, double* out, bool fin_chol, double* R, int* status,
         const XtyWs& ws, cudaStream_t st) {
     if (jx <= 0 || w <= 0 || w > 32 || n < 0) return -1;
     const bool same = (X == Y) && (ldx == ldy) && (jx == w);
-    const Geo o = geometry(d, n, jx, w, same);
+    Geo o = geometry(d, n, jx, w, same);
     if (size_t(o.gx) * o.gy * o.chunk * w > ws.cap) return -1;
     XtyArgs a{n, X, ldx, jx, Y, ldy, w, o.chunk, ws.part, out, ws.counter, fin_chol ? 1 : 0, R, status};
+    const bool aligned = ((reinterpret_cast<uintptr_t>(X) | reinterpret_cast<uintptr_t>(Y)) % 16 == 0) &&
+                         (ldx % 2 == 0) && (ldy % 2 == 0);
+    if (aligned && n >= 32 * 64) {
+        // per-warp cp.async pipeline: size the warps so the rings use ~200 KB of smem
+        constexpr int TW = 32;
+        const int ncol = w + ((o.sym || X == Y) ? 0 : std::min(o.chunk, jx));
+        const size_t ring_w = size_t(PIPE_S) * ncol * (TW + 4) * sizeof(double);
+        int nw = int((200 * 1024) / ring_w);
+        nw = nw < 2 ? 2 : (nw > 16 ? 16 : nw);
+        size_t smem = size_t(nw) * ring_w;
+        const size_t red = size_t(nw) * o.MT * o.NTN * 64 * sizeof(double);
+        if (smem < red) smem = red;
+        if (smem < size_t(32 * nw) * sizeof(double)) smem = size_t(32 * nw) * sizeof(double);
+        o.gx = std::max(1, d.sms / o.gy);
+        if (size_t(o.gx) * o.gy * o.chunk * w > ws.cap) return -1;
+        if (o.sym) {
+            if (o.NTN == 1) launch_pipe(k_xty_pipe<1, 1, true, TW>, o, nw, smem, a, st);
+            else if (o.NTN == 2) launch_pipe(k_xty_pipe<2, 2, true, TW>, o, nw, smem, a, st);
+            else launch_pipe(k_xty_pipe<4, 4, true, TW>, o, nw, smem, a, st);
+            return 0;
+        }
+        switch (o.MT * 10 + o.NTN) {
+            case 11: launch_pipe(k_xty_pipe<1, 1, false, TW>, o, nw, smem, a, st); break;
+            case 21: launch_pipe(k_xty_pipe<2, 1, false, TW>, o, nw, smem, a, st); break;
+            case 41: launch_pipe(k_xty_pipe<4, 1, false, TW>, o, nw, smem, a, st); break;
+            case 81: launch_pipe(k_xty_pipe<8, 1, false, TW>, o, nw, smem, a, st); break;
+            case 12: launch_pipe(k_xty_pipe<1, 2, false, TW>, o, nw, smem, a, st); break;
+            case 22: launch_pipe(k_xty_pipe<2, 2, false, TW>, o, nw, smem, a, st); break;
+            case 42: launch_pipe(k_xty_pipe<4, 2, false, TW>, o, nw, smem, a, st); break;
+            case 82: launch_pipe(k_xty_pipe<8, 2, false, TW>, o, nw, smem, a, st); break;
+            case 14: launch_pipe(k_xty_pipe<1, 4, false, TW>, o, nw, smem, a, st); break;
+            case 24: launch_pipe(k_xty_pipe<2, 4, false, TW>, o, nw, smem, a, st); break;
+            default: launch_pipe(k_xty_pipe<4, 4, false, TW>, o, nw, smem, a, st); break;
+        }
+        return 0;
+    }
     if (o.sym) {
         if (o.NTN == 1) launch(k_xty_mma<1, 1, 16, true>, o, a, st);
         else if (o.NTN == 2) launch(k_xty_mma<2, 2, 8, true>, o, a, st);
