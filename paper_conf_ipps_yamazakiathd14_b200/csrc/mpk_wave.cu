@@ -24,6 +24,7 @@ namespace kern {
 
 namespace {
 constexpr int NT = 256;
+constexpr int RPT = 4;                  // rows per thread in flight (memory-level parallelism)
 
 __device__ __forceinline__ int ld_acquire(const int* p) {
     int v;
@@ -66,18 +67,51 @@ __global__ void __launch_bounds__(NT) k_mpk_wave(WaveArgs a) {
         double* y = a.V + a.ldv * (a.j + k);
         const double th = a.theta[k - 1], b2 = a.b2[k - 1];
         const double* xp = a.kind[k - 1] == 2 ? a.V + a.ldv * (a.j + k - 2) : nullptr;
-        for (int64_t r = r0 + threadIdx.x; r < r1; r += NT) {
-            const int64_t sl = r >> 5;
-            const int ln = int(r & 31);
-            int64_t o = __ldg(a.sptr + sl) + ln;
-            const int64_t e = __ldg(a.sptr + sl + 1);
-            double acc = 0.0;
-#pragma unroll 4
-            for (; o < e; o += 32) acc = fma(__ldg(a.val + o), __ldca(x + __ldg(a.col + o)), acc);
-            double out = acc;
-            if (th != 0.0) out = fma(-th, __ldca(x + r), out);
-            if (xp) out = fma(b2, __ldca(xp + r), out);
-            __stcg(y + r, out);
+        // RPT rows per thread, loads of all RPT rows issued together per stored column
+        for (int64_t rb = r0 + threadIdx.x; rb < r1; rb += int64_t(NT) * RPT) {
+            int64_t o[RPT], e[RPT];
+            double acc[RPT];
+#pragma unroll
+            for (int u = 0; u < RPT; ++u) {
+                const int64_t r = rb + int64_t(NT) * u;
+                acc[u] = 0.0;
+                if (r < r1) {
+                    o[u] = __ldg(a.sptr + (r >> 5)) + (r & 31);
+                    e[u] = __ldg(a.sptr + (r >> 5) + 1);
+                } else {
+                    o[u] = 0; e[u] = 0;
+                }
+            }
+            bool more = true;
+            while (more) {
+                more = false;
+                double vv[RPT], xv[RPT];
+#pragma unroll
+                for (int u = 0; u < RPT; ++u) {
+                    if (o[u] < e[u]) {
+                        vv[u] = __ldg(a.val + o[u]);
+                        xv[u] = __ldca(x + __ldg(a.col + o[u]));
+                    }
+                }
+#pragma unroll
+                for (int u = 0; u < RPT; ++u) {
+                    if (o[u] < e[u]) {
+                        acc[u] = fma(vv[u], xv[u], acc[u]);
+                        o[u] += 32;
+                        more |= o[u] < e[u];
+                    }
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < RPT; ++u) {
+                const int64_t r = rb + int64_t(NT) * u;
+                if (r < r1) {
+                    double out = acc[u];
+                    if (th != 0.0) out = fma(-th, __ldca(x + r), out);
+                    if (xp) out = fma(b2, __ldca(xp + r), out);
+                    __stcg(y + r, out);
+                }
+            }
         }
         __syncthreads();
         if (threadIdx.x == 0) {

@@ -111,7 +111,7 @@ struct cagmres {
     bool wave_ok = false, wave_on = false;   // off until it beats the stepwise MPK
     bool wave_force = false;               // option value 2: skip the L2-fit heuristic
     int64_t wave_bw = 0;
-    int wave_CH = 1024, wave_ctas = 2, wave_lag = 0, wave_nC = 0, wave_epoch = 0;
+    int wave_CH = 1024, wave_ctas = 4, wave_lag = 0, wave_nC = 0, wave_epoch = 0;
     int* d_done = nullptr;
     std::vector<int2*> d_pairs;            // indexed by sb (built lazily)
     std::vector<int> npairs;
