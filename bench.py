@@ -240,7 +240,8 @@ def run_ours(args):
                        "l2": "inputs larger than L2 (A 175 MB, V 520 MB) + 256 MB flush between steps",
                        "setup_s": round(setup_s, 2)},
             "e2e": {"value": round(e2e, 4), "unit": "ms", "h2d_bytes_per_step": 8 * len(b_host),
-                    "d2h_bytes_per_step": 8 * len(b_host)},
+                    "d2h_bytes_per_step": 8 * len(b_host), "each_ms": [round(v, 3) for v in e2e_ms]},
+            "value_each_ms": [round(float(v), 3) for v in ms],
             "gpu_launches": int(launches_first),
             "roofline": {"bound": "hbm", "kernel": "k_spmv_sell32 (MPK SpMV step)",
                          "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",

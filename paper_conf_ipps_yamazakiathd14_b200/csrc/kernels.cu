@@ -33,7 +33,8 @@ long long g_launches = 0;
 // ------------------------------------------------------------------------------------
 template <int MODE>   // 0: Ax   1: Ax + bu u   2: Ax + bu u + bw w   3: u - Ax
 __global__ void __launch_bounds__(NT) k_spmv_sell32(int64_t nrows, const int64_t* __restrict__ sptr,
-                                                    const int32_t* __restrict__ col,
+                                                    const int64_t* __restrict__ sinfo,
+                                                    const int32_t* __restrict__ dcol, int64_t ncols,
                                                     const double* __restrict__ val,
                                                     const double* __restrict__ x,
                                                     const double* __restrict__ u, double bu,
@@ -43,11 +44,14 @@ __global__ void __launch_bounds__(NT) k_spmv_sell32(int64_t nrows, const int64_t
     if (r >= nrows) return;
     const int64_t sl = r >> 5;
     const int lane = int(r & 31);
-    int64_t o = __ldg(sptr + sl) + lane;
-    const int64_t e = __ldg(sptr + sl + 1);
+    const int64_t b = __ldg(sptr + sl), e = __ldg(sptr + sl + 1);
+    const int64_t info = __ldg(sinfo + sl);
+    const bool dia = info & 1;
+    const int64_t dp = info >> 1;
     double acc = 0.0;
 #pragma unroll 4
-    for (; o < e; o += 32) acc = fma(__ldg(val + o), __ldg(x + __ldg(col + o)), acc);
+    for (int64_t o = b + lane; o < e; o += 32)
+        acc = fma(__ldg(val + o), __ldg(x + sell_col(r, o, b, dia, dp, dcol, ncols)), acc);
     double out;
     if constexpr (MODE == 3) {
         out = __ldg(u + r) - acc;
@@ -67,11 +71,11 @@ void spmv(const Dev& d, const Sell& A, int64_t nrows, const double* x, double* y
     ++g_launches;
     if (w && !u) { u = x; bu = 0.0; }             // pair step with a == 0: keep MODE 2 well formed
     if (w)
-        k_spmv_sell32<2><<<grid, NT, 0, st>>>(nrows, A.sptr, A.col, A.val, x, u, bu, w, bw, y);
+        k_spmv_sell32<2><<<grid, NT, 0, st>>>(nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, u, bu, w, bw, y);
     else if (u)
-        k_spmv_sell32<1><<<grid, NT, 0, st>>>(nrows, A.sptr, A.col, A.val, x, u, bu, nullptr, 0.0, y);
+        k_spmv_sell32<1><<<grid, NT, 0, st>>>(nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, u, bu, nullptr, 0.0, y);
     else
-        k_spmv_sell32<0><<<grid, NT, 0, st>>>(nrows, A.sptr, A.col, A.val, x, nullptr, 0.0, nullptr, 0.0, y);
+        k_spmv_sell32<0><<<grid, NT, 0, st>>>(nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, nullptr, 0.0, nullptr, 0.0, y);
 }
 
 void residual(const Dev& d, const Sell& A, int64_t nrows, const double* x, const double* b,
@@ -79,7 +83,7 @@ void residual(const Dev& d, const Sell& A, int64_t nrows, const double* x, const
     (void)d;
     if (nrows <= 0) return;
     const unsigned grid = unsigned((nrows + NT - 1) / NT);
-    ++g_launches; k_spmv_sell32<3><<<grid, NT, 0, st>>>(nrows, A.sptr, A.col, A.val, x, b, 1.0, nullptr, 0.0, r);
+    ++g_launches; k_spmv_sell32<3><<<grid, NT, 0, st>>>(nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, b, 1.0, nullptr, 0.0, r);
 }
 
 // ------------------------------------------------------------------------------------

@@ -14,20 +14,36 @@ struct Dev {
     int device = 0;
 };
 
-// Sliced ELLPACK, slice height 32 (one warp), column-major inside a slice.
+// Sliced ELLPACK, slice height 32 (one warp), column-major inside a slice, with per-slice
+// diagonal-offset column compression: sinfo[sl] = (dptr << 1) | dia.
+//   dia == 1: entry t of row r has column clamp(r + dcol[dptr + t]) (zero value if absent)
+//   dia == 0: entry t of lane l has column dcol[dptr + 32 t + l]
 struct Sell {
     int64_t nrows = 0;          // stored rows (extended rows at distance <= s-1)
     int64_t nslices = 0;
-    int64_t nstored = 0;        // stored entries incl. padding
+    int64_t nstored = 0;        // stored values incl. padding
     int64_t nnz = 0;            // true nonzeros
-    int64_t* sptr = nullptr;    // nslices+1 offsets (elements)
-    int32_t* col = nullptr;     // local (extended) column ids
+    int64_t ncols = 0;          // valid x entries (clamp bound for DIA slices)
+    int64_t ndcol = 0, ndia = 0;
+    int64_t* sptr = nullptr;    // nslices+1 value offsets
+    int64_t* sinfo = nullptr;   // nslices
+    int32_t* dcol = nullptr;    // DIA offsets / explicit column ids
     double* val = nullptr;
 };
 
+// column of stored entry o (slice base b) of row r
+__device__ __forceinline__ int64_t sell_col(int64_t r, int64_t o, int64_t b, bool dia, int64_t dp,
+                                            const int32_t* __restrict__ dcol, int64_t ncols) {
+    if (dia) {
+        int64_t c = r + __ldg(dcol + dp + ((o - b) >> 5));
+        return c < 0 ? 0 : (c >= ncols ? ncols - 1 : c);
+    }
+    return __ldg(dcol + dp + (o - b));
+}
+
 // Single-GPU temporally blocked MPK (mpk_wave.cu).
 struct WaveArgs {
-    const int64_t* sptr; const int32_t* col; const double* val;
+    const int64_t* sptr; const int64_t* sinfo; const int32_t* dcol; const double* val; int64_t ncols;
     double* V; int64_t ldv; int j;
     int64_t n; int64_t bw; int CH, nC;    // rows, half-bandwidth, rows per chunk, chunks
     const int2* pairs; int npairs;        // (chunk, step) items in wavefront order

@@ -69,17 +69,22 @@ __global__ void __launch_bounds__(NT) k_mpk_wave(WaveArgs a) {
         const double* xp = a.kind[k - 1] == 2 ? a.V + a.ldv * (a.j + k - 2) : nullptr;
         // RPT rows per thread, loads of all RPT rows issued together per stored column
         for (int64_t rb = r0 + threadIdx.x; rb < r1; rb += int64_t(NT) * RPT) {
-            int64_t o[RPT], e[RPT];
+            int64_t o[RPT], e[RPT], bs[RPT], dp[RPT];
+            bool dia[RPT];
             double acc[RPT];
 #pragma unroll
             for (int u = 0; u < RPT; ++u) {
                 const int64_t r = rb + int64_t(NT) * u;
                 acc[u] = 0.0;
                 if (r < r1) {
-                    o[u] = __ldg(a.sptr + (r >> 5)) + (r & 31);
+                    bs[u] = __ldg(a.sptr + (r >> 5));
+                    o[u] = bs[u] + (r & 31);
                     e[u] = __ldg(a.sptr + (r >> 5) + 1);
+                    const int64_t info = __ldg(a.sinfo + (r >> 5));
+                    dia[u] = info & 1;
+                    dp[u] = info >> 1;
                 } else {
-                    o[u] = 0; e[u] = 0;
+                    o[u] = 0; e[u] = 0; bs[u] = 0; dp[u] = 0; dia[u] = false;
                 }
             }
             bool more = true;
@@ -89,8 +94,9 @@ __global__ void __launch_bounds__(NT) k_mpk_wave(WaveArgs a) {
 #pragma unroll
                 for (int u = 0; u < RPT; ++u) {
                     if (o[u] < e[u]) {
+                        const int64_t r = rb + int64_t(NT) * u;
                         vv[u] = __ldg(a.val + o[u]);
-                        xv[u] = __ldca(x + __ldg(a.col + o[u]));
+                        xv[u] = __ldca(x + sell_col(r, o[u], bs[u], dia[u], dp[u], a.dcol, a.ncols));
                     }
                 }
 #pragma unroll

@@ -11,6 +11,7 @@
 //         block (and of the reorthogonalisation pass); copied to the host once per cycle
 //         for the Hessenberg update and the least-squares solve.
 #include <algorithm>
+#include <climits>
 #include <cmath>
 #include <cstring>
 #include <new>
@@ -119,7 +120,7 @@ struct cagmres {
     ~cagmres() {
         cudaFree(d_done);
         for (int2* p : d_pairs) cudaFree(p);
-        cudaFree(A.sptr); cudaFree(A.col); cudaFree(A.val);
+        cudaFree(A.sptr); cudaFree(A.sinfo); cudaFree(A.dcol); cudaFree(A.val);
         cudaFree(V); cudaFree(xe); cudaFree(tab); cudaFree(gbuf); cudaFree(ybuf); cudaFree(caqr_ws);
         cudaFreeHost(h_tab); cudaFreeHost(h_y); cudaFreeHost(h_beta); cudaFreeHost(h_stat);
         if (ev_tab) cudaEventDestroy(ev_tab);
@@ -153,45 +154,90 @@ struct Scope {
 int64_t round_up(int64_t a, int64_t b) { return (a + b - 1) / b * b; }
 
 // ---- SELL-32 build (host) + upload ------------------------------------------------------
+// SELL-32 with per-slice diagonal-offset column compression.  A slice
+// (32 consecutive rows, one warp) whose rows' column offsets col - row take few distinct
+// values (stencils, banded and most PDE matrices) is stored DIA-style: one int32 offset per
+// stored "diagonal" plus 32 values per diagonal (exact zeros where a row lacks it), so the
+// column stream drops from 4 B to ~4/32 B per stored entry.  Other slices keep explicit
+// column indices.  Entries of a row are visited in increasing column order in both modes.
 int build_sell(cagmres* h, const cagmres_plan& p) {
     const int64_t nr = p.n_mat;
     const int64_t ns = (nr + 31) / 32;
-    std::vector<int64_t> sptr(size_t(ns) + 1, 0);
+    std::vector<int64_t> sptr(size_t(ns) + 1, 0), sinfo(static_cast<size_t>(ns));
+    std::vector<std::vector<int32_t>> offs(static_cast<size_t>(ns));
+    std::vector<char> dia(static_cast<size_t>(ns), 0);
+    int64_t ndcol = 0, ndia = 0;
     for (int64_t sl = 0; sl < ns; ++sl) {
         int64_t wmax = 0;
-        for (int64_t r = sl * 32; r < std::min(nr, sl * 32 + 32); ++r)
+        std::vector<int64_t> o;
+        for (int64_t r = sl * 32; r < std::min(nr, sl * 32 + 32); ++r) {
             wmax = std::max(wmax, p.rowptr[size_t(r) + 1] - p.rowptr[size_t(r)]);
-        sptr[size_t(sl) + 1] = sptr[size_t(sl)] + 32 * wmax;
+            for (int64_t e = p.rowptr[size_t(r)]; e < p.rowptr[size_t(r) + 1]; ++e)
+                o.push_back(int64_t(p.colind[size_t(e)]) - r);
+        }
+        std::sort(o.begin(), o.end());
+        o.erase(std::unique(o.begin(), o.end()), o.end());
+        const bool use_dia = int64_t(o.size()) <= wmax + (wmax + 3) / 4 &&
+                             (o.empty() || (o.front() > INT32_MIN / 2 && o.back() < INT32_MAX / 2));
+        int64_t wdt = wmax;
+        if (use_dia) {
+            dia[size_t(sl)] = 1;
+            ++ndia;
+            wdt = int64_t(o.size());
+            offs[size_t(sl)].assign(o.begin(), o.end());
+            sinfo[size_t(sl)] = (ndcol << 1) | 1;
+            ndcol += wdt;
+        } else {
+            sinfo[size_t(sl)] = ndcol << 1;
+            ndcol += 32 * wdt;
+        }
+        sptr[size_t(sl) + 1] = sptr[size_t(sl)] + 32 * wdt;
     }
     const int64_t tot = sptr[size_t(ns)];
-    std::vector<int32_t> col(static_cast<size_t>(tot));
-    std::vector<double> val(static_cast<size_t>(tot));
+    std::vector<int32_t> dcol(static_cast<size_t>(std::max<int64_t>(ndcol, 1)));
+    std::vector<double> val(static_cast<size_t>(std::max<int64_t>(tot, 1)), 0.0);
     for (int64_t sl = 0; sl < ns; ++sl) {
         const int64_t wdt = (sptr[size_t(sl) + 1] - sptr[size_t(sl)]) / 32;
-        for (int lane = 0; lane < 32; ++lane) {
-            const int64_t r = sl * 32 + lane;
-            const int64_t b = r < nr ? p.rowptr[size_t(r)] : 0, e = r < nr ? p.rowptr[size_t(r) + 1] : 0;
-            for (int64_t t = 0; t < wdt; ++t) {
-                const int64_t o = sptr[size_t(sl)] + 32 * t + lane;
-                if (b + t < e) {
-                    col[size_t(o)] = p.colind[size_t(b + t)];
-                    val[size_t(o)] = p.val[size_t(b + t)];
-                } else {
-                    col[size_t(o)] = int32_t(r < nr ? r : 0);
-                    val[size_t(o)] = 0.0;
+        const int64_t dp = sinfo[size_t(sl)] >> 1;
+        if (dia[size_t(sl)]) {
+            const std::vector<int32_t>& of = offs[size_t(sl)];
+            for (int64_t t = 0; t < wdt; ++t) dcol[size_t(dp + t)] = of[size_t(t)];
+            for (int lane = 0; lane < 32; ++lane) {
+                const int64_t r = sl * 32 + lane;
+                if (r >= nr) continue;
+                int64_t t = 0;
+                for (int64_t e = p.rowptr[size_t(r)]; e < p.rowptr[size_t(r) + 1]; ++e) {
+                    const int64_t off = int64_t(p.colind[size_t(e)]) - r;
+                    while (of[size_t(t)] != off) ++t;          // offsets and columns both ascend
+                    val[size_t(sptr[size_t(sl)] + 32 * t + lane)] = p.val[size_t(e)];
+                }
+            }
+        } else {
+            for (int lane = 0; lane < 32; ++lane) {
+                const int64_t r = sl * 32 + lane;
+                const int64_t b = r < nr ? p.rowptr[size_t(r)] : 0, e = r < nr ? p.rowptr[size_t(r) + 1] : 0;
+                for (int64_t t = 0; t < wdt; ++t) {
+                    const int64_t o = sptr[size_t(sl)] + 32 * t + lane;
+                    if (b + t < e) {
+                        dcol[size_t(dp + 32 * t + lane)] = p.colind[size_t(b + t)];
+                        val[size_t(o)] = p.val[size_t(b + t)];
+                    } else {
+                        dcol[size_t(dp + 32 * t + lane)] = int32_t(r < nr ? r : 0);
+                    }
                 }
             }
         }
     }
     h->A.nrows = nr; h->A.nslices = ns; h->A.nstored = tot; h->A.nnz = p.nnz_mat;
+    h->A.ncols = p.n_ext; h->A.ndcol = ndcol; h->A.ndia = ndia;
     CU(cudaMalloc(&h->A.sptr, sizeof(int64_t) * size_t(ns + 1)));
-    CU(cudaMalloc(&h->A.col, sizeof(int32_t) * size_t(std::max<int64_t>(tot, 1))));
+    CU(cudaMalloc(&h->A.sinfo, sizeof(int64_t) * size_t(std::max<int64_t>(ns, 1))));
+    CU(cudaMalloc(&h->A.dcol, sizeof(int32_t) * size_t(std::max<int64_t>(ndcol, 1))));
     CU(cudaMalloc(&h->A.val, sizeof(double) * size_t(std::max<int64_t>(tot, 1))));
     CU(cudaMemcpy(h->A.sptr, sptr.data(), sizeof(int64_t) * size_t(ns + 1), cudaMemcpyHostToDevice));
-    if (tot) {
-        CU(cudaMemcpy(h->A.col, col.data(), sizeof(int32_t) * size_t(tot), cudaMemcpyHostToDevice));
-        CU(cudaMemcpy(h->A.val, val.data(), sizeof(double) * size_t(tot), cudaMemcpyHostToDevice));
-    }
+    if (ns) CU(cudaMemcpy(h->A.sinfo, sinfo.data(), sizeof(int64_t) * size_t(ns), cudaMemcpyHostToDevice));
+    if (ndcol) CU(cudaMemcpy(h->A.dcol, dcol.data(), sizeof(int32_t) * size_t(ndcol), cudaMemcpyHostToDevice));
+    if (tot) CU(cudaMemcpy(h->A.val, val.data(), sizeof(double) * size_t(tot), cudaMemcpyHostToDevice));
     // nnz of the first level_len[h] rows (algorithmic byte model of a prefix SpMV)
     h->nnz_prefix.assign(size_t(h->s) + 1, 0);
     for (int hh = 0; hh <= h->s; ++hh) {
@@ -454,7 +500,7 @@ int mpk_block(cagmres* h, int j, int sb, const std::vector<host::Step>& steps) {
     if (h->wave_on && h->nranks == 1 && sb >= 2 && wave_fits(h)) {
         TRY(wave_pairs(h, sb));
         kern::WaveArgs a{};
-        a.sptr = h->A.sptr; a.col = h->A.col; a.val = h->A.val;
+        a.sptr = h->A.sptr; a.sinfo = h->A.sinfo; a.dcol = h->A.dcol; a.val = h->A.val; a.ncols = h->A.ncols;
         a.V = h->V; a.ldv = h->ldv; a.j = j;
         a.n = h->n_loc; a.bw = h->wave_bw; a.CH = h->wave_CH; a.nC = h->wave_nC;
         a.pairs = h->d_pairs[size_t(sb)]; a.npairs = h->npairs[size_t(sb)];

@@ -303,133 +303,6 @@ __global__ void __launch_bounds__(NT, 1) k_xty_pipe(XtyArgs a) {
 }
 
 // ======================================================================================
-// Same per-warp cp.async ring, scalar DFMA compute with exact-size register blocking.
-// ncu on the DMMA variant: tensor pipe 61-70 % busy with math_pipe_throttle stalls — the
-// FP64 MMA path sustains ~12 TFLOP/s here and 8x8x4 tiles waste 2.5-3x on w = 11 panels
-// (Gram: 192 FMA/row issued for 66 useful).  Scalar blocking issues exactly the needed FMAs.
-//   SYM (Gram): lane = row of the 32-row tile; each lane accumulates the upper triangle of
-//               its rows (WM(WM+1)/2 registers); one smem load per panel element.
-//   general   : CG column groups x 32/CG row lanes; a lane owns JB X-columns x all w
-//               Y-columns (JB*WM accumulators) for CG rows of each tile.
-// ======================================================================================
-constexpr int SC_S = 4;
-
-template <int JB, int WM, bool SYM>
-__global__ void __launch_bounds__(256, 1) k_xty_sc(XtyArgs a, int CG) {
-    extern __shared__ __align__(16) double smp[];
-    constexpr int TW = 32, SP = TW + 4;
-    constexpr int NACC = SYM ? WM * (WM + 1) / 2 : JB * WM;
-    const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    const int w = a.w;
-    const int colbase = SYM ? 0 : blockIdx.y * a.chunk;
-    const int nxc = SYM ? w : min(a.chunk, a.jx - colbase);
-    const bool xsame = !SYM && a.X == a.Y;
-    const int nx = (SYM || xsame) ? 0 : nxc;
-    const int ncol = w + nx;
-    const int64_t stage_d = int64_t(ncol) * SP;
-    double* ring = smp + int64_t(wp) * SC_S * stage_d;
-    const int64_t T = a.n / TW;
-    const int64_t W = int64_t(gridDim.x) * nw;
-    const int64_t g = int64_t(blockIdx.x) * nw + wp;
-    const int64_t t0 = g * T / W, t1 = (g + 1) * T / W;
-    const double* xbase = xsame ? a.Y + a.ldy * colbase : a.X + a.ldx * colbase;
-    auto colptr = [&](int c) -> const double* { return c < w ? a.Y + a.ldy * c : xbase + a.ldx * (c - w); };
-    constexpr int CPC = TW * 8 / 16;
-    auto issue = [&](int64_t t, int stage) {
-        if (t < t1) {
-            double* dst = ring + stage * stage_d;
-            const int64_t r0 = t * TW;
-            for (int q = lane; q < ncol * CPC; q += 32) {
-                const int c = q / CPC, part = q - c * CPC;
-                ptx::cp_async16(dst + c * SP + part * 2, colptr(c) + r0 + part * 2);
-            }
-        }
-        ptx::cp_async_commit();
-    };
-    // lane roles (general): column group cg, row lane rl, rows rl + (32/CG)*i, i < CG
-    const int cg = SYM ? 0 : lane % CG, rl = SYM ? lane : lane / CG;
-    const int rstep = SYM ? 32 : 32 / CG;
-    int xc[JB];
-    bool xok[JB];
-#pragma unroll
-    for (int jb = 0; jb < JB; ++jb) {
-        const int il = cg * JB + jb;
-        xok[jb] = !SYM && il < nxc;
-        xc[jb] = (nx ? w : 0) + (il < nxc ? il : 0);      // slot column (X from the Y slot if xsame)
-    }
-    double acc[NACC];
-#pragma unroll
-    for (int e = 0; e < NACC; ++e) acc[e] = 0.0;
-    auto row_fma = [&](auto getp, auto getx) {
-        double p[WM];
-#pragma unroll
-        for (int c = 0; c < WM; ++c) p[c] = c < w ? getp(c) : 0.0;
-        if constexpr (SYM) {
-            int idx = 0;
-#pragma unroll
-            for (int i = 0; i < WM; ++i)
-#pragma unroll
-                for (int c = i; c < WM; ++c) { acc[idx] = fma(p[i], p[c], acc[idx]); ++idx; }
-        } else {
-#pragma unroll
-            for (int jb = 0; jb < JB; ++jb) {
-                const double xv = xok[jb] ? getx(jb) : 0.0;
-#pragma unroll
-                for (int c = 0; c < WM; ++c) acc[jb * WM + c] = fma(xv, p[c], acc[jb * WM + c]);
-            }
-        }
-    };
-#pragma unroll
-    for (int s = 0; s < SC_S - 1; ++s) issue(t0 + s, s);
-    int stage = 0;
-    for (int64_t t = t0; t < t1; ++t) {
-        issue(t + SC_S - 1, (stage + SC_S - 1) % SC_S);
-        ptx::cp_async_wait<SC_S - 1>();
-        __syncwarp();
-        const double* sl = ring + stage * stage_d;
-        for (int r = rl; r < TW; r += rstep)
-            row_fma([&](int c) { return sl[c * SP + r]; }, [&](int jb) { return sl[xc[jb] * SP + r]; });
-        __syncwarp();
-        stage = (stage + 1) % SC_S;
-    }
-    ptx::cp_async_wait<0>();
-    if (blockIdx.x == 0 && wp == 0) {                          // ragged tail, direct loads
-        for (int64_t r = T * TW + rl; r < a.n; r += rstep)
-            row_fma([&](int c) { return colptr(c)[r]; }, [&](int jb) { return colptr(xc[jb])[r]; });
-    }
-    // ---- CTA reduction: warp butterfly over lanes of the same column group, smem over warps
-    __syncthreads();
-    double* red = smp;                                           // nw x CG x NACC
-#pragma unroll
-    for (int e = 0; e < NACC; ++e) {
-        double v = acc[e];
-        for (int off = 16; off >= (SYM ? 1 : CG); off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
-        if (lane < (SYM ? 1 : CG)) red[(int64_t(wp) * (SYM ? 1 : CG) + lane) * NACC + e] = v;
-    }
-    __syncthreads();
-    const int nent = a.chunk * w;
-    double* part = a.part + (int64_t(blockIdx.y) * gridDim.x + blockIdx.x) * nent;
-    for (int e = threadIdx.x; e < nent; e += blockDim.x) {
-        const int il = e % a.chunk, c = e / a.chunk;
-        double sum = 0.0;
-        if (SYM) {
-            const int lo = min(il, c), hi = max(il, c);
-            if (hi < WM) {
-                const int idx = lo * WM - lo * (lo - 1) / 2 + (hi - lo);
-                for (int q = 0; q < nw; ++q) sum += red[int64_t(q) * NACC + idx];
-            }
-        } else {
-            const int gi = il / JB, jb = il - gi * JB;
-            if (gi < CG)
-                for (int q = 0; q < nw; ++q) sum += red[(int64_t(q) * CG + gi) * NACC + jb * WM + c];
-        }
-        part[il + int64_t(a.chunk) * c] = sum;
-    }
-    __syncthreads();
-    xty_finish(a, nent);
-}
-
-// ======================================================================================
 // host side
 // ======================================================================================
 namespace {
@@ -497,46 +370,6 @@ int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const dou
     XtyArgs a{n, X, ldx, jx, Y, ldy, w, o.chunk, ws.part, out, ws.counter, fin_chol ? 1 : 0, R, status};
     const bool aligned = ((reinterpret_cast<uintptr_t>(X) | reinterpret_cast<uintptr_t>(Y)) % 16 == 0) &&
                          (ldx % 2 == 0) && (ldy % 2 == 0);
-    if (aligned && n >= 32 * 64 && w <= 12 && (same || jx <= 64)) {
-        // per-warp cp.async ring + scalar register blocking (exact FMA count)
-        const int WMv = w <= 4 ? 4 : (w <= 8 ? 8 : 12);
-        int CG = 1, chunk = w;
-        if (!same) {
-            const int need = (jx + 3) / 4;                        // JB = 4 X-columns per lane
-            CG = 1;
-            while (CG < need) CG *= 2;                            // <= 16 for jx <= 64
-            chunk = 4 * CG;
-        }
-        Geo g2 = o;
-        g2.chunk = same ? w : chunk;
-        g2.gy = 1;
-        g2.gx = d.sms;
-        XtyArgs b2 = a;
-        b2.chunk = g2.chunk;
-        const int ncol = w + ((same || X == Y) ? 0 : std::min(g2.chunk, jx));
-        const size_t ring_w = size_t(SC_S) * ncol * (32 + 4) * sizeof(double);
-        int nw = int((200 * 1024) / ring_w);
-        nw = nw < 2 ? 2 : (nw > 8 ? 8 : nw);
-        const int nacc = same ? WMv * (WMv + 1) / 2 : 4 * WMv;
-        size_t smem = std::max(size_t(nw) * ring_w, size_t(nw) * (same ? 1 : CG) * nacc * sizeof(double));
-        smem = std::max(smem, size_t(32 * nw) * sizeof(double));
-        if (size_t(g2.gx) * g2.chunk * w > ws.cap) return -1;
-        auto go = [&](auto kfn) {
-            cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
-            ++g_launches;
-            kfn<<<dim3(g2.gx, 1), 32 * nw, smem, st>>>(b2, CG);
-        };
-        if (same) {
-            if (WMv == 4) go(k_xty_sc<1, 4, true>);
-            else if (WMv == 8) go(k_xty_sc<1, 8, true>);
-            else go(k_xty_sc<1, 12, true>);
-        } else {
-            if (WMv == 4) go(k_xty_sc<4, 4, false>);
-            else if (WMv == 8) go(k_xty_sc<4, 8, false>);
-            else go(k_xty_sc<4, 12, false>);
-        }
-        return 0;
-    }
     if (aligned && n >= 32 * 64) {
         // per-warp cp.async pipeline: size the warps so the rings use ~200 KB of smem
         constexpr int TW = 32;
