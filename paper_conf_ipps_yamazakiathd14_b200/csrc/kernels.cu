@@ -32,7 +32,7 @@ long long g_launches = 0;
 // not depend on the partition.
 // ------------------------------------------------------------------------------------
 template <int MODE>   // 0: Ax   1: Ax + bu u   2: Ax + bu u + bw w   3: u - Ax
-__global__ void __launch_bounds__(NT) k_spmv_sell32(int64_t nrows, const int64_t* __restrict__ sptr,
+__global__ void __launch_bounds__(NT, 4) k_spmv_sell32(int64_t nrows, const int64_t* __restrict__ sptr,
                                                     const int64_t* __restrict__ sinfo,
                                                     const int32_t* __restrict__ dcol, int64_t ncols,
                                                     const double* __restrict__ val,
@@ -41,17 +41,11 @@ __global__ void __launch_bounds__(NT) k_spmv_sell32(int64_t nrows, const int64_t
                                                     const double* __restrict__ w, double bw,
                                                     double* __restrict__ y) {
     const int64_t r = int64_t(blockIdx.x) * NT + threadIdx.x;
+    if ((r & ~int64_t(31)) >= nrows) return;           // whole warp beyond the matrix
+    // every lane of the warp takes part (shuffles); rows >= nrows compute but do not store
+    const int64_t rr = r < nrows ? r : nrows - 1;
+    const double acc = sell_row_dot(rr, sptr, sinfo, dcol, ncols, val, x, false);
     if (r >= nrows) return;
-    const int64_t sl = r >> 5;
-    const int lane = int(r & 31);
-    const int64_t b = __ldg(sptr + sl), e = __ldg(sptr + sl + 1);
-    const int64_t info = __ldg(sinfo + sl);
-    const bool dia = info & 1;
-    const int64_t dp = info >> 1;
-    double acc = 0.0;
-#pragma unroll 4
-    for (int64_t o = b + lane; o < e; o += 32)
-        acc = fma(__ldg(val + o), __ldg(x + sell_col(r, o, b, dia, dp, dcol, ncols)), acc);
     double out;
     if constexpr (MODE == 3) {
         out = __ldg(u + r) - acc;

@@ -15,8 +15,9 @@ struct Dev {
 };
 
 // Sliced ELLPACK, slice height 32 (one warp), column-major inside a slice, with per-slice
-// diagonal-offset column compression: sinfo[sl] = (dptr << 1) | dia.
-//   dia == 1: entry t of row r has column clamp(r + dcol[dptr + t]) (zero value if absent)
+// diagonal-offset column compression: sinfo[sl] = dptr << 2 | clamp << 1 | dia.
+//   dia == 1: entry t of row r has column r + dcol[dptr + t] (<= 32 diagonals; zero value if the
+//             row lacks it; clamped into [0, ncols) only in slices flagged `clamp`)
 //   dia == 0: entry t of lane l has column dcol[dptr + 32 t + l]
 struct Sell {
     int64_t nrows = 0;          // stored rows (extended rows at distance <= s-1)
@@ -31,14 +32,61 @@ struct Sell {
     double* val = nullptr;
 };
 
-// column of stored entry o (slice base b) of row r
-__device__ __forceinline__ int64_t sell_col(int64_t r, int64_t o, int64_t b, bool dia, int64_t dp,
-                                            const int32_t* __restrict__ dcol, int64_t ncols) {
-    if (dia) {
-        int64_t c = r + __ldg(dcol + dp + ((o - b) >> 5));
-        return c < 0 ? 0 : (c >= ncols ? ncols - 1 : c);
+// y_r = sum over the stored entries of row r (one lane of a 32-row slice), in stored order.
+// Loads of 8 entries are issued before their FMAs; DIA offsets are loaded once per slice (lane
+// t holds offset t) and broadcast with shuffles, so no column index is loaded per entry.
+__device__ __forceinline__ double sell_row_dot(int64_t r, const int64_t* __restrict__ sptr,
+                                               const int64_t* __restrict__ sinfo,
+                                               const int32_t* __restrict__ dcol, int64_t ncols,
+                                               const double* __restrict__ val,
+                                               const double* __restrict__ x, bool coherent) {
+    const int64_t sl = r >> 5;
+    const int lane = int(r & 31);
+    const int64_t b = __ldg(sptr + sl), e = __ldg(sptr + sl + 1);
+    const int W = int((e - b) >> 5);
+    const int64_t info = __ldg(sinfo + sl);
+    const int64_t dp = info >> 2;
+    double acc = 0.0;
+    auto ldx = [&](int64_t c) { return coherent ? __ldca(x + c) : __ldg(x + c); };
+    if (info & 1) {
+        const int myoff = lane < W ? __ldg(dcol + dp + lane) : 0;
+        const bool clamp = (info & 2) != 0;
+        for (int t0 = 0; t0 < W; t0 += 8) {
+            double v[8], xv[8];
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+                const int off = __shfl_sync(0xffffffffu, myoff, (t0 + u) & 31);
+                if (t0 + u < W) {
+                    int64_t c = r + off;
+                    if (clamp) c = c < 0 ? 0 : (c >= ncols ? ncols - 1 : c);
+                    v[u] = __ldg(val + b + 32 * (t0 + u) + lane);
+                    xv[u] = ldx(c);
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < 8; ++u)
+                if (t0 + u < W) acc = fma(v[u], xv[u], acc);
+        }
+    } else {
+        for (int t0 = 0; t0 < W; t0 += 8) {
+            double v[8];
+            int c[8];
+#pragma unroll
+            for (int u = 0; u < 8; ++u)
+                if (t0 + u < W) {
+                    v[u] = __ldg(val + b + 32 * (t0 + u) + lane);
+                    c[u] = __ldg(dcol + dp + 32 * (t0 + u) + lane);
+                }
+            double xv[8];
+#pragma unroll
+            for (int u = 0; u < 8; ++u)
+                if (t0 + u < W) xv[u] = ldx(c[u]);
+#pragma unroll
+            for (int u = 0; u < 8; ++u)
+                if (t0 + u < W) acc = fma(v[u], xv[u], acc);
+        }
     }
-    return __ldg(dcol + dp + (o - b));
+    return acc;
 }
 
 // Single-GPU temporally blocked MPK (mpk_wave.cu).

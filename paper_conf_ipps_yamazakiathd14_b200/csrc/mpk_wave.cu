@@ -24,7 +24,6 @@ namespace kern {
 
 namespace {
 constexpr int NT = 256;
-constexpr int RPT = 4;                  // rows per thread in flight (memory-level parallelism)
 
 __device__ __forceinline__ int ld_acquire(const int* p) {
     int v;
@@ -67,56 +66,15 @@ __global__ void __launch_bounds__(NT) k_mpk_wave(WaveArgs a) {
         double* y = a.V + a.ldv * (a.j + k);
         const double th = a.theta[k - 1], b2 = a.b2[k - 1];
         const double* xp = a.kind[k - 1] == 2 ? a.V + a.ldv * (a.j + k - 2) : nullptr;
-        // RPT rows per thread, loads of all RPT rows issued together per stored column
-        for (int64_t rb = r0 + threadIdx.x; rb < r1; rb += int64_t(NT) * RPT) {
-            int64_t o[RPT], e[RPT], bs[RPT], dp[RPT];
-            bool dia[RPT];
-            double acc[RPT];
-#pragma unroll
-            for (int u = 0; u < RPT; ++u) {
-                const int64_t r = rb + int64_t(NT) * u;
-                acc[u] = 0.0;
-                if (r < r1) {
-                    bs[u] = __ldg(a.sptr + (r >> 5));
-                    o[u] = bs[u] + (r & 31);
-                    e[u] = __ldg(a.sptr + (r >> 5) + 1);
-                    const int64_t info = __ldg(a.sinfo + (r >> 5));
-                    dia[u] = info & 1;
-                    dp[u] = info >> 1;
-                } else {
-                    o[u] = 0; e[u] = 0; bs[u] = 0; dp[u] = 0; dia[u] = false;
-                }
-            }
-            bool more = true;
-            while (more) {
-                more = false;
-                double vv[RPT], xv[RPT];
-#pragma unroll
-                for (int u = 0; u < RPT; ++u) {
-                    if (o[u] < e[u]) {
-                        const int64_t r = rb + int64_t(NT) * u;
-                        vv[u] = __ldg(a.val + o[u]);
-                        xv[u] = __ldca(x + sell_col(r, o[u], bs[u], dia[u], dp[u], a.dcol, a.ncols));
-                    }
-                }
-#pragma unroll
-                for (int u = 0; u < RPT; ++u) {
-                    if (o[u] < e[u]) {
-                        acc[u] = fma(vv[u], xv[u], acc[u]);
-                        o[u] += 32;
-                        more |= o[u] < e[u];
-                    }
-                }
-            }
-#pragma unroll
-            for (int u = 0; u < RPT; ++u) {
-                const int64_t r = rb + int64_t(NT) * u;
-                if (r < r1) {
-                    double out = acc[u];
-                    if (th != 0.0) out = fma(-th, __ldca(x + r), out);
-                    if (xp) out = fma(b2, __ldca(xp + r), out);
-                    __stcg(y + r, out);
-                }
+        // same row computation as k_spmv_sell32 (sell_row_dot), x through L1 (see header)
+        for (int64_t r = r0 + threadIdx.x; (r & ~int64_t(31)) < r1; r += NT) {
+            const int64_t rr = r < r1 ? r : r1 - 1;
+            const double acc = sell_row_dot(rr, a.sptr, a.sinfo, a.dcol, a.ncols, a.val, x, true);
+            if (r < r1) {
+                double out = acc;
+                if (th != 0.0) out = fma(-th, __ldca(x + r), out);
+                if (xp) out = fma(b2, __ldca(xp + r), out);
+                __stcg(y + r, out);
             }
         }
         __syncthreads();

@@ -177,7 +177,7 @@ int build_sell(cagmres* h, const cagmres_plan& p) {
         }
         std::sort(o.begin(), o.end());
         o.erase(std::unique(o.begin(), o.end()), o.end());
-        const bool use_dia = int64_t(o.size()) <= wmax + (wmax + 3) / 4 &&
+        const bool use_dia = int64_t(o.size()) <= wmax + (wmax + 3) / 4 && o.size() <= 32 &&
                              (o.empty() || (o.front() > INT32_MIN / 2 && o.back() < INT32_MAX / 2));
         int64_t wdt = wmax;
         if (use_dia) {
@@ -185,10 +185,13 @@ int build_sell(cagmres* h, const cagmres_plan& p) {
             ++ndia;
             wdt = int64_t(o.size());
             offs[size_t(sl)].assign(o.begin(), o.end());
-            sinfo[size_t(sl)] = (ndcol << 1) | 1;
+            // clamp flag: some row + offset of this slice leaves [0, n_ext)
+            const int64_t r0 = sl * 32, r1 = sl * 32 + 31;
+            const bool clamp = !o.empty() && (r0 + o.front() < 0 || r1 + o.back() >= p.n_ext);
+            sinfo[size_t(sl)] = (ndcol << 2) | (clamp ? 2 : 0) | 1;
             ndcol += wdt;
         } else {
-            sinfo[size_t(sl)] = ndcol << 1;
+            sinfo[size_t(sl)] = ndcol << 2;
             ndcol += 32 * wdt;
         }
         sptr[size_t(sl) + 1] = sptr[size_t(sl)] + 32 * wdt;
@@ -198,7 +201,7 @@ int build_sell(cagmres* h, const cagmres_plan& p) {
     std::vector<double> val(static_cast<size_t>(std::max<int64_t>(tot, 1)), 0.0);
     for (int64_t sl = 0; sl < ns; ++sl) {
         const int64_t wdt = (sptr[size_t(sl) + 1] - sptr[size_t(sl)]) / 32;
-        const int64_t dp = sinfo[size_t(sl)] >> 1;
+        const int64_t dp = sinfo[size_t(sl)] >> 2;
         if (dia[size_t(sl)]) {
             const std::vector<int32_t>& of = offs[size_t(sl)];
             for (int64_t t = 0; t < wdt; ++t) dcol[size_t(dp + t)] = of[size_t(t)];
