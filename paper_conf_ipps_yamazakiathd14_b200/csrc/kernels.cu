@@ -21,6 +21,7 @@
 namespace kern {
 
 constexpr int NT = 256;
+constexpr int SPMV_BATCH = 4;           // entries whose loads are issued together
 long long g_launches = 0;
 
 // ------------------------------------------------------------------------------------
@@ -32,7 +33,7 @@ long long g_launches = 0;
 // not depend on the partition.
 // ------------------------------------------------------------------------------------
 template <int MODE>   // 0: Ax   1: Ax + bu u   2: Ax + bu u + bw w   3: u - Ax
-__global__ void __launch_bounds__(NT, 4) k_spmv_sell32(int64_t nrows, const int64_t* __restrict__ sptr,
+__global__ void __launch_bounds__(NT, 6) k_spmv_sell32(int64_t nrows, const int64_t* __restrict__ sptr,
                                                     const int64_t* __restrict__ sinfo,
                                                     const int32_t* __restrict__ dcol, int64_t ncols,
                                                     const double* __restrict__ val,
@@ -44,7 +45,7 @@ __global__ void __launch_bounds__(NT, 4) k_spmv_sell32(int64_t nrows, const int6
     if ((r & ~int64_t(31)) >= nrows) return;           // whole warp beyond the matrix
     // every lane of the warp takes part (shuffles); rows >= nrows compute but do not store
     const int64_t rr = r < nrows ? r : nrows - 1;
-    const double acc = sell_row_dot(rr, sptr, sinfo, dcol, ncols, val, x, false);
+    const double acc = sell_row_dot<SPMV_BATCH>(rr, sptr, sinfo, dcol, ncols, val, x, false);
     if (r >= nrows) return;
     double out;
     if constexpr (MODE == 3) {

@@ -35,6 +35,7 @@ struct Sell {
 // y_r = sum over the stored entries of row r (one lane of a 32-row slice), in stored order.
 // Loads of 8 entries are issued before their FMAs; DIA offsets are loaded once per slice (lane
 // t holds offset t) and broadcast with shuffles, so no column index is loaded per entry.
+template <int BATCH>
 __device__ __forceinline__ double sell_row_dot(int64_t r, const int64_t* __restrict__ sptr,
                                                const int64_t* __restrict__ sinfo,
                                                const int32_t* __restrict__ dcol, int64_t ncols,
@@ -51,10 +52,10 @@ __device__ __forceinline__ double sell_row_dot(int64_t r, const int64_t* __restr
     if (info & 1) {
         const int myoff = lane < W ? __ldg(dcol + dp + lane) : 0;
         const bool clamp = (info & 2) != 0;
-        for (int t0 = 0; t0 < W; t0 += 8) {
-            double v[8], xv[8];
+        for (int t0 = 0; t0 < W; t0 += BATCH) {
+            double v[BATCH], xv[BATCH];
 #pragma unroll
-            for (int u = 0; u < 8; ++u) {
+            for (int u = 0; u < BATCH; ++u) {
                 const int off = __shfl_sync(0xffffffffu, myoff, (t0 + u) & 31);
                 if (t0 + u < W) {
                     int64_t c = r + off;
@@ -64,25 +65,25 @@ __device__ __forceinline__ double sell_row_dot(int64_t r, const int64_t* __restr
                 }
             }
 #pragma unroll
-            for (int u = 0; u < 8; ++u)
+            for (int u = 0; u < BATCH; ++u)
                 if (t0 + u < W) acc = fma(v[u], xv[u], acc);
         }
     } else {
-        for (int t0 = 0; t0 < W; t0 += 8) {
-            double v[8];
-            int c[8];
+        for (int t0 = 0; t0 < W; t0 += BATCH) {
+            double v[BATCH];
+            int c[BATCH];
 #pragma unroll
-            for (int u = 0; u < 8; ++u)
+            for (int u = 0; u < BATCH; ++u)
                 if (t0 + u < W) {
                     v[u] = __ldg(val + b + 32 * (t0 + u) + lane);
                     c[u] = __ldg(dcol + dp + 32 * (t0 + u) + lane);
                 }
-            double xv[8];
+            double xv[BATCH];
 #pragma unroll
-            for (int u = 0; u < 8; ++u)
+            for (int u = 0; u < BATCH; ++u)
                 if (t0 + u < W) xv[u] = ldx(c[u]);
 #pragma unroll
-            for (int u = 0; u < 8; ++u)
+            for (int u = 0; u < BATCH; ++u)
                 if (t0 + u < W) acc = fma(v[u], xv[u], acc);
         }
     }
