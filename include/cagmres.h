@@ -116,6 +116,10 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
  *                          temporally blocked MPK when A is banded enough and the reuse
  *                          window fits L2 ("reducing communication of MPK on a single
  *                          GPU"); 2 = force it whenever A is banded.  Bitwise identical.
+ *   CAGMRES_OPT_SPMV     : SpMV kernel: 0 (default) = one SELL-32 slice per warp; 1, 2, 3 = two
+ *                          slices per warp with load batches 4/8/4 at 4/2/3 CTAs per SM.
+ *   CAGMRES_OPT_FUSE     : bit 0 (default 0) = BOrth pass 2 fused with the CholQR Gram;
+ *                          bit 1 (default 1) = fused first-cycle Arnoldi passes.
  *   CAGMRES_OPT_WAVE_CHUNK / _WAVE_CTAS / _WAVE_LAG : temporal-blocking tuning (rows per
  *                          chunk, multiple of 256; resident CTAs per SM; wavefront lag in
  *                          chunks, 0 = automatic). */
@@ -123,6 +127,8 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
 #define CAGMRES_OPT_WAVE_CHUNK 3
 #define CAGMRES_OPT_WAVE_CTAS  4
 #define CAGMRES_OPT_WAVE_LAG   5
+#define CAGMRES_OPT_FUSE       6
+#define CAGMRES_OPT_SPMV       7
 int cagmres_set_option(cagmres_t h, int opt, int64_t value);
 
 /* Sizes: n_loc owned rows, n_ext owned+ghost rows (P:60 i^(d,1)), ldv = leading dim of V. */

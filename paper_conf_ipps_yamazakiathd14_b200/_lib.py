@@ -17,7 +17,7 @@ EINVAL, ECUDA, ENCCL, EBREAKDOWN, ENOMEM, EGHOST, ENOTSUP = -1, -2, -3, -4, -5, 
 MONOMIAL, NEWTON = 0, 1
 CHOLQR, SVQR, CGS, MGS, CAQR = 0, 1, 2, 3, 4
 REORTH, BORTH_MGS = 0x100, 0x200
-OPT_MPK_WAVE, OPT_WAVE_CHUNK, OPT_WAVE_CTAS, OPT_WAVE_LAG = 1, 3, 4, 5
+OPT_MPK_WAVE, OPT_WAVE_CHUNK, OPT_WAVE_CTAS, OPT_WAVE_LAG, OPT_FUSE, OPT_SPMV = 1, 3, 4, 5, 6, 7
 
 
 class CSRStruct(C.Structure):

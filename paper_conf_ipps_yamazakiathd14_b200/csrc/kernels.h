@@ -22,6 +22,7 @@ struct Dev {
 struct Sell {
     int64_t nrows = 0;          // stored rows (extended rows at distance <= s-1)
     int64_t nslices = 0;
+    int variant = 0;            // SpMV kernel: 0 one slice per warp (default); 1..3 two slices per warp
     int64_t nstored = 0;        // stored values incl. padding
     int64_t nnz = 0;            // true nonzeros
     int64_t ncols = 0;          // valid x entries (clamp bound for DIA slices)
@@ -33,7 +34,9 @@ struct Sell {
 };
 
 // y_r = sum over the stored entries of row r (one lane of a 32-row slice), in stored order.
-// Loads of 8 entries are issued before their FMAs; DIA offsets are loaded once per slice (lane
+// All 32 lanes of the warp call it together with the 32 rows of one slice (r & 31 == lane,
+// padding rows of the last slice included), because lane t loads the slice's DIA offset t.
+// Loads of BATCH entries are issued before their FMAs; DIA offsets are loaded once per slice (lane
 // t holds offset t) and broadcast with shuffles, so no column index is loaded per entry.
 template <int BATCH>
 __device__ __forceinline__ double sell_row_dot(int64_t r, const int64_t* __restrict__ sptr,
@@ -48,40 +51,59 @@ __device__ __forceinline__ double sell_row_dot(int64_t r, const int64_t* __restr
     const int64_t info = __ldg(sinfo + sl);
     const int64_t dp = info >> 2;
     double acc = 0.0;
-    auto ldx = [&](int64_t c) { return coherent ? __ldca(x + c) : __ldg(x + c); };
+    auto ldx = [&](const double* p) { return coherent ? __ldca(p) : __ldg(p); };
+    const double* vp = val + b + lane;              // entry t of this row: vp[32 t]
     if (info & 1) {
         const int myoff = lane < W ? __ldg(dcol + dp + lane) : 0;
-        const bool clamp = (info & 2) != 0;
-        for (int t0 = 0; t0 < W; t0 += BATCH) {
-            double v[BATCH], xv[BATCH];
+        if (!(info & 2)) {                          // no clamping: x address = x + r + offset
+            const double* xr = x + r;
+            for (int t0 = 0; t0 < W; t0 += BATCH, vp += 32 * BATCH) {
+                double v[BATCH], xv[BATCH];
 #pragma unroll
-            for (int u = 0; u < BATCH; ++u) {
-                const int off = __shfl_sync(0xffffffffu, myoff, (t0 + u) & 31);
-                if (t0 + u < W) {
-                    int64_t c = r + off;
-                    if (clamp) c = c < 0 ? 0 : (c >= ncols ? ncols - 1 : c);
-                    v[u] = __ldg(val + b + 32 * (t0 + u) + lane);
-                    xv[u] = ldx(c);
+                for (int u = 0; u < BATCH; ++u) {
+                    const int off = __shfl_sync(0xffffffffu, myoff, (t0 + u) & 31);
+                    if (t0 + u < W) {
+                        v[u] = __ldg(vp + 32 * u);
+                        xv[u] = ldx(xr + off);
+                    }
                 }
-            }
 #pragma unroll
-            for (int u = 0; u < BATCH; ++u)
-                if (t0 + u < W) acc = fma(v[u], xv[u], acc);
+                for (int u = 0; u < BATCH; ++u)
+                    if (t0 + u < W) acc = fma(v[u], xv[u], acc);
+            }
+        } else {
+            for (int t0 = 0; t0 < W; t0 += BATCH, vp += 32 * BATCH) {
+                double v[BATCH], xv[BATCH];
+#pragma unroll
+                for (int u = 0; u < BATCH; ++u) {
+                    const int off = __shfl_sync(0xffffffffu, myoff, (t0 + u) & 31);
+                    if (t0 + u < W) {
+                        int64_t c = r + off;
+                        c = c < 0 ? 0 : (c >= ncols ? ncols - 1 : c);
+                        v[u] = __ldg(vp + 32 * u);
+                        xv[u] = ldx(x + c);
+                    }
+                }
+#pragma unroll
+                for (int u = 0; u < BATCH; ++u)
+                    if (t0 + u < W) acc = fma(v[u], xv[u], acc);
+            }
         }
     } else {
-        for (int t0 = 0; t0 < W; t0 += BATCH) {
+        const int32_t* cp = dcol + dp + lane;
+        for (int t0 = 0; t0 < W; t0 += BATCH, vp += 32 * BATCH, cp += 32 * BATCH) {
             double v[BATCH];
             int c[BATCH];
 #pragma unroll
             for (int u = 0; u < BATCH; ++u)
                 if (t0 + u < W) {
-                    v[u] = __ldg(val + b + 32 * (t0 + u) + lane);
-                    c[u] = __ldg(dcol + dp + 32 * (t0 + u) + lane);
+                    v[u] = __ldg(vp + 32 * u);
+                    c[u] = __ldg(cp + 32 * u);
                 }
             double xv[BATCH];
 #pragma unroll
             for (int u = 0; u < BATCH; ++u)
-                if (t0 + u < W) xv[u] = ldx(c[u]);
+                if (t0 + u < W) xv[u] = ldx(x + c[u]);
 #pragma unroll
             for (int u = 0; u < BATCH; ++u)
                 if (t0 + u < W) acc = fma(v[u], xv[u], acc);
@@ -125,6 +147,25 @@ size_t arnoldi_ws_doubles(const Dev& d);
 size_t caqr_ws_doubles(int64_t n, int w);
 int caqr(const Dev& d, int64_t n, double* P, int64_t ldp, int w, double* R, int c0, double* ws,
          cudaStream_t st);
+
+// BOrth pass 2 fused with the CholQR Gram (fused.cu): P := P - X C (P: n x w, X: n x jx,
+// C: jx x w ld jx) and out = [q0 P]^T [q0 P] ((w+1) x (w+1), ld w+1), R = chol(out) if
+// fin_chol.  Returns -1 when not applicable (unaligned, jx > 64, w + 1 > 16, tiny n).
+struct UpdGramArgs {
+    int64_t n;
+    const double* X; int64_t ldx; int jx;
+    double* P; int64_t ldp; int w;
+    const double* q0;
+    const double* C;
+    double* part;
+    double* out;
+    unsigned int* counter;
+    int fin_chol;
+    double* R;
+    int* status;
+};
+int update_gram(const Dev& d, const UpdGramArgs& a, cudaStream_t st);
+size_t update_gram_ws_doubles(const Dev& d);
 
 // Status bits written by device kernels into the handle's status word.
 enum : int { ST_CHOL = 1, ST_SVQR = 2, ST_NORM = 4 };

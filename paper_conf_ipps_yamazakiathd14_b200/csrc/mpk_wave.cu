@@ -68,8 +68,7 @@ __global__ void __launch_bounds__(NT) k_mpk_wave(WaveArgs a) {
         const double* xp = a.kind[k - 1] == 2 ? a.V + a.ldv * (a.j + k - 2) : nullptr;
         // same row computation as k_spmv_sell32 (sell_row_dot), x through L1 (see header)
         for (int64_t r = r0 + threadIdx.x; (r & ~int64_t(31)) < r1; r += NT) {
-            const int64_t rr = r < r1 ? r : r1 - 1;
-            const double acc = sell_row_dot<4>(rr, a.sptr, a.sinfo, a.dcol, a.ncols, a.val, x, true);
+            const double acc = sell_row_dot<4>(r, a.sptr, a.sinfo, a.dcol, a.ncols, a.val, x, true);
             if (r < r1) {
                 double out = acc;
                 if (th != 0.0) out = fma(-th, __ldca(x + r), out);

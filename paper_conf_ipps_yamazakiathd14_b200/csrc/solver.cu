@@ -93,6 +93,7 @@ struct cagmres {
     double* arn_part = nullptr;            // fused Arnoldi partials
     unsigned int* arn_counter = nullptr;
     bool arnoldi_fuse = true;
+    bool fuse_borth_gram = false;          // BOrth pass 2 + CholQR Gram in one pass (fused.cu; slower)
     int* status = nullptr;
     // halo (distributed)
     std::vector<int64_t> send_off, recv_off;
@@ -655,6 +656,33 @@ int ca_cycle(cagmres* h, const std::vector<Block>& bl) {
         for (int pass = 0; pass < (re2 ? 2 : 1); ++pass) {
             double* C = h->tab + (pass ? b.c2 : b.c1);
             double* R = h->tab + (pass ? b.r2 : b.r1);
+            if (j > 0 && !mgs && kind == CAGMRES_CHOLQR && h->fuse_borth_gram) {
+                // BOrth pass 1, then [P -= Q C  fused with  B = [q_j P]^T [q_j P] (+ chol)]
+                const double nl = double(h->n_loc);
+                int fused = -1;
+                {
+                    Scope sc(h, PH_BORTH);
+                    TRY(xty_global(h, h->V, h->ldv, j, Pj + h->ldv, h->ldv, sb, C, false, nullptr));
+                    kern::UpdGramArgs ua{h->n_loc, h->V, h->ldv, j, Pj + h->ldv, h->ldv, sb, Pj, C, h->ws.part,
+                                         h->gbuf, h->ws.counter, h->nranks == 1 ? 1 : 0, R, h->status};
+                    fused = kern::update_gram(h->dev, ua, h->stream);
+                    if (fused == 0) h->bytes[PH_BORTH] += 8.0 * nl * (2.0 * j + 3.0 * sb);
+                    else kern::update(h->dev, h->n_loc, h->V, h->ldv, j, Pj + h->ldv, h->ldv, sb, C, h->stream);
+                }
+                if (fused == 0) {
+                    Scope sc(h, PH_TSQR);
+                    if (h->nranks > 1) {
+                        TRY(allreduce(h, h->gbuf, size_t(w) * size_t(w)));
+                        kern::chol(h->gbuf, w, R, h->status, h->stream);
+                    }
+                    kern::trsm(h->dev, h->n_loc, Pj, h->ldv, w, R, 1, h->stream);
+                    h->bytes[PH_TSQR] += 8.0 * nl * (2.0 * w + double(w - 1));   // Gram bytes as if unfused
+                    continue;
+                }
+                h->bytes[PH_BORTH] += 8.0 * nl * (2.0 * j + 3.0 * sb);
+                TRY(tsqr_panel(h, Pj, h->ldv, w, R, kind, 1));
+                continue;
+            }
             TRY(borth_panel(h, h->V, h->ldv, j, Pj + h->ldv, h->ldv, sb, C, mgs));
             TRY(tsqr_panel(h, Pj, h->ldv, w, R, kind, 1));
         }
@@ -846,6 +874,8 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
     if (!h) return CAGMRES_EINVAL;
     switch (opt) {
         case CAGMRES_OPT_MPK_WAVE: h->wave_on = value != 0; h->wave_force = value == 2; return CAGMRES_OK;
+        case CAGMRES_OPT_SPMV: if (value < 0 || value > 3) return CAGMRES_EINVAL; h->A.variant = value; return CAGMRES_OK;
+        case CAGMRES_OPT_FUSE: h->fuse_borth_gram = (value & 1) != 0; h->arnoldi_fuse = (value & 2) != 0; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK:
             if (value < 256 || value % 256) return CAGMRES_EINVAL;
             h->wave_CH = int(value); wave_reset_pairs(h); return CAGMRES_OK;

@@ -116,8 +116,8 @@ class Solver:
         L.check(self._lib.cagmres_set_stream(self._h, C.c_void_p(s.cuda_stream)), "set_stream")
 
     def set_option(self, opt, value):
-        """opt: "mpk_wave", "wave_chunk", "wave_ctas", "wave_lag" (CAGMRES_OPT_*)."""
-        code = {"mpk_wave": 1, "wave_chunk": 3, "wave_ctas": 4, "wave_lag": 5}[opt]
+        """opt: "mpk_wave", "wave_chunk", "wave_ctas", "wave_lag", "fuse", "spmv" (CAGMRES_OPT_*)."""
+        code = {"mpk_wave": 1, "wave_chunk": 3, "wave_ctas": 4, "wave_lag": 5, "fuse": 6, "spmv": 7}[opt]
         L.check(self._lib.cagmres_set_option(self._h, code, int(value)), "set_option")
 
     def close(self):

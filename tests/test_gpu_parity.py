@@ -74,11 +74,15 @@ SHIFTS = (np.array([7.9, 7.9, 0.09, 0.09, 3.8, 5.5, 1.2, 6.6, 2.5, 4.4]),
 
 # ----------------------------------------------------------------------------- MPK
 @pytest.mark.parametrize("basis", ["monomial", "newton"])
-@pytest.mark.parametrize("gen", ["C1", "cd27_ragged", "g3_small"])
+@pytest.mark.parametrize("gen", ["C1", "cd27_ragged", "g3_small", "banded_1row_tail", "cd7_ragged"])
 def test_mpk_parity(basis, gen):
+    """Last-slice cases: banded n = 300001 leaves ONE valid row in a DIA slice of 14 diagonals
+    (lanes 1..13 must still load their offsets), 2025 = 63*32 + 9 rows for the 5-pt stencil."""
     A = {"C1": lambda: G.convection_diffusion(32, 2, 5),
          "cd27_ragged": lambda: G.convection_diffusion(13, 3, 27),       # n = 2197, ragged tail
-         "g3_small": lambda: G.g3_shaped(n=50001, width=250)}[gen]()
+         "g3_small": lambda: G.g3_shaped(n=50001, width=250),
+         "banded_1row_tail": lambda: G.banded(n=300001),
+         "cd7_ragged": lambda: G.convection_diffusion(45, 2, 5)}[gen]()
     As = A.to_scipy()
     s = 6
     S = Solver(A, s=s, m=12, basis=basis)
@@ -113,12 +117,32 @@ def test_mpk_wave_bitwise_equals_stepwise(gen):
     q = dev(G.u(5, np.arange(A.n)))
     S1 = Solver(A, s=10, m=30, basis="newton")
     S2 = Solver(A, s=10, m=30, basis="newton")
+    S1.set_option("mpk_wave", 2)                   # forced on (off by default)
     S2.set_option("mpk_wave", 0)
     for S in (S1, S2):
         S.set_shifts(*SHIFTS)
     for sb in (10, 4, 2):
         W1, W2 = S1.mpk(q, sb), S2.mpk(q, sb)
         assert torch.equal(W1, W2), (gen, sb)
+
+
+@pytest.mark.parametrize("gen", ["cd27_ragged", "g3_small", "banded"])
+def test_spmv_variants_bitwise(gen):
+    """Every SpMV kernel variant (CAGMRES_OPT_SPMV: one or two SELL-32 slices per warp, load
+    batches 4/8) sums each row in the same order: the MPK bases are bitwise identical; the
+    parity of variant 0 against the oracle is test_mpk_parity."""
+    A = {"cd27_ragged": lambda: G.convection_diffusion(17, 3, 27),
+         "g3_small": lambda: G.g3_shaped(n=40000, width=200),
+         "banded": lambda: G.banded(n=300001)}[gen]()
+    q = dev(G.u(6, np.arange(A.n)))
+    S = Solver(A, s=6, m=30, basis="newton")
+    S.set_shifts(*SHIFTS)
+    Ws = []
+    for v in range(4):
+        S.set_option("spmv", v)
+        Ws.append(S.mpk(q, 6))
+    for v in range(1, 4):
+        assert torch.equal(Ws[v], Ws[0]), v
 
 
 def test_mpk_full_size_C2():
@@ -274,3 +298,23 @@ def test_solve_full_size_C2():
     assert hist_within_envelope(st.hist, ref, env)
     r = b - As @ x.cpu().numpy()
     assert np.linalg.norm(r) <= 1.01e-8 * np.linalg.norm(b)
+
+
+@pytest.mark.parametrize("fuse", [0, 1])
+@pytest.mark.parametrize("s,m,reorth", [(5, 30, False), (15, 60, True), (10, 80, False)])
+def test_solve_fused_borth_gram(fuse, s, m, reorth):
+    """BOrth pass 2 fused with the CholQR Gram (fused.cu; j up to 60 -> 16 k-tiles, w+1 = 16)
+    against the unfused path, both vs the oracle; m = 80 exceeds the fused kernel's j <= 64
+    and falls back to the separate update + Gram inside a cycle.  n = 2500 (ragged tail)."""
+    A = G.convection_diffusion(50, 2, 5)
+    As = A.to_scipy()
+    b = G.rhs(A.n)
+    sh = O.modified_leja(O.ritz_values(O.arnoldi_cgs2(As, b, m)[1], m), s)
+    S = Solver(A, s=s, m=m, basis="newton", reorth=reorth)
+    S.set_option("fuse", fuse | 2)
+    S.set_shifts(*sh)
+    x, st = S.solve(dev(b), tol=1e-8, maxit=40)
+    ref, env = rounding_envelope(As, b, s=s, m=m, basis="newton", reorth=reorth, tol=1e-8, shifts=sh)
+    assert st.status == 0
+    assert abs(st.cycles - len(ref)) <= 1
+    assert hist_within_envelope(st.hist, ref, env)
