@@ -117,7 +117,9 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
  *                          window fits L2 ("reducing communication of MPK on a single
  *                          GPU"); 2 = force it whenever A is banded.  Bitwise identical.
  *   CAGMRES_OPT_SPMV     : SpMV kernel: 0 (default) = one SELL-32 slice per warp; 1, 2, 3 = two
- *                          slices per warp with load batches 4/8/4 at 4/2/3 CTAs per SM.
+ *                          slices per warp with load batches 4/8/4 at 4/2/3 CTAs per SM;
+ *                          4, 5 = persistent grid, slice descriptors software-pipelined two
+ *                          slices ahead, load batches 8/4.  All variants are bitwise identical.
  *   CAGMRES_OPT_FUSE     : bit 0 (default 0) = BOrth pass 2 fused with the CholQR Gram;
  *                          bit 1 (default 1) = fused first-cycle Arnoldi passes.
  *   CAGMRES_OPT_WAVE_CHUNK / _WAVE_CTAS / _WAVE_LAG : temporal-blocking tuning (rows per

@@ -55,16 +55,32 @@ def build(verbose: bool = False, force: bool = False) -> str:
     nccl_so = sorted(glob.glob(os.path.join(lib, "libnccl.so*")))
     link = ["-L", libdir, "-l:" + os.path.basename(nccl_so[0])] if not os.path.exists(
         os.path.join(libdir, "libnccl.so")) else ["-L", libdir, "-lnccl"]
-    cmd = [nvcc, "-O3", *ARCH, "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC,-O3",
-           "-Xptxas", "-v" if verbose else "-O3",
-           "-I", os.path.join(ROOT, "include"), "-I", inc,
-           *sources(), *link, "-Xlinker", "-rpath," + libdir, "-lcudart", "-o", LIB + ".tmp"]
+    common = ["-O3", *ARCH, "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3",
+              "-Xptxas", "-v" if verbose else "-O3", "-I", os.path.join(ROOT, "include"), "-I", inc]
+    objdir = os.path.join(ROOT, "build", "obj")
+    os.makedirs(objdir, exist_ok=True)
+
+    def compile_one(src):
+        obj = os.path.join(objdir, os.path.basename(src) + ".o")
+        r = subprocess.run([nvcc, *common, "-c", src, "-o", obj], capture_output=True, text=True)
+        return src, obj, r
+
+    # one nvcc per translation unit, in parallel (no cross-TU device code: no -rdc needed)
+    from concurrent.futures import ThreadPoolExecutor
+    with ThreadPoolExecutor(max_workers=min(16, os.cpu_count() or 4)) as ex:
+        results = list(ex.map(compile_one, sources()))
+    for src, _, r in results:
+        if r.returncode != 0:
+            sys.stderr.write(r.stdout + r.stderr)
+            raise RuntimeError(f"nvcc build of {os.path.basename(src)} failed")
+        if verbose:
+            sys.stderr.write(r.stderr)
+    cmd = [nvcc, *ARCH, "-shared", "-Xcompiler", "-fPIC", *[o for _, o, _ in results], *link,
+           "-Xlinker", "-rpath," + libdir, "-lcudart", "-o", LIB + ".tmp"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)
-        raise RuntimeError("nvcc build of libcagmres.so failed")
-    if verbose:
-        sys.stderr.write(r.stderr)
+        raise RuntimeError("link of libcagmres.so failed")
     os.replace(LIB + ".tmp", LIB)
     return LIB
 

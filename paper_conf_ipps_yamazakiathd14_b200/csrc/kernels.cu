@@ -141,12 +141,90 @@ __global__ void __launch_bounds__(NT, MINB) k_spmv_sell32_x2(int64_t nrows, cons
     }
 }
 
+// Persistent SpMV with a software-pipelined slice descriptor.  In k_spmv_sell32 every warp
+// pays a chain of dependent loads before its first x gather (sptr/sinfo -> DIA offsets ->
+// x), ~3 L2/HBM latencies for 32 rows of ~7 entries.  Here a grid of (SMs x resident CTAs)
+// warps strides over the slices and, while slice i's values and x are in flight, already
+// holds slice i+1's (b, W, info) and offsets and loads slice i+2's (b, W, info): one latency
+// per slice.  Per row the FMA order is t = 0..W-1 exactly as sell_row_dot: results are
+// bitwise identical to k_spmv_sell32.
+template <int MODE, int PB, int MINB>
+__global__ void __launch_bounds__(NT, MINB) k_spmv_sell32_persist(int64_t nrows, const int64_t* __restrict__ sptr,
+                                                             const int64_t* __restrict__ sinfo,
+                                                             const int32_t* __restrict__ dcol, int64_t ncols,
+                                                             const double* __restrict__ val,
+                                                             const double* __restrict__ x,
+                                                             const double* __restrict__ u, double bu,
+                                                             const double* __restrict__ w, double bw,
+                                                             double* __restrict__ y) {
+    const int lane = threadIdx.x & 31;
+    const int64_t nsl = (nrows + 31) >> 5;
+    const int64_t stride = int64_t(gridDim.x) * (NT / 32);
+    int64_t sl = (int64_t(blockIdx.x) * NT + threadIdx.x) >> 5;
+    if (sl >= nsl) return;
+    // descriptors: current slice (b0, W0, i0, o0), next (b1, W1, i1, o1), after next (b2, W2, i2)
+    int64_t b0, i0, b1 = 0, i1 = 1, b2, i2;
+    int W0, W1 = 0, W2, o0, o1;
+    sell_slice_meta(sl, sptr, sinfo, b0, W0, i0);
+    if (sl + stride < nsl) sell_slice_meta(sl + stride, sptr, sinfo, b1, W1, i1);
+    o0 = sell_slice_off(lane, W0, i0, dcol);
+#pragma unroll 1
+    for (; sl < nsl; sl += stride) {
+        b2 = 0; W2 = 0; i2 = 1;
+        if (sl + 2 * stride < nsl) sell_slice_meta(sl + 2 * stride, sptr, sinfo, b2, W2, i2);
+        o1 = sell_slice_off(lane, W1, i1, dcol);
+        const int64_t r = sl * 32 + lane;
+        const double acc = sell_slice_dot<PB, true>(r, b0, W0, i0, o0, dcol, ncols, val, x, false);
+        if (r < nrows) {
+            double out;
+            if constexpr (MODE == 3) {
+                out = __ldg(u + r) - acc;
+            } else {
+                out = acc;
+                if constexpr (MODE >= 1) out = fma(bu, __ldg(u + r), out);
+                if constexpr (MODE >= 2) out = fma(bw, __ldg(w + r), out);
+            }
+            y[r] = out;
+        }
+        b0 = b1; W0 = W1; i0 = i1; o0 = o1;
+        b1 = b2; W1 = W2; i1 = i2;
+    }
+}
+
+template <int MODE, int PB, int MINB>
+static void launch_persist(const Dev& d, const Sell& A, int64_t nrows, const double* x, double* y,
+                           const double* u, double bu, const double* w, double bw, cudaStream_t st) {
+    static int occ = 0;
+    if (occ == 0) {
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_spmv_sell32_persist<MODE, PB, MINB>, NT, 0);
+        if (occ < 1) occ = 1;
+    }
+    const int64_t nsl = (nrows + 31) >> 5;
+    int64_t g = int64_t(d.sms) * occ;
+    const int64_t need = (nsl + NT / 32 - 1) / (NT / 32);
+    if (g > need) g = need;
+    k_spmv_sell32_persist<MODE, PB, MINB><<<unsigned(g), NT, 0, st>>>(nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val,
+                                                                 x, u, bu, w, bw, y);
+}
+
 void spmv(const Dev& d, const Sell& A, int64_t nrows, const double* x, double* y,
           const double* u, double bu, const double* w, double bw, cudaStream_t st) {
     (void)d;
     if (nrows <= 0) return;
     ++g_launches;
     if (w && !u) { u = x; bu = 0.0; }             // pair step with a == 0: keep MODE 2 well formed
+    if (A.variant == 4 || A.variant == 5) {
+        if (A.variant == 4) {
+            if (w) launch_persist<2, 8, 3>(d, A, nrows, x, y, u, bu, w, bw, st);
+            else if (u) launch_persist<1, 8, 3>(d, A, nrows, x, y, u, bu, nullptr, 0.0, st);
+            else launch_persist<0, 8, 3>(d, A, nrows, x, y, nullptr, 0.0, nullptr, 0.0, st);
+        } else {
+            if (w) launch_persist<2, 4, 4>(d, A, nrows, x, y, u, bu, w, bw, st);
+            else if (u) launch_persist<1, 4, 4>(d, A, nrows, x, y, u, bu, nullptr, 0.0, st);
+            else launch_persist<0, 4, 4>(d, A, nrows, x, y, nullptr, 0.0, nullptr, 0.0, st);
+        }
+        return;
+    }
     if (A.variant >= 1) {
         const int64_t nsl = (nrows + 31) >> 5;
         const unsigned grid = unsigned((nsl + 2 * (NT / 32) - 1) / (2 * (NT / 32)));
@@ -174,6 +252,10 @@ void residual(const Dev& d, const Sell& A, int64_t nrows, const double* x, const
     (void)d;
     if (nrows <= 0) return;
     ++g_launches;
+    if (A.variant == 4 || A.variant == 5) {
+        launch_persist<3, 8, 3>(d, A, nrows, x, r, b, 1.0, nullptr, 0.0, st);
+        return;
+    }
     if (A.variant >= 1) {
         const int64_t nsl = (nrows + 31) >> 5;
         const unsigned grid = unsigned((nsl + 2 * (NT / 32) - 1) / (2 * (NT / 32)));

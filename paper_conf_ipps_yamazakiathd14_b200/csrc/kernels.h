@@ -38,23 +38,18 @@ struct Sell {
 // padding rows of the last slice included), because lane t loads the slice's DIA offset t.
 // Loads of BATCH entries are issued before their FMAs; DIA offsets are loaded once per slice (lane
 // t holds offset t) and broadcast with shuffles, so no column index is loaded per entry.
-template <int BATCH>
-__device__ __forceinline__ double sell_row_dot(int64_t r, const int64_t* __restrict__ sptr,
-                                               const int64_t* __restrict__ sinfo,
-                                               const int32_t* __restrict__ dcol, int64_t ncols,
-                                               const double* __restrict__ val,
-                                               const double* __restrict__ x, bool coherent) {
-    const int64_t sl = r >> 5;
+// SEL: load with selects (arrays always assigned) instead of guarded assignments; same FMAs.
+template <int BATCH, bool SEL = false>
+__device__ __forceinline__ double sell_slice_dot(int64_t r, int64_t b, int W, int64_t info, int myoff,
+                                                 const int32_t* __restrict__ dcol, int64_t ncols,
+                                                 const double* __restrict__ val,
+                                                 const double* __restrict__ x, bool coherent) {
     const int lane = int(r & 31);
-    const int64_t b = __ldg(sptr + sl), e = __ldg(sptr + sl + 1);
-    const int W = int((e - b) >> 5);
-    const int64_t info = __ldg(sinfo + sl);
     const int64_t dp = info >> 2;
     double acc = 0.0;
     auto ldx = [&](const double* p) { return coherent ? __ldca(p) : __ldg(p); };
     const double* vp = val + b + lane;              // entry t of this row: vp[32 t]
     if (info & 1) {
-        const int myoff = lane < W ? __ldg(dcol + dp + lane) : 0;
         if (!(info & 2)) {                          // no clamping: x address = x + r + offset
             const double* xr = x + r;
             for (int t0 = 0; t0 < W; t0 += BATCH, vp += 32 * BATCH) {
@@ -62,7 +57,11 @@ __device__ __forceinline__ double sell_row_dot(int64_t r, const int64_t* __restr
 #pragma unroll
                 for (int u = 0; u < BATCH; ++u) {
                     const int off = __shfl_sync(0xffffffffu, myoff, (t0 + u) & 31);
-                    if (t0 + u < W) {
+                    if (SEL) {                      // arrays fully assigned (stay in registers
+                        const bool ok = t0 + u < W; //  inside the persistent kernel's loop)
+                        v[u] = ok ? __ldg(vp + 32 * u) : 0.0;
+                        xv[u] = ok ? ldx(xr + off) : 0.0;
+                    } else if (t0 + u < W) {
                         v[u] = __ldg(vp + 32 * u);
                         xv[u] = ldx(xr + off);
                     }
@@ -77,9 +76,13 @@ __device__ __forceinline__ double sell_row_dot(int64_t r, const int64_t* __restr
 #pragma unroll
                 for (int u = 0; u < BATCH; ++u) {
                     const int off = __shfl_sync(0xffffffffu, myoff, (t0 + u) & 31);
-                    if (t0 + u < W) {
-                        int64_t c = r + off;
-                        c = c < 0 ? 0 : (c >= ncols ? ncols - 1 : c);
+                    const bool ok = t0 + u < W;
+                    int64_t c = r + off;
+                    c = c < 0 ? 0 : (c >= ncols ? ncols - 1 : c);
+                    if (SEL) {
+                        v[u] = ok ? __ldg(vp + 32 * u) : 0.0;
+                        xv[u] = ok ? ldx(x + c) : 0.0;
+                    } else if (ok) {
                         v[u] = __ldg(vp + 32 * u);
                         xv[u] = ldx(x + c);
                     }
@@ -95,21 +98,54 @@ __device__ __forceinline__ double sell_row_dot(int64_t r, const int64_t* __restr
             double v[BATCH];
             int c[BATCH];
 #pragma unroll
-            for (int u = 0; u < BATCH; ++u)
-                if (t0 + u < W) {
+            for (int u = 0; u < BATCH; ++u) {
+                const bool ok = t0 + u < W;
+                if (SEL) {
+                    v[u] = ok ? __ldg(vp + 32 * u) : 0.0;
+                    c[u] = ok ? __ldg(cp + 32 * u) : 0;
+                } else if (ok) {
                     v[u] = __ldg(vp + 32 * u);
                     c[u] = __ldg(cp + 32 * u);
                 }
+            }
             double xv[BATCH];
 #pragma unroll
-            for (int u = 0; u < BATCH; ++u)
-                if (t0 + u < W) xv[u] = ldx(x + c[u]);
+            for (int u = 0; u < BATCH; ++u) {
+                if (SEL) xv[u] = t0 + u < W ? ldx(x + c[u]) : 0.0;
+                else if (t0 + u < W) xv[u] = ldx(x + c[u]);
+            }
 #pragma unroll
             for (int u = 0; u < BATCH; ++u)
                 if (t0 + u < W) acc = fma(v[u], xv[u], acc);
         }
     }
     return acc;
+}
+
+// Slice descriptor of the slice holding row r: value offset b, width W (entries per row),
+// sinfo word, and (DIA slices) this lane's diagonal offset (lane t holds offset t).
+__device__ __forceinline__ void sell_slice_meta(int64_t sl, const int64_t* __restrict__ sptr,
+                                                const int64_t* __restrict__ sinfo, int64_t& b, int& W,
+                                                int64_t& info) {
+    b = __ldg(sptr + sl);
+    W = int((__ldg(sptr + sl + 1) - b) >> 5);
+    info = __ldg(sinfo + sl);
+}
+__device__ __forceinline__ int sell_slice_off(int lane, int W, int64_t info, const int32_t* __restrict__ dcol) {
+    return ((info & 1) && lane < W) ? __ldg(dcol + (info >> 2) + lane) : 0;
+}
+
+template <int BATCH>
+__device__ __forceinline__ double sell_row_dot(int64_t r, const int64_t* __restrict__ sptr,
+                                               const int64_t* __restrict__ sinfo,
+                                               const int32_t* __restrict__ dcol, int64_t ncols,
+                                               const double* __restrict__ val,
+                                               const double* __restrict__ x, bool coherent) {
+    int64_t b, info;
+    int W;
+    sell_slice_meta(r >> 5, sptr, sinfo, b, W, info);
+    const int myoff = sell_slice_off(int(r & 31), W, info, dcol);
+    return sell_slice_dot<BATCH>(r, b, W, info, myoff, dcol, ncols, val, x, coherent);
 }
 
 // Single-GPU temporally blocked MPK (mpk_wave.cu).

@@ -874,7 +874,7 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
     if (!h) return CAGMRES_EINVAL;
     switch (opt) {
         case CAGMRES_OPT_MPK_WAVE: h->wave_on = value != 0; h->wave_force = value == 2; return CAGMRES_OK;
-        case CAGMRES_OPT_SPMV: if (value < 0 || value > 3) return CAGMRES_EINVAL; h->A.variant = value; return CAGMRES_OK;
+        case CAGMRES_OPT_SPMV: if (value < 0 || value > 5) return CAGMRES_EINVAL; h->A.variant = value; return CAGMRES_OK;
         case CAGMRES_OPT_FUSE: h->fuse_borth_gram = (value & 1) != 0; h->arnoldi_fuse = (value & 2) != 0; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK:
             if (value < 256 || value % 256) return CAGMRES_EINVAL;

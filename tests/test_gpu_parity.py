@@ -129,7 +129,7 @@ def test_mpk_wave_bitwise_equals_stepwise(gen):
 @pytest.mark.parametrize("gen", ["cd27_ragged", "g3_small", "banded"])
 def test_spmv_variants_bitwise(gen):
     """Every SpMV kernel variant (CAGMRES_OPT_SPMV: one or two SELL-32 slices per warp, load
-    batches 4/8) sums each row in the same order: the MPK bases are bitwise identical; the
+    batches 4/8, persistent with pipelined slice descriptors) sums each row in the same order: the MPK bases are bitwise identical; the
     parity of variant 0 against the oracle is test_mpk_parity."""
     A = {"cd27_ragged": lambda: G.convection_diffusion(17, 3, 27),
          "g3_small": lambda: G.g3_shaped(n=40000, width=200),
@@ -138,10 +138,10 @@ def test_spmv_variants_bitwise(gen):
     S = Solver(A, s=6, m=30, basis="newton")
     S.set_shifts(*SHIFTS)
     Ws = []
-    for v in range(4):
+    for v in range(6):
         S.set_option("spmv", v)
         Ws.append(S.mpk(q, 6))
-    for v in range(1, 4):
+    for v in range(1, 6):
         assert torch.equal(Ws[v], Ws[0]), v
 
 
