@@ -150,6 +150,9 @@ def run_ours(args):
         S = Solver(A, cfg["s"], cfg["m"], basis=cfg["basis"], tsqr=cfg["tsqr"], reorth=cfg["reorth"],
                    group=group, row_starts=rs)
         b_host = G.rhs(cfg["n"], rows=(rs[rank], rs[rank + 1]))
+    for kv in args.opt:
+        k_, v_ = kv.split("=")
+        S.set_option(k_, int(v_))
     setup_s = time.time() - t0
     stream = torch.cuda.current_stream()
     b = torch.tensor(b_host, device="cuda")
@@ -251,12 +254,13 @@ def run_ours(args):
             "config": {"workload": cfg["workload"], "n": cfg["n"], "s": cfg["s"], "m": cfg["m"],
                        "tol": TOL, "cycles": stats[-1].cycles, "parallelism": f"rows{ws}",
                        "l2": "inputs larger than L2 (A 175 MB, V 520 MB) + 256 MB flush between steps",
-                       "setup_s": round(setup_s, 2)},
+                       "setup_s": round(setup_s, 2), "options": args.opt,
+                       "kernels": {k_: S.get_option(k_) for k_ in ("spmv", "gram", "fuse", "mpk_wave")}},
             "e2e": {"value": round(e2e, 4), "unit": "ms", "h2d_bytes_per_step": 8 * len(b_host),
                     "d2h_bytes_per_step": 8 * len(b_host), "each_ms": [round(v, 3) for v in e2e_ms]},
             "value_each_ms": [round(float(v), 3) for v in ms],
             "gpu_launches": int(launches_first),
-            "roofline": {"bound": "hbm", "kernel": "k_spmv_sell32 (MPK SpMV step)",
+            "roofline": {"bound": "hbm", "kernel": f"SELL-32 SpMV (MPK step), CAGMRES_OPT_SPMV variant {S.get_option('spmv')}",
                          "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(achieved / peak, 4), "traffic": traffic,
                          "peak_source": peak_kind, "bytes_per_launch": spmv_bytes,
@@ -353,6 +357,9 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C2", choices=sorted(CFG))
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--opt", action="append", default=[],
+                    help="solver option NAME=VALUE (CAGMRES_OPT_*: spmv, gram, fuse, mpk_wave, ...); "
+                         "default: the library's defaults")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":

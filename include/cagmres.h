@@ -116,10 +116,15 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
  *                          temporally blocked MPK when A is banded enough and the reuse
  *                          window fits L2 ("reducing communication of MPK on a single
  *                          GPU"); 2 = force it whenever A is banded.  Bitwise identical.
- *   CAGMRES_OPT_SPMV     : SpMV kernel: 0 (default) = one SELL-32 slice per warp; 1, 2, 3 = two
+ *   CAGMRES_OPT_SPMV     : SpMV kernel (default: the fastest on this matrix, timed once at create;
+ *                          -1 re-runs that selection): 0 = one SELL-32 slice per warp; 1, 2, 3 = two
  *                          slices per warp with load batches 4/8/4 at 4/2/3 CTAs per SM;
- *                          4, 5 = persistent grid, slice descriptors software-pipelined two
- *                          slices ahead, load batches 8/4.  All variants are bitwise identical.
+ *                          4..9 = persistent grid, slice descriptors software-pipelined two
+ *                          slices ahead, (load batch, CTAs/SM) = (8,3) (4,4) (4,5) (4,6) (2,6)
+ *                          (2,8).  All variants are bitwise identical.
+ *   CAGMRES_OPT_GRAM     : CholQR Gram kernel: 0 = FP64 tensor core (DMMA m8n8k4) on a per-warp
+ *                          cp.async ring; 1 (default) = scalar DFMA on a deeper ring (w <= 12,
+ *                          else the DMMA kernel).
  *   CAGMRES_OPT_FUSE     : bit 0 (default 0) = BOrth pass 2 fused with the CholQR Gram;
  *                          bit 1 (default 1) = fused first-cycle Arnoldi passes.
  *   CAGMRES_OPT_WAVE_CHUNK / _WAVE_CTAS / _WAVE_LAG : temporal-blocking tuning (rows per
@@ -131,7 +136,11 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
 #define CAGMRES_OPT_WAVE_LAG   5
 #define CAGMRES_OPT_FUSE       6
 #define CAGMRES_OPT_SPMV       7
+#define CAGMRES_OPT_GRAM       8
 int cagmres_set_option(cagmres_t h, int opt, int64_t value);
+/* Current value of an option (e.g. the SpMV variant the create-time selection picked).
+ * EINVAL for a null handle / pointer or an unknown option. */
+int cagmres_get_option(cagmres_t h, int opt, int64_t* value);
 
 /* Sizes: n_loc owned rows, n_ext owned+ghost rows (P:60 i^(d,1)), ldv = leading dim of V. */
 int cagmres_sizes(cagmres_t h, int64_t* n_loc, int64_t* n_ext, int64_t* ldv);

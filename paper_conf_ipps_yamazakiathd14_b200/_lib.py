@@ -61,6 +61,7 @@ SIGNATURES = {
     "cagmres_destroy": ([_P], C.c_int),
     "cagmres_set_stream": ([_P, _P], C.c_int),
     "cagmres_set_option": ([_P, C.c_int, C.c_int64], C.c_int),
+    "cagmres_get_option": ([_P, C.c_int, C.POINTER(C.c_int64)], C.c_int),
     "cagmres_sizes": ([_P, _PI64, _PI64, _PI64], C.c_int),
     "cagmres_set_shifts": ([_P, _PD, _PD, C.c_int], C.c_int),
     "cagmres_get_shifts": ([_P, _PD, _PD, C.c_int, C.POINTER(C.c_int)], C.c_int),

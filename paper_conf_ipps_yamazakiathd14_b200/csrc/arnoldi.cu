@@ -26,7 +26,6 @@ template <int JX, int MODE>
 __global__ void __launch_bounds__(NT) k_arnoldi_fused(ArnoldiArgs a) {
     __shared__ double sc[JX];
     __shared__ double sred[NWARP][JX];
-    __shared__ bool s_last;
     const int jx = a.jx;
     for (int i = threadIdx.x; i < JX; i += NT) sc[i] = (MODE != 0 && i < jx) ? a.c_in[i] : 0.0;
     __syncthreads();
@@ -66,22 +65,15 @@ __global__ void __launch_bounds__(NT) k_arnoldi_fused(ArnoldiArgs a) {
         for (int q = 0; q < NWARP; ++q) s += sred[q][i];
         part[i] = s;
     }
-    __threadfence();
-    __syncthreads();
-    if (threadIdx.x == 0) s_last = atomicAdd(a.counter, 1u) == gridDim.x - 1;
-    __syncthreads();
-    if (!s_last) return;
-    __threadfence();
     const int nout = MODE == 2 ? 1 : jx;
-    __shared__ double sfin[NT];
-    final_reduce(a.part, int(gridDim.x), NA, nout, sfin, [&](int i, double s) {
-        if (MODE == 2 && a.sqrt_out) {
-            if (!(s > 0.0)) atomicOr(a.status, ST_NORM);
-            s = sqrt(s);
-        }
-        a.c_out[i] = s;
-    });
-    if (threadIdx.x == 0) *a.counter = 0u;
+    tree_reduce(a.part, a.part + int64_t(gridDim.x) * NA, int(gridDim.x), int(blockIdx.x), NA, nout, a.counter,
+                [&](int i, double s) {
+                    if (MODE == 2 && a.sqrt_out) {
+                        if (!(s > 0.0)) atomicOr(a.status, ST_NORM);
+                        s = sqrt(s);
+                    }
+                    a.c_out[i] = s;
+                });
 }
 
 int arnoldi_fused(const Dev& d, const ArnoldiArgs& a, int mode, cudaStream_t st) {
@@ -112,6 +104,6 @@ int arnoldi_fused(const Dev& d, const ArnoldiArgs& a, int mode, cudaStream_t st)
     return 0;
 }
 
-size_t arnoldi_ws_doubles(const Dev& d) { return size_t(d.sms) * 8 * 32; }
+size_t arnoldi_ws_doubles(const Dev& d) { return 2 * size_t(d.sms) * 8 * 32; }
 
 }  // namespace kern

@@ -175,18 +175,11 @@ __global__ void __launch_bounds__(512, 1) k_update_gram(UpdGramArgs a) {
         for (int q = 0; q < nw; ++q) sum += red[q * FR + (mt * NTG + nt) * 64 + ln * 2 + h];
         part[e] = sum;
     }
-    __shared__ bool s_last;
-    __threadfence();
-    __syncthreads();
-    if (threadIdx.x == 0) s_last = atomicAdd(a.counter, 1u) == gridDim.x - 1;
-    __syncthreads();
-    if (!s_last) return;
-    __threadfence();
-    final_reduce(a.part, int(gridDim.x), nent, nent, red, [&](int e, double tot) { a.out[e] = tot; });
-    if (threadIdx.x == 0) *a.counter = 0u;
-    if (a.fin_chol) {
-        __syncthreads();
-        if (threadIdx.x == 0) chol_upper_serial(a.out, wg, wg, a.R, a.status);
+    const bool fin = tree_reduce(a.part, a.part + int64_t(gridDim.x) * nent, int(gridDim.x), int(blockIdx.x),
+                                 nent, nent, a.counter, [&](int e, double tot) { a.out[e] = tot; });
+    if (fin && a.fin_chol && threadIdx.x < 32) {
+        __threadfence_block();
+        chol_upper_warp(a.out, wg, wg, a.R, a.status, smp);
     }
 }
 
@@ -230,6 +223,6 @@ int update_gram(const Dev& d, const UpdGramArgs& a, cudaStream_t st) {
     return 0;
 }
 
-size_t update_gram_ws_doubles(const Dev& d) { return size_t(d.sms) * 16 * 16; }
+size_t update_gram_ws_doubles(const Dev& d) { return 2 * size_t(d.sms) * 16 * 16; }
 
 }  // namespace kern

@@ -213,15 +213,19 @@ void spmv(const Dev& d, const Sell& A, int64_t nrows, const double* x, double* y
     if (nrows <= 0) return;
     ++g_launches;
     if (w && !u) { u = x; bu = 0.0; }             // pair step with a == 0: keep MODE 2 well formed
-    if (A.variant == 4 || A.variant == 5) {
-        if (A.variant == 4) {
-            if (w) launch_persist<2, 8, 3>(d, A, nrows, x, y, u, bu, w, bw, st);
-            else if (u) launch_persist<1, 8, 3>(d, A, nrows, x, y, u, bu, nullptr, 0.0, st);
-            else launch_persist<0, 8, 3>(d, A, nrows, x, y, nullptr, 0.0, nullptr, 0.0, st);
-        } else {
-            if (w) launch_persist<2, 4, 4>(d, A, nrows, x, y, u, bu, w, bw, st);
-            else if (u) launch_persist<1, 4, 4>(d, A, nrows, x, y, u, bu, nullptr, 0.0, st);
-            else launch_persist<0, 4, 4>(d, A, nrows, x, y, nullptr, 0.0, nullptr, 0.0, st);
+    if (A.variant >= 4) {
+        auto go = [&](auto k0, auto k1, auto k2) {
+            if (w) k2(d, A, nrows, x, y, u, bu, w, bw, st);
+            else if (u) k1(d, A, nrows, x, y, u, bu, nullptr, 0.0, st);
+            else k0(d, A, nrows, x, y, nullptr, 0.0, nullptr, 0.0, st);
+        };
+        switch (A.variant) {   // (load batch, min CTAs per SM)
+            case 4: go(launch_persist<0, 8, 3>, launch_persist<1, 8, 3>, launch_persist<2, 8, 3>); break;
+            case 5: go(launch_persist<0, 4, 4>, launch_persist<1, 4, 4>, launch_persist<2, 4, 4>); break;
+            case 6: go(launch_persist<0, 4, 5>, launch_persist<1, 4, 5>, launch_persist<2, 4, 5>); break;
+            case 7: go(launch_persist<0, 4, 6>, launch_persist<1, 4, 6>, launch_persist<2, 4, 6>); break;
+            case 8: go(launch_persist<0, 2, 6>, launch_persist<1, 2, 6>, launch_persist<2, 2, 6>); break;
+            default: go(launch_persist<0, 2, 8>, launch_persist<1, 2, 8>, launch_persist<2, 2, 8>); break;
         }
         return;
     }
@@ -252,8 +256,8 @@ void residual(const Dev& d, const Sell& A, int64_t nrows, const double* x, const
     (void)d;
     if (nrows <= 0) return;
     ++g_launches;
-    if (A.variant == 4 || A.variant == 5) {
-        launch_persist<3, 8, 3>(d, A, nrows, x, r, b, 1.0, nullptr, 0.0, st);
+    if (A.variant >= 4) {
+        launch_persist<3, 4, 4>(d, A, nrows, x, r, b, 1.0, nullptr, 0.0, st);
         return;
     }
     if (A.variant >= 1) {
@@ -270,7 +274,8 @@ void residual(const Dev& d, const Sell& A, int64_t nrows, const double* x, const
 // Small dense factorizations on one thread / one CTA (w <= 32).
 // ------------------------------------------------------------------------------------
 __global__ void k_chol(const double* G, int w, double* R, int* status) {
-    if (threadIdx.x == 0) chol_upper_serial(G, w, w, R, status);
+    __shared__ double sm[32 * 32];
+    chol_upper_warp(G, w, w, R, status, sm);
 }
 
 void chol(const double* G, int w, double* R, int* status, cudaStream_t st) {

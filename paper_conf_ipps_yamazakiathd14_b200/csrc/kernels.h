@@ -12,6 +12,7 @@ extern long long g_launches;
 struct Dev {
     int sms = 148;
     int device = 0;
+    int gram = 1;               // CholQR Gram kernel: 0 = FP64 tensor core (DMMA), 1 = scalar DFMA ring
 };
 
 // Sliced ELLPACK, slice height 32 (one warp), column-major inside a slice, with per-slice
@@ -218,11 +219,27 @@ void residual(const Dev& d, const Sell& A, int64_t nrows, const double* x, const
 // to out (jx x w, ld jx).  fin_chol: out is the Gram (X == Y, jx == w) and R = chol(out)
 // (upper, ld w) is computed in the same launch; breakdown sets ST_CHOL in *status.
 // ws: workspace of at least xty_ws_doubles() doubles; counter: a zeroed device uint.
+// counter: XTY_COUNTERS zeroed uints (tree_reduce tickets, reduce.cuh; left zeroed).
+constexpr int XTY_COUNTERS = 4096;
 struct XtyWs { double* part = nullptr; size_t cap = 0; unsigned int* counter = nullptr; };
 size_t xty_ws_doubles(const Dev& d, int jx, int w);
 int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const double* Y,
         int64_t ldy, int w, double* out, bool fin_chol, double* R, int* status,
         const XtyWs& ws, cudaStream_t st);
+
+// Scalar-DFMA Gram G = P^T P (gram.cu; P 16-B aligned, ld even, w <= 12), same final
+// reduction / in-launch Cholesky contract as xty with X == Y.  Returns -1 if not applicable.
+struct GramArgs {
+    int64_t n;
+    const double* P; int64_t ldp; int w;
+    double* part;               // >= sms * w * w doubles
+    double* out;                // w x w, ld w
+    unsigned int* counter;
+    int fin_chol;
+    double* R;
+    int* status;
+};
+int gram_dfma(const Dev& d, const GramArgs& a, cudaStream_t st);
 
 // R = chol(G) (upper, ld w), one tiny launch (used after a cross-rank allreduce of G).
 void chol(const double* G, int w, double* R, int* status, cudaStream_t st);

@@ -42,3 +42,70 @@ __device__ __forceinline__ void final_reduce(const double* part, int nblk, int64
 }
 
 }  // namespace kern
+
+namespace kern {
+
+// Two-level deterministic reduction of per-CTA partials, replacing "last CTA sums all
+// partials" (a ~148 x nent serial read by one SM: 8-20 us, tools/reduce_probe.cu).
+// CTA b (of nblk) has written part[b * stride + e], e < nent, and calls this with every
+// thread.  CTAs form groups of TR_GS consecutive ids; the last CTA of a group to arrive
+// (atomic ticket) sums its group's partials in id order into gpart[g * stride + e]; the last
+// group to finish sums the group partials in group order and calls store(e, total).
+// Each thread keeps all of its <= TR_GS loads in flight, so each level costs about one L2
+// round trip.  Fixed summation order: bitwise reproducible for a given grid.  cnt: >= 65
+// zeroed counters (left zeroed on exit).  Returns true only in the CTA that stored.
+constexpr int TR_GS = 16;
+constexpr int TR_TOP = 64;            // index of the top-level counter (nblk <= 64 * TR_GS)
+constexpr int TR_CNT = 72;            // counters per independent reduction
+
+template <class Store>
+__device__ __forceinline__ bool tree_reduce(const double* part, double* gpart, int nblk, int b, int64_t stride,
+                                            int nent, unsigned int* cnt, Store store) {
+    const int ng = (nblk + TR_GS - 1) / TR_GS;
+    const int g = b / TR_GS;
+    const int gsz = min(TR_GS, nblk - g * TR_GS);
+    __shared__ int s_flag;
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) s_flag = atomicAdd(cnt + g, 1u) == unsigned(gsz - 1);
+    __syncthreads();
+    if (!s_flag) return false;
+    __threadfence();
+    const double* pg = part + int64_t(g) * TR_GS * stride;
+    for (int e = threadIdx.x; e < nent; e += blockDim.x) {
+        double v[TR_GS];
+#pragma unroll
+        for (int u = 0; u < TR_GS; ++u) v[u] = u < gsz ? __ldcg(pg + int64_t(u) * stride + e) : 0.0;
+        double s = v[0];
+#pragma unroll
+        for (int u = 1; u < TR_GS; ++u)
+            if (u < gsz) s += v[u];
+        if (ng == 1) store(e, s);
+        else __stcg(gpart + int64_t(g) * stride + e, s);
+    }
+    if (threadIdx.x == 0) cnt[g] = 0u;
+    if (ng == 1) { __syncthreads(); return true; }
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) s_flag = atomicAdd(cnt + TR_TOP, 1u) == unsigned(ng - 1);
+    __syncthreads();
+    if (!s_flag) return false;
+    __threadfence();
+    for (int e = threadIdx.x; e < nent; e += blockDim.x) {
+        double s = 0.0;
+        for (int g0 = 0; g0 < ng; g0 += TR_GS) {
+            double v[TR_GS];
+#pragma unroll
+            for (int u = 0; u < TR_GS; ++u) v[u] = g0 + u < ng ? __ldcg(gpart + int64_t(g0 + u) * stride + e) : 0.0;
+#pragma unroll
+            for (int u = 0; u < TR_GS; ++u)
+                if (g0 + u < ng) s = (g0 + u == 0) ? v[u] : s + v[u];
+        }
+        store(e, s);
+    }
+    if (threadIdx.x == 0) cnt[TR_TOP] = 0u;
+    __syncthreads();
+    return true;
+}
+
+}  // namespace kern

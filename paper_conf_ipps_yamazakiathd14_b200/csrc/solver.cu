@@ -74,6 +74,7 @@ struct cagmres {
     kern::Dev dev;
     cudaStream_t stream = nullptr, own_stream = nullptr;
     kern::Sell A;
+    double spmv_tuned_us = 0.0;            // setup-time SpMV autotune result (diagnostic)
     std::vector<int64_t> level_len;        // ext rows with distance <= h
     std::vector<int64_t> nnz_prefix;       // nnz of stored rows with distance <= h (h <= s-1)
     double* V = nullptr;
@@ -278,13 +279,15 @@ int common_alloc(cagmres* h) {
     CU(cudaEventCreateWithFlags(&h->ev_beta, cudaEventDisableTiming));
     size_t cap = 0;
     for (int w = 1; w <= 32; ++w) cap = std::max(cap, kern::xty_ws_doubles(h->dev, h->m + 1, w));
+    cap = std::max(cap, kern::update_gram_ws_doubles(h->dev));
+    cap = std::max(cap, size_t(2) * size_t(h->dev.sms) * 12 * 12);     // scalar Gram (+ group partials)
     h->ws.cap = cap;
     CU(cudaMalloc(&h->ws.part, sizeof(double) * cap));
-    CU(cudaMalloc(&h->ws.counter, sizeof(unsigned int)));
-    CU(cudaMemset(h->ws.counter, 0, sizeof(unsigned int)));
+    CU(cudaMalloc(&h->ws.counter, sizeof(unsigned int) * kern::XTY_COUNTERS));
+    CU(cudaMemset(h->ws.counter, 0, sizeof(unsigned int) * kern::XTY_COUNTERS));
     CU(cudaMalloc(&h->arn_part, sizeof(double) * kern::arnoldi_ws_doubles(h->dev)));
-    CU(cudaMalloc(&h->arn_counter, sizeof(unsigned int)));
-    CU(cudaMemset(h->arn_counter, 0, sizeof(unsigned int)));
+    CU(cudaMalloc(&h->arn_counter, sizeof(unsigned int) * kern::XTY_COUNTERS));
+    CU(cudaMemset(h->arn_counter, 0, sizeof(unsigned int) * kern::XTY_COUNTERS));
     CU(cudaMalloc(&h->status, sizeof(int)));
     CU(cudaMemset(h->status, 0, sizeof(int)));
     return CAGMRES_OK;
@@ -354,6 +357,43 @@ void wave_reset_pairs(cagmres* h) {
     h->wave_nC = 0;
 }
 
+// SpMV kernel selection (setup, once): every CAGMRES_OPT_SPMV variant computes each row with
+// the same operations in the same order (bitwise identical results), so the fastest one on
+// this matrix is picked by timing y = A x over all stored rows (x = V[:,0], y = V[:,1]).
+int spmv_autotune(cagmres* h) {
+    static const int cand[] = {0, 3, 5, 6, 8};
+    if (h->m < 1 || h->A.nrows <= 0) return CAGMRES_OK;
+    double* x = h->V;
+    double* y = h->V + h->ldv;
+    cudaEvent_t e0, e1;
+    CU(cudaEventCreate(&e0));
+    CU(cudaEventCreate(&e1));
+    float best = 1e30f;
+    int pick = 0;
+    for (int v : cand) {
+        h->A.variant = v;
+        kern::spmv(h->dev, h->A, h->A.nrows, x, y, nullptr, 0.0, nullptr, 0.0, h->stream);   // warm-up
+        float tmin = 1e30f;
+        for (int r = 0; r < 3; ++r) {
+            CU(cudaEventRecord(e0, h->stream));
+            kern::spmv(h->dev, h->A, h->A.nrows, x, y, nullptr, 0.0, nullptr, 0.0, h->stream);
+            CU(cudaEventRecord(e1, h->stream));
+            CU(cudaEventSynchronize(e1));
+            float ms = 0.f;
+            CU(cudaEventElapsedTime(&ms, e0, e1));
+            tmin = std::min(tmin, ms);
+        }
+        if (tmin < best) { best = tmin; pick = v; }
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    h->A.variant = pick;
+    h->spmv_tuned_us = double(best) * 1e3;
+    CU(cudaMemsetAsync(h->V, 0, sizeof(double) * size_t(h->ldv) * 2, h->stream));
+    CU(cudaStreamSynchronize(h->stream));
+    return CAGMRES_OK;
+}
+
 int init_common(cagmres* h, const cagmres_csr* A, const int64_t* row_starts, int s, int m,
                 int basis, int orth) {
     if (s < 1 || m < 1 || s > m || s > 31 || (basis != CAGMRES_MONOMIAL && basis != CAGMRES_NEWTON))
@@ -378,6 +418,7 @@ int init_common(cagmres* h, const cagmres_csr* A, const int64_t* row_starts, int
     h->level_len = plan.level_len;
     TRY(build_sell(h, plan));
     TRY(common_alloc(h));
+    TRY(spmv_autotune(h));
     if (h->nranks == 1) TRY(wave_setup(h, plan));
     if (h->nranks > 1) {
         // ---- exchange request lists (setup, "compress ... needed by other GPUs") ----
@@ -874,13 +915,32 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
     if (!h) return CAGMRES_EINVAL;
     switch (opt) {
         case CAGMRES_OPT_MPK_WAVE: h->wave_on = value != 0; h->wave_force = value == 2; return CAGMRES_OK;
-        case CAGMRES_OPT_SPMV: if (value < 0 || value > 5) return CAGMRES_EINVAL; h->A.variant = value; return CAGMRES_OK;
+        case CAGMRES_OPT_SPMV:
+            if (value < -1 || value > 9) return CAGMRES_EINVAL;
+            if (value == -1) return spmv_autotune(h);
+            h->A.variant = int(value);
+            return CAGMRES_OK;
+        case CAGMRES_OPT_GRAM: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->dev.gram = int(value); return CAGMRES_OK;
         case CAGMRES_OPT_FUSE: h->fuse_borth_gram = (value & 1) != 0; h->arnoldi_fuse = (value & 2) != 0; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK:
             if (value < 256 || value % 256) return CAGMRES_EINVAL;
             h->wave_CH = int(value); wave_reset_pairs(h); return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CTAS: h->wave_ctas = int(value); wave_reset_pairs(h); return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_LAG: h->wave_lag = int(value); wave_reset_pairs(h); return CAGMRES_OK;
+        default: return CAGMRES_EINVAL;
+    }
+}
+
+int cagmres_get_option(cagmres_t h, int opt, int64_t* value) {
+    if (!h || !value) return CAGMRES_EINVAL;
+    switch (opt) {
+        case CAGMRES_OPT_MPK_WAVE: *value = h->wave_on ? (h->wave_force ? 2 : 1) : 0; return CAGMRES_OK;
+        case CAGMRES_OPT_SPMV: *value = h->A.variant; return CAGMRES_OK;
+        case CAGMRES_OPT_GRAM: *value = h->dev.gram; return CAGMRES_OK;
+        case CAGMRES_OPT_FUSE: *value = (h->fuse_borth_gram ? 1 : 0) | (h->arnoldi_fuse ? 2 : 0); return CAGMRES_OK;
+        case CAGMRES_OPT_WAVE_CHUNK: *value = h->wave_CH; return CAGMRES_OK;
+        case CAGMRES_OPT_WAVE_CTAS: *value = h->wave_ctas; return CAGMRES_OK;
+        case CAGMRES_OPT_WAVE_LAG: *value = h->wave_lag; return CAGMRES_OK;
         default: return CAGMRES_EINVAL;
     }
 }

@@ -41,31 +41,24 @@ struct XtyArgs {
     int* status;
 };
 
-// ---- CTA partial -> last-CTA fixed-order total (+ Cholesky) ---------------------------
+// ---- CTA partial -> two-level fixed-order total (+ Cholesky) ---------------------------
+// Partials of y-chunk `by` live at part[(by * gx + bx) * nent]; its group partials after all
+// CTA partials; its counters at counter[by * TR_CNT].
 __device__ __forceinline__ void xty_finish(const XtyArgs& a, int nent_cta) {
-    __shared__ bool s_last;
-    __threadfence();
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        const unsigned total = gridDim.x * gridDim.y;
-        s_last = (atomicAdd(a.counter, 1u) == total - 1);
-    }
-    __syncthreads();
-    if (!s_last) return;
-    __threadfence();
+    const int gx = int(gridDim.x), by = int(blockIdx.y);
+    const int ng = (gx + TR_GS - 1) / TR_GS;
+    const double* pb = a.part + int64_t(by) * gx * nent_cta;
+    double* gp = a.part + int64_t(gridDim.y) * gx * nent_cta + int64_t(by) * ng * nent_cta;
     const int jx = a.jx, w = a.w;
-    extern __shared__ double red[];
-    for (int by = 0; by < int(gridDim.y); ++by) {
-        const double* pb = a.part + int64_t(by) * gridDim.x * int64_t(nent_cta);
-        final_reduce(pb, int(gridDim.x), nent_cta, a.chunk * w, red, [&](int e, double tot) {
-            const int il = e % a.chunk, c = e / a.chunk, i = by * a.chunk + il;
-            if (i < jx) a.out[i + int64_t(jx) * c] = tot;
-        });
-    }
-    if (threadIdx.x == 0) *a.counter = 0u;         // ready for the next launch (stream order)
-    if (a.fin_chol) {
-        __syncthreads();
-        if (threadIdx.x == 0) chol_upper_serial(a.out, jx, w, a.R, a.status);
+    const bool fin = tree_reduce(pb, gp, gx, int(blockIdx.x), nent_cta, a.chunk * w, a.counter + by * TR_CNT,
+                                 [&](int e, double tot) {
+                                     const int il = e % a.chunk, c = e / a.chunk, i = by * a.chunk + il;
+                                     if (i < jx) a.out[i + int64_t(jx) * c] = tot;
+                                 });
+    if (fin && a.fin_chol && threadIdx.x < 32) {                 // gy == 1 for the Gram
+        extern __shared__ double red[];
+        __threadfence_block();
+        chol_upper_warp(a.out, jx, w, a.R, a.status, red);
     }
 }
 
@@ -347,7 +340,7 @@ size_t xty_ws_doubles(const Dev& d, int jx, int w) {
     size_t m = 0;
     for (int same = 0; same < 2; ++same) {
         const Geo o = geometry(d, int64_t(1) << 40, same ? w : jx, w, same != 0);
-        const size_t v = size_t(o.gx) * o.gy * o.chunk * w;
+        const size_t v = 2 * size_t(std::max(o.gx, d.sms / o.gy)) * o.gy * o.chunk * w;   // + group partials
         m = v > m ? v : m;
     }
     return m;
@@ -365,8 +358,12 @@ int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const dou
         const XtyWs& ws, cudaStream_t st) {
     if (jx <= 0 || w <= 0 || w > 32 || n < 0) return -1;
     const bool same = (X == Y) && (ldx == ldy) && (jx == w);
+    if (same && d.gram == 1 && size_t(d.sms) * w * w * 2 <= ws.cap) {
+        GramArgs g{n, X, ldx, w, ws.part, out, ws.counter, fin_chol ? 1 : 0, R, status};
+        if (gram_dfma(d, g, st) == 0) return 0;
+    }
     Geo o = geometry(d, n, jx, w, same);
-    if (size_t(o.gx) * o.gy * o.chunk * w > ws.cap) return -1;
+    if (size_t(o.gx) * o.gy * o.chunk * w * 2 > ws.cap || o.gy * TR_CNT > XTY_COUNTERS) return -1;
     XtyArgs a{n, X, ldx, jx, Y, ldy, w, o.chunk, ws.part, out, ws.counter, fin_chol ? 1 : 0, R, status};
     const bool aligned = ((reinterpret_cast<uintptr_t>(X) | reinterpret_cast<uintptr_t>(Y)) % 16 == 0) &&
                          (ldx % 2 == 0) && (ldy % 2 == 0);
@@ -382,7 +379,7 @@ int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const dou
         if (smem < red) smem = red;
         if (smem < size_t(32 * nw) * sizeof(double)) smem = size_t(32 * nw) * sizeof(double);
         o.gx = std::max(1, d.sms / o.gy);
-        if (size_t(o.gx) * o.gy * o.chunk * w > ws.cap) return -1;
+        if (size_t(o.gx) * o.gy * o.chunk * w * 2 > ws.cap) return -1;
         if (o.sym) {
             if (o.NTN == 1) launch_pipe(k_xty_pipe<1, 1, true, TW>, o, nw, smem, a, st);
             else if (o.NTN == 2) launch_pipe(k_xty_pipe<2, 2, true, TW>, o, nw, smem, a, st);

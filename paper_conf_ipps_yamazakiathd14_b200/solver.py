@@ -115,10 +115,16 @@ class Solver:
         s = torch.cuda.current_stream(self.device)
         L.check(self._lib.cagmres_set_stream(self._h, C.c_void_p(s.cuda_stream)), "set_stream")
 
+    OPTIONS = {"mpk_wave": 1, "wave_chunk": 3, "wave_ctas": 4, "wave_lag": 5, "fuse": 6, "spmv": 7, "gram": 8}
+
     def set_option(self, opt, value):
-        """opt: "mpk_wave", "wave_chunk", "wave_ctas", "wave_lag", "fuse", "spmv" (CAGMRES_OPT_*)."""
-        code = {"mpk_wave": 1, "wave_chunk": 3, "wave_ctas": 4, "wave_lag": 5, "fuse": 6, "spmv": 7}[opt]
-        L.check(self._lib.cagmres_set_option(self._h, code, int(value)), "set_option")
+        """opt: "mpk_wave", "wave_chunk", "wave_ctas", "wave_lag", "fuse", "spmv", "gram" (CAGMRES_OPT_*)."""
+        L.check(self._lib.cagmres_set_option(self._h, self.OPTIONS[opt], int(value)), "set_option")
+
+    def get_option(self, opt):
+        v = C.c_int64(0)
+        L.check(self._lib.cagmres_get_option(self._h, self.OPTIONS[opt], C.byref(v)), "get_option")
+        return int(v.value)
 
     def close(self):
         if self._h:

@@ -138,10 +138,10 @@ def test_spmv_variants_bitwise(gen):
     S = Solver(A, s=6, m=30, basis="newton")
     S.set_shifts(*SHIFTS)
     Ws = []
-    for v in range(6):
+    for v in range(10):
         S.set_option("spmv", v)
         Ws.append(S.mpk(q, 6))
-    for v in range(1, 6):
+    for v in range(1, 10):
         assert torch.equal(Ws[v], Ws[0]), v
 
 
@@ -177,9 +177,12 @@ def test_borth_parity(n, j, w):
 @pytest.mark.parametrize("kind,reorth", [("cholqr", False), ("cholqr", True), ("svqr", False),
                                          ("cgs", False), ("mgs", False), ("caqr", False)])
 @pytest.mark.parametrize("n,w", [(100002, 11), (100003, 11), (777, 6), (4096, 1), (20000, 16), (65538, 13)])
-def test_tsqr_parity(kind, reorth, n, w):
+@pytest.mark.parametrize("gram", [0, 1])
+def test_tsqr_parity(kind, reorth, n, w, gram):
+    """gram: CAGMRES_OPT_GRAM (0 = DMMA tensor-core Gram, 1 = scalar DFMA ring Gram)."""
     A = G.banded(n=n)
     S = Solver(A, s=1, m=2, basis="monomial")
+    S.set_option("gram", gram)
     P = G.random_panel(n, w, 31)
     if w > 2:
         P[:, 2] += 0.3 * P[:, 1]
@@ -318,3 +321,24 @@ def test_solve_fused_borth_gram(fuse, s, m, reorth):
     assert st.status == 0
     assert abs(st.cycles - len(ref)) <= 1
     assert hist_within_envelope(st.hist, ref, env)
+
+
+@pytest.mark.parametrize("spmv,gram", [(4, 1), (5, 0), (0, 1)])
+def test_solve_kernel_options(spmv, gram):
+    """Solve with the persistent SpMV (CAGMRES_OPT_SPMV 4/5) and the scalar-DFMA Gram
+    (CAGMRES_OPT_GRAM 1) against the oracle: 3D 7-point 40^3 (n = 64,000), s = 10, m = 30."""
+    A = G.convection_diffusion(40, 3, 7)
+    As = A.to_scipy()
+    b = G.rhs(A.n)
+    sh = O.modified_leja(O.ritz_values(O.arnoldi_cgs2(As, b, 30)[1], 30), 10)
+    S = Solver(A, s=10, m=30, basis="newton")
+    S.set_option("spmv", spmv)
+    S.set_option("gram", gram)
+    S.set_shifts(*sh)
+    x, st = S.solve(dev(b), tol=1e-8, maxit=40)
+    ref, env = rounding_envelope(As, b, s=10, m=30, basis="newton", tol=1e-8, shifts=sh)
+    assert st.status == 0
+    assert abs(st.cycles - len(ref)) <= 1
+    assert hist_within_envelope(st.hist, ref, env)
+    r = b - As @ x.cpu().numpy()
+    assert np.linalg.norm(r) <= 1.01e-8 * np.linalg.norm(b)

@@ -53,7 +53,8 @@ def main():
         t = timeit(lambda: S.borth(Q, j, P, w))
         by = 8.0 * n * (2 * j + 3 * w)
         out[f"borth j={j} w={w}"] = dict(ms=round(t, 4), gbs=round(by / t / 1e6, 1))
-    for w in [1, 6, 11, 16]:
+    for w, gram in [(1, 0), (6, 0), (11, 0), (16, 0), (1, 1), (6, 1), (11, 1), (12, 1)]:
+        S.set_option("gram", gram)
         Pt = torch.randn(w, ld, dtype=torch.float64, device="cuda")
         P = Pt.t()[:n]                           # fresh column-major panel, ld = ld
 
@@ -62,9 +63,9 @@ def main():
         try:
             t = timeit(f)
             by = 8.0 * n * (3 * w)
-            out[f"tsqr cholqr w={w}"] = dict(ms=round(t, 4), gbs=round(by / t / 1e6, 1))
+            out[f"tsqr cholqr w={w} gram={gram}"] = dict(ms=round(t, 4), gbs=round(by / t / 1e6, 1))
         except Exception as e:                   # report, keep going
-            out[f"tsqr cholqr w={w}"] = dict(error=str(e), norms=[float(P[:, c].norm()) for c in range(w)])
+            out[f"tsqr cholqr w={w} gram={gram}"] = dict(error=str(e), norms=[float(P[:, c].norm()) for c in range(w)])
     q = torch.tensor(G.rhs(n), device="cuda")
     W = torch.empty(11, n, dtype=torch.float64, device="cuda").t()
     t = timeit(lambda: S.mpk(q, 10, out=W))
