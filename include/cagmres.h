@@ -44,6 +44,11 @@ extern "C" {
 
 /* ---- options ----------------------------------------------------------------------- */
 enum { CAGMRES_MONOMIAL = 0, CAGMRES_NEWTON = 1 };               /* MPK basis      */
+/* Standard GMRES(m) baseline (the "GMRES" rows of Fig. 14/15): every
+ * restart cycle is m Arnoldi steps, each one SpMV (1-deep halo) plus CGS orthogonalisation
+ * of width 1 (CGS2 when CAGMRES_REORTH is set) on the same kernels; s is not used (pass 1).
+ * Not a CA method — it is the comparator the paper's speedups are quoted against. */
+#define CAGMRES_GMRES 2
 enum { CAGMRES_CHOLQR = 0, CAGMRES_SVQR = 1, CAGMRES_CGS = 2,     /* TSQR, Fig. 9/10     */
        CAGMRES_MGS = 3, CAGMRES_CAQR = 4 };
 #define CAGMRES_TSQR_MASK   0xff
@@ -90,7 +95,7 @@ typedef struct {
 /* ---- lifetime ---------------------------------------------------------------------- */
 /* Single-GPU handle on the current CUDA device.  A: all n rows (row_begin=own_begin=0,
  * row_end=own_end=n).  s >= 1 block size, m >= 1 restart length, s <= m; basis
- * CAGMRES_MONOMIAL|NEWTON; orth = TSQR kind | flags.  Copies A to the device (sliced-ELL
+ * CAGMRES_MONOMIAL|NEWTON|GMRES; orth = TSQR kind | flags.  Copies A to the device (sliced-ELL
  * layout) and allocates the basis V (n x (m+1)) and all workspace.
  * Errors: EINVAL, ECUDA, ENOMEM. */
 int cagmres_create(cagmres_t* h, const cagmres_csr* A, int s, int m, int basis, int orth);
@@ -121,10 +126,14 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
  *                          slices per warp with load batches 4/8/4 at 4/2/3 CTAs per SM;
  *                          4..9 = persistent grid, slice descriptors software-pipelined two
  *                          slices ahead, (load batch, CTAs/SM) = (8,3) (4,4) (4,5) (4,6) (2,6)
- *                          (2,8).  All variants are bitwise identical.
+ *                          (2,8); 10..13 = persistent, fully unrolled body for the matrix's most
+ *                          common DIA slice width, >= 3/4/5/6 CTAs per SM.  All variants are
+ *                          bitwise identical.
  *   CAGMRES_OPT_GRAM     : CholQR Gram kernel: 0 = FP64 tensor core (DMMA m8n8k4) on a per-warp
  *                          cp.async ring; 1 (default) = scalar DFMA on a deeper ring (w <= 12,
  *                          else the DMMA kernel).
+ *   CAGMRES_OPT_ARNOLDI  : width-1 Arnoldi passes (first Newton cycle, GMRES baseline): 0 = one
+ *                          thread per row, register loads; 1 (default) = per-warp cp.async ring.
  *   CAGMRES_OPT_FUSE     : bit 0 (default 0) = BOrth pass 2 fused with the CholQR Gram;
  *                          bit 1 (default 1) = fused first-cycle Arnoldi passes.
  *   CAGMRES_OPT_WAVE_CHUNK / _WAVE_CTAS / _WAVE_LAG : temporal-blocking tuning (rows per
@@ -137,6 +146,7 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
 #define CAGMRES_OPT_FUSE       6
 #define CAGMRES_OPT_SPMV       7
 #define CAGMRES_OPT_GRAM       8
+#define CAGMRES_OPT_ARNOLDI    9
 int cagmres_set_option(cagmres_t h, int opt, int64_t value);
 /* Current value of an option (e.g. the SpMV variant the create-time selection picked).
  * EINVAL for a null handle / pointer or an unknown option. */

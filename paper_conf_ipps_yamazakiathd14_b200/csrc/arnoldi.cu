@@ -13,6 +13,7 @@
 #include <cstdint>
 
 #include "kernels.h"
+#include "ptx.h"
 #include "reduce.cuh"
 
 namespace kern {
@@ -76,8 +77,131 @@ __global__ void __launch_bounds__(NT) k_arnoldi_fused(ArnoldiArgs a) {
                 });
 }
 
+// Ring version (aligned columns, n >= 64 tiles): the register-load kernel above keeps one row's
+// jx loads in flight per thread with <= 16 warps per SM and no prefetch across rows (ncu:
+// 2.2-3.6 TB/s at jx ~ 24).  Here each warp streams its own contiguous range of 32-row tiles
+// of [Q | v] through an AR_S-stage shared-memory ring with 16-B cp.async (no registers held),
+// lane l owns row l of a tile and reads its Q row from the ring (column c at c*32 + l:
+// conflict-free).  Same per-row operations as k_arnoldi_fused; partials reduced in a fixed order.
+constexpr int AR_S = 3;
+template <int JX, int MODE>
+__global__ void __launch_bounds__(512, 1) k_arnoldi_ring(ArnoldiArgs a) {
+    extern __shared__ __align__(16) double sma[];
+    __shared__ double sc[JX > 0 ? JX : 1];
+    __shared__ double sred[16][JX > 0 ? JX : 1];
+    const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    const int jx = a.jx;
+    for (int i = threadIdx.x; i < JX; i += blockDim.x) sc[i] = (MODE != 0 && i < jx) ? a.c_in[i] : 0.0;
+    __syncthreads();
+    constexpr int NA = MODE == 2 ? 1 : JX;
+    double acc[NA];
+#pragma unroll
+    for (int i = 0; i < NA; ++i) acc[i] = 0.0;
+    const int ncol = jx + 1;                                   // Q columns, then v
+    const int64_t stage_d = int64_t(ncol) * 32;
+    double* ring = sma + int64_t(wp) * AR_S * stage_d;
+    const int64_t T = a.n / 32;
+    const int64_t Wn = int64_t(gridDim.x) * nw;
+    const int64_t g = int64_t(blockIdx.x) * nw + wp;
+    const int64_t t0 = g * T / Wn, t1 = (g + 1) * T / Wn;
+    auto issue = [&](int64_t t, int stage) {
+        if (t < t1) {
+            double* dst = ring + stage * stage_d;
+            const int64_t r0 = t * 32;
+            for (int q = lane; q < ncol * 16; q += 32) {
+                const int c = q >> 4, part = q & 15;
+                const double* src = (c < jx ? a.Q + a.ldq * c : a.v) + r0 + part * 2;
+                ptx::cp_async16(dst + c * 32 + part * 2, src);
+            }
+        }
+        ptx::cp_async_commit();
+    };
+    auto row = [&](const double* sq, double vv, int64_t r) {
+        if constexpr (MODE != 0) {
+#pragma unroll
+            for (int i = 0; i < JX; ++i)
+                if (i < jx) vv = fma(-sq[i * 32], sc[i], vv);
+            if (jx > 0) a.v[r] = vv;
+        }
+        if constexpr (MODE != 2) {
+#pragma unroll
+            for (int i = 0; i < JX; ++i)
+                if (i < jx) acc[i] = fma(sq[i * 32], vv, acc[i]);
+        } else {
+            acc[0] = fma(vv, vv, acc[0]);
+        }
+    };
+#pragma unroll
+    for (int s = 0; s < AR_S - 1; ++s) issue(t0 + s, s);
+    int stage = 0;
+    for (int64_t t = t0; t < t1; ++t) {
+        issue(t + AR_S - 1, (stage + AR_S - 1) % AR_S);
+        ptx::cp_async_wait<AR_S - 1>();
+        __syncwarp();
+        const double* sl = ring + stage * stage_d + lane;
+        row(sl, sl[jx * 32], t * 32 + lane);
+        __syncwarp();
+        stage = (stage + 1) % AR_S;
+    }
+    ptx::cp_async_wait<0>();
+    if (blockIdx.x == 0 && wp == 0) {                          // ragged tail rows [32 T, n)
+        const int64_t r = T * 32 + lane;
+        if (r < a.n) {
+            double* sl = ring + lane;                          // ring idle: stage this lane's row
+            for (int c = 0; c < jx; ++c) sl[c * 32] = a.Q[a.ldq * c + r];
+            row(sl, a.v[r], r);
+        }
+    }
+#pragma unroll
+    for (int i = 0; i < NA; ++i) {
+        double x = acc[i];
+        for (int off = 16; off > 0; off >>= 1) x += __shfl_xor_sync(0xffffffffu, x, off);
+        if (lane == 0) sred[wp][i] = x;
+    }
+    __syncthreads();
+    double* part = a.part + int64_t(blockIdx.x) * NA;
+    for (int i = threadIdx.x; i < NA; i += blockDim.x) {
+        double s = 0.0;
+        for (int q = 0; q < nw; ++q) s += sred[q][i];
+        part[i] = s;
+    }
+    const int nout = MODE == 2 ? 1 : jx;
+    tree_reduce(a.part, a.part + int64_t(gridDim.x) * NA, int(gridDim.x), int(blockIdx.x), NA, nout, a.counter,
+                [&](int i, double s) {
+                    if (MODE == 2 && a.sqrt_out) {
+                        if (!(s > 0.0)) atomicOr(a.status, ST_NORM);
+                        s = sqrt(s);
+                    }
+                    a.c_out[i] = s;
+                });
+}
+
+namespace {
+template <int JX, int MODE>
+bool go_ring(const Dev& d, const ArnoldiArgs& a, cudaStream_t st) {
+    const bool aligned = ((reinterpret_cast<uintptr_t>(a.v) | reinterpret_cast<uintptr_t>(a.Q)) % 16 == 0) &&
+                         (a.ldq % 2 == 0 || a.jx == 0);
+    if (!aligned || a.n < 64 * 32) return false;
+    const size_t ring_w = size_t(AR_S) * size_t(a.jx + 1) * 32 * sizeof(double);
+    int nw = int((200 * 1024) / ring_w);
+    nw = nw < 2 ? 2 : (nw > 16 ? 16 : nw);
+    const size_t smem = size_t(nw) * ring_w;
+    cudaFuncSetAttribute(k_arnoldi_ring<JX, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    ++g_launches;
+    k_arnoldi_ring<JX, MODE><<<unsigned(d.sms), 32 * nw, smem, st>>>(a);
+    return true;
+}
+}  // namespace
+
 int arnoldi_fused(const Dev& d, const ArnoldiArgs& a, int mode, cudaStream_t st) {
     if (a.jx < (mode == 2 ? 0 : 1) || a.jx > 32) return -1;   // wider: caller uses unfused passes
+    if (d.arnoldi_ring) {
+        bool ok;
+        if (mode == 0) ok = a.jx <= 8 ? go_ring<8, 0>(d, a, st) : (a.jx <= 16 ? go_ring<16, 0>(d, a, st) : go_ring<32, 0>(d, a, st));
+        else if (mode == 1) ok = a.jx <= 8 ? go_ring<8, 1>(d, a, st) : (a.jx <= 16 ? go_ring<16, 1>(d, a, st) : go_ring<32, 1>(d, a, st));
+        else ok = a.jx <= 8 ? go_ring<8, 2>(d, a, st) : (a.jx <= 16 ? go_ring<16, 2>(d, a, st) : go_ring<32, 2>(d, a, st));
+        if (ok) return 0;
+    }
     const int64_t blocks = (a.n + NT - 1) / NT;
     auto go = [&](auto kfn) {
         int occ = 0;
@@ -104,6 +228,6 @@ int arnoldi_fused(const Dev& d, const ArnoldiArgs& a, int mode, cudaStream_t st)
     return 0;
 }
 
-size_t arnoldi_ws_doubles(const Dev& d) { return 2 * size_t(d.sms) * 8 * 32; }
+size_t arnoldi_ws_doubles(const Dev& d) { return 2 * size_t(d.sms) * 8 * 32; }   // >= 2 * sms * 32 (ring)
 
 }  // namespace kern

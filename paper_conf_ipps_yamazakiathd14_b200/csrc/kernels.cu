@@ -213,6 +213,10 @@ void spmv(const Dev& d, const Sell& A, int64_t nrows, const double* x, double* y
     if (nrows <= 0) return;
     ++g_launches;
     if (w && !u) { u = x; bu = 0.0; }             // pair step with a == 0: keep MODE 2 well formed
+    if (A.variant >= 10) {
+        spmv_dia(d, A, A.variant, nrows, x, y, u, bu, w, bw, w ? 2 : (u ? 1 : 0), st);
+        return;
+    }
     if (A.variant >= 4) {
         auto go = [&](auto k0, auto k1, auto k2) {
             if (w) k2(d, A, nrows, x, y, u, bu, w, bw, st);
@@ -256,6 +260,10 @@ void residual(const Dev& d, const Sell& A, int64_t nrows, const double* x, const
     (void)d;
     if (nrows <= 0) return;
     ++g_launches;
+    if (A.variant >= 10) {
+        spmv_dia(d, A, A.variant, nrows, x, r, b, 1.0, nullptr, 0.0, 3, st);
+        return;
+    }
     if (A.variant >= 4) {
         launch_persist<3, 4, 4>(d, A, nrows, x, r, b, 1.0, nullptr, 0.0, st);
         return;

@@ -13,6 +13,7 @@ struct Dev {
     int sms = 148;
     int device = 0;
     int gram = 1;               // CholQR Gram kernel: 0 = FP64 tensor core (DMMA), 1 = scalar DFMA ring
+    int arnoldi_ring = 1;       // first-cycle / GMRES Arnoldi passes: 1 = cp.async ring kernels
 };
 
 // Sliced ELLPACK, slice height 32 (one warp), column-major inside a slice, with per-slice
@@ -28,6 +29,7 @@ struct Sell {
     int64_t nnz = 0;            // true nonzeros
     int64_t ncols = 0;          // valid x entries (clamp bound for DIA slices)
     int64_t ndcol = 0, ndia = 0;
+    int dia_w = 0;              // most common width of the unclamped DIA slices (spmv_dia.cu)
     int64_t* sptr = nullptr;    // nslices+1 value offsets
     int64_t* sinfo = nullptr;   // nslices
     int32_t* dcol = nullptr;    // DIA offsets / explicit column ids
@@ -211,6 +213,10 @@ enum : int { ST_CHOL = 1, ST_SVQR = 2, ST_NORM = 4 };
 // second step of a complex pair: w = x_prev, bw = b^2.
 void spmv(const Dev& d, const Sell& A, int64_t nrows, const double* x, double* y,
           const double* u, double bu, const double* w, double bw, cudaStream_t st);
+// DIA-width-specialised SpMV (spmv_dia.cu), CAGMRES_OPT_SPMV 10..13; mode as k_spmv_sell32
+// (3 = u - A x).
+void spmv_dia(const Dev& d, const Sell& A, int variant, int64_t nrows, const double* x, double* y,
+              const double* u, double bu, const double* w, double bw, int mode, cudaStream_t st);
 // r[0:nrows) = b - A x
 void residual(const Dev& d, const Sell& A, int64_t nrows, const double* x, const double* b,
               double* r, cudaStream_t st);

@@ -235,6 +235,15 @@ int build_sell(cagmres* h, const cagmres_plan& p) {
     }
     h->A.nrows = nr; h->A.nslices = ns; h->A.nstored = tot; h->A.nnz = p.nnz_mat;
     h->A.ncols = p.n_ext; h->A.ndcol = ndcol; h->A.ndia = ndia;
+    {   // most common width among unclamped DIA slices (the specialised SpMV's fast path)
+        std::vector<int64_t> cnt(33, 0);
+        for (int64_t sl = 0; sl < ns; ++sl)
+            if ((sinfo[size_t(sl)] & 3) == 1) {
+                const int64_t wdt = (sptr[size_t(sl) + 1] - sptr[size_t(sl)]) / 32;
+                if (wdt <= 32) ++cnt[size_t(wdt)];
+            }
+        h->A.dia_w = int(std::max_element(cnt.begin(), cnt.end()) - cnt.begin());
+    }
     CU(cudaMalloc(&h->A.sptr, sizeof(int64_t) * size_t(ns + 1)));
     CU(cudaMalloc(&h->A.sinfo, sizeof(int64_t) * size_t(std::max<int64_t>(ns, 1))));
     CU(cudaMalloc(&h->A.dcol, sizeof(int32_t) * size_t(std::max<int64_t>(ndcol, 1))));
@@ -361,7 +370,7 @@ void wave_reset_pairs(cagmres* h) {
 // the same operations in the same order (bitwise identical results), so the fastest one on
 // this matrix is picked by timing y = A x over all stored rows (x = V[:,0], y = V[:,1]).
 int spmv_autotune(cagmres* h) {
-    static const int cand[] = {0, 3, 5, 6, 8};
+    static const int cand[] = {0, 3, 5, 6, 8, 10, 11, 12, 13};
     if (h->m < 1 || h->A.nrows <= 0) return CAGMRES_OK;
     double* x = h->V;
     double* y = h->V + h->ldv;
@@ -396,7 +405,7 @@ int spmv_autotune(cagmres* h) {
 
 int init_common(cagmres* h, const cagmres_csr* A, const int64_t* row_starts, int s, int m,
                 int basis, int orth) {
-    if (s < 1 || m < 1 || s > m || s > 31 || (basis != CAGMRES_MONOMIAL && basis != CAGMRES_NEWTON))
+    if (s < 1 || m < 1 || s > m || s > 31 || (basis != CAGMRES_MONOMIAL && basis != CAGMRES_NEWTON && basis != CAGMRES_GMRES))
         return CAGMRES_EINVAL;
     const int kind = orth & CAGMRES_TSQR_MASK;
     if (kind > CAGMRES_CAQR) return CAGMRES_EINVAL;
@@ -733,7 +742,8 @@ int ca_cycle(cagmres* h, const std::vector<Block>& bl) {
 
 // First Newton cycle = GMRES(m) with CGS2 Arnoldi (reading G12), on the
 // same kernels with panel width 1.  tab layout: per k: c1 (m+1), c2 (m+1), r (1).
-int arnoldi_cycle(cagmres* h) {
+// cgs2 = false (GMRES baseline without CAGMRES_REORTH): one CGS pass, c2 = 0.
+int arnoldi_cycle(cagmres* h, bool cgs2) {
     const int m = h->m;
     const size_t stride = 2 * size_t(m + 1) + 1;
     for (int k = 0; k < m; ++k) {
@@ -760,14 +770,18 @@ int arnoldi_cycle(cagmres* h) {
                 aa.c_out = c1;
                 if (kern::arnoldi_fused(h->dev, aa, 0, h->stream)) return CAGMRES_EINVAL;
                 TRY(allreduce(h, c1, size_t(k + 1)));
-                aa.c_in = c1; aa.c_out = c2;
-                if (kern::arnoldi_fused(h->dev, aa, 1, h->stream)) return CAGMRES_EINVAL;
-                TRY(allreduce(h, c2, size_t(k + 1)));
-                h->bytes[PH_BORTH] += 8.0 * nl * (3.0 * (k + 1) + 4.0);
+                if (cgs2) {
+                    aa.c_in = c1; aa.c_out = c2;
+                    if (kern::arnoldi_fused(h->dev, aa, 1, h->stream)) return CAGMRES_EINVAL;
+                    TRY(allreduce(h, c2, size_t(k + 1)));
+                    h->bytes[PH_BORTH] += 8.0 * nl * (3.0 * (k + 1) + 4.0);
+                } else {
+                    h->bytes[PH_BORTH] += 8.0 * nl * ((k + 1) + 1.0);
+                }
             }
             {
                 Scope sc(h, PH_TSQR);
-                aa.c_in = c2; aa.c_out = r;
+                aa.c_in = cgs2 ? c2 : c1; aa.c_out = r;
                 if (kern::arnoldi_fused(h->dev, aa, 2, h->stream)) return CAGMRES_EINVAL;
                 if (h->nranks > 1) {
                     TRY(allreduce(h, r, 1));
@@ -779,7 +793,7 @@ int arnoldi_cycle(cagmres* h) {
             continue;
         }
         TRY(borth_panel(h, h->V, h->ldv, k + 1, v, h->ldv, 1, c1, false));
-        TRY(borth_panel(h, h->V, h->ldv, k + 1, v, h->ldv, 1, c2, false));
+        if (cgs2) TRY(borth_panel(h, h->V, h->ldv, k + 1, v, h->ldv, 1, c2, false));
         TRY(tsqr_panel(h, v, h->ldv, 1, r, CAGMRES_CHOLQR, 0));
     }
     return CAGMRES_OK;
@@ -815,9 +829,10 @@ int residual_norm_async(cagmres* h, const double* b, const double* x) {
 }
 
 // One restart cycle's GPU work plus the async copy of its coefficient table and status.
-int enqueue_cycle(cagmres* h, bool first_newton, const std::vector<Block>& bl) {
-    if (first_newton) {
-        TRY(arnoldi_cycle(h));
+int enqueue_cycle(cagmres* h, bool arnoldi, const std::vector<Block>& bl) {
+    if (arnoldi) {
+        // the shift-finding Newton cycle is CGS2 (G12); the GMRES baseline follows the flag
+        TRY(arnoldi_cycle(h, h->basis != CAGMRES_GMRES || (h->orth & CAGMRES_REORTH) != 0));
     } else {
         TRY(ca_cycle(h, bl));
     }
@@ -916,11 +931,12 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
     switch (opt) {
         case CAGMRES_OPT_MPK_WAVE: h->wave_on = value != 0; h->wave_force = value == 2; return CAGMRES_OK;
         case CAGMRES_OPT_SPMV:
-            if (value < -1 || value > 9) return CAGMRES_EINVAL;
+            if (value < -1 || value > 13 || (value > 9 && value < 10)) return CAGMRES_EINVAL;
             if (value == -1) return spmv_autotune(h);
             h->A.variant = int(value);
             return CAGMRES_OK;
         case CAGMRES_OPT_GRAM: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->dev.gram = int(value); return CAGMRES_OK;
+        case CAGMRES_OPT_ARNOLDI: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->dev.arnoldi_ring = int(value); return CAGMRES_OK;
         case CAGMRES_OPT_FUSE: h->fuse_borth_gram = (value & 1) != 0; h->arnoldi_fuse = (value & 2) != 0; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK:
             if (value < 256 || value % 256) return CAGMRES_EINVAL;
@@ -937,6 +953,7 @@ int cagmres_get_option(cagmres_t h, int opt, int64_t* value) {
         case CAGMRES_OPT_MPK_WAVE: *value = h->wave_on ? (h->wave_force ? 2 : 1) : 0; return CAGMRES_OK;
         case CAGMRES_OPT_SPMV: *value = h->A.variant; return CAGMRES_OK;
         case CAGMRES_OPT_GRAM: *value = h->dev.gram; return CAGMRES_OK;
+        case CAGMRES_OPT_ARNOLDI: *value = h->dev.arnoldi_ring; return CAGMRES_OK;
         case CAGMRES_OPT_FUSE: *value = (h->fuse_borth_gram ? 1 : 0) | (h->arnoldi_fuse ? 2 : 0); return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK: *value = h->wave_CH; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CTAS: *value = h->wave_ctas; return CAGMRES_OK;
@@ -976,7 +993,7 @@ int cagmres_mpk(cagmres_t h, const double* q, double* W, int64_t ldw, int sb) {
     if (!h || !q || !W || sb < 1 || sb > h->s || ldw < h->n_loc || sb > h->m) return CAGMRES_EINVAL;
     if (h->basis == CAGMRES_NEWTON && !h->have_shifts) return CAGMRES_EINVAL;
     CU(cudaMemcpyAsync(h->V, q, sizeof(double) * size_t(h->n_loc), cudaMemcpyDeviceToDevice, h->stream));
-    const std::vector<host::Step> steps = h->basis == CAGMRES_MONOMIAL
+    const std::vector<host::Step> steps = h->basis != CAGMRES_NEWTON
         ? host::block_steps({}, {}, sb) : host::block_steps(h->sh_re, h->sh_im, sb);
     TRY(mpk_block(h, 0, sb, steps));
     CU(cudaMemcpy2DAsync(W, sizeof(double) * size_t(ldw), h->V, sizeof(double) * size_t(h->ldv),
@@ -1052,17 +1069,19 @@ int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit
     bool pending = false;                    // next cycle already enqueued (speculation)
     for (; cyc < maxit && rc != CAGMRES_OK; ++cyc) {
         const bool first_newton = h->basis == CAGMRES_NEWTON && !h->have_shifts;
+        const bool arnoldi = first_newton || h->basis == CAGMRES_GMRES;
+        const bool cgs2 = h->basis != CAGMRES_GMRES || (h->orth & CAGMRES_REORTH) != 0;
         std::fill(H.begin(), H.end(), 0.0);
-        if (!pending) TRY(enqueue_cycle(h, first_newton, bl));
+        if (!pending) TRY(enqueue_cycle(h, arnoldi, bl));
         pending = false;
         CU(cudaEventSynchronize(h->ev_tab));
         if (*h->h_stat) { rc = CAGMRES_EBREAKDOWN; break; }
         // ---- Hessenberg matrix (host) ----
-        if (first_newton) {
+        if (arnoldi) {
             const size_t stride = 2 * size_t(m + 1) + 1;
             for (int k = 0; k < m; ++k) {
                 const double* c1 = htab + stride * k;
-                for (int i = 0; i <= k; ++i) H[size_t(i) + size_t(m + 1) * k] = c1[i] + c1[i + m + 1];
+                for (int i = 0; i <= k; ++i) H[size_t(i) + size_t(m + 1) * k] = c1[i] + (cgs2 ? c1[i + m + 1] : 0.0);
                 H[size_t(k + 1) + size_t(m + 1) * k] = c1[2 * (m + 1)];
             }
         } else {
@@ -1125,7 +1144,7 @@ int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit
         // waiting for beta unless the least-squares residual estimate says this cycle has
         // (almost) converged — hides the host round trip of the convergence test.
         if (cyc + 1 < maxit && res[size_t(m - 1)] > 2.0 * tol * rho0) {
-            TRY(enqueue_cycle(h, false, bl));
+            TRY(enqueue_cycle(h, h->basis == CAGMRES_GMRES, bl));
             pending = true;
         }
         CU(cudaEventSynchronize(h->ev_beta));

@@ -1,0 +1,140 @@
+// spmv_dia.cu — MPK SpMV step (Fig. 4; Newton shift fused) specialised for the
+// dominant DIA slice width of the matrix (CAGMRES_OPT_SPMV 10..13).
+//
+// The persistent kernel of kernels.cu (variant 5) is latency-bound (ncu: issue active 56 %,
+// long-scoreboard the top stall, ~255 instructions per 32-row slice): its generic batched loop
+// pays predicates, selects and 64-bit index arithmetic per entry and issues the shift operand
+// loads only after the dot product.  Here a slice whose width equals the matrix's most common
+// DIA width WT (7 for the 7-point stencil, 5 / 27 for the 5- and 27-point ones; A.dia_w) and
+// needs no clamping runs a fully unrolled body: WT value loads, WT x gathers and the u / w
+// loads are all in flight together (one dependent latency per slice), no predicates.  Other
+// slices take the generic sell_slice_dot path.  The slice descriptors are software-pipelined
+// one / two grid strides ahead exactly as in k_spmv_sell32_persist.
+// Per row the FMAs run t = 0..W-1 from 0.0 and the epilogue is out = fma(bu, u, acc), then
+// fma(bw, w, .): the same operations in the same order as every other variant (bitwise
+// identical results; tests/test_gpu_parity.py::test_spmv_variants_bitwise).
+// (A cp.async shared-memory ring version of this step — every value, x gather and shift
+// operand staged per slice — was measured 2x slower: 8 warps/SM, issue-latency bound.)
+#include <cstdint>
+
+#include "kernels.h"
+
+namespace kern {
+
+namespace {
+constexpr int DT_NT = 256;
+
+struct DiaArgs {
+    int64_t nrows;
+    const int64_t* sptr; const int64_t* sinfo; const int32_t* dcol; int64_t ncols;
+    const double* val;
+    const double* x;
+    const double* u; double bu;
+    const double* w; double bw;
+    double* y;
+};
+}  // namespace
+
+template <int MODE, int WT, int MINB>   // MODE 0: Ax  1: Ax + bu u  2: + bw w  3: u - Ax
+__global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
+    const int lane = threadIdx.x & 31;
+    const int64_t nsl = (a.nrows + 31) >> 5;
+    const int64_t stride = int64_t(gridDim.x) * (DT_NT / 32);
+    int64_t sl = (int64_t(blockIdx.x) * DT_NT + threadIdx.x) >> 5;
+    if (sl >= nsl) return;
+    int64_t b0, i0, b1 = 0, i1 = 1, b2, i2;
+    int W0, W1 = 0, W2, o0, o1;
+    sell_slice_meta(sl, a.sptr, a.sinfo, b0, W0, i0);
+    if (sl + stride < nsl) sell_slice_meta(sl + stride, a.sptr, a.sinfo, b1, W1, i1);
+    o0 = sell_slice_off(lane, W0, i0, a.dcol);
+#pragma unroll 1
+    for (; sl < nsl; sl += stride) {
+        b2 = 0; W2 = 0; i2 = 1;
+        if (sl + 2 * stride < nsl) sell_slice_meta(sl + 2 * stride, a.sptr, a.sinfo, b2, W2, i2);
+        o1 = sell_slice_off(lane, W1, i1, a.dcol);
+        const int64_t r = sl * 32 + lane;
+        const bool live = r < a.nrows;
+        double uu = 0.0, ww = 0.0, acc = 0.0;
+        if (W0 == WT && (i0 & 3) == 1) {
+            const double* vp = a.val + b0 + lane;
+            const double* xr = a.x + r;
+            double v[WT], xv[WT];
+#pragma unroll
+            for (int t = 0; t < WT; ++t) {
+                const int o = __shfl_sync(0xffffffffu, o0, t);
+                v[t] = __ldg(vp + 32 * t);
+                xv[t] = __ldg(xr + o);
+            }
+            if (MODE >= 1 && live) uu = __ldg(a.u + r);
+            if (MODE == 2 && live) ww = __ldg(a.w + r);
+#pragma unroll
+            for (int t = 0; t < WT; ++t) acc = fma(v[t], xv[t], acc);
+        } else {
+            acc = sell_slice_dot<4, true>(r, b0, W0, i0, o0, a.dcol, a.ncols, a.val, a.x, false);
+            if (MODE >= 1 && live) uu = __ldg(a.u + r);
+            if (MODE == 2 && live) ww = __ldg(a.w + r);
+        }
+        if (live) {
+            double out;
+            if constexpr (MODE == 3) {
+                out = uu - acc;
+            } else {
+                out = acc;
+                if constexpr (MODE >= 1) out = fma(a.bu, uu, out);
+                if constexpr (MODE >= 2) out = fma(a.bw, ww, out);
+            }
+            a.y[r] = out;
+        }
+        b0 = b1; W0 = W1; i0 = i1; o0 = o1;
+        b1 = b2; W1 = W2; i1 = i2;
+    }
+}
+
+namespace {
+template <int MODE, int WT, int MINB>
+void go_dia(const Dev& d, const DiaArgs& a, cudaStream_t st) {
+    static int occ = 0;
+    if (occ == 0) {
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_spmv_dia<MODE, WT, MINB>, DT_NT, 0);
+        if (occ < 1) occ = 1;
+    }
+    const int64_t nsl = (a.nrows + 31) >> 5;
+    int64_t g = int64_t(d.sms) * occ;
+    const int64_t need = (nsl + DT_NT / 32 - 1) / (DT_NT / 32);
+    if (g > need) g = need;
+    k_spmv_dia<MODE, WT, MINB><<<unsigned(g), DT_NT, 0, st>>>(a);
+}
+
+template <int WT, int MINB>
+void go_modes(const Dev& d, const DiaArgs& a, cudaStream_t st, int mode) {
+    switch (mode) {
+        case 0: go_dia<0, WT, MINB>(d, a, st); break;
+        case 1: go_dia<1, WT, MINB>(d, a, st); break;
+        case 2: go_dia<2, WT, MINB>(d, a, st); break;
+        default: go_dia<3, WT, MINB>(d, a, st); break;
+    }
+}
+
+template <int MINB>
+void go_width(const Dev& d, const DiaArgs& a, int wt, cudaStream_t st, int mode) {
+    switch (wt) {
+        case 5: go_modes<5, MINB>(d, a, st, mode); break;
+        case 27: go_modes<27, MINB>(d, a, st, mode); break;
+        default: go_modes<7, MINB>(d, a, st, mode); break;     // other widths: generic path
+    }
+}
+}  // namespace
+
+// variants 10 / 11 / 12 / 13: at least 3 / 4 / 5 / 6 CTAs per SM (register cap)
+void spmv_dia(const Dev& d, const Sell& A, int variant, int64_t nrows, const double* x, double* y,
+              const double* u, double bu, const double* w, double bw, int mode, cudaStream_t st) {
+    DiaArgs a{nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, u, bu, w, bw, y};
+    switch (variant) {
+        case 10: go_width<3>(d, a, A.dia_w, st, mode); break;
+        case 11: go_width<4>(d, a, A.dia_w, st, mode); break;
+        case 12: go_width<5>(d, a, A.dia_w, st, mode); break;
+        default: go_width<6>(d, a, A.dia_w, st, mode); break;
+    }
+}
+
+}  // namespace kern

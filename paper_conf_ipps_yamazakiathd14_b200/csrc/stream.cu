@@ -309,6 +309,28 @@ int dispatch(const Dev& d, const StreamArgs& a, cudaStream_t st) {
         default: return -1;
     }
 }
+// w = 1 TRSM (Arnoldi normalisation v /= h, q_0 = r / beta): P[:,0] *= 1 / R[0].  A DMMA
+// tile would waste 7/8 of its work and 12 M instructions on 2 M rows; this is a plain
+// vectorised stream (16-B loads/stores, grid = SMs x 4).  The product p * (1/r) is rounded once,
+// exactly like the DMMA path (fma(p, 1/r, 0)), so results are bitwise identical.
+__global__ void __launch_bounds__(256) k_scale1(int64_t n, double* __restrict__ p, const double* __restrict__ r) {
+    const double inv = 1.0 / __ldg(r);
+    const int64_t i0 = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    const int64_t stride = int64_t(gridDim.x) * blockDim.x;
+    const bool al = (reinterpret_cast<uintptr_t>(p) & 15) == 0;
+    if (al) {
+        double2* p2 = reinterpret_cast<double2*>(p);
+        const int64_t n2 = n >> 1;
+        for (int64_t i = i0; i < n2; i += stride) {
+            double2 v = __ldcs(p2 + i);
+            v.x *= inv; v.y *= inv;
+            p2[i] = v;
+        }
+        if (i0 == 0 && (n & 1)) p[n - 1] *= inv;
+    } else {
+        for (int64_t i = i0; i < n; i += stride) p[i] *= inv;
+    }
+}
 }  // namespace
 
 void update(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, double* P,
@@ -325,6 +347,14 @@ void update(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, doubl
 void trsm(const Dev& d, int64_t n, double* P, int64_t ldp, int w, const double* R, int c0,
           cudaStream_t st) {
     if (n <= 0 || w <= 0) return;
+    if (w == 1 && c0 == 0) {
+        int64_t g = int64_t(d.sms) * 4;
+        const int64_t need = ((n >> 1) + 255) / 256;
+        if (g > need) g = need < 1 ? 1 : need;
+        ++g_launches;
+        k_scale1<<<unsigned(g), 256, 0, st>>>(n, P, R);
+        return;
+    }
     StreamArgs a{n, nullptr, 0, 0, P, ldp, w, R, w, c0};
     dispatch<1>(d, a, st);
 }

@@ -13,7 +13,7 @@ import numpy as np
 
 from . import _lib as L
 
-_BASIS = {"monomial": L.MONOMIAL, "newton": L.NEWTON}
+_BASIS = {"monomial": L.MONOMIAL, "newton": L.NEWTON, "gmres": L.GMRES}
 _TSQR = {"cholqr": L.CHOLQR, "svqr": L.SVQR, "cgs": L.CGS, "mgs": L.MGS, "caqr": L.CAQR}
 
 
@@ -115,10 +115,11 @@ class Solver:
         s = torch.cuda.current_stream(self.device)
         L.check(self._lib.cagmres_set_stream(self._h, C.c_void_p(s.cuda_stream)), "set_stream")
 
-    OPTIONS = {"mpk_wave": 1, "wave_chunk": 3, "wave_ctas": 4, "wave_lag": 5, "fuse": 6, "spmv": 7, "gram": 8}
+    OPTIONS = {"mpk_wave": 1, "wave_chunk": 3, "wave_ctas": 4, "wave_lag": 5, "fuse": 6, "spmv": 7, "gram": 8,
+               "arnoldi": 9}
 
     def set_option(self, opt, value):
-        """opt: "mpk_wave", "wave_chunk", "wave_ctas", "wave_lag", "fuse", "spmv", "gram" (CAGMRES_OPT_*)."""
+        """opt: "mpk_wave", "wave_chunk", "wave_ctas", "wave_lag", "fuse", "spmv", "gram", "arnoldi" (CAGMRES_OPT_*)."""
         L.check(self._lib.cagmres_set_option(self._h, self.OPTIONS[opt], int(value)), "set_option")
 
     def get_option(self, opt):

@@ -126,23 +126,25 @@ def test_mpk_wave_bitwise_equals_stepwise(gen):
         assert torch.equal(W1, W2), (gen, sb)
 
 
-@pytest.mark.parametrize("gen", ["cd27_ragged", "g3_small", "banded"])
+@pytest.mark.parametrize("gen", ["cd27_ragged", "g3_small", "banded", "cd7_ragged"])
 def test_spmv_variants_bitwise(gen):
     """Every SpMV kernel variant (CAGMRES_OPT_SPMV: one or two SELL-32 slices per warp, load
     batches 4/8, persistent with pipelined slice descriptors) sums each row in the same order: the MPK bases are bitwise identical; the
     parity of variant 0 against the oracle is test_mpk_parity."""
     A = {"cd27_ragged": lambda: G.convection_diffusion(17, 3, 27),
          "g3_small": lambda: G.g3_shaped(n=40000, width=200),
-         "banded": lambda: G.banded(n=300001)}[gen]()
+         "banded": lambda: G.banded(n=300001),
+         "cd7_ragged": lambda: G.convection_diffusion(45, 3, 7)}[gen]()
     q = dev(G.u(6, np.arange(A.n)))
     S = Solver(A, s=6, m=30, basis="newton")
     S.set_shifts(*SHIFTS)
     Ws = []
-    for v in range(10):
+    variants = list(range(10)) + [10, 11, 12, 13]       # 10..13: cp.async ring-staged slices
+    for v in variants:
         S.set_option("spmv", v)
         Ws.append(S.mpk(q, 6))
-    for v in range(1, 10):
-        assert torch.equal(Ws[v], Ws[0]), v
+    for i, v in enumerate(variants[1:], 1):
+        assert torch.equal(Ws[i], Ws[0]), v
 
 
 def test_mpk_full_size_C2():
@@ -340,5 +342,36 @@ def test_solve_kernel_options(spmv, gram):
     assert st.status == 0
     assert abs(st.cycles - len(ref)) <= 1
     assert hist_within_envelope(st.hist, ref, env)
+    r = b - As @ x.cpu().numpy()
+    assert np.linalg.norm(r) <= 1.01e-8 * np.linalg.norm(b)
+
+
+# ----------------------------------------------------------------------------- GMRES baseline
+@pytest.mark.parametrize("reorth,arnoldi", [(False, 1), (True, 1), (False, 0)])
+@pytest.mark.parametrize("gen", ["C1", "g3_small"])
+def test_solve_gmres_baseline(gen, reorth, arnoldi):
+    """basis="gmres": the standard GMRES(m) comparator of Fig. 14/15 on the GPU —
+    SpMV + CGS (CGS2 with reorth) per iteration.  Restarted GMRES's per-cycle residuals are
+    fixed by the Krylov space, so they must match the oracle's MGS GMRES(m) [3] to rounding
+    (its own sensitivity to summation order measured by symmetric permutations)."""
+    if gen == "C1":
+        A, m = G.convection_diffusion(32, 2, 5), 30
+    else:
+        A, m = G.g3_shaped(n=40000, width=200), 60
+    As = A.to_scipy()
+    b = G.rhs(A.n)
+    S = Solver(A, s=1, m=m, basis="gmres", reorth=reorth)
+    S.set_option("arnoldi", arnoldi)          # 1: cp.async ring Arnoldi passes (n >= 2048), 0: register kernel
+    x, st = S.solve(dev(b), tol=1e-8, maxit=200)
+    ref = O.gmres(As, b, m, tol=1e-8, maxcyc=200)["hist"]
+    env = np.zeros(len(ref))
+    p = np.argsort(G.u(1000, np.arange(A.n)))
+    hp = O.gmres(As[p][:, p], b[p], m, tol=1e-8, maxcyc=200)["hist"]
+    k = min(len(hp), len(ref))
+    env[:k] = np.abs(hp[:k] - ref[:k]) / ref[:k]
+    env = np.maximum.accumulate(env)
+    assert st.status == 0 and abs(st.cycles - len(ref)) <= 1
+    assert hist_within_envelope(st.hist, ref, env, factor=100.0)
+    assert np.all(np.diff(st.hist) <= 1e-14)                      # restarted GMRES is monotone
     r = b - As @ x.cpu().numpy()
     assert np.linalg.norm(r) <= 1.01e-8 * np.linalg.norm(b)

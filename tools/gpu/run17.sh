@@ -1,7 +1,5 @@
 #!/bin/bash
 cd $GRAFT_REPO_ROOT
 mkdir -p gpurun_out
-timeout 900 python -m pytest tests/test_gpu_parity.py -m gpu -q -k "mpk or spmv or solve_C1 or fused" > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
-timeout 600 python tools/spmv_variants.py > gpurun_out/spmv_variants.json 2> gpurun_out/spmv_variants.log
-timeout 600 python bench.py --steps 5 --warmup 3 --no-cpu > gpurun_out/bench.log 2>&1; echo "bench rc=$?" >> gpurun_out/bench.log
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:spmv_sell32 -s 40 -c 1 -o gpurun_out/prof_spmv2 python bench.py --steps 1 --warmup 3 --no-cpu > gpurun_out/ncu_full.log 2>&1
+timeout 300 ncu --set full --clock-control none --import-source on -k regex:spmv_ring -s 40 -c 1 -o gpurun_out/prof_ring python tools/kprof.py --opt spmv=10 > gpurun_out/prof_ring.log 2>&1
+timeout 300 ncu --set full --clock-control none --import-source on -k regex:spmv_sell32_persist -s 40 -c 1 -o gpurun_out/prof_persist python tools/kprof.py --opt spmv=5 > gpurun_out/prof_persist.log 2>&1
