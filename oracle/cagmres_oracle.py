@@ -127,6 +127,28 @@ def tsqr_cholqr(P):
     return _trsm_right(P, R), R
 
 
+def borth_cholqr_onepass(Q, P):
+    """One-pass BOrth + CholQR (the fused-CGS direction of P:176 and
+    the one-reduction tall-skinny kernels of P:275 fn 7).  P = [q_j, W_1..W_sb]:
+      M  = [Q P]^T P                       (one product: C and the Gram of the raw panel)
+      Cf = M[0:j, :] with column 0 := 0     (q_j is not re-orthogonalised, G2)
+      G  = M[j:, :] - Cf^T Cf               (Pythagoras: = (P - Q Cf)^T (P - Q Cf) when Q^T Q = I)
+      R  = chol(G) ;  Q_hat = (P - Q Cf) R^{-1}
+    Returns (C = Cf[:, 1:], Q_hat, R).  Equal to borth_cgs + tsqr_cholqr in exact arithmetic
+    when Q has orthonormal columns."""
+    j = Q.shape[1]
+    M = np.column_stack([Q, P]).T @ P
+    Cf = M[:j, :].copy()
+    Cf[:, 0] = 0.0
+    G = M[j:, :] - Cf.T @ Cf
+    try:
+        L = np.linalg.cholesky(G)
+    except np.linalg.LinAlgError as e:
+        raise Breakdown("one-pass CholQR: Gram matrix not positive definite") from e
+    R = L.T.copy()
+    return Cf[:, 1:], _trsm_right(P - Q @ Cf, R), R
+
+
 def tsqr_svqr(P):
     """SVQR (P:172, P:221; G14): B = P^T P ; D = diag(B)^{-1/2} ; D B D = U S U^T ;
     s_i <- max(s_i, eps*s_max) ; R_hat = R of qr(S^{1/2} U^T) with positive diagonal ;
@@ -366,34 +388,36 @@ def gmres(A, b, m, tol=1e-8, maxcyc=100, x0=None):
 # CA-GMRES(s, m) (Fig. 2 reconstructed per SURVEY §8(c) / DESIGN.md)
 # ---------------------------------------------------------------------------------------
 def ca_cycle(A, Q, H, s, m, re, im, tsqr="cholqr", borth="cgs", reorth=False,
-             caqr_blocks=1, diag=None):
+             caqr_blocks=1, diag=None, onepass=False):
     """One restart cycle's basis generation: fills Q[:,1:m+1] and H ((m+1) x m) given
-    Q[:,0] = r/beta.  Blocks of sb = min(s, m-j)."""
+    Q[:,0] = r/beta.  Blocks of sb = min(s, m-j).  onepass: panels with j > 0 use
+    borth_cholqr_onepass (CholQR only) for each BOrth+TSQR pass."""
     j = 0
     tsqr_f = TSQR[tsqr]
     borth_f = BORTH[borth]
+    if onepass and (tsqr != "cholqr" or borth != "cgs"):
+        raise ValueError("onepass needs tsqr='cholqr', borth='cgs'")
+
+    def bt_pass(P):                                          # one BOrth + TSQR pass on P
+        Cc = np.zeros((j, P.shape[1]))
+        if onepass and j > 0:
+            Cc[:, 1:], Qh_, R_ = borth_cholqr_onepass(Q[:, :j], P)
+            return Cc, Qh_, R_
+        P = P.copy()
+        if j > 0:                                            # BOrth (P:156), col 0 skipped
+            Cp, P1 = borth_f(Q[:, :j], P[:, 1:])
+            Cc[:, 1:] = Cp
+            P[:, 1:] = P1
+        Qh_, R_ = tsqr_caqr(P, caqr_blocks) if tsqr == "caqr" else tsqr_f(P)   # TSQR (Fig. 9)
+        return Cc, Qh_, R_
+
     while j < m:
         sb = min(s, m - j)
         W = mpk(A, Q[:, j], sb, re, im)                          # MPK (Fig. 4)
         B = change_of_basis(sb, re, im)
-        C = np.zeros((j, sb + 1))
-        P = W.copy()
-        if j > 0:                                                # BOrth (P:156), col 0 skipped
-            Cp, P1 = borth_f(Q[:, :j], W[:, 1:])
-            C[:, 1:] = Cp
-            P[:, 1:] = P1
-        if tsqr == "caqr":
-            Qh, R = tsqr_caqr(P, caqr_blocks)
-        else:
-            Qh, R = tsqr_f(P)                                    # TSQR (Fig. 9)
+        C, Qh, R = bt_pass(W)
         if reorth:                                               # "2x" (P:158, P:273, G16)
-            P2 = np.column_stack([Q[:, j], Qh[:, 1:]])
-            C2 = np.zeros((j, sb + 1))
-            if j > 0:
-                Cp, P2b = borth_f(Q[:, :j], P2[:, 1:])
-                C2[:, 1:] = Cp
-                P2[:, 1:] = P2b
-            Qh, R2 = (tsqr_caqr(P2, caqr_blocks) if tsqr == "caqr" else tsqr_f(P2))
+            C2, Qh, R2 = bt_pass(np.column_stack([Q[:, j], Qh[:, 1:]]))
             C = C + C2 @ R
             R = R2 @ R
         Q[:, j + 1:j + sb + 1] = Qh[:, 1:]                       # q_j kept (G2)
@@ -410,7 +434,7 @@ def ca_cycle(A, Q, H, s, m, re, im, tsqr="cholqr", borth="cgs", reorth=False,
 
 def cagmres(A, b, s, m, basis="newton", tsqr="cholqr", borth="cgs", reorth=False,
             tol=1e-8, maxcyc=100, x0=None, shifts=None, caqr_blocks=1, diag=None,
-            keep_last=False):
+            keep_last=False, onepass=False):
     """CA-GMRES(s, m) solve.  x0 = 0 by default (G17).
     basis 'newton': first cycle is GMRES(m) (Arnoldi CGS2) unless shifts are given; its
     Ritz values in modified Leja order become the shifts.  'monomial': theta = 0
@@ -440,7 +464,7 @@ def cagmres(A, b, s, m, basis="newton", tsqr="cholqr", borth="cgs", reorth=False
             Q, H, _ = arnoldi_cgs2(A, r, m)
             re, im = modified_leja(ritz_values(H, m), s)
         else:
-            ca_cycle(A, Q, H, s, m, re, im, tsqr, borth, reorth, caqr_blocks, diag)
+            ca_cycle(A, Q, H, s, m, re, im, tsqr, borth, reorth, caqr_blocks, diag, onepass)
         y, _ = givens_ls(H, beta)                        # LS on the CPU
         x = x + Q[:, :m] @ y                             # x := x + V_{1:m} y
         rho = np.linalg.norm(b - A @ x)                  # explicit residual (G17)

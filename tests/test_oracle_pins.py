@@ -80,6 +80,26 @@ def test_borth_projects_out(kind):
     assert np.allclose(C, Q.T @ P, atol=1e-13)
 
 
+def test_onepass_borth_cholqr_equals_two_pass():
+    """One-pass BOrth+CholQR (NEXT-2) equals CGS BOrth followed by CholQR when Q^T Q = I
+    (Pythagoras); pinned against the two-pass composition and against Householder QR of the
+    explicitly projected panel."""
+    Q, _ = np.linalg.qr(G.random_panel(3000, 20, 4))
+    P = G.random_panel(3000, 6, 5)
+    P[:, 0] = np.linalg.qr(np.column_stack([Q, P[:, 0]]))[0][:, -1]      # q_j orthonormal, _|_ Q
+    P[:, 2] += 0.3 * Q[:, 5] + 0.2 * P[:, 1]
+    C1, Qh1, R1 = O.borth_cholqr_onepass(Q, P)
+    Cp, Pp = O.borth_cgs(Q, P[:, 1:])
+    Qh2, R2 = O.tsqr_cholqr(np.column_stack([P[:, 0], Pp]))
+    assert np.abs(C1 - Q.T @ P[:, 1:]).max() < 1e-13
+    assert np.abs(C1 - Cp).max() < 1e-13
+    assert np.abs(R1 - R2).max() < 1e-12 * np.abs(R2).max()
+    assert np.abs(Qh1 - Qh2).max() < 1e-11
+    Qr, Rr = _ref_qr(np.column_stack([P[:, 0], P[:, 1:] - Q @ (Q.T @ P[:, 1:])]))
+    assert np.abs(R1 - Rr).max() < 1e-12 * np.abs(Rr).max()
+    assert O.orth_error(np.column_stack([Q, Qh1])) < 1e-12
+
+
 # ----------------------------------------------------------------------------- TSQR (Fig. 9/10)
 def _ref_qr(P):
     Q, R = np.linalg.qr(P)
@@ -149,16 +169,18 @@ def test_givens_ls_matches_lstsq():
 
 
 # ----------------------------------------------------------------------------- H update (G1)
-@pytest.mark.parametrize("tsqr,reorth", [("cholqr", False), ("cholqr", True), ("svqr", False),
-                                         ("mgs", False), ("caqr", False), ("cgs", True)])
-def test_ca_cycle_arnoldi_relation_and_gmres_equivalence(cd2, tsqr, reorth):
+@pytest.mark.parametrize("tsqr,reorth,onepass", [("cholqr", False, False), ("cholqr", True, False),
+                                                 ("svqr", False, False), ("mgs", False, False),
+                                                 ("caqr", False, False), ("cgs", True, False),
+                                                 ("cholqr", False, True), ("cholqr", True, True)])
+def test_ca_cycle_arnoldi_relation_and_gmres_equivalence(cd2, tsqr, reorth, onepass):
     n = cd2.shape[0]
     b = G.rhs(n)
     m, s = 30, 5
     re, im = O.modified_leja(O.ritz_values(O.arnoldi_cgs2(cd2, b, m)[1], m), s)
     Q = np.zeros((n, m + 1), order="F"); Q[:, 0] = b / np.linalg.norm(b)
     H = np.zeros((m + 1, m))
-    O.ca_cycle(cd2, Q, H, s, m, re, im, tsqr=tsqr, reorth=reorth)
+    O.ca_cycle(cd2, Q, H, s, m, re, im, tsqr=tsqr, reorth=reorth, onepass=onepass)
     Aop = sp.linalg.norm(cd2)
     assert np.linalg.norm(cd2 @ Q[:, :m] - Q @ H) / Aop < 1e-12
     assert np.allclose(np.tril(H, -2), 0.0)            # exactly upper Hessenberg
@@ -198,13 +220,14 @@ def test_s1_is_gmres(cd2):
 
 
 # ----------------------------------------------------------------------------- whole solve
-@pytest.mark.parametrize("basis,tsqr,reorth", [("newton", "cholqr", False),
-                                               ("monomial", "cholqr", False),
-                                               ("newton", "cholqr", True),
-                                               ("newton", "svqr", False)])
-def test_solve_matches_dense_direct(cd2, basis, tsqr, reorth):
+@pytest.mark.parametrize("basis,tsqr,reorth,onepass", [("newton", "cholqr", False, False),
+                                                       ("monomial", "cholqr", False, False),
+                                                       ("newton", "cholqr", True, False),
+                                                       ("newton", "svqr", False, False),
+                                                       ("newton", "cholqr", True, True)])
+def test_solve_matches_dense_direct(cd2, basis, tsqr, reorth, onepass):
     b = G.rhs(cd2.shape[0])
-    r = O.cagmres(cd2, b, 5, 30, basis=basis, tsqr=tsqr, reorth=reorth, tol=1e-8)
+    r = O.cagmres(cd2, b, 5, 30, basis=basis, tsqr=tsqr, reorth=reorth, tol=1e-8, onepass=onepass)
     xs = np.linalg.solve(cd2.toarray(), b)
     kappa = np.linalg.cond(cd2.toarray())
     assert r["hist"][-1] <= 1e-8
