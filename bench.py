@@ -142,13 +142,14 @@ def run_ours(args):
     t0 = time.time()
     if ws == 1:
         A = cfg["build"]()
-        S = Solver(A, cfg["s"], cfg["m"], basis=cfg["basis"], tsqr=cfg["tsqr"], reorth=cfg["reorth"])
+        S = Solver(A, cfg["s"], cfg["m"], basis=cfg["basis"], tsqr=cfg["tsqr"], reorth=cfg["reorth"] or args.reorth,
+                   onepass=args.onepass)
         b_host = G.rhs(cfg["n"])
     else:
         rs = np.array([(p * cfg["n"]) // ws for p in range(ws + 1)], dtype=np.int64)
         A = ghost_rows(cfg, rs, rank, cfg["s"])
-        S = Solver(A, cfg["s"], cfg["m"], basis=cfg["basis"], tsqr=cfg["tsqr"], reorth=cfg["reorth"],
-                   group=group, row_starts=rs)
+        S = Solver(A, cfg["s"], cfg["m"], basis=cfg["basis"], tsqr=cfg["tsqr"], reorth=cfg["reorth"] or args.reorth,
+                   group=group, row_starts=rs, onepass=args.onepass)
         b_host = G.rhs(cfg["n"], rows=(rs[rank], rs[rank + 1]))
     for kv in args.opt:
         k_, v_ = kv.split("=")
@@ -242,35 +243,44 @@ def run_ours(args):
         t = torch.tensor([e2e], device="cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e = float(t.item())
-    # ---- the paper's comparator (Fig. 14/15): standard GMRES(m) on the same GPU kernels ----
-    gm = None
-    if not args.no_gmres:
-        Sg = (Solver(A, 1, cfg["m"], basis="gmres", tsqr="cholqr", reorth=False) if ws == 1 else
-              Solver(A, 1, cfg["m"], basis="gmres", tsqr="cholqr", reorth=False, group=group, row_starts=rs))
-        xg = torch.zeros_like(b)
-        Sg.solve(b, xg, tol=TOL, maxit=400)
-        g_ms, g_st = [], None
+    # ---- comparators on the same GPU kernels, timed like `value` (not part of it) ----
+    def time_other(S2, maxit):
+        x2 = torch.zeros_like(b)
+        S2.solve(b, x2, tol=TOL, maxit=maxit)
+        o_ms, o_st = [], None
         for k in range(max(1, min(args.steps, 3))):
             flush.fill_(float(k))
             if group is not None:
                 dist.barrier()
             torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            xg.zero_()
+            x2.zero_()
             e0.record(stream)
-            _, g_st = Sg.solve(b, xg, tol=TOL, maxit=400)
+            _, o_st = S2.solve(b, x2, tol=TOL, maxit=maxit)
             e1.record(stream)
             torch.cuda.synchronize()
-            g_ms.append(e0.elapsed_time(e1))
-        gv = float(np.mean(g_ms))
+            o_ms.append(e0.elapsed_time(e1))
+        v = float(np.mean(o_ms))
         if group is not None:
-            t = torch.tensor([gv], device="cuda")
+            t = torch.tensor([v], device="cuda")
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            gv = float(t.item())
+            v = float(t.item())
+        S2.close()
+        return v, o_st
+
+    kw = {} if ws == 1 else dict(group=group, row_starts=rs)
+    gm = None
+    if not args.no_gmres:      # the paper's comparator (Fig. 14/15): standard GMRES(m)
+        gv, g_st = time_other(Solver(A, 1, cfg["m"], basis="gmres", tsqr="cholqr", reorth=False, **kw), 400)
         gm = {"value": round(gv, 4), "unit": "ms", "cycles": int(g_st.cycles),
               "method": f"GMRES({cfg['m']}) with CGS, one SpMV + CGS pass per iteration (basis='gmres')",
               "ca_speedup": round(gv / ms_step, 3)}
-        Sg.close()
+    op = None
+    if not args.no_gmres and not args.onepass:   # SURVEY NEXT-2 variant of the same solve
+        ov, o_st = time_other(Solver(A, cfg["s"], cfg["m"], basis=cfg["basis"], tsqr=cfg["tsqr"],
+                                     reorth=cfg["reorth"] or args.reorth, onepass=True, **kw), 200)
+        op = {"value": round(ov, 4), "unit": "ms", "cycles": int(o_st.cycles),
+              "method": "one-pass BOrth+CholQR (CAGMRES_ONEPASS: [Q P]^T P, Pythagorean Gram, (P-QC)R^-1 in one pass)"}
     clocks = clk.summary()
     out = None
     if rank == 0:
@@ -284,6 +294,8 @@ def run_ours(args):
                        "tol": TOL, "cycles": stats[-1].cycles, "parallelism": f"rows{ws}",
                        "l2": "inputs larger than L2 (A 175 MB, V 520 MB) + 256 MB flush between steps",
                        "setup_s": round(setup_s, 2), "options": args.opt,
+                       "orth": ("CholQR" + ("2 (reorth)" if (cfg["reorth"] or args.reorth) else "")
+                                + (", one-pass BOrth+CholQR (NEXT-2)" if args.onepass else ", BOrth CGS")),
                        "kernels": {k_: S.get_option(k_) for k_ in ("spmv", "gram", "fuse", "mpk_wave")}},
             "e2e": {"value": round(e2e, 4), "unit": "ms", "h2d_bytes_per_step": 8 * len(b_host),
                     "d2h_bytes_per_step": 8 * len(b_host), "each_ms": [round(v, 3) for v in e2e_ms]},
@@ -300,6 +312,7 @@ def run_ours(args):
             "phases_note": "one extra untimed solve with CUDA events around every phase",
             "phases_gbs": {k: (round(v, 1) if v else None) for k, v in phase_gbs.items()},
             "gmres_baseline": gm,
+            "onepass_variant": op,
             "clocks": clocks,
             "cpu_baseline": cpu,
         }
@@ -388,6 +401,8 @@ def main():
     ap.add_argument("--config", default="C2", choices=sorted(CFG))
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-gmres", action="store_true", help="skip the GPU GMRES(m) comparator")
+    ap.add_argument("--reorth", action="store_true", help="2x BOrth+TSQR (CholQR2)")
+    ap.add_argument("--onepass", action="store_true", help="one-pass BOrth+CholQR (CAGMRES_ONEPASS, NEXT-2)")
     ap.add_argument("--opt", action="append", default=[],
                     help="solver option NAME=VALUE (CAGMRES_OPT_*: spmv, gram, fuse, mpk_wave, ...); "
                          "default: the library's defaults")

@@ -54,6 +54,12 @@ enum { CAGMRES_CHOLQR = 0, CAGMRES_SVQR = 1, CAGMRES_CGS = 2,     /* TSQR, Fig. 
 #define CAGMRES_TSQR_MASK   0xff
 #define CAGMRES_REORTH      0x100   /* "2x": BOrth+TSQR twice (Fig. 14)       */
 #define CAGMRES_BORTH_MGS   0x200   /* BOrth by MGS instead of CGS      */
+/* One-pass BOrth + CholQR (fused CGS; one-reduction kernels, P:275 fn 7):
+ * for panels with j > 0, one pass [C; B] = [Q P]^T P, R = chol(B - C^T C) (Pythagoras, exact
+ * when Q^T Q = I), then P := (P - Q C) R^{-1} in one pass.  Reads the panel twice instead of
+ * four times and needs one reduction instead of two.  CholQR only (else EINVAL); less stable
+ * than the two-pass method (use with CAGMRES_REORTH); j + s + 1 <= 64. */
+#define CAGMRES_ONEPASS     0x400
 
 typedef struct cagmres* cagmres_t;
 
@@ -147,6 +153,13 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
 #define CAGMRES_OPT_SPMV       7
 #define CAGMRES_OPT_GRAM       8
 #define CAGMRES_OPT_ARNOLDI    9
+#define CAGMRES_OPT_PANEL_TW   10   /* wide panel kernels: 16 (default: 16-row ring tiles where
+                                       measured faster) or 32 (always 32-row tiles) */
+#define CAGMRES_OPT_PDL        12   /* process-wide: 1 (default) = programmatic dependent launch of
+                                       the hot kernels (next kernel's CTAs scheduled while the
+                                       previous one drains), 0 = plain stream order */
+#define CAGMRES_OPT_TRSM       11   /* CholQR/SVQR panel update V R^{-1}: 1 (default) = scalar
+                                       FP64 on a cp.async ring (w <= 16), 0 = FP64 tensor core */
 int cagmres_set_option(cagmres_t h, int opt, int64_t value);
 /* Current value of an option (e.g. the SpMV variant the create-time selection picked).
  * EINVAL for a null handle / pointer or an unknown option. */

@@ -16,7 +16,7 @@ OK, NOT_CONVERGED = 0, 1
 EINVAL, ECUDA, ENCCL, EBREAKDOWN, ENOMEM, EGHOST, ENOTSUP = -1, -2, -3, -4, -5, -6, -7
 MONOMIAL, NEWTON, GMRES = 0, 1, 2
 CHOLQR, SVQR, CGS, MGS, CAQR = 0, 1, 2, 3, 4
-REORTH, BORTH_MGS = 0x100, 0x200
+REORTH, BORTH_MGS, ONEPASS = 0x100, 0x200, 0x400
 OPT_MPK_WAVE, OPT_WAVE_CHUNK, OPT_WAVE_CTAS, OPT_WAVE_LAG, OPT_FUSE, OPT_SPMV = 1, 3, 4, 5, 6, 7
 
 

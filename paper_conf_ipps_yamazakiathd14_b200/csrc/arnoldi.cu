@@ -89,6 +89,8 @@ __global__ void __launch_bounds__(512, 1) k_arnoldi_ring(ArnoldiArgs a) {
     extern __shared__ __align__(16) double sma[];
     __shared__ double sc[JX > 0 ? JX : 1];
     __shared__ double sred[16][JX > 0 ? JX : 1];
+    pdl_wait();
+    pdl_trigger();
     const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const int jx = a.jx;
     for (int i = threadIdx.x; i < JX; i += blockDim.x) sc[i] = (MODE != 0 && i < jx) ? a.c_in[i] : 0.0;
@@ -188,7 +190,7 @@ bool go_ring(const Dev& d, const ArnoldiArgs& a, cudaStream_t st) {
     const size_t smem = size_t(nw) * ring_w;
     cudaFuncSetAttribute(k_arnoldi_ring<JX, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
     ++g_launches;
-    k_arnoldi_ring<JX, MODE><<<unsigned(d.sms), 32 * nw, smem, st>>>(a);
+    launch_pdl(k_arnoldi_ring<JX, MODE>, dim3(unsigned(d.sms)), dim3(32 * nw), smem, st, a);
     return true;
 }
 }  // namespace

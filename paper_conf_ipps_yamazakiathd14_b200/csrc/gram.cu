@@ -7,10 +7,11 @@
 // per row, a fraction of the DFMA pipe.
 //
 // Data movement: the warps of a CTA work in pairs; each pair streams its own contiguous
-// range of 32-row tiles of the W columns through an S-stage shared-memory ring with 16-B
+// range of 64-row tiles of the W columns through an S-stage shared-memory ring with 16-B
 // cp.async copies (both warps issue half of every tile's copies), so the bytes in flight
-// (~150 KB per SM) live in shared memory, not in registers.  Lane l of both warps owns row l
-// of a tile (column c, row l at c*32 + l: conflict-free reads); the W(W+1)/2 upper-triangle
+// (~150 KB per SM) live in shared memory, not in registers.  Lane l of both warps owns rows
+// 2l, 2l+1 of a tile (one 16-B shared load per column; 32-row tiles with one row per lane
+// measured 49 us for W = 11 at n = 2.1M: barrier / MIO-throttle bound); the W(W+1)/2 upper-triangle
 // products are split between the two warps (33 + 33 sums at W = 11), which halves the
 // registers per thread and so doubles the warps per SM that hide the latencies.  One named
 // barrier per tile and pair publishes the tile and frees the slot read in the previous step.
@@ -30,28 +31,33 @@ namespace kern {
 
 namespace {
 constexpr int GR_NT = 512;               // 16 warps = 8 pairs, one CTA per SM
-constexpr int GR_TW = 32;                // rows per tile
+constexpr int GR_TW = 64;                // rows per tile (2 per lane: one LDS.128 per column)
 constexpr int GR_NP = GR_NT / 64;        // warp pairs
 
 template <int W>
-__host__ __device__ constexpr int gram_stages() { return W <= 6 ? 12 : (W <= 8 ? 10 : 8); }
+__host__ __device__ constexpr int gram_stages() { return W <= 6 ? 6 : (W <= 8 ? 5 : 4); }
 
 __device__ __forceinline__ void pair_sync(int pair) {
     asm volatile("bar.sync %0, 64;" ::"r"(pair + 1) : "memory");
 }
 
-// acc[e - lo] += v_i v_k for the upper-triangle entries e in [lo, hi) (row-major order)
+// acc[e - lo] += v_i v_k for the upper-triangle entries e in [lo, hi) (row-major order), for
+// the two rows 2 lane, 2 lane + 1 of the tile (in that order)
 template <int W, int LO, int HI>
 __device__ __forceinline__ void rank1_part(const double* __restrict__ sl, int lane, double (&acc)[HI - LO]) {
-    double v[W];
+    double2 v[W];
 #pragma unroll
-    for (int c = 0; c < W; ++c) v[c] = sl[c * GR_TW + lane];      // unused columns: dead code
+    for (int c = 0; c < W; ++c)                                    // unused columns: dead code
+        v[c] = *reinterpret_cast<const double2*>(sl + c * GR_TW + 2 * lane);
     int e = 0;
 #pragma unroll
     for (int i = 0; i < W; ++i)
 #pragma unroll
         for (int k = i; k < W; ++k, ++e)
-            if (e >= LO && e < HI) acc[e - LO] = fma(v[i], v[k], acc[e - LO]);
+            if (e >= LO && e < HI) {
+                acc[e - LO] = fma(v[i].x, v[k].x, acc[e - LO]);
+                acc[e - LO] = fma(v[i].y, v[k].y, acc[e - LO]);
+            }
 }
 }  // namespace
 
@@ -69,7 +75,7 @@ __device__ __forceinline__ void gram_pair_body(const GramArgs& a, double* smg, d
     const int64_t NPg = int64_t(gridDim.x) * GR_NP;
     const int64_t g = int64_t(blockIdx.x) * GR_NP + pair;
     const int64_t t0 = g * T / NPg, t1 = (g + 1) * T / NPg;
-    // this thread's 16-B chunks of a tile (pair-thread q = 64 c' + ...): fixed offsets
+    // this thread's 16-B chunks of a tile (pair-thread q = 64 k + pt): fixed offsets
     constexpr int CPC = GR_TW * 8 / 16;                            // 16-B chunks per column tile
     constexpr int NCH = W * CPC;
     constexpr int KC = (NCH + 63) / 64;
@@ -109,7 +115,7 @@ __device__ __forceinline__ void gram_pair_body(const GramArgs& a, double* smg, d
         nxt += stage_d; if (nxt == rend) nxt = ring;
     }
     ptx::cp_async_wait<0>();
-    if (blockIdx.x == 0 && pair == 0 && T * GR_TW < a.n) {         // ragged tail rows [T*32, n)
+    if (blockIdx.x == 0 && pair == 0 && T * GR_TW < a.n) {         // ragged tail rows [T*64, n)
         pair_sync(pair);
         double* sl = ring;                                         // ring idle: stage the tail
         const int64_t r0 = T * GR_TW;
@@ -135,6 +141,8 @@ __global__ void __launch_bounds__(GR_NT, 1) k_gram_ring(GramArgs a) {
     constexpr int NE = W * (W + 1) / 2;
     __shared__ double red[GR_NP * NE];                             // per-pair sums (not aliased)
     const int wp = threadIdx.x >> 5, pair = wp >> 1, h = wp & 1;
+    pdl_wait();
+    pdl_trigger();
     if (h == 0) gram_pair_body<W, 0>(a, smg, red, pair, 0);
     else gram_pair_body<W, 1>(a, smg, red, pair, 1);
     __syncthreads();
@@ -166,7 +174,7 @@ int gram_dfma(const Dev& d, const GramArgs& a, cudaStream_t st) {
         smem = smem < need ? need : smem;
         cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
         ++g_launches;
-        kfn<<<unsigned(d.sms), GR_NT, smem, st>>>(a);
+        launch_pdl(kfn, dim3(unsigned(d.sms)), dim3(GR_NT), smem, st, a);
     };
     switch (a.w) {
         case 1: go(k_gram_ring<1>, gram_stages<1>()); break;

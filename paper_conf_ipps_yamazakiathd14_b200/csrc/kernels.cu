@@ -23,6 +23,7 @@ namespace kern {
 constexpr int NT = 256;
 constexpr int SPMV_BATCH = 4;           // entries whose loads are issued together
 long long g_launches = 0;
+int g_pdl = 1;
 
 // ------------------------------------------------------------------------------------
 // K1: y = A x + bu*u + bw*w on the first nrows rows of a SELL-32 matrix.
@@ -161,13 +162,16 @@ __global__ void __launch_bounds__(NT, MINB) k_spmv_sell32_persist(int64_t nrows,
     const int64_t nsl = (nrows + 31) >> 5;
     const int64_t stride = int64_t(gridDim.x) * (NT / 32);
     int64_t sl = (int64_t(blockIdx.x) * NT + threadIdx.x) >> 5;
-    if (sl >= nsl) return;
+    if (sl >= nsl) { pdl_wait(); pdl_trigger(); return; }
     // descriptors: current slice (b0, W0, i0, o0), next (b1, W1, i1, o1), after next (b2, W2, i2)
+    // (the matrix is never written during a solve: loaded before the PDL wait)
     int64_t b0, i0, b1 = 0, i1 = 1, b2, i2;
     int W0, W1 = 0, W2, o0, o1;
     sell_slice_meta(sl, sptr, sinfo, b0, W0, i0);
     if (sl + stride < nsl) sell_slice_meta(sl + stride, sptr, sinfo, b1, W1, i1);
     o0 = sell_slice_off(lane, W0, i0, dcol);
+    pdl_wait();
+    pdl_trigger();
 #pragma unroll 1
     for (; sl < nsl; sl += stride) {
         b2 = 0; W2 = 0; i2 = 1;
@@ -203,8 +207,8 @@ static void launch_persist(const Dev& d, const Sell& A, int64_t nrows, const dou
     int64_t g = int64_t(d.sms) * occ;
     const int64_t need = (nsl + NT / 32 - 1) / (NT / 32);
     if (g > need) g = need;
-    k_spmv_sell32_persist<MODE, PB, MINB><<<unsigned(g), NT, 0, st>>>(nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val,
-                                                                 x, u, bu, w, bw, y);
+    launch_pdl(k_spmv_sell32_persist<MODE, PB, MINB>, dim3(unsigned(g)), dim3(NT), 0, st, nrows, A.sptr, A.sinfo,
+               A.dcol, A.ncols, A.val, x, u, bu, w, bw, y);
 }
 
 void spmv(const Dev& d, const Sell& A, int64_t nrows, const double* x, double* y,
@@ -283,11 +287,13 @@ void residual(const Dev& d, const Sell& A, int64_t nrows, const double* x, const
 // ------------------------------------------------------------------------------------
 __global__ void k_chol(const double* G, int w, double* R, int* status) {
     __shared__ double sm[32 * 32];
+    pdl_wait();
+    pdl_trigger();
     chol_upper_warp(G, w, w, R, status, sm);
 }
 
 void chol(const double* G, int w, double* R, int* status, cudaStream_t st) {
-    ++g_launches; k_chol<<<1, 32, 0, st>>>(G, w, R, status);
+    ++g_launches; launch_pdl(k_chol, dim3(1), dim3(32), 0, st, G, w, R, status);
 }
 
 // SVQR (reading G14): D = diag(G)^{-1/2}; D G D = U S U^T (cyclic

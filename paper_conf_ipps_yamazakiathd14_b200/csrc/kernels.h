@@ -8,12 +8,38 @@ namespace kern {
 // Process-wide count of kernel launches issued by this library (bench.py gpu_launches).
 extern long long g_launches;
 
+// Programmatic dependent launch (PDL, sm_90+): the hot kernels are launched with
+// programmaticStreamSerializationAllowed, so their CTAs are scheduled while the previous
+// kernel in the stream drains (its tail / last-CTA reduction); each such kernel executes
+// pdl_wait() (griddepcontrol.wait: the previous grid has completed and its memory is
+// visible) before it touches any data a predecessor writes, then pdl_trigger().
+// Process-wide switch (CAGMRES_OPT_PDL); 1 by default.
+extern int g_pdl;
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+template <typename... KArgs, typename... Args>
+inline void launch_pdl(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = g_pdl ? 1 : 0;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...);
+}
+
 // Device properties used for grid sizing (filled once per handle).
 struct Dev {
     int sms = 148;
     int device = 0;
     int gram = 1;               // CholQR Gram kernel: 0 = FP64 tensor core (DMMA), 1 = scalar DFMA ring
     int arnoldi_ring = 1;       // first-cycle / GMRES Arnoldi passes: 1 = cp.async ring kernels
+    int trsm_scalar = 1;        // CholQR/SVQR update: 1 = scalar DFMA ring (w <= 16), 0 = DMMA
+    int panel_tw16 = 1;         // panel ring kernels: 16-row tiles when >= 24 columns are streamed
 };
 
 // Sliced ELLPACK, slice height 32 (one warp), column-major inside a slice, with per-slice
@@ -255,6 +281,14 @@ void svqr_factor(const double* G, int w, double* R, int* status, cudaStream_t st
 // P[:, 0:w] -= X C  (C: jx x w, ld jx)      (BOrth pass 2)
 void update(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, double* P,
             int64_t ldp, int w, const double* C, cudaStream_t st);
+// P[:, c0:w] = (X M)[:, c0:w]  (X: n x K, ld ldx, contiguous columns that contain P; M: K x w,
+// ld ldm; P written in place)  — one-pass BOrth+CholQR update.  -1 if K > 64 or w > 32.
+int gemm_rows(const Dev& d, int64_t n, const double* X, int64_t ldx, int K, double* P, int64_t ldp, int w,
+              const double* M, int64_t ldm, int c0, cudaStream_t st);
+// one-pass BOrth+CholQR small step (onepass.cu): from Mx = [Q P]^T P ((j+w) x w, ld j+w) write
+// C (j x (w-1), ld j), R = chol(Mx[j:, :] - Cf^T Cf) (ld w), Mo = [-Cf R^{-1}; R^{-1}] (ld j+w).
+void onepass_finalize(const double* Mx, int j, int w, double* C, double* R, double* Mo, int* status,
+                      cudaStream_t st);
 // P[:, c0:w] = (P R^{-1})[:, c0:w]   (R upper w x w, ld w)
 void trsm(const Dev& d, int64_t n, double* P, int64_t ldp, int w, const double* R, int c0,
           cudaStream_t st);

@@ -83,6 +83,7 @@ struct cagmres {
     double* gbuf = nullptr;                // Gram / small scratch
     double* ybuf = nullptr;                // LS solution (m)
     double* caqr_ws = nullptr;             // CAQR tree workspace (lazy)
+    double* op_M = nullptr;                // one-pass BOrth+CholQR: [-C R^{-1}; R^{-1}] (64 x 32)
     // pinned host mirrors + events of the per-cycle host <-> device exchange
     double* h_tab = nullptr;
     double* h_y = nullptr;
@@ -123,7 +124,7 @@ struct cagmres {
         cudaFree(d_done);
         for (int2* p : d_pairs) cudaFree(p);
         cudaFree(A.sptr); cudaFree(A.sinfo); cudaFree(A.dcol); cudaFree(A.val);
-        cudaFree(V); cudaFree(xe); cudaFree(tab); cudaFree(gbuf); cudaFree(ybuf); cudaFree(caqr_ws);
+        cudaFree(V); cudaFree(xe); cudaFree(tab); cudaFree(gbuf); cudaFree(ybuf); cudaFree(caqr_ws); cudaFree(op_M);
         cudaFreeHost(h_tab); cudaFreeHost(h_y); cudaFreeHost(h_beta); cudaFreeHost(h_stat);
         if (ev_tab) cudaEventDestroy(ev_tab);
         if (ev_beta) cudaEventDestroy(ev_beta);
@@ -280,6 +281,7 @@ int common_alloc(cagmres* h) {
     CU(cudaMemset(h->tab, 0, sizeof(double) * h->tab_cap));
     CU(cudaMalloc(&h->gbuf, sizeof(double) * size_t(h->m + 2) * size_t(std::max(h->m, 32) + 2)));
     CU(cudaMalloc(&h->ybuf, sizeof(double) * size_t(h->m + 2)));
+    CU(cudaMalloc(&h->op_M, sizeof(double) * 64 * 32));
     CU(cudaMallocHost(&h->h_tab, sizeof(double) * h->tab_cap));
     CU(cudaMallocHost(&h->h_y, sizeof(double) * size_t(h->m + 2)));
     CU(cudaMallocHost(&h->h_beta, sizeof(double) * 2));
@@ -409,6 +411,7 @@ int init_common(cagmres* h, const cagmres_csr* A, const int64_t* row_starts, int
         return CAGMRES_EINVAL;
     const int kind = orth & CAGMRES_TSQR_MASK;
     if (kind > CAGMRES_CAQR) return CAGMRES_EINVAL;
+    if ((orth & CAGMRES_ONEPASS) && (kind != CAGMRES_CHOLQR || (orth & CAGMRES_BORTH_MGS))) return CAGMRES_EINVAL;
     if (kind == CAGMRES_CAQR && h->nranks > 1) return CAGMRES_ENOTSUP;   // single-GPU tree only
     h->s = s; h->m = m; h->basis = basis; h->orth = orth;
     int dv = 0;
@@ -706,6 +709,22 @@ int ca_cycle(cagmres* h, const std::vector<Block>& bl) {
         for (int pass = 0; pass < (re2 ? 2 : 1); ++pass) {
             double* C = h->tab + (pass ? b.c2 : b.c1);
             double* R = h->tab + (pass ? b.r2 : b.r1);
+            if (j > 0 && (h->orth & CAGMRES_ONEPASS) && j + w <= 64) {
+                // one-pass BOrth + CholQR (NEXT-2): [Q P]^T P ; small step ; P := [Q P] M
+                const double nl = double(h->n_loc);
+                {
+                    Scope sc(h, PH_BORTH);
+                    TRY(xty_global(h, h->V, h->ldv, j + w, Pj, h->ldv, w, h->gbuf, false, nullptr));
+                    h->bytes[PH_BORTH] += 8.0 * nl * (j + w);
+                }
+                Scope sc(h, PH_TSQR);
+                kern::onepass_finalize(h->gbuf, j, w, C, R, h->op_M, h->status, h->stream);
+                if (kern::gemm_rows(h->dev, h->n_loc, h->V, h->ldv, j + w, Pj, h->ldv, w, h->op_M, j + w, 1,
+                                    h->stream))
+                    return CAGMRES_EINVAL;
+                h->bytes[PH_TSQR] += 8.0 * nl * (j + w + (w - 1));
+                continue;
+            }
             if (j > 0 && !mgs && kind == CAGMRES_CHOLQR && h->fuse_borth_gram) {
                 // BOrth pass 1, then [P -= Q C  fused with  B = [q_j P]^T [q_j P] (+ chol)]
                 const double nl = double(h->n_loc);
@@ -937,6 +956,9 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
             return CAGMRES_OK;
         case CAGMRES_OPT_GRAM: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->dev.gram = int(value); return CAGMRES_OK;
         case CAGMRES_OPT_ARNOLDI: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->dev.arnoldi_ring = int(value); return CAGMRES_OK;
+        case CAGMRES_OPT_PANEL_TW: if (value != 16 && value != 32) return CAGMRES_EINVAL; h->dev.panel_tw16 = value == 16; return CAGMRES_OK;
+        case CAGMRES_OPT_TRSM: if (value < 0 || value > 4) return CAGMRES_EINVAL; h->dev.trsm_scalar = int(value); return CAGMRES_OK;
+        case CAGMRES_OPT_PDL: if (value < 0 || value > 1) return CAGMRES_EINVAL; kern::g_pdl = int(value); return CAGMRES_OK;
         case CAGMRES_OPT_FUSE: h->fuse_borth_gram = (value & 1) != 0; h->arnoldi_fuse = (value & 2) != 0; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK:
             if (value < 256 || value % 256) return CAGMRES_EINVAL;
@@ -954,6 +976,9 @@ int cagmres_get_option(cagmres_t h, int opt, int64_t* value) {
         case CAGMRES_OPT_SPMV: *value = h->A.variant; return CAGMRES_OK;
         case CAGMRES_OPT_GRAM: *value = h->dev.gram; return CAGMRES_OK;
         case CAGMRES_OPT_ARNOLDI: *value = h->dev.arnoldi_ring; return CAGMRES_OK;
+        case CAGMRES_OPT_PANEL_TW: *value = h->dev.panel_tw16 ? 16 : 32; return CAGMRES_OK;
+        case CAGMRES_OPT_TRSM: *value = h->dev.trsm_scalar; return CAGMRES_OK;
+        case CAGMRES_OPT_PDL: *value = kern::g_pdl; return CAGMRES_OK;
         case CAGMRES_OPT_FUSE: *value = (h->fuse_borth_gram ? 1 : 0) | (h->arnoldi_fuse ? 2 : 0); return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK: *value = h->wave_CH; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CTAS: *value = h->wave_ctas; return CAGMRES_OK;

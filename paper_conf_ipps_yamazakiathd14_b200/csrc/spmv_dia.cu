@@ -41,12 +41,15 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
     const int64_t nsl = (a.nrows + 31) >> 5;
     const int64_t stride = int64_t(gridDim.x) * (DT_NT / 32);
     int64_t sl = (int64_t(blockIdx.x) * DT_NT + threadIdx.x) >> 5;
-    if (sl >= nsl) return;
+    if (sl >= nsl) { pdl_wait(); pdl_trigger(); return; }
     int64_t b0, i0, b1 = 0, i1 = 1, b2, i2;
     int W0, W1 = 0, W2, o0, o1;
+    // slice descriptors (static during a solve) are loaded before the PDL wait
     sell_slice_meta(sl, a.sptr, a.sinfo, b0, W0, i0);
     if (sl + stride < nsl) sell_slice_meta(sl + stride, a.sptr, a.sinfo, b1, W1, i1);
     o0 = sell_slice_off(lane, W0, i0, a.dcol);
+    pdl_wait();
+    pdl_trigger();
 #pragma unroll 1
     for (; sl < nsl; sl += stride) {
         b2 = 0; W2 = 0; i2 = 1;
@@ -102,7 +105,7 @@ void go_dia(const Dev& d, const DiaArgs& a, cudaStream_t st) {
     int64_t g = int64_t(d.sms) * occ;
     const int64_t need = (nsl + DT_NT / 32 - 1) / (DT_NT / 32);
     if (g > need) g = need;
-    k_spmv_dia<MODE, WT, MINB><<<unsigned(g), DT_NT, 0, st>>>(a);
+    launch_pdl(k_spmv_dia<MODE, WT, MINB>, dim3(unsigned(g)), dim3(DT_NT), 0, st, a);
 }
 
 template <int WT, int MINB>

@@ -1,6 +1,8 @@
 // stream.cu — row-streaming panel kernels on the FP64 tensor core (sm_100a DMMA).
 //   K9  update : P[:, 0:w] -= X C                 (BOrth pass 2; x += V y)
 //   K8  trsm   : P[:, c0:w] = (P R^{-1})[:, c0:w] (CholQR/SVQR update)
+//       gemm   : P[:, c0:w] = (X M)[:, c0:w], X = [Q | P] contiguous (one-pass BOrth+CholQR
+//                update (P - Q C) R^{-1} = [Q P] [-C R^{-1}; R^{-1}])
 // Each warp forms 8-row x w output tiles with mma.sync.m8n8k4.f64 against the small
 // right-hand matrix (C, or R^{-1}), whose B-fragments live in registers for the whole
 // kernel.  A fragments (8 rows x 4 columns) and the P tile are loaded straight from global
@@ -45,14 +47,15 @@ __device__ __forceinline__ void upper_inverse(const double* R, int w, double* sR
     __syncthreads();
 }
 
-// MODE 0: update (A = X, B = C, D = P - A B); MODE 1: trsm (A = P, B = R^{-1}, D = A B).
+// MODE 0: update (A = X, B = C, D = P - A B); MODE 1: trsm (A = P, B = R^{-1}, D = A B);
+// MODE 2: gemm (A = X with jx = K columns that include P, B = M, D = A B).
 template <int MODE, int KTM, int NTN, int U>
 __global__ void __launch_bounds__(NT) k_rows_mma(StreamArgs a) {
     __shared__ double sB[32 * 32 + 32];
     const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5;
     const int gid = lane >> 2, tig = lane & 3;
     const int w = a.w;
-    const int K = MODE == 0 ? a.jx : w;
+    const int K = MODE == 1 ? w : a.jx;
     if (MODE == 1) upper_inverse(a.M, w, sB, sB + 32 * 32);   // (ldm == w for R)
     // B fragments: b[kt][nt] = B[4kt + tig][8nt + gid]
     double b[KTM][NTN];
@@ -62,13 +65,13 @@ __global__ void __launch_bounds__(NT) k_rows_mma(StreamArgs a) {
         for (int nt = 0; nt < NTN; ++nt) {
             const int k = 4 * kt + tig, c = 8 * nt + gid;
             double v = 0.0;
-            if (k < K && c < w) v = MODE == 0 ? a.M[k + a.ldm * c] : sB[k * 32 + c];
+            if (k < K && c < w) v = MODE != 1 ? a.M[k + a.ldm * c] : sB[k * 32 + c];
             b[kt][nt] = v;
         }
     // per-lane column pointers (clamped: the matching B rows / stored columns are masked)
     const double* acol[KTM];
-    const double* Abase = MODE == 0 ? a.X : a.P;
-    const int64_t ldA = MODE == 0 ? a.ldx : a.ldp;
+    const double* Abase = MODE != 1 ? a.X : a.P;
+    const int64_t ldA = MODE != 1 ? a.ldx : a.ldp;
 #pragma unroll
     for (int kt = 0; kt < KTM; ++kt) acol[kt] = Abase + ldA * min(4 * kt + tig, K - 1);
     double* pcol[NTN][2];
@@ -85,6 +88,8 @@ __global__ void __launch_bounds__(NT) k_rows_mma(StreamArgs a) {
             wcol[nt][h] = c < w && (MODE == 0 || c >= a.c0);
         }
     const int KT = (K + 3) / 4;
+    // MODE 2 writes P in place: every output row depends only on the same row of X (which
+    // holds P), loaded by the same warp before it stores — rows are private to a warp.
 
     const int64_t ngroups = (a.n + 7) / 8;
     const int64_t nsg = (ngroups + U - 1) / U;
@@ -136,10 +141,12 @@ __global__ void __launch_bounds__(512, 1) k_rows_pipe(StreamArgs a) {
     extern __shared__ __align__(16) double smp[];
     constexpr int SP = TW + 8;
     __shared__ double sB[32 * 32 + 32];
+    pdl_wait();
+    pdl_trigger();
     const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const int gid = lane >> 2, tig = lane & 3;
     const int w = a.w;
-    const int K = MODE == 0 ? a.jx : w;
+    const int K = MODE == 1 ? w : a.jx;
     if (MODE == 1) upper_inverse(a.M, w, sB, sB + 32 * 32);
     double b[KTM][NTN];
 #pragma unroll
@@ -148,11 +155,11 @@ __global__ void __launch_bounds__(512, 1) k_rows_pipe(StreamArgs a) {
         for (int nt = 0; nt < NTN; ++nt) {
             const int k = 4 * kt + tig, c = 8 * nt + gid;
             double v = 0.0;
-            if (k < K && c < w) v = MODE == 0 ? a.M[k + a.ldm * c] : sB[k * 32 + c];
+            if (k < K && c < w) v = MODE != 1 ? a.M[k + a.ldm * c] : sB[k * 32 + c];
             b[kt][nt] = v;
         }
-    const int jxl = MODE == 0 ? a.jx : 0;
-    const int ncol = jxl + w;
+    const int jxl = MODE != 1 ? a.jx : 0;
+    const int ncol = MODE == 2 ? a.jx : jxl + w;               // gemm: P is inside X
     const int64_t stage_d = int64_t(ncol) * SP;
     double* ring = smp + int64_t(wp) * RP_S * stage_d;
     const int64_t T = a.n / TW;
@@ -175,7 +182,7 @@ __global__ void __launch_bounds__(512, 1) k_rows_pipe(StreamArgs a) {
     const int KT = (K + 3) / 4;
     int acol[KTM];
 #pragma unroll
-    for (int kt = 0; kt < KTM; ++kt) acol[kt] = (MODE == 0 ? 0 : jxl) + min(4 * kt + tig, K - 1);
+    for (int kt = 0; kt < KTM; ++kt) acol[kt] = (MODE == 1 ? jxl : 0) + min(4 * kt + tig, K - 1);
     int pcol[NTN][2];
     bool wcol[NTN][2];
 #pragma unroll
@@ -235,7 +242,7 @@ __global__ void __launch_bounds__(512, 1) k_rows_pipe(StreamArgs a) {
 #pragma unroll
             for (int kt = 0; kt < KTM; ++kt) {
                 if (kt < KT) {
-                    const double* src = acol[kt] < jxl ? a.X + a.ldx * acol[kt] : a.P + a.ldp * (acol[kt] - jxl);
+                    const double* src = (MODE == 2 || acol[kt] < jxl) ? a.X + a.ldx * acol[kt] : a.P + a.ldp * (acol[kt] - jxl);
                     const double av = ok ? src[row] : 0.0;
                     const double am = MODE == 0 ? -av : av;
 #pragma unroll
@@ -253,21 +260,30 @@ __global__ void __launch_bounds__(512, 1) k_rows_pipe(StreamArgs a) {
     }
 }
 
-template <int MODE, int KTM, int NTN>
-bool run_pipe(const Dev& d, const StreamArgs& a, cudaStream_t st) {
-    constexpr int TW = 32;
-    const bool aligned = ((reinterpret_cast<uintptr_t>(a.P) | reinterpret_cast<uintptr_t>(MODE == 0 ? a.X : a.P)) % 16 == 0) &&
+template <int MODE, int KTM, int NTN, int TW>
+bool run_pipe_tw(const Dev& d, const StreamArgs& a, cudaStream_t st) {
+    const bool aligned = ((reinterpret_cast<uintptr_t>(a.P) | reinterpret_cast<uintptr_t>(MODE != 1 ? a.X : a.P)) % 16 == 0) &&
                          (a.ldp % 2 == 0) && (MODE == 1 || a.ldx % 2 == 0);
     if (!aligned || a.n < 64 * TW) return false;
-    const int ncol = (MODE == 0 ? a.jx : 0) + a.w;
+    const int ncol = MODE == 2 ? a.jx : (MODE == 0 ? a.jx : 0) + a.w;
     const size_t ring_w = size_t(RP_S) * ncol * (TW + 8) * sizeof(double);
     int nw = int((200 * 1024) / ring_w);
     nw = nw < 2 ? 2 : (nw > 16 ? 16 : nw);
     const size_t smem = size_t(nw) * ring_w;
     cudaFuncSetAttribute(k_rows_pipe<MODE, KTM, NTN, TW>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
     ++g_launches;
-    k_rows_pipe<MODE, KTM, NTN, TW><<<unsigned(d.sms), 32 * nw, smem, st>>>(a);
+    launch_pdl(k_rows_pipe<MODE, KTM, NTN, TW>, dim3(unsigned(d.sms)), dim3(32 * nw), smem, st, a);
     return true;
+}
+
+// wide panels: 16-row tiles, about twice the warps per SM
+template <int MODE, int KTM, int NTN>
+bool run_pipe(const Dev& d, const StreamArgs& a, cudaStream_t st) {
+    // measured (profiles/r1_launches_C2_tw*.txt): 16-row tiles win for wide light-compute
+    // panels (x += V y, w = 1) and the one-pass gemm, lose for the BOrth update (w = 10)
+    const int ncol = MODE == 2 ? a.jx : (MODE == 0 ? a.jx : 0) + a.w;
+    if (d.panel_tw16 && ncol >= 24 && (MODE == 2 || a.w <= 8)) return run_pipe_tw<MODE, KTM, NTN, 16>(d, a, st);
+    return run_pipe_tw<MODE, KTM, NTN, 32>(d, a, st);
 }
 
 template <int MODE, int KTM, int NTN, int U>
@@ -287,7 +303,7 @@ void run(const Dev& d, const StreamArgs& a, cudaStream_t st) {
 
 template <int MODE>
 int dispatch(const Dev& d, const StreamArgs& a, cudaStream_t st) {
-    const int w = a.w, K = MODE == 0 ? a.jx : w;
+    const int w = a.w, K = MODE == 1 ? w : a.jx;
     const int ntn = w <= 8 ? 1 : (w <= 16 ? 2 : 4);
     const int ktm = K <= 4 ? 1 : (K <= 8 ? 2 : (K <= 16 ? 4 : (K <= 32 ? 8 : (K <= 64 ? 16 : 0))));
     switch (ktm * 10 + ntn) {
@@ -314,6 +330,8 @@ int dispatch(const Dev& d, const StreamArgs& a, cudaStream_t st) {
 // vectorised stream (16-B loads/stores, grid = SMs x 4).  The product p * (1/r) is rounded once,
 // exactly like the DMMA path (fma(p, 1/r, 0)), so results are bitwise identical.
 __global__ void __launch_bounds__(256) k_scale1(int64_t n, double* __restrict__ p, const double* __restrict__ r) {
+    pdl_wait();
+    pdl_trigger();
     const double inv = 1.0 / __ldg(r);
     const int64_t i0 = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
     const int64_t stride = int64_t(gridDim.x) * blockDim.x;
@@ -331,6 +349,122 @@ __global__ void __launch_bounds__(256) k_scale1(int64_t n, double* __restrict__ 
         for (int64_t i = i0; i < n; i += stride) p[i] *= inv;
     }
 }
+// Scalar-FP64 TRSM on a per-warp cp.async ring (CAGMRES_OPT_TRSM = 1, default for w <= 16).
+// The DMMA form pads the w x w triangular R^{-1} to 16 x 16 tiles (34 % useful MACs at w = 11)
+// and was tensor-pipe co-limited (ncu: 67 us, 4.4 TB/s at n = 2.1M, w = 11); here lane l owns
+// row l of a 32-row tile, reads its W panel values from the ring once and forms
+// out[c] = sum_{k <= c} p[k] Ri[k][c] for c >= c0 with R^{-1} broadcast from shared memory:
+// w(w+1)/2 DFMAs per row, no padding.
+template <int W, int RS>
+__global__ void __launch_bounds__(512, 1) k_trsm_ring(StreamArgs a) {
+    extern __shared__ __align__(16) double smt[];
+    __shared__ double sB[32 * 32 + 32];
+    __shared__ double sRi[W * W];
+    const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    pdl_wait();
+    pdl_trigger();
+    upper_inverse(a.M, W, sB, sB + 32 * 32);
+    for (int q = threadIdx.x; q < W * W; q += blockDim.x) sRi[q] = sB[(q / W) * 32 + (q % W)];   // [k*W + c]
+    __syncthreads();
+    constexpr int SD = W * 32;
+    double* ring = smt + int64_t(wp) * RS * SD;
+    const int64_t T = a.n / 32;
+    const int64_t Wn = int64_t(gridDim.x) * nw;
+    const int64_t g = int64_t(blockIdx.x) * nw + wp;
+    const int64_t t0 = g * T / Wn, t1 = (g + 1) * T / Wn;
+    const int c0 = a.c0;
+    auto issue = [&](int64_t t, int stage) {
+        if (t < t1) {
+            double* dst = ring + stage * SD;
+            const int64_t r0 = t * 32;
+            for (int q = lane; q < W * 16; q += 32) {
+                const int c = q >> 4, part = q & 15;
+                ptx::cp_async16(dst + c * 32 + part * 2, a.P + a.ldp * c + r0 + part * 2);
+            }
+        }
+        ptx::cp_async_commit();
+    };
+    auto rowout = [&](const double (&v)[W], double* out) {
+#pragma unroll
+        for (int c = 0; c < W; ++c) {
+            if (c < c0) continue;
+            double acc = 0.0;
+#pragma unroll
+            for (int k = 0; k <= c; ++k) acc = fma(v[k], sRi[k * W + c], acc);
+            out[a.ldp * c] = acc;
+        }
+    };
+#pragma unroll
+    for (int s = 0; s < RS - 1; ++s) issue(t0 + s, s);
+    int stage = 0;
+    for (int64_t t = t0; t < t1; ++t) {
+        issue(t + RS - 1, stage == 0 ? RS - 1 : stage - 1);
+        ptx::cp_async_wait<RS - 1>();
+        __syncwarp();
+        const double* sl = ring + stage * SD + lane;
+        double v[W];
+#pragma unroll
+        for (int k = 0; k < W; ++k) v[k] = sl[k * 32];
+        rowout(v, a.P + t * 32 + lane);
+        __syncwarp();
+        stage = stage == RS - 1 ? 0 : stage + 1;
+    }
+    ptx::cp_async_wait<0>();
+    if (blockIdx.x == 0 && wp == 0) {                          // ragged tail rows [32 T, n)
+        const int64_t r = T * 32 + lane;
+        if (r < a.n) {
+            double v[W];
+#pragma unroll
+            for (int k = 0; k < W; ++k) v[k] = a.P[a.ldp * k + r];
+            rowout(v, a.P + r);
+        }
+    }
+}
+
+template <int W, int RS>
+bool go_trsm_rs(const Dev& d, const StreamArgs& a, cudaStream_t st) {
+    const size_t ring_w = size_t(RS) * W * 32 * sizeof(double);
+    int nw = int((200 * 1024) / ring_w);
+    nw = nw < 2 ? 2 : (nw > 16 ? 16 : nw);
+    const size_t smem = size_t(nw) * ring_w;
+    cudaFuncSetAttribute(k_trsm_ring<W, RS>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    ++g_launches;
+    launch_pdl(k_trsm_ring<W, RS>, dim3(unsigned(d.sms)), dim3(32 * nw), smem, st, a);
+    return true;
+}
+
+template <int W>
+bool go_trsm_ring(const Dev& d, const StreamArgs& a, cudaStream_t st) {
+    const bool aligned = (reinterpret_cast<uintptr_t>(a.P) % 16 == 0) && (a.ldp % 2 == 0);
+    if (!aligned || a.n < 64 * 32) return false;
+    switch (d.trsm_scalar) {             // ring stages (CAGMRES_OPT_TRSM 1..4 -> 3, 4, 6, 8)
+        case 2: return go_trsm_rs<W, 4>(d, a, st);
+        case 3: return go_trsm_rs<W, 6>(d, a, st);
+        case 4: return go_trsm_rs<W, 8>(d, a, st);
+        default: return go_trsm_rs<W, 3>(d, a, st);
+    }
+}
+
+bool trsm_ring(const Dev& d, const StreamArgs& a, cudaStream_t st) {
+    switch (a.w) {
+        case 2: return go_trsm_ring<2>(d, a, st);
+        case 3: return go_trsm_ring<3>(d, a, st);
+        case 4: return go_trsm_ring<4>(d, a, st);
+        case 5: return go_trsm_ring<5>(d, a, st);
+        case 6: return go_trsm_ring<6>(d, a, st);
+        case 7: return go_trsm_ring<7>(d, a, st);
+        case 8: return go_trsm_ring<8>(d, a, st);
+        case 9: return go_trsm_ring<9>(d, a, st);
+        case 10: return go_trsm_ring<10>(d, a, st);
+        case 11: return go_trsm_ring<11>(d, a, st);
+        case 12: return go_trsm_ring<12>(d, a, st);
+        case 13: return go_trsm_ring<13>(d, a, st);
+        case 14: return go_trsm_ring<14>(d, a, st);
+        case 15: return go_trsm_ring<15>(d, a, st);
+        case 16: return go_trsm_ring<16>(d, a, st);
+        default: return false;
+    }
+}
 }  // namespace
 
 void update(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, double* P,
@@ -344,6 +478,14 @@ void update(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, doubl
     }
 }
 
+int gemm_rows(const Dev& d, int64_t n, const double* X, int64_t ldx, int K, double* P, int64_t ldp, int w,
+              const double* M, int64_t ldm, int c0, cudaStream_t st) {
+    if (n <= 0 || w <= 0) return 0;
+    if (K > 64 || w > 32) return -1;
+    StreamArgs a{n, X, ldx, K, P, ldp, w, M, ldm, c0};
+    return dispatch<2>(d, a, st);
+}
+
 void trsm(const Dev& d, int64_t n, double* P, int64_t ldp, int w, const double* R, int c0,
           cudaStream_t st) {
     if (n <= 0 || w <= 0) return;
@@ -352,10 +494,11 @@ void trsm(const Dev& d, int64_t n, double* P, int64_t ldp, int w, const double* 
         const int64_t need = ((n >> 1) + 255) / 256;
         if (g > need) g = need < 1 ? 1 : need;
         ++g_launches;
-        k_scale1<<<unsigned(g), 256, 0, st>>>(n, P, R);
+        launch_pdl(k_scale1, dim3(unsigned(g)), dim3(256), 0, st, n, P, R);
         return;
     }
     StreamArgs a{n, nullptr, 0, 0, P, ldp, w, R, w, c0};
+    if (d.trsm_scalar && trsm_ring(d, a, st)) return;
     dispatch<1>(d, a, st);
 }
 

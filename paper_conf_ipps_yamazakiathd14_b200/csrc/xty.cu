@@ -168,6 +168,8 @@ constexpr int PIPE_S = 3;
 template <int MT, int NTN, bool SYM, int TW>
 __global__ void __launch_bounds__(NT, 1) k_xty_pipe(XtyArgs a) {
     extern __shared__ __align__(16) double smp[];
+    pdl_wait();
+    pdl_trigger();
     constexpr int SP = TW + 4;
     const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const int gid = lane >> 2, tig = lane & 3;
@@ -350,7 +352,40 @@ template <typename K>
 void launch_pipe(K kfn, const Geo& o, int nw, size_t smem, const XtyArgs& a, cudaStream_t st) {
     cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
     ++g_launches;
-    kfn<<<dim3(o.gx, o.gy), 32 * nw, smem, st>>>(a);
+    launch_pdl(kfn, dim3(o.gx, o.gy), dim3(32 * nw), smem, st, a);
+}
+
+template <int TW>
+int xty_pipe_launch(const Dev& d, Geo o, const XtyArgs& a, int ncol, const XtyWs& ws, cudaStream_t st) {
+    const size_t ring_w = size_t(PIPE_S) * ncol * (TW + 4) * sizeof(double);
+    int nw = int((200 * 1024) / ring_w);
+    nw = nw < 2 ? 2 : (nw > 16 ? 16 : nw);
+    size_t smem = size_t(nw) * ring_w;
+    const size_t red = size_t(nw) * o.MT * o.NTN * 64 * sizeof(double);
+    if (smem < red) smem = red;
+    if (smem < size_t(32 * nw) * sizeof(double)) smem = size_t(32 * nw) * sizeof(double);
+    o.gx = std::max(1, d.sms / o.gy);
+    if (size_t(o.gx) * o.gy * o.chunk * a.w * 2 > ws.cap) return -1;
+    if (o.sym) {
+        if (o.NTN == 1) launch_pipe(k_xty_pipe<1, 1, true, TW>, o, nw, smem, a, st);
+        else if (o.NTN == 2) launch_pipe(k_xty_pipe<2, 2, true, TW>, o, nw, smem, a, st);
+        else launch_pipe(k_xty_pipe<4, 4, true, TW>, o, nw, smem, a, st);
+        return 0;
+    }
+    switch (o.MT * 10 + o.NTN) {
+        case 11: launch_pipe(k_xty_pipe<1, 1, false, TW>, o, nw, smem, a, st); break;
+        case 21: launch_pipe(k_xty_pipe<2, 1, false, TW>, o, nw, smem, a, st); break;
+        case 41: launch_pipe(k_xty_pipe<4, 1, false, TW>, o, nw, smem, a, st); break;
+        case 81: launch_pipe(k_xty_pipe<8, 1, false, TW>, o, nw, smem, a, st); break;
+        case 12: launch_pipe(k_xty_pipe<1, 2, false, TW>, o, nw, smem, a, st); break;
+        case 22: launch_pipe(k_xty_pipe<2, 2, false, TW>, o, nw, smem, a, st); break;
+        case 42: launch_pipe(k_xty_pipe<4, 2, false, TW>, o, nw, smem, a, st); break;
+        case 82: launch_pipe(k_xty_pipe<8, 2, false, TW>, o, nw, smem, a, st); break;
+        case 14: launch_pipe(k_xty_pipe<1, 4, false, TW>, o, nw, smem, a, st); break;
+        case 24: launch_pipe(k_xty_pipe<2, 4, false, TW>, o, nw, smem, a, st); break;
+        default: launch_pipe(k_xty_pipe<4, 4, false, TW>, o, nw, smem, a, st); break;
+    }
+    return 0;
 }
 
 int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const double* Y,
@@ -368,38 +403,11 @@ int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const dou
     const bool aligned = ((reinterpret_cast<uintptr_t>(X) | reinterpret_cast<uintptr_t>(Y)) % 16 == 0) &&
                          (ldx % 2 == 0) && (ldy % 2 == 0);
     if (aligned && n >= 32 * 64) {
-        // per-warp cp.async pipeline: size the warps so the rings use ~200 KB of smem
-        constexpr int TW = 32;
+        // per-warp cp.async pipeline: size the warps so the rings use ~200 KB of smem; very
+        // wide panels (>= 36 streamed columns, < 6 warps at 32 rows) use 16-row tiles
         const int ncol = w + ((o.sym || X == Y) ? 0 : std::min(o.chunk, jx));
-        const size_t ring_w = size_t(PIPE_S) * ncol * (TW + 4) * sizeof(double);
-        int nw = int((200 * 1024) / ring_w);
-        nw = nw < 2 ? 2 : (nw > 16 ? 16 : nw);
-        size_t smem = size_t(nw) * ring_w;
-        const size_t red = size_t(nw) * o.MT * o.NTN * 64 * sizeof(double);
-        if (smem < red) smem = red;
-        if (smem < size_t(32 * nw) * sizeof(double)) smem = size_t(32 * nw) * sizeof(double);
-        o.gx = std::max(1, d.sms / o.gy);
-        if (size_t(o.gx) * o.gy * o.chunk * w * 2 > ws.cap) return -1;
-        if (o.sym) {
-            if (o.NTN == 1) launch_pipe(k_xty_pipe<1, 1, true, TW>, o, nw, smem, a, st);
-            else if (o.NTN == 2) launch_pipe(k_xty_pipe<2, 2, true, TW>, o, nw, smem, a, st);
-            else launch_pipe(k_xty_pipe<4, 4, true, TW>, o, nw, smem, a, st);
-            return 0;
-        }
-        switch (o.MT * 10 + o.NTN) {
-            case 11: launch_pipe(k_xty_pipe<1, 1, false, TW>, o, nw, smem, a, st); break;
-            case 21: launch_pipe(k_xty_pipe<2, 1, false, TW>, o, nw, smem, a, st); break;
-            case 41: launch_pipe(k_xty_pipe<4, 1, false, TW>, o, nw, smem, a, st); break;
-            case 81: launch_pipe(k_xty_pipe<8, 1, false, TW>, o, nw, smem, a, st); break;
-            case 12: launch_pipe(k_xty_pipe<1, 2, false, TW>, o, nw, smem, a, st); break;
-            case 22: launch_pipe(k_xty_pipe<2, 2, false, TW>, o, nw, smem, a, st); break;
-            case 42: launch_pipe(k_xty_pipe<4, 2, false, TW>, o, nw, smem, a, st); break;
-            case 82: launch_pipe(k_xty_pipe<8, 2, false, TW>, o, nw, smem, a, st); break;
-            case 14: launch_pipe(k_xty_pipe<1, 4, false, TW>, o, nw, smem, a, st); break;
-            case 24: launch_pipe(k_xty_pipe<2, 4, false, TW>, o, nw, smem, a, st); break;
-            default: launch_pipe(k_xty_pipe<4, 4, false, TW>, o, nw, smem, a, st); break;
-        }
-        return 0;
+        if (d.panel_tw16 && ncol >= 36) return xty_pipe_launch<16>(d, o, a, ncol, ws, st);
+        return xty_pipe_launch<32>(d, o, a, ncol, ws, st);
     }
     if (o.sym) {
         if (o.NTN == 1) launch(k_xty_mma<1, 1, 16, true>, o, a, st);

@@ -17,10 +17,12 @@ _BASIS = {"monomial": L.MONOMIAL, "newton": L.NEWTON, "gmres": L.GMRES}
 _TSQR = {"cholqr": L.CHOLQR, "svqr": L.SVQR, "cgs": L.CGS, "mgs": L.MGS, "caqr": L.CAQR}
 
 
-def orth_flags(tsqr="cholqr", reorth=False, borth="cgs"):
+def orth_flags(tsqr="cholqr", reorth=False, borth="cgs", onepass=False):
     f = _TSQR[tsqr]
     if reorth:
         f |= L.REORTH
+    if onepass:
+        f |= L.ONEPASS
     if borth == "mgs":
         f |= L.BORTH_MGS
     return f
@@ -59,12 +61,12 @@ class Solver:
     """
 
     def __init__(self, A, s, m, basis="newton", tsqr="cholqr", reorth=False, borth="cgs",
-                 group=None, row_starts=None, device=None):
+                 group=None, row_starts=None, device=None, onepass=False):
         import torch
         self._lib = L.load()
         self.s, self.m = int(s), int(m)
         self.basis = basis
-        self.orth = orth_flags(tsqr, reorth, borth)
+        self.orth = orth_flags(tsqr, reorth, borth, onepass)
         self._h = C.c_void_p()
         if device is None:
             device = torch.cuda.current_device()
@@ -116,7 +118,7 @@ class Solver:
         L.check(self._lib.cagmres_set_stream(self._h, C.c_void_p(s.cuda_stream)), "set_stream")
 
     OPTIONS = {"mpk_wave": 1, "wave_chunk": 3, "wave_ctas": 4, "wave_lag": 5, "fuse": 6, "spmv": 7, "gram": 8,
-               "arnoldi": 9}
+               "arnoldi": 9, "panel_tw": 10, "trsm": 11, "pdl": 12}
 
     def set_option(self, opt, value):
         """opt: "mpk_wave", "wave_chunk", "wave_ctas", "wave_lag", "fuse", "spmv", "gram", "arnoldi" (CAGMRES_OPT_*)."""

@@ -375,3 +375,41 @@ def test_solve_gmres_baseline(gen, reorth, arnoldi):
     assert np.all(np.diff(st.hist) <= 1e-14)                      # restarted GMRES is monotone
     r = b - As @ x.cpu().numpy()
     assert np.linalg.norm(r) <= 1.01e-8 * np.linalg.norm(b)
+
+
+# ----------------------------------------------------------------------------- one-pass BOrth+CholQR
+@pytest.mark.parametrize("s,m,reorth,gen", [(5, 30, False, "C1"), (5, 30, True, "C1"), (10, 30, True, "cd7"),
+                                             (5, 60, False, "g3_small"), (7, 30, True, "cd27_ragged")])
+def test_solve_onepass(s, m, reorth, gen):
+    """CAGMRES_ONEPASS (NEXT-2): per-cycle residuals vs oracle cagmres(onepass=True) with the same
+    injected shifts; rounding envelope of the oracle as in the other solve tests."""
+    A = {"C1": lambda: G.convection_diffusion(32, 2, 5),
+         "cd7": lambda: G.convection_diffusion(40, 3, 7),
+         "g3_small": lambda: G.g3_shaped(n=40000, width=200),
+         "cd27_ragged": lambda: G.convection_diffusion(13, 3, 27)}[gen]()
+    As = A.to_scipy()
+    b = G.rhs(A.n)
+    re, im = O.modified_leja(O.ritz_values(O.arnoldi_cgs2(As, b, m)[1], m), s)
+    S = Solver(A, s=s, m=m, basis="newton", reorth=reorth, onepass=True)
+    S.set_shifts(re, im)
+    x, st = S.solve(dev(b), tol=1e-8, maxit=200)
+    ref, env = rounding_envelope(As, b, nperm=1, s=s, m=m, basis="newton", reorth=reorth, tol=1e-8,
+                                 maxcyc=200, shifts=(re, im), onepass=True)
+    assert st.status == 0 and abs(st.cycles - len(ref)) <= 1
+    assert hist_within_envelope(st.hist, ref, env)
+    r = b - As @ x.cpu().numpy()
+    assert np.linalg.norm(r) <= 1.01e-8 * np.linalg.norm(b)
+
+
+def test_onepass_cycle_basis_matches_two_pass():
+    """One cycle, same shifts: the one-pass basis spans the same space as the two-pass one —
+    residual histories agree to rounding (Pythagoras exact when Q^T Q = I)."""
+    A = G.convection_diffusion(64, 3, 7)
+    b = G.rhs(A.n)
+    out = []
+    for op in (False, True):
+        S = Solver(A, s=10, m=30, basis="newton", reorth=True, onepass=op)
+        S.set_shifts(*SHIFTS)
+        _, st = S.solve(dev(b), tol=0.0, maxit=3)
+        out.append(st.hist)
+    assert np.allclose(out[0], out[1], rtol=1e-8)
