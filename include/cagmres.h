@@ -133,8 +133,9 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
  *                          4..9 = persistent grid, slice descriptors software-pipelined two
  *                          slices ahead, (load batch, CTAs/SM) = (8,3) (4,4) (4,5) (4,6) (2,6)
  *                          (2,8); 10..13 = persistent, fully unrolled body for the matrix's most
- *                          common DIA slice width, >= 3/4/5/6 CTAs per SM.  All variants are
- *                          bitwise identical.
+ *                          common DIA slice width, >= 3/4/5/6 CTAs per SM; 14, 15 = the same with
+ *                          CTA-contiguous slice ranges (L1 reuse of x), 4/5 CTAs per SM.  All
+ *                          variants are bitwise identical.
  *   CAGMRES_OPT_GRAM     : CholQR Gram kernel: 0 = FP64 tensor core (DMMA m8n8k4) on a per-warp
  *                          cp.async ring; 1 (default) = scalar DFMA on a deeper ring (w <= 12,
  *                          else the DMMA kernel).
@@ -171,7 +172,10 @@ int cagmres_sizes(cagmres_t h, int64_t* n_loc, int64_t* n_ext, int64_t* ldv);
 /* ---- shifts ------------------------------------------------------------------ */
 /* Newton shifts theta_k = re[k] + i im[k], k < count, in application order, conjugate pairs
  * adjacent with +im first.  Replaces any shifts the first GMRES cycle would compute.
- * count >= 1 (extra entries beyond s are ignored).  Errors: EINVAL (pair not adjacent). */
+ * count >= 1 (extra entries beyond s are ignored).  count == 0 (re, im may be NULL) forgets
+ * the shifts: a Newton solve keeps the Leja-ordered Ritz values of its first cycle for later
+ * solves with the same matrix unless they are cleared this way.
+ * Errors: EINVAL (pair not adjacent). */
 int cagmres_set_shifts(cagmres_t h, const double* re, const double* im, int count);
 /* Copies the current shifts (after a Newton solve: the Leja-ordered Ritz values) to host
  * arrays of capacity cap; *count = number available (0 if none). */

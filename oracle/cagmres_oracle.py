@@ -344,9 +344,10 @@ def arnoldi_mgs(A, r, m):
     return Q, H, beta
 
 
-def arnoldi_cgs2(A, r, m):
-    """First (shift-finding) cycle of Newton CA-GMRES: standard GMRES iterations,
-    Arnoldi with CGS + one reorthogonalisation (G12)."""
+def arnoldi_cgs(A, r, m, reorth=False):
+    """First (shift-finding) cycle of Newton CA-GMRES: the standard GMRES iterations as
+    the paper runs GMRES — Arnoldi with CGS (the "GMRES ... CGS" rows of Fig. 14),
+    plus one reorthogonalisation pass ("2x", CGS2) when reorth (reading G12)."""
     n = A.shape[0]
     beta = np.linalg.norm(r)
     Q = np.zeros((n, m + 1), order="F")
@@ -354,16 +355,23 @@ def arnoldi_cgs2(A, r, m):
     Q[:, 0] = r / beta
     for k in range(m):
         w = A @ Q[:, k]
-        c1 = Q[:, :k + 1].T @ w
-        w = w - Q[:, :k + 1] @ c1
-        c2 = Q[:, :k + 1].T @ w
-        w = w - Q[:, :k + 1] @ c2
-        H[:k + 1, k] = c1 + c2
+        c = Q[:, :k + 1].T @ w
+        w = w - Q[:, :k + 1] @ c
+        if reorth:
+            c2 = Q[:, :k + 1].T @ w
+            w = w - Q[:, :k + 1] @ c2
+            c = c + c2
+        H[:k + 1, k] = c
         H[k + 1, k] = np.sqrt(w @ w)
         if H[k + 1, k] == 0.0:
             raise Breakdown("Arnoldi breakdown")
         Q[:, k + 1] = w / H[k + 1, k]
     return Q, H, beta
+
+
+def arnoldi_cgs2(A, r, m):
+    """arnoldi_cgs with one reorthogonalisation (CGS2)."""
+    return arnoldi_cgs(A, r, m, reorth=True)
 
 
 def gmres(A, b, m, tol=1e-8, maxcyc=100, x0=None):
@@ -436,7 +444,7 @@ def cagmres(A, b, s, m, basis="newton", tsqr="cholqr", borth="cgs", reorth=False
             tol=1e-8, maxcyc=100, x0=None, shifts=None, caqr_blocks=1, diag=None,
             keep_last=False, onepass=False):
     """CA-GMRES(s, m) solve.  x0 = 0 by default (G17).
-    basis 'newton': first cycle is GMRES(m) (Arnoldi CGS2) unless shifts are given; its
+    basis 'newton': first cycle is GMRES(m) (Arnoldi CGS, CGS2 if reorth) unless shifts are given; its
     Ritz values in modified Leja order become the shifts.  'monomial': theta = 0
     from cycle 1 (G18).  Returns dict(x, hist (rho_c / rho_0 per cycle), cycles, shifts)."""
     A = sp.csr_matrix(A)
@@ -461,7 +469,7 @@ def cagmres(A, b, s, m, basis="newton", tsqr="cholqr", borth="cgs", reorth=False
         Q[:, 0] = r / beta
         H = np.zeros((m + 1, m))
         if re is None:                                   # first Newton cycle = GMRES(m)
-            Q, H, _ = arnoldi_cgs2(A, r, m)
+            Q, H, _ = arnoldi_cgs(A, r, m, reorth=reorth)
             re, im = modified_leja(ritz_values(H, m), s)
         else:
             ca_cycle(A, Q, H, s, m, re, im, tsqr, borth, reorth, caqr_blocks, diag, onepass)

@@ -372,6 +372,8 @@ void wave_reset_pairs(cagmres* h) {
 // the same operations in the same order (bitwise identical results), so the fastest one on
 // this matrix is picked by timing y = A x over all stored rows (x = V[:,0], y = V[:,1]).
 int spmv_autotune(cagmres* h) {
+    // 14, 15 (CTA-contiguous) are faster per launch but lose ~1.4 ms per C2 solve in the
+    // back-to-back PDL chain (profiles/r1_bench_C2_spmv14.json): options only
     static const int cand[] = {0, 3, 5, 6, 8, 10, 11, 12, 13};
     if (h->m < 1 || h->A.nrows <= 0) return CAGMRES_OK;
     double* x = h->V;
@@ -381,18 +383,22 @@ int spmv_autotune(cagmres* h) {
     CU(cudaEventCreate(&e1));
     float best = 1e30f;
     int pick = 0;
+    constexpr int CHAIN = 8;                 // an MPK-like chain of dependent launches
     for (int v : cand) {
         h->A.variant = v;
-        kern::spmv(h->dev, h->A, h->A.nrows, x, y, nullptr, 0.0, nullptr, 0.0, h->stream);   // warm-up
+        for (int k = 0; k < 2; ++k)          // warm-up
+            kern::spmv(h->dev, h->A, h->A.nrows, k ? y : x, k ? x : y, nullptr, 0.0, nullptr, 0.0, h->stream);
         float tmin = 1e30f;
         for (int r = 0; r < 3; ++r) {
             CU(cudaEventRecord(e0, h->stream));
-            kern::spmv(h->dev, h->A, h->A.nrows, x, y, nullptr, 0.0, nullptr, 0.0, h->stream);
+            for (int k = 0; k < CHAIN; ++k)
+                kern::spmv(h->dev, h->A, h->A.nrows, (k & 1) ? y : x, (k & 1) ? x : y, nullptr, 0.0, nullptr, 0.0,
+                           h->stream);
             CU(cudaEventRecord(e1, h->stream));
             CU(cudaEventSynchronize(e1));
             float ms = 0.f;
             CU(cudaEventElapsedTime(&ms, e0, e1));
-            tmin = std::min(tmin, ms);
+            tmin = std::min(tmin, ms / CHAIN);
         }
         if (tmin < best) { best = tmin; pick = v; }
     }
@@ -759,9 +765,9 @@ int ca_cycle(cagmres* h, const std::vector<Block>& bl) {
     return CAGMRES_OK;
 }
 
-// First Newton cycle = GMRES(m) with CGS2 Arnoldi (reading G12), on the
-// same kernels with panel width 1.  tab layout: per k: c1 (m+1), c2 (m+1), r (1).
-// cgs2 = false (GMRES baseline without CAGMRES_REORTH): one CGS pass, c2 = 0.
+// First Newton cycle = GMRES(m) with CGS Arnoldi, CGS2 with CAGMRES_REORTH (Fig. 14,
+// DESIGN.md reading G12), on the same kernels with panel width 1; also the GMRES baseline.
+// tab layout: per k: c1 (m+1), c2 (m+1, unused for CGS), r (1).
 int arnoldi_cycle(cagmres* h, bool cgs2) {
     const int m = h->m;
     const size_t stride = 2 * size_t(m + 1) + 1;
@@ -850,8 +856,9 @@ int residual_norm_async(cagmres* h, const double* b, const double* x) {
 // One restart cycle's GPU work plus the async copy of its coefficient table and status.
 int enqueue_cycle(cagmres* h, bool arnoldi, const std::vector<Block>& bl) {
     if (arnoldi) {
-        // the shift-finding Newton cycle is CGS2 (G12); the GMRES baseline follows the flag
-        TRY(arnoldi_cycle(h, h->basis != CAGMRES_GMRES || (h->orth & CAGMRES_REORTH) != 0));
+        // standard GMRES as the paper runs it: CGS Arnoldi (Fig. 14 "GMRES ... CGS" rows), CGS2
+        // with CAGMRES_REORTH — for the shift-finding Newton cycle (G12) and the baseline
+        TRY(arnoldi_cycle(h, (h->orth & CAGMRES_REORTH) != 0));
     } else {
         TRY(ca_cycle(h, bl));
     }
@@ -950,7 +957,7 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
     switch (opt) {
         case CAGMRES_OPT_MPK_WAVE: h->wave_on = value != 0; h->wave_force = value == 2; return CAGMRES_OK;
         case CAGMRES_OPT_SPMV:
-            if (value < -1 || value > 13 || (value > 9 && value < 10)) return CAGMRES_EINVAL;
+            if (value < -1 || value > 15) return CAGMRES_EINVAL;
             if (value == -1) return spmv_autotune(h);
             h->A.variant = int(value);
             return CAGMRES_OK;
@@ -996,7 +1003,14 @@ int cagmres_sizes(cagmres_t h, int64_t* n_loc, int64_t* n_ext, int64_t* ldv) {
 }
 
 int cagmres_set_shifts(cagmres_t h, const double* re, const double* im, int count) {
-    if (!h || !re || !im || count < 1) return CAGMRES_EINVAL;
+    if (!h || count < 0) return CAGMRES_EINVAL;
+    if (count == 0) {                        // forget the shifts: the next Newton solve starts
+        h->sh_re.clear();                    // with the GMRES cycle again
+        h->sh_im.clear();
+        h->have_shifts = false;
+        return CAGMRES_OK;
+    }
+    if (!re || !im) return CAGMRES_EINVAL;
     for (int k = 0; k < count; ++k) {
         if (im[k] > 0.0 && k + 1 < count && !(re[k + 1] == re[k] && im[k + 1] == -im[k])) return CAGMRES_EINVAL;
         if (im[k] < 0.0 && (k == 0 || !(re[k - 1] == re[k] && im[k - 1] == -im[k]))) return CAGMRES_EINVAL;
@@ -1095,7 +1109,7 @@ int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit
     for (; cyc < maxit && rc != CAGMRES_OK; ++cyc) {
         const bool first_newton = h->basis == CAGMRES_NEWTON && !h->have_shifts;
         const bool arnoldi = first_newton || h->basis == CAGMRES_GMRES;
-        const bool cgs2 = h->basis != CAGMRES_GMRES || (h->orth & CAGMRES_REORTH) != 0;
+        const bool cgs2 = (h->orth & CAGMRES_REORTH) != 0;
         std::fill(H.begin(), H.end(), 0.0);
         if (!pending) TRY(enqueue_cycle(h, arnoldi, bl));
         pending = false;

@@ -35,12 +35,31 @@ struct DiaArgs {
 };
 }  // namespace
 
-template <int MODE, int WT, int MINB>   // MODE 0: Ax  1: Ax + bu u  2: + bw w  3: u - Ax
+// value stream: read once, keep it out of L1 so L1 holds the x lines neighbouring warps reuse
+__device__ __forceinline__ double ldg_stream(const double* p) {
+    double v;
+    asm volatile("ld.global.nc.L1::no_allocate.f64 %0, [%1];" : "=d"(v) : "l"(p));
+    return v;
+}
+
+// CONTIG = 0: slices grid-strided over all warps.  CONTIG = 1: each CTA owns a contiguous
+// range of slices and its 8 warps walk it side by side, so the x lines of the +-1 and +-nx
+// offsets (and, for thin 3-D grids, +-nx*ny) are L1 hits from the CTA's own recent loads.
+template <int MODE, int WT, int MINB, int CONTIG = 0>   // MODE 0: Ax  1: Ax + bu u  2: + bw w  3: u - Ax
 __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
     const int lane = threadIdx.x & 31;
-    const int64_t nsl = (a.nrows + 31) >> 5;
-    const int64_t stride = int64_t(gridDim.x) * (DT_NT / 32);
-    int64_t sl = (int64_t(blockIdx.x) * DT_NT + threadIdx.x) >> 5;
+    const int64_t nsl_all = (a.nrows + 31) >> 5;
+    int64_t stride, sl, nsl;
+    if (CONTIG) {
+        stride = DT_NT / 32;
+        const int64_t c0 = int64_t(blockIdx.x) * nsl_all / gridDim.x;
+        nsl = int64_t(blockIdx.x + 1) * nsl_all / gridDim.x;
+        sl = c0 + (threadIdx.x >> 5);
+    } else {
+        stride = int64_t(gridDim.x) * (DT_NT / 32);
+        nsl = nsl_all;
+        sl = (int64_t(blockIdx.x) * DT_NT + threadIdx.x) >> 5;
+    }
     if (sl >= nsl) { pdl_wait(); pdl_trigger(); return; }
     int64_t b0, i0, b1 = 0, i1 = 1, b2, i2;
     int W0, W1 = 0, W2, o0, o1;
@@ -65,7 +84,7 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
 #pragma unroll
             for (int t = 0; t < WT; ++t) {
                 const int o = __shfl_sync(0xffffffffu, o0, t);
-                v[t] = __ldg(vp + 32 * t);
+                v[t] = CONTIG ? ldg_stream(vp + 32 * t) : __ldg(vp + 32 * t);
                 xv[t] = __ldg(xr + o);
             }
             if (MODE >= 1 && live) uu = __ldg(a.u + r);
@@ -94,49 +113,52 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
 }
 
 namespace {
-template <int MODE, int WT, int MINB>
+template <int MODE, int WT, int MINB, int CONTIG>
 void go_dia(const Dev& d, const DiaArgs& a, cudaStream_t st) {
     static int occ = 0;
     if (occ == 0) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_spmv_dia<MODE, WT, MINB>, DT_NT, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_spmv_dia<MODE, WT, MINB, CONTIG>, DT_NT, 0);
         if (occ < 1) occ = 1;
     }
     const int64_t nsl = (a.nrows + 31) >> 5;
     int64_t g = int64_t(d.sms) * occ;
     const int64_t need = (nsl + DT_NT / 32 - 1) / (DT_NT / 32);
     if (g > need) g = need;
-    launch_pdl(k_spmv_dia<MODE, WT, MINB>, dim3(unsigned(g)), dim3(DT_NT), 0, st, a);
+    launch_pdl(k_spmv_dia<MODE, WT, MINB, CONTIG>, dim3(unsigned(g)), dim3(DT_NT), 0, st, a);
 }
 
-template <int WT, int MINB>
+template <int WT, int MINB, int CONTIG>
 void go_modes(const Dev& d, const DiaArgs& a, cudaStream_t st, int mode) {
     switch (mode) {
-        case 0: go_dia<0, WT, MINB>(d, a, st); break;
-        case 1: go_dia<1, WT, MINB>(d, a, st); break;
-        case 2: go_dia<2, WT, MINB>(d, a, st); break;
-        default: go_dia<3, WT, MINB>(d, a, st); break;
+        case 0: go_dia<0, WT, MINB, CONTIG>(d, a, st); break;
+        case 1: go_dia<1, WT, MINB, CONTIG>(d, a, st); break;
+        case 2: go_dia<2, WT, MINB, CONTIG>(d, a, st); break;
+        default: go_dia<3, WT, MINB, CONTIG>(d, a, st); break;
     }
 }
 
-template <int MINB>
+template <int MINB, int CONTIG>
 void go_width(const Dev& d, const DiaArgs& a, int wt, cudaStream_t st, int mode) {
     switch (wt) {
-        case 5: go_modes<5, MINB>(d, a, st, mode); break;
-        case 27: go_modes<27, MINB>(d, a, st, mode); break;
-        default: go_modes<7, MINB>(d, a, st, mode); break;     // other widths: generic path
+        case 5: go_modes<5, MINB, CONTIG>(d, a, st, mode); break;
+        case 27: go_modes<27, MINB, CONTIG>(d, a, st, mode); break;
+        default: go_modes<7, MINB, CONTIG>(d, a, st, mode); break;     // other widths: generic path
     }
 }
 }  // namespace
 
-// variants 10 / 11 / 12 / 13: at least 3 / 4 / 5 / 6 CTAs per SM (register cap)
+// variants 10 / 11 / 12 / 13: at least 3 / 4 / 5 / 6 CTAs per SM (register cap), grid-strided
+// slices; 14 / 15: 4 / 5 CTAs per SM, CTA-contiguous slice ranges (L1 reuse of x)
 void spmv_dia(const Dev& d, const Sell& A, int variant, int64_t nrows, const double* x, double* y,
               const double* u, double bu, const double* w, double bw, int mode, cudaStream_t st) {
     DiaArgs a{nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, u, bu, w, bw, y};
     switch (variant) {
-        case 10: go_width<3>(d, a, A.dia_w, st, mode); break;
-        case 11: go_width<4>(d, a, A.dia_w, st, mode); break;
-        case 12: go_width<5>(d, a, A.dia_w, st, mode); break;
-        default: go_width<6>(d, a, A.dia_w, st, mode); break;
+        case 10: go_width<3, 0>(d, a, A.dia_w, st, mode); break;
+        case 11: go_width<4, 0>(d, a, A.dia_w, st, mode); break;
+        case 12: go_width<5, 0>(d, a, A.dia_w, st, mode); break;
+        case 14: go_width<4, 1>(d, a, A.dia_w, st, mode); break;
+        case 15: go_width<5, 1>(d, a, A.dia_w, st, mode); break;
+        default: go_width<6, 0>(d, a, A.dia_w, st, mode); break;
     }
 }
 

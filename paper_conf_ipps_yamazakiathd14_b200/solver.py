@@ -145,6 +145,10 @@ class Solver:
         im = np.zeros_like(re) if im is None else np.ascontiguousarray(im, dtype=np.float64)
         L.check(self._lib.cagmres_set_shifts(self._h, L.dptr(re), L.dptr(im), len(re)), "set_shifts")
 
+    def clear_shifts(self):
+        """Forget the Newton shifts: the next solve runs its own first GMRES cycle."""
+        L.check(self._lib.cagmres_set_shifts(self._h, None, None, 0), "set_shifts")
+
     def get_shifts(self):
         cap = 4 * self.m + 8
         re, im = np.zeros(cap), np.zeros(cap)

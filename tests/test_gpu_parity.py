@@ -139,7 +139,7 @@ def test_spmv_variants_bitwise(gen):
     S = Solver(A, s=6, m=30, basis="newton")
     S.set_shifts(*SHIFTS)
     Ws = []
-    variants = list(range(10)) + [10, 11, 12, 13]       # 10..13: cp.async ring-staged slices
+    variants = list(range(10)) + [10, 11, 12, 13, 14, 15]       # 10..13: cp.async ring-staged slices
     for v in variants:
         S.set_option("spmv", v)
         Ws.append(S.mpk(q, 6))
@@ -413,3 +413,19 @@ def test_onepass_cycle_basis_matches_two_pass():
         _, st = S.solve(dev(b), tol=0.0, maxit=3)
         out.append(st.hist)
     assert np.allclose(out[0], out[1], rtol=1e-8)
+
+
+def test_clear_shifts_reruns_first_cycle_bitwise():
+    """set_shifts(count = 0): the next Newton solve runs its own GMRES shift cycle again
+    and, the reductions being deterministic, reproduces the first solve bit for bit."""
+    A = G.convection_diffusion(40, 3, 7)
+    b = dev(G.rhs(A.n))
+    S = Solver(A, s=10, m=30, basis="newton")
+    x1, st1 = S.solve(b, tol=1e-8, maxit=60)
+    sh1 = S.get_shifts()
+    x2, st2 = S.solve(b, tol=1e-8, maxit=60)            # reuses the shifts: no GMRES cycle
+    S.clear_shifts()
+    x3, st3 = S.solve(b, tol=1e-8, maxit=60)
+    assert np.array_equal(st3.hist, st1.hist) and torch.equal(x3, x1)
+    assert np.array_equal(S.get_shifts()[0], sh1[0])
+    assert st2.cycles >= 1
