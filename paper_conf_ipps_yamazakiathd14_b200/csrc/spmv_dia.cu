@@ -42,10 +42,17 @@ __device__ __forceinline__ double ldg_stream(const double* p) {
     return v;
 }
 
+__device__ __forceinline__ void prefetch_l2(const void* p) {
+    asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+}
+
+// PF = 1: while slice i is computed, the value lines of slice i + stride (descriptor already in
+// registers) are prefetched into L2, so next iteration's value loads are L2 hits: one more
+// slice of HBM requests in flight per warp without holding registers.
 // CONTIG = 0: slices grid-strided over all warps.  CONTIG = 1: each CTA owns a contiguous
 // range of slices and its 8 warps walk it side by side, so the x lines of the +-1 and +-nx
 // offsets (and, for thin 3-D grids, +-nx*ny) are L1 hits from the CTA's own recent loads.
-template <int MODE, int WT, int MINB, int CONTIG = 0>   // MODE 0: Ax  1: Ax + bu u  2: + bw w  3: u - Ax
+template <int MODE, int WT, int MINB, int CONTIG = 0, int PF = 0>   // MODE 0: Ax  1: + bu u  2: + bw w  3: u - Ax
 __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
     const int lane = threadIdx.x & 31;
     const int64_t nsl_all = (a.nrows + 31) >> 5;
@@ -74,6 +81,7 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
         b2 = 0; W2 = 0; i2 = 1;
         if (sl + 2 * stride < nsl) sell_slice_meta(sl + 2 * stride, a.sptr, a.sinfo, b2, W2, i2);
         o1 = sell_slice_off(lane, W1, i1, a.dcol);
+        if (PF && lane < 2 * W1) prefetch_l2(a.val + b1 + 16 * lane);     // 128-B lines of slice +1
         const int64_t r = sl * 32 + lane;
         const bool live = r < a.nrows;
         double uu = 0.0, ww = 0.0, acc = 0.0;
@@ -113,42 +121,43 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
 }
 
 namespace {
-template <int MODE, int WT, int MINB, int CONTIG>
+template <int MODE, int WT, int MINB, int CONTIG, int PF>
 void go_dia(const Dev& d, const DiaArgs& a, cudaStream_t st) {
     static int occ = 0;
     if (occ == 0) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_spmv_dia<MODE, WT, MINB, CONTIG>, DT_NT, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_spmv_dia<MODE, WT, MINB, CONTIG, PF>, DT_NT, 0);
         if (occ < 1) occ = 1;
     }
     const int64_t nsl = (a.nrows + 31) >> 5;
     int64_t g = int64_t(d.sms) * occ;
     const int64_t need = (nsl + DT_NT / 32 - 1) / (DT_NT / 32);
     if (g > need) g = need;
-    launch_pdl(k_spmv_dia<MODE, WT, MINB, CONTIG>, dim3(unsigned(g)), dim3(DT_NT), 0, st, a);
+    launch_pdl(k_spmv_dia<MODE, WT, MINB, CONTIG, PF>, dim3(unsigned(g)), dim3(DT_NT), 0, st, a);
 }
 
-template <int WT, int MINB, int CONTIG>
+template <int WT, int MINB, int CONTIG, int PF>
 void go_modes(const Dev& d, const DiaArgs& a, cudaStream_t st, int mode) {
     switch (mode) {
-        case 0: go_dia<0, WT, MINB, CONTIG>(d, a, st); break;
-        case 1: go_dia<1, WT, MINB, CONTIG>(d, a, st); break;
-        case 2: go_dia<2, WT, MINB, CONTIG>(d, a, st); break;
-        default: go_dia<3, WT, MINB, CONTIG>(d, a, st); break;
+        case 0: go_dia<0, WT, MINB, CONTIG, PF>(d, a, st); break;
+        case 1: go_dia<1, WT, MINB, CONTIG, PF>(d, a, st); break;
+        case 2: go_dia<2, WT, MINB, CONTIG, PF>(d, a, st); break;
+        default: go_dia<3, WT, MINB, CONTIG, PF>(d, a, st); break;
     }
 }
 
-template <int MINB, int CONTIG>
+template <int MINB, int CONTIG, int PF = 0>
 void go_width(const Dev& d, const DiaArgs& a, int wt, cudaStream_t st, int mode) {
     switch (wt) {
-        case 5: go_modes<5, MINB, CONTIG>(d, a, st, mode); break;
-        case 27: go_modes<27, MINB, CONTIG>(d, a, st, mode); break;
-        default: go_modes<7, MINB, CONTIG>(d, a, st, mode); break;     // other widths: generic path
+        case 5: go_modes<5, MINB, CONTIG, PF>(d, a, st, mode); break;
+        case 27: go_modes<27, MINB, CONTIG, PF>(d, a, st, mode); break;
+        default: go_modes<7, MINB, CONTIG, PF>(d, a, st, mode); break;     // other widths: generic path
     }
 }
 }  // namespace
 
 // variants 10 / 11 / 12 / 13: at least 3 / 4 / 5 / 6 CTAs per SM (register cap), grid-strided
-// slices; 14 / 15: 4 / 5 CTAs per SM, CTA-contiguous slice ranges (L1 reuse of x)
+// slices; 14 / 15: 4 / 5 CTAs per SM, CTA-contiguous slice ranges (L1 reuse of x); 16 / 17:
+// 4 / 5 CTAs per SM, grid-strided, L2 prefetch of the next slice's values
 void spmv_dia(const Dev& d, const Sell& A, int variant, int64_t nrows, const double* x, double* y,
               const double* u, double bu, const double* w, double bw, int mode, cudaStream_t st) {
     DiaArgs a{nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, u, bu, w, bw, y};
@@ -158,6 +167,8 @@ void spmv_dia(const Dev& d, const Sell& A, int variant, int64_t nrows, const dou
         case 12: go_width<5, 0>(d, a, A.dia_w, st, mode); break;
         case 14: go_width<4, 1>(d, a, A.dia_w, st, mode); break;
         case 15: go_width<5, 1>(d, a, A.dia_w, st, mode); break;
+        case 16: go_width<4, 0, 1>(d, a, A.dia_w, st, mode); break;
+        case 17: go_width<5, 0, 1>(d, a, A.dia_w, st, mode); break;
         default: go_width<6, 0>(d, a, A.dia_w, st, mode); break;
     }
 }
