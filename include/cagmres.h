@@ -160,6 +160,8 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
 #define CAGMRES_OPT_PDL        12   /* process-wide: 1 (default) = programmatic dependent launch of
                                        the hot kernels (next kernel's CTAs scheduled while the
                                        previous one drains), 0 = plain stream order */
+#define CAGMRES_OPT_PANEL_PF   13   /* 1 (default) = panel ring kernels also prefetch tiles beyond
+                                       their cp.async window into L2; 0 = off */
 #define CAGMRES_OPT_TRSM       11   /* CholQR/SVQR panel update V R^{-1}: 1 (default) = scalar
                                        FP64 on a cp.async ring (w <= 16), 0 = FP64 tensor core */
 int cagmres_set_option(cagmres_t h, int opt, int64_t value);

@@ -106,15 +106,17 @@ __global__ void __launch_bounds__(512, 1) k_arnoldi_ring(ArnoldiArgs a) {
     const int64_t Wn = int64_t(gridDim.x) * nw;
     const int64_t g = int64_t(blockIdx.x) * nw + wp;
     const int64_t t0 = g * T / Wn, t1 = (g + 1) * T / Wn;
+    const int part2 = 2 * (lane & 15), cfirst = lane >> 4;
+    const int64_t cstride = 2 * a.ldq;
     auto issue = [&](int64_t t, int stage) {
         if (t < t1) {
-            double* dst = ring + stage * stage_d;
-            const int64_t r0 = t * 32;
-            for (int q = lane; q < ncol * 16; q += 32) {
-                const int c = q >> 4, part = q & 15;
-                const double* src = (c < jx ? a.Q + a.ldq * c : a.v) + r0 + part * 2;
-                ptx::cp_async16(dst + c * 32 + part * 2, src);
-            }
+            double* dst = ring + stage * stage_d + cfirst * 32 + part2;
+            const int64_t r0 = t * 32 + part2;
+            const double* src = a.Q + a.ldq * cfirst + r0;
+            int c = cfirst;
+#pragma unroll 4
+            for (; c < jx; c += 2, dst += 64, src += cstride) ptx::cp_async16(dst, src);
+            if (c == jx) ptx::cp_async16(dst, a.v + r0);             // v is slot column jx
         }
         ptx::cp_async_commit();
     };
@@ -138,6 +140,11 @@ __global__ void __launch_bounds__(512, 1) k_arnoldi_ring(ArnoldiArgs a) {
     int stage = 0;
     for (int64_t t = t0; t < t1; ++t) {
         issue(t + AR_S - 1, (stage + AR_S - 1) % AR_S);
+        if (a.pf && t + AR_S - 1 + ptx::PF_DIST < t1) {
+            const int64_t rp = (t + AR_S - 1 + ptx::PF_DIST) * 32;
+            for (int q = lane; q < ncol * 2; q += 32)
+                ptx::prefetch_l2((q >> 1 < jx ? a.Q + a.ldq * (q >> 1) : a.v) + rp + 16 * (q & 1));
+        }
         ptx::cp_async_wait<AR_S - 1>();
         __syncwarp();
         const double* sl = ring + stage * stage_d + lane;

@@ -33,6 +33,7 @@ namespace {
 constexpr int GR_NT = 512;               // 16 warps = 8 pairs, one CTA per SM
 constexpr int GR_TW = 64;                // rows per tile (2 per lane: one LDS.128 per column)
 constexpr int GR_NP = GR_NT / 64;        // warp pairs
+constexpr bool GR_PF = false;            // L2 prefetch beyond the ring: measured no gain (50.8 vs 50.2 us)
 
 template <int W>
 __host__ __device__ constexpr int gram_stages() { return W <= 6 ? 6 : (W <= 8 ? 5 : 4); }
@@ -110,6 +111,9 @@ __device__ __forceinline__ void gram_pair_body(const GramArgs& a, double* smg, d
         ptx::cp_async_wait<S - 2>();                               // my copies of tile t landed
         pair_sync(pair);                                           // ... and my partner's; slot
         issue(t + S - 1, nxt);                                     //  of step t-1 is free
+        if (GR_PF && a.pf && t + S - 1 + ptx::PF_DIST < t1 && pt < W * (GR_TW / 16))   // 128-B lines, tile +PF
+            ptx::prefetch_l2(a.P + a.ldp * (pt / (GR_TW / 16)) + (t + S - 1 + ptx::PF_DIST) * GR_TW +
+                             16 * (pt % (GR_TW / 16)));
         if (HI > LO) rank1_part<W, LO, (HI > LO ? HI : LO + 1)>(cur, lane, acc);
         cur += stage_d; if (cur == rend) cur = ring;
         nxt += stage_d; if (nxt == rend) nxt = ring;

@@ -39,7 +39,8 @@ struct Dev {
     int gram = 1;               // CholQR Gram kernel: 0 = FP64 tensor core (DMMA), 1 = scalar DFMA ring
     int arnoldi_ring = 1;       // first-cycle / GMRES Arnoldi passes: 1 = cp.async ring kernels
     int trsm_scalar = 1;        // CholQR/SVQR update: 1 = scalar DFMA ring (w <= 16), 0 = DMMA
-    int panel_tw16 = 1;         // panel ring kernels: 16-row tiles when >= 24 columns are streamed
+    int panel_tw16 = 1;
+    int panel_pf = 1;           // panel rings: L2 prefetch PF_DIST tiles beyond the cp.async window         // panel ring kernels: 16-row tiles when >= 24 columns are streamed
 };
 
 // Sliced ELLPACK, slice height 32 (one warp), column-major inside a slice, with per-slice
@@ -194,6 +195,7 @@ void mpk_wave(const Dev& d, const WaveArgs& a, int ctas_per_sm, cudaStream_t st)
 // c_out = Q^T v; mode 2: v -= Q c_in and c_out[0] = v^T v (sqrt if sqrt_out).  jx <= 32
 // (returns -1 otherwise).  part: >= arnoldi_ws_doubles() doubles; counter: zeroed uint.
 struct ArnoldiArgs {
+    int pf;                     // L2 prefetch ahead of the ring (ring kernels)
     int64_t n;
     const double* Q; int64_t ldq; int jx;
     double* v;
@@ -264,6 +266,7 @@ int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const dou
 struct GramArgs {
     int64_t n;
     const double* P; int64_t ldp; int w;
+    int pf;                     // L2 prefetch ahead of the ring
     double* part;               // >= sms * w * w doubles
     double* out;                // w x w, ld w
     unsigned int* counter;

@@ -49,6 +49,11 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         : "memory");
 }
 
+// L2 prefetch of one line (no registers, no completion tracking): the panel rings prefetch a
+// tile PF_DIST tiles beyond their cp.async window so more HBM requests are in flight per SM
+__device__ __forceinline__ void prefetch_l2(const void* p) { asm volatile("prefetch.global.L2 [%0];" ::"l"(p)); }
+constexpr int PF_DIST = 3;              // tiles beyond the last one issued by cp.async
+
 // 16-byte asynchronous global -> shared copy (LDGSTS), L2-only (.cg), commit / wait groups.
 __device__ __forceinline__ void cp_async16(void* dst, const void* src) {
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");

@@ -788,7 +788,7 @@ int arnoldi_cycle(cagmres* h, bool cgs2) {
         if (h->arnoldi_fuse && k + 1 <= 32) {
             // c1 = Q^T v ; [v -= Q c1, c2 = Q^T v] ; [v -= Q c2, r = ||v||] ; v /= r
             const double nl = double(h->n_loc);
-            kern::ArnoldiArgs aa{h->n_loc, h->V, h->ldv, k + 1, v, nullptr, nullptr, h->arn_part,
+            kern::ArnoldiArgs aa{h->dev.panel_pf, h->n_loc, h->V, h->ldv, k + 1, v, nullptr, nullptr, h->arn_part,
                                  h->arn_counter, h->status, h->nranks == 1 ? 1 : 0};
             {
                 Scope sc(h, PH_BORTH);
@@ -838,7 +838,7 @@ int residual_norm_async(cagmres* h, const double* b, const double* x) {
     kern::residual(h->dev, h->A, h->n_loc, xx, b, h->V, h->stream);
     double* rr = h->gbuf + 8;
     {   // ||r|| by the scalar reduction kernel (mode 2 with no Q columns)
-        kern::ArnoldiArgs aa{h->n_loc, h->V, h->ldv, 0, h->V, nullptr, rr, h->arn_part, h->arn_counter,
+        kern::ArnoldiArgs aa{h->dev.panel_pf, h->n_loc, h->V, h->ldv, 0, h->V, nullptr, rr, h->arn_part, h->arn_counter,
                              h->status, h->nranks == 1 ? 1 : 0};
         if (kern::arnoldi_fused(h->dev, aa, 2, h->stream)) return CAGMRES_EINVAL;
         if (h->nranks > 1) {
@@ -966,6 +966,7 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
         case CAGMRES_OPT_PANEL_TW: if (value != 16 && value != 32) return CAGMRES_EINVAL; h->dev.panel_tw16 = value == 16; return CAGMRES_OK;
         case CAGMRES_OPT_TRSM: if (value < 0 || value > 4) return CAGMRES_EINVAL; h->dev.trsm_scalar = int(value); return CAGMRES_OK;
         case CAGMRES_OPT_PDL: if (value < 0 || value > 1) return CAGMRES_EINVAL; kern::g_pdl = int(value); return CAGMRES_OK;
+        case CAGMRES_OPT_PANEL_PF: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->dev.panel_pf = int(value); return CAGMRES_OK;
         case CAGMRES_OPT_FUSE: h->fuse_borth_gram = (value & 1) != 0; h->arnoldi_fuse = (value & 2) != 0; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK:
             if (value < 256 || value % 256) return CAGMRES_EINVAL;
@@ -986,6 +987,7 @@ int cagmres_get_option(cagmres_t h, int opt, int64_t* value) {
         case CAGMRES_OPT_PANEL_TW: *value = h->dev.panel_tw16 ? 16 : 32; return CAGMRES_OK;
         case CAGMRES_OPT_TRSM: *value = h->dev.trsm_scalar; return CAGMRES_OK;
         case CAGMRES_OPT_PDL: *value = kern::g_pdl; return CAGMRES_OK;
+        case CAGMRES_OPT_PANEL_PF: *value = h->dev.panel_pf; return CAGMRES_OK;
         case CAGMRES_OPT_FUSE: *value = (h->fuse_borth_gram ? 1 : 0) | (h->arnoldi_fuse ? 2 : 0); return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK: *value = h->wave_CH; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CTAS: *value = h->wave_ctas; return CAGMRES_OK;

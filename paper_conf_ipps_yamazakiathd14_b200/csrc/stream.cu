@@ -28,6 +28,7 @@ struct StreamArgs {
     double* P; int64_t ldp; int w;
     const double* M; int64_t ldm;             // C (jx x w) or R (w x w), leading dim ldm
     int c0;                                   // trsm: first column written
+    int pf = 0;                               // L2 prefetch ahead of the ring (Dev::panel_pf)
 };
 
 // R^{-1} (upper, w x w) into sRi[k*32 + c]; one thread per column (back substitution)
@@ -136,18 +137,25 @@ __global__ void __launch_bounds__(NT) k_rows_mma(StreamArgs a) {
 // of TW+8 doubles (== 8 mod 16: conflict free for that pattern) and store results directly.
 constexpr int RP_S = 3;
 
-template <int MODE, int KTM, int NTN, int TW>
-__global__ void __launch_bounds__(512, 1) k_rows_pipe(StreamArgs a) {
+template <int MODE, int KTM, int NTN, int TW, int MAXT = 512>   // MAXT 256: up to 255 registers
+__global__ void __launch_bounds__(MAXT, 1) k_rows_pipe(StreamArgs a) {
     extern __shared__ __align__(16) double smp[];
     constexpr int SP = TW + 8;
     __shared__ double sB[32 * 32 + 32];
+    __shared__ const double* sCol[96];                         // column base pointers (ncol <= 96)
     pdl_wait();
     pdl_trigger();
     const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const int gid = lane >> 2, tig = lane & 3;
     const int w = a.w;
     const int K = MODE == 1 ? w : a.jx;
-    if (MODE == 1) upper_inverse(a.M, w, sB, sB + 32 * 32);
+    const int jxl = MODE != 1 ? a.jx : 0;
+    const int ncol = MODE == 2 ? a.jx : jxl + w;               // gemm: P is inside X
+    for (int c = threadIdx.x; c < ncol; c += blockDim.x)
+        sCol[c] = c < jxl ? a.X + a.ldx * c : a.P + a.ldp * (c - jxl);
+    if (MODE == 1) upper_inverse(a.M, w, sB, sB + 32 * 32);  // (has __syncthreads)
+    else __syncthreads();
+    // B fragments (update: -C, so d = P + A (-C) needs no per-element negation)
     double b[KTM][NTN];
 #pragma unroll
     for (int kt = 0; kt < KTM; ++kt)
@@ -156,77 +164,96 @@ __global__ void __launch_bounds__(512, 1) k_rows_pipe(StreamArgs a) {
             const int k = 4 * kt + tig, c = 8 * nt + gid;
             double v = 0.0;
             if (k < K && c < w) v = MODE != 1 ? a.M[k + a.ldm * c] : sB[k * 32 + c];
-            b[kt][nt] = v;
+            b[kt][nt] = MODE == 0 ? -v : v;
         }
-    const int jxl = MODE != 1 ? a.jx : 0;
-    const int ncol = MODE == 2 ? a.jx : jxl + w;               // gemm: P is inside X
+    // measured (profiles/r1_launches_C2_pf.txt): prefetch helps narrow panels, hurts wide ones
+    const bool d_pf = a.pf != 0 && TW == 32 && ncol <= 24;
     const int64_t stage_d = int64_t(ncol) * SP;
     double* ring = smp + int64_t(wp) * RP_S * stage_d;
     const int64_t T = a.n / TW;
     const int64_t W = int64_t(gridDim.x) * nw;
     const int64_t g = int64_t(blockIdx.x) * nw + wp;
     const int64_t t0 = g * T / W, t1 = (g + 1) * T / W;
-    auto colptr = [&](int c) -> const double* { return c < jxl ? a.X + a.ldx * c : a.P + a.ldp * (c - jxl); };
+    auto colptr = [&](int c) -> const double* { return sCol[c]; };
+    // copy slots: lane covers 16-B part (lane % CPC) of columns lane / CPC, + 32 / CPC, ...
     constexpr int CPC = TW * 8 / 16;
+    constexpr int CSTEP = 32 / CPC;
+    const int part2 = 2 * (lane % CPC), cfirst = lane / CPC;
     auto issue = [&](int64_t t, int stage) {
         if (t < t1) {
-            double* dst = ring + stage * stage_d;
-            const int64_t r0 = t * TW;
-            for (int q = lane; q < ncol * CPC; q += 32) {
-                const int c = q / CPC, part = q - c * CPC;
-                ptx::cp_async16(dst + c * SP + part * 2, colptr(c) + r0 + part * 2);
-            }
+            double* dst = ring + stage * stage_d + part2;
+            const int64_t r0 = t * TW + part2;
+#pragma unroll 4
+            for (int c = cfirst; c < ncol; c += CSTEP) ptx::cp_async16(dst + c * SP, sCol[c] + r0);
         }
         ptx::cp_async_commit();
     };
     const int KT = (K + 3) / 4;
     int acol[KTM];
 #pragma unroll
-    for (int kt = 0; kt < KTM; ++kt) acol[kt] = (MODE == 1 ? jxl : 0) + min(4 * kt + tig, K - 1);
+    for (int kt = 0; kt < KTM; ++kt) acol[kt] = ((MODE == 1 ? jxl : 0) + min(4 * kt + tig, K - 1)) * SP;
     int pcol[NTN][2];
     bool wcol[NTN][2];
+    double* pst[NTN][2];                                       // per-lane output column pointers
 #pragma unroll
     for (int nt = 0; nt < NTN; ++nt)
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
             const int c = 8 * nt + 2 * tig + h;
-            pcol[nt][h] = min(c, w - 1);
+            pcol[nt][h] = (jxl + min(c, w - 1)) * SP;
             wcol[nt][h] = c < w && (MODE == 0 || c >= a.c0);
+            pst[nt][h] = a.P + a.ldp * min(c, w - 1) + gid + t0 * TW;
         }
 #pragma unroll
     for (int s = 0; s < RP_S - 1; ++s) issue(t0 + s, s);
-    int stage = 0;
+    int stage = 0, stage_in = RP_S - 1;
     for (int64_t t = t0; t < t1; ++t) {
-        issue(t + RP_S - 1, (stage + RP_S - 1) % RP_S);
+        issue(t + RP_S - 1, stage_in);
+        if (d_pf && t + RP_S - 1 + ptx::PF_DIST < t1) {
+            const int64_t rp = (t + RP_S - 1 + ptx::PF_DIST) * TW;
+            constexpr int LPC = TW / 16;                        // 128-B lines per column tile
+            for (int q = lane; q < ncol * LPC; q += 32) ptx::prefetch_l2(colptr(q / LPC) + rp + 16 * (q % LPC));
+        }
         ptx::cp_async_wait<RP_S - 1>();
         __syncwarp();
-        const double* sl = ring + stage * stage_d;
-        double* outb = a.P + t * TW;
-#pragma unroll 1
+        const double* sl = ring + stage * stage_d + gid;
+        // per-tile operand pointers; the 8-row groups below are unrolled, so every shared load
+        // and global store is [register + immediate]
+        const double* sa[KTM];
+#pragma unroll
+        for (int kt = 0; kt < KTM; ++kt) sa[kt] = sl + acol[kt];
+        const double* sd[NTN][2];
+#pragma unroll
+        for (int nt = 0; nt < NTN; ++nt)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) sd[nt][h] = sl + pcol[nt][h];
+#pragma unroll
         for (int g8 = 0; g8 < TW / 8; ++g8) {
-            const int row = 8 * g8 + gid;
             double d[NTN][2];
 #pragma unroll
             for (int nt = 0; nt < NTN; ++nt)
 #pragma unroll
-                for (int h = 0; h < 2; ++h) d[nt][h] = MODE == 0 ? sl[(jxl + pcol[nt][h]) * SP + row] : 0.0;
+                for (int h = 0; h < 2; ++h) d[nt][h] = MODE == 0 ? sd[nt][h][8 * g8] : 0.0;
 #pragma unroll
             for (int kt = 0; kt < KTM; ++kt) {
-                if (kt < KT) {
-                    const double av = sl[acol[kt] * SP + row];
-                    const double am = MODE == 0 ? -av : av;
+                if (kt >= KT) break;                            // uniform: skip padded k-steps
+                const double av = sa[kt][8 * g8];
 #pragma unroll
-                    for (int nt = 0; nt < NTN; ++nt) ptx::dmma(d[nt][0], d[nt][1], am, b[kt][nt]);
-                }
+                for (int nt = 0; nt < NTN; ++nt) ptx::dmma(d[nt][0], d[nt][1], av, b[kt][nt]);
             }
 #pragma unroll
             for (int nt = 0; nt < NTN; ++nt)
 #pragma unroll
                 for (int h = 0; h < 2; ++h)
-                    if (wcol[nt][h]) __stcs(outb + a.ldp * (8 * nt + 2 * tig + h) + row, d[nt][h]);
+                    if (wcol[nt][h]) __stcs(pst[nt][h] + 8 * g8, d[nt][h]);
         }
+#pragma unroll
+        for (int nt = 0; nt < NTN; ++nt)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) pst[nt][h] += TW;
         __syncwarp();
-        stage = (stage + 1) % RP_S;
+        stage = stage == RP_S - 1 ? 0 : stage + 1;
+        stage_in = stage_in == RP_S - 1 ? 0 : stage_in + 1;
     }
     ptx::cp_async_wait<0>();
     // ragged tail rows [T*TW, n): warp 0 of CTA 0, direct zero-padded loads
@@ -238,15 +265,13 @@ __global__ void __launch_bounds__(512, 1) k_rows_pipe(StreamArgs a) {
 #pragma unroll
             for (int nt = 0; nt < NTN; ++nt)
 #pragma unroll
-                for (int h = 0; h < 2; ++h) d[nt][h] = (MODE == 0 && ok) ? a.P[a.ldp * pcol[nt][h] + row] : 0.0;
+                for (int h = 0; h < 2; ++h) d[nt][h] = (MODE == 0 && ok) ? sCol[pcol[nt][h] / SP][row] : 0.0;
 #pragma unroll
             for (int kt = 0; kt < KTM; ++kt) {
                 if (kt < KT) {
-                    const double* src = (MODE == 2 || acol[kt] < jxl) ? a.X + a.ldx * acol[kt] : a.P + a.ldp * (acol[kt] - jxl);
-                    const double av = ok ? src[row] : 0.0;
-                    const double am = MODE == 0 ? -av : av;
+                    const double av = ok ? sCol[acol[kt] / SP][row] : 0.0;
 #pragma unroll
-                    for (int nt = 0; nt < NTN; ++nt) ptx::dmma(d[nt][0], d[nt][1], am, b[kt][nt]);
+                    for (int nt = 0; nt < NTN; ++nt) ptx::dmma(d[nt][0], d[nt][1], av, b[kt][nt]);
                 }
             }
             if (ok) {
@@ -270,9 +295,14 @@ bool run_pipe_tw(const Dev& d, const StreamArgs& a, cudaStream_t st) {
     int nw = int((200 * 1024) / ring_w);
     nw = nw < 2 ? 2 : (nw > 16 ? 16 : nw);
     const size_t smem = size_t(nw) * ring_w;
-    cudaFuncSetAttribute(k_rows_pipe<MODE, KTM, NTN, TW>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
     ++g_launches;
-    launch_pdl(k_rows_pipe<MODE, KTM, NTN, TW>, dim3(unsigned(d.sms)), dim3(32 * nw), smem, st, a);
+    if (nw <= 8) {      // wide panels: few warps fit anyway -> let them keep every pointer in registers
+        cudaFuncSetAttribute(k_rows_pipe<MODE, KTM, NTN, TW, 256>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+        launch_pdl(k_rows_pipe<MODE, KTM, NTN, TW, 256>, dim3(unsigned(d.sms)), dim3(32 * nw), smem, st, a);
+    } else {
+        cudaFuncSetAttribute(k_rows_pipe<MODE, KTM, NTN, TW, 512>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+        launch_pdl(k_rows_pipe<MODE, KTM, NTN, TW, 512>, dim3(unsigned(d.sms)), dim3(32 * nw), smem, st, a);
+    }
     return true;
 }
 
@@ -373,14 +403,15 @@ __global__ void __launch_bounds__(512, 1) k_trsm_ring(StreamArgs a) {
     const int64_t g = int64_t(blockIdx.x) * nw + wp;
     const int64_t t0 = g * T / Wn, t1 = (g + 1) * T / Wn;
     const int c0 = a.c0;
+    const int part2 = 2 * (lane & 15), cfirst = lane >> 4;
+    const double* srcl = a.P + a.ldp * cfirst + part2;         // this lane's copy slots: columns
+    const int64_t cstride = 2 * a.ldp;                          // cfirst, cfirst + 2, ...
     auto issue = [&](int64_t t, int stage) {
         if (t < t1) {
-            double* dst = ring + stage * SD;
-            const int64_t r0 = t * 32;
-            for (int q = lane; q < W * 16; q += 32) {
-                const int c = q >> 4, part = q & 15;
-                ptx::cp_async16(dst + c * 32 + part * 2, a.P + a.ldp * c + r0 + part * 2);
-            }
+            double* dst = ring + stage * SD + cfirst * 32 + part2;
+            const double* src = srcl + t * 32;
+#pragma unroll
+            for (int c = cfirst; c < W; c += 2, dst += 64, src += cstride) ptx::cp_async16(dst, src);
         }
         ptx::cp_async_commit();
     };
@@ -399,6 +430,8 @@ __global__ void __launch_bounds__(512, 1) k_trsm_ring(StreamArgs a) {
     int stage = 0;
     for (int64_t t = t0; t < t1; ++t) {
         issue(t + RS - 1, stage == 0 ? RS - 1 : stage - 1);
+        if (a.pf && t + RS - 1 + ptx::PF_DIST < t1 && lane < 2 * W)
+            ptx::prefetch_l2(a.P + a.ldp * (lane >> 1) + (t + RS - 1 + ptx::PF_DIST) * 32 + 16 * (lane & 1));
         ptx::cp_async_wait<RS - 1>();
         __syncwarp();
         const double* sl = ring + stage * SD + lane;
@@ -473,7 +506,7 @@ void update(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, doubl
     // wide X (> 64 columns): P -= X[:, s] C[s, :] in 64-column slabs (C viewed with ld jx)
     for (int s0 = 0; s0 < jx; s0 += 64) {
         const int js = jx - s0 < 64 ? jx - s0 : 64;
-        StreamArgs a{n, X + ldx * s0, ldx, js, P, ldp, w, C + s0, jx, 0};
+        StreamArgs a{n, X + ldx * s0, ldx, js, P, ldp, w, C + s0, jx, 0, d.panel_pf};
         dispatch<0>(d, a, st);
     }
 }
@@ -482,7 +515,7 @@ int gemm_rows(const Dev& d, int64_t n, const double* X, int64_t ldx, int K, doub
               const double* M, int64_t ldm, int c0, cudaStream_t st) {
     if (n <= 0 || w <= 0) return 0;
     if (K > 64 || w > 32) return -1;
-    StreamArgs a{n, X, ldx, K, P, ldp, w, M, ldm, c0};
+    StreamArgs a{n, X, ldx, K, P, ldp, w, M, ldm, c0, d.panel_pf};
     return dispatch<2>(d, a, st);
 }
 
@@ -497,7 +530,7 @@ void trsm(const Dev& d, int64_t n, double* P, int64_t ldp, int w, const double* 
         launch_pdl(k_scale1, dim3(unsigned(g)), dim3(256), 0, st, n, P, R);
         return;
     }
-    StreamArgs a{n, nullptr, 0, 0, P, ldp, w, R, w, c0};
+    StreamArgs a{n, nullptr, 0, 0, P, ldp, w, R, w, c0, d.panel_pf};
     if (d.trsm_scalar && trsm_ring(d, a, st)) return;
     dispatch<1>(d, a, st);
 }

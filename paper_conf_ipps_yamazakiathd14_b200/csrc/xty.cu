@@ -39,6 +39,7 @@ struct XtyArgs {
     int fin_chol;
     double* R;
     int* status;
+    int pf = 0;                 // L2 prefetch ahead of the ring (Dev::panel_pf)
 };
 
 // ---- CTA partial -> two-level fixed-order total (+ Cholesky) ---------------------------
@@ -186,18 +187,19 @@ __global__ void __launch_bounds__(NT, 1) k_xty_pipe(XtyArgs a) {
     const int64_t t0 = g * T / W, t1 = (g + 1) * T / W;
     // columns: Y cols 0..w-1 at slot cols 0..w-1; X cols (if streamed) at w..w+nx-1
     const double* xbase = a.X == a.Y && !SYM ? a.Y + a.ldy * colbase : a.X + a.ldx * colbase;
-    auto colptr = [&](int c) -> const double* {
-        return c < w ? a.Y + a.ldy * c : xbase + a.ldx * (c - w);
-    };
+    __shared__ const double* sCol[96];                             // column base pointers
+    for (int c = threadIdx.x; c < ncol; c += blockDim.x) sCol[c] = c < w ? a.Y + a.ldy * c : xbase + a.ldx * (c - w);
+    __syncthreads();
+    auto colptr = [&](int c) -> const double* { return sCol[c]; };
     constexpr int CPC = TW * 8 / 16;                               // 16-B chunks per column
+    constexpr int CSTEP = 32 / CPC;
+    const int part2 = 2 * (lane % CPC), cfirst = lane / CPC;
     auto issue = [&](int64_t t, int stage) {
         if (t < t1) {
-            double* dst = ring + stage * stage_d;
-            const int64_t r0 = t * TW;
-            for (int q = lane; q < ncol * CPC; q += 32) {
-                const int c = q / CPC, part = q - c * CPC;
-                ptx::cp_async16(dst + c * SP + part * 2, colptr(c) + r0 + part * 2);
-            }
+            double* dst = ring + stage * stage_d + part2;
+            const int64_t r0 = t * TW + part2;
+#pragma unroll 4
+            for (int c = cfirst; c < ncol; c += CSTEP) ptx::cp_async16(dst + c * SP, sCol[c] + r0);
         }
         ptx::cp_async_commit();
     };
@@ -219,6 +221,11 @@ __global__ void __launch_bounds__(NT, 1) k_xty_pipe(XtyArgs a) {
     int stage = 0;
     for (int64_t t = t0; t < t1; ++t) {
         issue(t + PIPE_S - 1, (stage + PIPE_S - 1) % PIPE_S);
+        if (a.pf && TW == 32 && ncol <= 24 && t + PIPE_S - 1 + ptx::PF_DIST < t1) {   // narrow panels only
+            const int64_t rp = (t + PIPE_S - 1 + ptx::PF_DIST) * TW;
+            constexpr int LPC = TW / 16;
+            for (int q = lane; q < ncol * LPC; q += 32) ptx::prefetch_l2(colptr(q / LPC) + rp + 16 * (q % LPC));
+        }
         ptx::cp_async_wait<PIPE_S - 1>();
         __syncwarp();
         const double* sl = ring + stage * stage_d;
@@ -394,12 +401,12 @@ int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const dou
     if (jx <= 0 || w <= 0 || w > 32 || n < 0) return -1;
     const bool same = (X == Y) && (ldx == ldy) && (jx == w);
     if (same && d.gram == 1 && size_t(d.sms) * w * w * 2 <= ws.cap) {
-        GramArgs g{n, X, ldx, w, ws.part, out, ws.counter, fin_chol ? 1 : 0, R, status};
+        GramArgs g{n, X, ldx, w, d.panel_pf, ws.part, out, ws.counter, fin_chol ? 1 : 0, R, status};
         if (gram_dfma(d, g, st) == 0) return 0;
     }
     Geo o = geometry(d, n, jx, w, same);
     if (size_t(o.gx) * o.gy * o.chunk * w * 2 > ws.cap || o.gy * TR_CNT > XTY_COUNTERS) return -1;
-    XtyArgs a{n, X, ldx, jx, Y, ldy, w, o.chunk, ws.part, out, ws.counter, fin_chol ? 1 : 0, R, status};
+    XtyArgs a{n, X, ldx, jx, Y, ldy, w, o.chunk, ws.part, out, ws.counter, fin_chol ? 1 : 0, R, status, d.panel_pf};
     const bool aligned = ((reinterpret_cast<uintptr_t>(X) | reinterpret_cast<uintptr_t>(Y)) % 16 == 0) &&
                          (ldx % 2 == 0) && (ldy % 2 == 0);
     if (aligned && n >= 32 * 64) {
