@@ -29,39 +29,52 @@ __device__ __forceinline__ void chol_upper_serial(const double* G, int ldg, int 
 
 namespace kern {
 
-// Same factorization by one full warp (right-looking; lane c owns column c of the upper
-// triangle, w <= 32).  Trailing updates G[i][c] -= R[k][i] R[k][c] are applied for
-// k = 0, 1, ... in the order chol_upper_serial's fma chain uses, so R is bitwise identical.
-// sm: w*w doubles of shared memory (scratch).  Must be called by all 32 lanes of a warp.
-__device__ __forceinline__ void chol_upper_warp(const double* G, int ldg, int w, double* R, int* status,
+// Same factorization by one full warp, register-resident (right-looking; lane c owns column c
+// of the upper triangle in registers, w <= WM <= 32).  Step k: the pivot comes from lane k by
+// shuffle, inv = rsqrt(pivot) (one MUFU + Newton steps; R[k][k] = pivot * inv), row k is scaled
+// by inv, and the trailing update g[i] -= R[k][i] R[k][c] takes R[k][i] from lane i by shuffle
+// — no shared-memory round trips or divisions on the serial chain (the shared-memory version
+// cost ~3-5 us in the Gram kernel's last CTA).  Writes R (w x w, ld w, zeros below the
+// diagonal) to R and to sm.  Must be called by all 32 lanes of a warp.
+template <int WM>
+__device__ __forceinline__ void chol_upper_regs(const double* G, int ldg, int w, double* R, int* status,
                                                 double* sm) {
     const int lane = threadIdx.x & 31;
-    for (int q = lane; q < w * w; q += 32) {
-        const int i = q % w, c = q / w;
-        sm[q] = i <= c ? G[i + ldg * c] : 0.0;
-    }
-    __syncwarp();
+    double g[WM];
+#pragma unroll
+    for (int i = 0; i < WM; ++i) g[i] = (i <= lane && lane < w) ? G[i + ldg * lane] : 0.0;
     bool bad = false;
-    for (int k = 0; k < w; ++k) {
-        double dkk = sm[k + w * k];
+#pragma unroll
+    for (int k = 0; k < WM; ++k) {
+        if (k >= w) break;
+        double dkk = __shfl_sync(0xffffffffu, g[k], k);
         if (!(dkk > 0.0)) { bad = true; dkk = DBL_MIN; }
-        const double rkk = sqrt(dkk);
-        const double inv = 1.0 / rkk;
-        __syncwarp();
-        if (lane == k) sm[k + w * k] = rkk;
-        if (lane > k && lane < w) sm[k + w * lane] *= inv;            // R[k][c]
-        __syncwarp();
-        if (lane > k && lane < w) {
-            const double rkc = sm[k + w * lane];
-            for (int i = k + 1; i <= lane; ++i) sm[i + w * lane] = fma(-sm[k + w * i], rkc, sm[i + w * lane]);
+        const double inv = rsqrt(dkk);
+        if (lane == k) g[k] = dkk * inv;
+        else if (lane > k) g[k] *= inv;                             // R[k][lane]
+#pragma unroll
+        for (int i = k + 1; i < WM; ++i) {
+            if (i >= w) break;
+            const double rki = __shfl_sync(0xffffffffu, g[k], i);  // R[k][i]
+            if (lane >= i) g[i] = fma(-rki, g[k], g[i]);
         }
-        __syncwarp();
     }
-    for (int q = lane; q < w * w; q += 32) {
-        const int i = q % w, c = q / w;
-        R[q] = i <= c ? sm[q] : 0.0;
+    if (lane < w) {
+#pragma unroll
+        for (int i = 0; i < WM; ++i)
+            if (i < w) {
+                const double v = i <= lane ? g[i] : 0.0;
+                R[i + w * lane] = v;
+                sm[i + w * lane] = v;
+            }
     }
     if (bad && lane == 0) atomicOr(status, ST_CHOL);
+}
+
+__device__ __forceinline__ void chol_upper_warp(const double* G, int ldg, int w, double* R, int* status,
+                                                double* sm) {
+    if (w <= 12) chol_upper_regs<12>(G, ldg, w, R, status, sm);
+    else chol_upper_regs<32>(G, ldg, w, R, status, sm);
 }
 
 }  // namespace kern

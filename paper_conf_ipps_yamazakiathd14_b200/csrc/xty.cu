@@ -228,13 +228,21 @@ __global__ void __launch_bounds__(NT, 1) k_xty_pipe(XtyArgs a) {
         }
         ptx::cp_async_wait<PIPE_S - 1>();
         __syncwarp();
-        const double* sl = ring + stage * stage_d;
+        const double* sl = ring + stage * stage_d + tig;
+        // per-tile fragment pointers: the unrolled k-steps below load [register + immediate]
+        const double* sy[NTN];
+#pragma unroll
+        for (int nt = 0; nt < NTN; ++nt) sy[nt] = sl + ycol[nt] * SP;
+        const double* sx[SYM ? 1 : MT];
+        if constexpr (!SYM) {
+#pragma unroll
+            for (int mt = 0; mt < MT; ++mt) sx[mt] = sl + xcol[mt] * SP;
+        }
 #pragma unroll
         for (int u = 0; u < TW / 4; ++u) {
-            const int row = 4 * u + tig;
             double bn[NTN];
 #pragma unroll
-            for (int nt = 0; nt < NTN; ++nt) bn[nt] = sl[ycol[nt] * SP + row];
+            for (int nt = 0; nt < NTN; ++nt) bn[nt] = sy[nt][4 * u];
             if constexpr (SYM) {
 #pragma unroll
                 for (int mt = 0; mt < MT; ++mt)
@@ -243,7 +251,7 @@ __global__ void __launch_bounds__(NT, 1) k_xty_pipe(XtyArgs a) {
             } else {
 #pragma unroll
                 for (int mt = 0; mt < MT; ++mt) {
-                    const double am = sl[xcol[mt] * SP + row];
+                    const double am = sx[mt][4 * u];
 #pragma unroll
                     for (int nt = 0; nt < NTN; ++nt) ptx::dmma(acc[mt][nt][0], acc[mt][nt][1], am, bn[nt]);
                 }
