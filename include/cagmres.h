@@ -136,7 +136,8 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
  *                          common DIA slice width, >= 3/4/5/6 CTAs per SM; 14, 15 = the same with
  *                          CTA-contiguous slice ranges (L1 reuse of x), 4/5 CTAs per SM; 16, 17 =
  *                          10..13's kernel with an L2 prefetch of the next slice's values, 4/5
- *                          CTAs per SM.  All variants are bitwise identical.
+ *                          CTAs per SM; 18 = prefetch two slices ahead.  All variants are bitwise
+ *                          identical.
  *   CAGMRES_OPT_GRAM     : CholQR Gram kernel: 0 = FP64 tensor core (DMMA m8n8k4) on a per-warp
  *                          cp.async ring; 1 (default) = scalar DFMA on a deeper ring (w <= 12,
  *                          else the DMMA kernel).

@@ -68,20 +68,27 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
         sl = (int64_t(blockIdx.x) * DT_NT + threadIdx.x) >> 5;
     }
     if (sl >= nsl) { pdl_wait(); pdl_trigger(); return; }
-    int64_t b0, i0, b1 = 0, i1 = 1, b2, i2;
-    int W0, W1 = 0, W2, o0, o1;
+    int64_t b0, i0, b1 = 0, i1 = 1, b2 = 0, i2 = 1, b3, i3;
+    int W0, W1 = 0, W2 = 0, W3, o0, o1;
     // slice descriptors (static during a solve) are loaded before the PDL wait
     sell_slice_meta(sl, a.sptr, a.sinfo, b0, W0, i0);
     if (sl + stride < nsl) sell_slice_meta(sl + stride, a.sptr, a.sinfo, b1, W1, i1);
+    if (PF == 2 && sl + 2 * stride < nsl) sell_slice_meta(sl + 2 * stride, a.sptr, a.sinfo, b2, W2, i2);
     o0 = sell_slice_off(lane, W0, i0, a.dcol);
     pdl_wait();
     pdl_trigger();
 #pragma unroll 1
     for (; sl < nsl; sl += stride) {
-        b2 = 0; W2 = 0; i2 = 1;
-        if (sl + 2 * stride < nsl) sell_slice_meta(sl + 2 * stride, a.sptr, a.sinfo, b2, W2, i2);
+        if (PF == 2) {                                                   // 3-deep descriptor pipeline
+            b3 = 0; W3 = 0; i3 = 1;
+            if (sl + 3 * stride < nsl) sell_slice_meta(sl + 3 * stride, a.sptr, a.sinfo, b3, W3, i3);
+            if (lane < 2 * W2) prefetch_l2(a.val + b2 + 16 * lane);      // 128-B lines of slice +2
+        } else {
+            b2 = 0; W2 = 0; i2 = 1;
+            if (sl + 2 * stride < nsl) sell_slice_meta(sl + 2 * stride, a.sptr, a.sinfo, b2, W2, i2);
+        }
         o1 = sell_slice_off(lane, W1, i1, a.dcol);
-        if (PF && lane < 2 * W1) prefetch_l2(a.val + b1 + 16 * lane);     // 128-B lines of slice +1
+        if (PF == 1 && lane < 2 * W1) prefetch_l2(a.val + b1 + 16 * lane);     // 128-B lines of slice +1
         const int64_t r = sl * 32 + lane;
         const bool live = r < a.nrows;
         double uu = 0.0, ww = 0.0, acc = 0.0;
@@ -92,7 +99,7 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
 #pragma unroll
             for (int t = 0; t < WT; ++t) {
                 const int o = __shfl_sync(0xffffffffu, o0, t);
-                v[t] = CONTIG ? ldg_stream(vp + 32 * t) : __ldg(vp + 32 * t);
+                v[t] = (CONTIG || PF) ? ldg_stream(vp + 32 * t) : __ldg(vp + 32 * t);
                 xv[t] = __ldg(xr + o);
             }
             if (MODE >= 1 && live) uu = __ldg(a.u + r);
@@ -117,6 +124,7 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
         }
         b0 = b1; W0 = W1; i0 = i1; o0 = o1;
         b1 = b2; W1 = W2; i1 = i2;
+        if (PF == 2) { b2 = b3; W2 = W3; i2 = i3; }
     }
 }
 
@@ -157,7 +165,8 @@ void go_width(const Dev& d, const DiaArgs& a, int wt, cudaStream_t st, int mode)
 
 // variants 10 / 11 / 12 / 13: at least 3 / 4 / 5 / 6 CTAs per SM (register cap), grid-strided
 // slices; 14 / 15: 4 / 5 CTAs per SM, CTA-contiguous slice ranges (L1 reuse of x); 16 / 17:
-// 4 / 5 CTAs per SM, grid-strided, L2 prefetch of the next slice's values
+// 4 / 5 CTAs per SM, grid-strided, L2 prefetch of the next slice's values (L1::no_allocate value
+// loads); 18: 4 CTAs per SM, prefetch two slices ahead (3-deep descriptor pipeline)
 void spmv_dia(const Dev& d, const Sell& A, int variant, int64_t nrows, const double* x, double* y,
               const double* u, double bu, const double* w, double bw, int mode, cudaStream_t st) {
     DiaArgs a{nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, u, bu, w, bw, y};
@@ -169,6 +178,7 @@ void spmv_dia(const Dev& d, const Sell& A, int variant, int64_t nrows, const dou
         case 15: go_width<5, 1>(d, a, A.dia_w, st, mode); break;
         case 16: go_width<4, 0, 1>(d, a, A.dia_w, st, mode); break;
         case 17: go_width<5, 0, 1>(d, a, A.dia_w, st, mode); break;
+        case 18: go_width<4, 0, 2>(d, a, A.dia_w, st, mode); break;
         default: go_width<6, 0>(d, a, A.dia_w, st, mode); break;
     }
 }
