@@ -95,7 +95,7 @@ __global__ void __launch_bounds__(512, 1) k_arnoldi_ring(ArnoldiArgs a) {
     const int jx = a.jx;
     for (int i = threadIdx.x; i < JX; i += blockDim.x) sc[i] = (MODE != 0 && i < jx) ? a.c_in[i] : 0.0;
     __syncthreads();
-    constexpr int NA = MODE == 2 ? 1 : JX;
+    constexpr int NA = (MODE == 2 || MODE == 3) ? 1 : JX;      // MODE 3: update only (x += V y)
     double acc[NA];
 #pragma unroll
     for (int i = 0; i < NA; ++i) acc[i] = 0.0;
@@ -127,11 +127,11 @@ __global__ void __launch_bounds__(512, 1) k_arnoldi_ring(ArnoldiArgs a) {
                 if (i < jx) vv = fma(-sq[i * 32], sc[i], vv);
             if (jx > 0) a.v[r] = vv;
         }
-        if constexpr (MODE != 2) {
+        if constexpr (MODE == 0 || MODE == 1) {
 #pragma unroll
             for (int i = 0; i < JX; ++i)
                 if (i < jx) acc[i] = fma(sq[i * 32], vv, acc[i]);
-        } else {
+        } else if constexpr (MODE == 2) {
             acc[0] = fma(vv, vv, acc[0]);
         }
     };
@@ -161,6 +161,7 @@ __global__ void __launch_bounds__(512, 1) k_arnoldi_ring(ArnoldiArgs a) {
             row(sl, a.v[r], r);
         }
     }
+    if constexpr (MODE == 3) return;                           // no reduction
 #pragma unroll
     for (int i = 0; i < NA; ++i) {
         double x = acc[i];
@@ -201,6 +202,16 @@ bool go_ring(const Dev& d, const ArnoldiArgs& a, cudaStream_t st) {
     return true;
 }
 }  // namespace
+
+// p -= X c for a single column p (x += V y at the end of a cycle): the ring kernel's
+// update-only mode, one lane per row (a DMMA tile would waste 7/8 of its columns).
+int update_w1(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, double* p, const double* c,
+              cudaStream_t st) {
+    if (!d.arnoldi_ring || jx < 1 || jx > 32) return -1;
+    ArnoldiArgs a{d.panel_pf, n, X, ldx, jx, p, c, nullptr, nullptr, nullptr, nullptr, 0};
+    const bool ok = jx <= 8 ? go_ring<8, 3>(d, a, st) : (jx <= 16 ? go_ring<16, 3>(d, a, st) : go_ring<32, 3>(d, a, st));
+    return ok ? 0 : -1;
+}
 
 int arnoldi_fused(const Dev& d, const ArnoldiArgs& a, int mode, cudaStream_t st) {
     if (a.jx < (mode == 2 ? 0 : 1) || a.jx > 32) return -1;   // wider: caller uses unfused passes

@@ -207,6 +207,9 @@ struct ArnoldiArgs {
     int sqrt_out;
 };
 int arnoldi_fused(const Dev& d, const ArnoldiArgs& a, int mode, cudaStream_t st);
+// p -= X c, p a single column (n), X n x jx (jx <= 32), c device jx-vector; -1 if not applicable
+int update_w1(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, double* p, const double* c,
+              cudaStream_t st);
 size_t arnoldi_ws_doubles(const Dev& d);
 
 // TSQR by CAQR (caqr.cu): P (n x w, w <= 32) := Q (columns >= c0 written), R (w x w, ld w,

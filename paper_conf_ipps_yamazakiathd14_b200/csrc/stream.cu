@@ -389,12 +389,16 @@ template <int W, int RS>
 __global__ void __launch_bounds__(512, 1) k_trsm_ring(StreamArgs a) {
     extern __shared__ __align__(16) double smt[];
     __shared__ double sB[32 * 32 + 32];
-    __shared__ double sRi[W * W];
+    constexpr int WP = W + (W & 1);                             // even row stride: 16-B pairs
+    __shared__ __align__(16) double sRi[W * WP];
     const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5, nw = blockDim.x >> 5;
     pdl_wait();
     pdl_trigger();
     upper_inverse(a.M, W, sB, sB + 32 * 32);
-    for (int q = threadIdx.x; q < W * W; q += blockDim.x) sRi[q] = sB[(q / W) * 32 + (q % W)];   // [k*W + c]
+    for (int q = threadIdx.x; q < W * WP; q += blockDim.x) {
+        const int k = q / WP, c = q - k * WP;
+        sRi[q] = c < W ? sB[k * 32 + c] : 0.0;                 // [k * WP + c] = R^{-1}[k][c]
+    }
     __syncthreads();
     constexpr int SD = W * 32;
     double* ring = smt + int64_t(wp) * RS * SD;
@@ -415,14 +419,21 @@ __global__ void __launch_bounds__(512, 1) k_trsm_ring(StreamArgs a) {
         }
         ptx::cp_async_commit();
     };
+    // two output columns per 16-B broadcast load of R^{-1}: out[c], out[c+1] = sum_k p[k] Ri[k][.]
+    // (Ri[c+1][c] = 0: the extra term adds an exact zero)
     auto rowout = [&](const double (&v)[W], double* out) {
 #pragma unroll
-        for (int c = 0; c < W; ++c) {
-            if (c < c0) continue;
-            double acc = 0.0;
+        for (int c = 0; c < W; c += 2) {
+            if (c + 1 < c0) continue;
+            double acc0 = 0.0, acc1 = 0.0;
 #pragma unroll
-            for (int k = 0; k <= c; ++k) acc = fma(v[k], sRi[k * W + c], acc);
-            out[a.ldp * c] = acc;
+            for (int k = 0; k <= c + 1 && k < W; ++k) {
+                const double2 r2 = *reinterpret_cast<const double2*>(&sRi[k * WP + c]);
+                acc0 = fma(v[k], r2.x, acc0);
+                acc1 = fma(v[k], r2.y, acc1);
+            }
+            if (c >= c0) out[a.ldp * c] = acc0;
+            if (c + 1 < W) out[a.ldp * (c + 1)] = acc1;
         }
     };
 #pragma unroll
@@ -503,6 +514,7 @@ bool trsm_ring(const Dev& d, const StreamArgs& a, cudaStream_t st) {
 void update(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, double* P,
             int64_t ldp, int w, const double* C, cudaStream_t st) {
     if (n <= 0 || w <= 0) return;
+    if (w == 1 && jx <= 32 && update_w1(d, n, X, ldx, jx, P, C, st) == 0) return;
     // wide X (> 64 columns): P -= X[:, s] C[s, :] in 64-column slabs (C viewed with ld jx)
     for (int s0 = 0; s0 < jx; s0 += 64) {
         const int js = jx - s0 < 64 ? jx - s0 : 64;
