@@ -203,13 +203,22 @@ bool go_ring(const Dev& d, const ArnoldiArgs& a, cudaStream_t st) {
 }
 }  // namespace
 
+// JX buckets of 8: the per-row loops are unrolled to JX with predicates i < jx
+template <int MODE>
+bool ring_dispatch(const Dev& d, const ArnoldiArgs& a, cudaStream_t st) {
+    if (a.jx <= 8) return go_ring<8, MODE>(d, a, st);
+    if (a.jx <= 16) return go_ring<16, MODE>(d, a, st);
+    if (a.jx <= 24) return go_ring<24, MODE>(d, a, st);
+    return go_ring<32, MODE>(d, a, st);
+}
+
 // p -= X c for a single column p (x += V y at the end of a cycle): the ring kernel's
 // update-only mode, one lane per row (a DMMA tile would waste 7/8 of its columns).
 int update_w1(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, double* p, const double* c,
               cudaStream_t st) {
     if (!d.arnoldi_ring || jx < 1 || jx > 32) return -1;
     ArnoldiArgs a{d.panel_pf, n, X, ldx, jx, p, c, nullptr, nullptr, nullptr, nullptr, 0};
-    const bool ok = jx <= 8 ? go_ring<8, 3>(d, a, st) : (jx <= 16 ? go_ring<16, 3>(d, a, st) : go_ring<32, 3>(d, a, st));
+    const bool ok = ring_dispatch<3>(d, a, st);
     return ok ? 0 : -1;
 }
 
@@ -217,9 +226,9 @@ int arnoldi_fused(const Dev& d, const ArnoldiArgs& a, int mode, cudaStream_t st)
     if (a.jx < (mode == 2 ? 0 : 1) || a.jx > 32) return -1;   // wider: caller uses unfused passes
     if (d.arnoldi_ring) {
         bool ok;
-        if (mode == 0) ok = a.jx <= 8 ? go_ring<8, 0>(d, a, st) : (a.jx <= 16 ? go_ring<16, 0>(d, a, st) : go_ring<32, 0>(d, a, st));
-        else if (mode == 1) ok = a.jx <= 8 ? go_ring<8, 1>(d, a, st) : (a.jx <= 16 ? go_ring<16, 1>(d, a, st) : go_ring<32, 1>(d, a, st));
-        else ok = a.jx <= 8 ? go_ring<8, 2>(d, a, st) : (a.jx <= 16 ? go_ring<16, 2>(d, a, st) : go_ring<32, 2>(d, a, st));
+        if (mode == 0) ok = ring_dispatch<0>(d, a, st);
+        else if (mode == 1) ok = ring_dispatch<1>(d, a, st);
+        else ok = ring_dispatch<2>(d, a, st);
         if (ok) return 0;
     }
     const int64_t blocks = (a.n + NT - 1) / NT;
