@@ -249,6 +249,18 @@ int cagmres_plan_set_sends(cagmres_plan_t p, const int64_t* counts, const int64_
 /* Send lists: owned local indices in request order (host, total = sum counts). */
 int cagmres_plan_send_index(cagmres_plan_t p, int64_t* local_idx);
 
+/* ---- host-only reordering for the row partition ------- */
+/* Reverse Cuthill-McKee order of the symmetrised pattern of A (n x n CSR, host): perm[new] =
+ * old.  Each connected component starts at a pseudo-peripheral node (repeated BFS from a
+ * minimum-degree node of the deepest level); neighbours are visited by increasing (degree,
+ * id); the Cuthill-McKee order is reversed.  Errors: EINVAL (column id out of range). */
+int cagmres_host_rcm(int64_t n, const int64_t* rowptr, const int32_t* colind, int64_t* perm);
+/* B = P A P^T: row i of B is row perm[i] of A with columns renumbered by the inverse
+ * permutation and sorted.  Output arrays caller-owned (out_rowptr n+1, out_colind/out_val nnz).
+ * Errors: EINVAL (perm not a permutation of 0..n-1, column out of range). */
+int cagmres_host_permute(int64_t n, const int64_t* rowptr, const int32_t* colind, const double* val,
+                         const int64_t* perm, int64_t* out_rowptr, int32_t* out_colind, double* out_val);
+
 /* ---- host-only small dense algorithms of the cycle (exported for tests) -------------- */
 /* Eigenvalues (Ritz values) of the upper Hessenberg H (m x m, ld ldh), Francis
  * double-shift QR; conjugate pairs returned adjacent (+im first).  EBREAKDOWN if the QR

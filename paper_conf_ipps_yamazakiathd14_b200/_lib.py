@@ -80,6 +80,8 @@ SIGNATURES = {
     "cagmres_plan_set_sends": ([_P, _PI64, _PI64, _PI32], C.c_int),
     "cagmres_plan_send_index": ([_P, _PI64], C.c_int),
     "cagmres_host_eigvals": ([_PD, C.c_int, C.c_int, _PD, _PD], C.c_int),
+    "cagmres_host_rcm": ([_I64, _PI64, _PI32, _PI64], C.c_int),
+    "cagmres_host_permute": ([_I64, _PI64, _PI32, _PD, _PI64, _PI64, _PI32, _PD], C.c_int),
     "cagmres_host_leja": ([_PD, _PD, C.c_int, C.c_int, _PD, _PD, C.c_int, C.POINTER(C.c_int)], C.c_int),
     "cagmres_host_change_of_basis": ([_PD, _PD, C.c_int, _PD], C.c_int),
     "cagmres_host_hessenberg_update": ([_PD, C.c_int, C.c_int, C.c_int, _PD, C.c_int, _PD], C.c_int),

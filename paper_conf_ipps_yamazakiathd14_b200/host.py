@@ -122,3 +122,31 @@ def givens_ls(H, beta):
     L.check(lib.cagmres_host_givens_ls(Hf.ctypes.data_as(L._PD), Hf.shape[0], k, float(beta),
                                        L.dptr(y), L.dptr(res)), "givens_ls")
     return y, res
+
+
+def rcm(A):
+    """Reverse Cuthill-McKee permutation (perm[new] = old) of the symmetrised pattern of the
+    n x n host CSR A (cagmres_host_rcm; NEXT-4 reordering for the MPK row partition)."""
+    lib = L.load()
+    rp = np.ascontiguousarray(A.rowptr, dtype=np.int64)
+    ci = np.ascontiguousarray(A.colind, dtype=np.int32)
+    perm = np.zeros(A.n, dtype=np.int64)
+    L.check(lib.cagmres_host_rcm(int(A.n), L.i64ptr(rp), ci.ctypes.data_as(L._PI32), L.i64ptr(perm)), "rcm")
+    return perm
+
+
+def permute(A, perm):
+    """B = P A P^T (cagmres_host_permute); returns a CSR of the same type as A."""
+    import dataclasses
+    lib = L.load()
+    rp = np.ascontiguousarray(A.rowptr, dtype=np.int64)
+    ci = np.ascontiguousarray(A.colind, dtype=np.int32)
+    va = np.ascontiguousarray(A.val, dtype=np.float64)
+    pm = np.ascontiguousarray(perm, dtype=np.int64)
+    orp = np.zeros(A.n + 1, dtype=np.int64)
+    oci = np.zeros(len(ci), dtype=np.int32)
+    ova = np.zeros(len(va), dtype=np.float64)
+    L.check(lib.cagmres_host_permute(int(A.n), L.i64ptr(rp), ci.ctypes.data_as(L._PI32), L.dptr(va),
+                                     L.i64ptr(pm), L.i64ptr(orp), oci.ctypes.data_as(L._PI32), L.dptr(ova)),
+            "permute")
+    return dataclasses.replace(A, rowptr=orp, colind=oci, val=ova)

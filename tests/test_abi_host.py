@@ -158,3 +158,45 @@ def test_plan_reports_missing_ghost_rows():
     with pytest.raises(L.CagmresError) as e:
         Plan(part, rs, 0, 3)                                        # s=3 needs 2 hops
     assert e.value.status == L.EGHOST
+
+
+# ----------------------------------------------------------------------------- NEXT-4 reordering
+def _bandwidth(S):
+    S = S.tocoo()
+    return int(np.max(np.abs(S.row - S.col))) if S.nnz else 0
+
+
+def test_rcm_restores_small_bandwidth_and_permute_matches_scipy():
+    """cagmres_host_rcm on a randomly permuted 2-D 5-pt grid: a valid permutation whose
+    bandwidth is within 10 % of SciPy's RCM (independent implementation); cagmres_host_permute
+    equals SciPy's P A P^T exactly."""
+    import scipy.sparse as sp
+    from scipy.sparse.csgraph import reverse_cuthill_mckee
+    from paper_conf_ipps_yamazakiathd14_b200 import host
+    A = G.convection_diffusion(40, 2, 5)
+    As = A.to_scipy()
+    rnd = np.argsort(G.u(77, np.arange(A.n)))
+    Ar = host.permute(A, rnd)                                   # scrambled
+    Ars = Ar.to_scipy()
+    assert (abs(Ars - As[rnd][:, rnd]) > 0).nnz == 0
+    p = host.rcm(Ar)
+    assert np.array_equal(np.sort(p), np.arange(A.n))
+    B = host.permute(Ar, p).to_scipy()
+    pr = reverse_cuthill_mckee(sp.csr_matrix(Ars), symmetric_mode=False)
+    assert _bandwidth(B) <= 1.1 * _bandwidth(Ars[pr][:, pr]) + 2
+    assert _bandwidth(B) < _bandwidth(Ars) / 10
+    assert (abs(B - Ars[p][:, p]) > 0).nnz == 0
+
+
+def test_rcm_disconnected_and_isolated_nodes():
+    """Two components plus isolated rows: every node appears exactly once."""
+    from paper_conf_ipps_yamazakiathd14_b200 import host
+    A1 = G.convection_diffusion(6, 2, 5).to_scipy()
+    import scipy.sparse as sp
+    S = sp.block_diag([A1, sp.identity(3), A1]).tocsr()
+    C = G.CSR(n=S.shape[0], row_begin=0, rowptr=S.indptr.astype(np.int64),
+              colind=S.indices.astype(np.int32), val=S.data.astype(np.float64))
+    p = host.rcm(C)
+    assert np.array_equal(np.sort(p), np.arange(C.n))
+    with pytest.raises(Exception):
+        host.permute(C, np.zeros(C.n, dtype=np.int64))          # not a permutation -> EINVAL
