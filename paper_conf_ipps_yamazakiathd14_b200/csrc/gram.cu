@@ -169,9 +169,120 @@ __global__ void __launch_bounds__(GR_NT, 1) k_gram_ring(GramArgs a) {
     }
 }
 
+// Per-warp variant (CAGMRES_OPT_GRAM = 2): every warp streams its own 32-row tiles through a
+// private cp.async ring (no pair barrier) and accumulates all W(W+1)/2 sums for its lane's row
+// (up to 78 accumulators: 8 warps per SM at <= 255 registers).
+constexpr int GW_NW = 8, GW_S = 4;
+template <int W>
+__global__ void __launch_bounds__(GW_NW * 32, 1) k_gram_warp(GramArgs a) {
+    extern __shared__ __align__(16) double smg[];
+    constexpr int NE = W * (W + 1) / 2;
+    __shared__ double red[GW_NW * NE];
+    const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5;
+    pdl_wait();
+    pdl_trigger();
+    constexpr int SD = W * 32;
+    double* ring = smg + int64_t(wp) * GW_S * SD;
+    const int64_t T = a.n / 32;
+    const int64_t Wn = int64_t(gridDim.x) * GW_NW;
+    const int64_t g = int64_t(blockIdx.x) * GW_NW + wp;
+    const int64_t t0 = g * T / Wn, t1 = (g + 1) * T / Wn;
+    const int part2 = 2 * (lane & 15), cfirst = lane >> 4;
+    const double* srcl = a.P + a.ldp * cfirst + part2;
+    const int64_t cstride = 2 * a.ldp;
+    auto issue = [&](int64_t t, int stage) {
+        if (t < t1) {
+            double* dst = ring + stage * SD + cfirst * 32 + part2;
+            const double* src = srcl + t * 32;
+#pragma unroll
+            for (int c = cfirst; c < W; c += 2, dst += 64, src += cstride) ptx::cp_async16(dst, src);
+        }
+        ptx::cp_async_commit();
+    };
+    double acc[NE];
+#pragma unroll
+    for (int e = 0; e < NE; ++e) acc[e] = 0.0;
+    auto rank1 = [&](const double* sl) {
+        double v[W];
+#pragma unroll
+        for (int c = 0; c < W; ++c) v[c] = sl[c * 32];
+        int e = 0;
+#pragma unroll
+        for (int i = 0; i < W; ++i)
+#pragma unroll
+            for (int k = i; k < W; ++k, ++e) acc[e] = fma(v[i], v[k], acc[e]);
+    };
+#pragma unroll
+    for (int s = 0; s < GW_S - 1; ++s) issue(t0 + s, s);
+    int stage = 0;
+    for (int64_t t = t0; t < t1; ++t) {
+        issue(t + GW_S - 1, stage == 0 ? GW_S - 1 : stage - 1);
+        ptx::cp_async_wait<GW_S - 1>();
+        __syncwarp();
+        rank1(ring + stage * SD + lane);
+        __syncwarp();
+        stage = stage == GW_S - 1 ? 0 : stage + 1;
+    }
+    ptx::cp_async_wait<0>();
+    if (blockIdx.x == 0 && wp == 0 && T * 32 + lane < a.n) {      // ragged tail rows [32 T, n)
+        double* sl = ring + lane;
+        const int64_t r = T * 32 + lane;
+        for (int c = 0; c < W; ++c) sl[c * 32] = a.P[a.ldp * c + r];
+        rank1(sl);
+    }
+#pragma unroll
+    for (int e = 0; e < NE; ++e) {
+        double sum = acc[e];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+        if (lane == 0) red[wp * NE + e] = sum;
+    }
+    __syncthreads();
+    constexpr int nent = W * W;
+    double* part = a.part + int64_t(blockIdx.x) * nent;
+    for (int q = threadIdx.x; q < nent; q += blockDim.x) {
+        int i = q % W, k = q / W;
+        if (i > k) { const int tt = i; i = k; k = tt; }
+        const int e = i * W - i * (i - 1) / 2 + (k - i);
+        double s = 0.0;
+#pragma unroll
+        for (int u = 0; u < GW_NW; ++u) s += red[u * NE + e];
+        part[q] = s;
+    }
+    const bool fin = tree_reduce(a.part, a.part + int64_t(gridDim.x) * nent, int(gridDim.x), int(blockIdx.x),
+                                 nent, nent, a.counter, [&](int q, double tot) { a.out[q] = tot; });
+    if (fin && a.fin_chol && threadIdx.x < 32) {
+        __threadfence_block();
+        chol_upper_warp(a.out, W, W, a.R, a.status, smg);
+    }
+}
+
+int gram_warp(const Dev& d, const GramArgs& a, cudaStream_t st) {
+    auto go = [&](auto kfn) {
+        size_t smem = size_t(GW_NW) * GW_S * a.w * 32 * sizeof(double);
+        const size_t need = size_t(32 * 32) * sizeof(double);
+        smem = smem < need ? need : smem;
+        cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+        ++g_launches;
+        launch_pdl(kfn, dim3(unsigned(d.sms)), dim3(GW_NW * 32), smem, st, a);
+    };
+    switch (a.w) {
+        case 6: go(k_gram_warp<6>); break;
+        case 7: go(k_gram_warp<7>); break;
+        case 8: go(k_gram_warp<8>); break;
+        case 9: go(k_gram_warp<9>); break;
+        case 10: go(k_gram_warp<10>); break;
+        case 11: go(k_gram_warp<11>); break;
+        case 12: go(k_gram_warp<12>); break;
+        default: return -1;
+    }
+    return 0;
+}
+
 int gram_dfma(const Dev& d, const GramArgs& a, cudaStream_t st) {
     const bool aligned = (reinterpret_cast<uintptr_t>(a.P) % 16 == 0) && a.ldp % 2 == 0;
     if (!aligned || a.w < 1 || a.w > 12 || a.n < 64 * GR_TW) return -1;
+    if (d.gram == 2 && gram_warp(d, a, st) == 0) return 0;
     auto go = [&](auto kfn, int S) {
         size_t smem = size_t(GR_NP) * S * a.w * GR_TW * sizeof(double);
         const size_t need = size_t(32 * 32) * sizeof(double);     // Cholesky scratch

@@ -961,7 +961,7 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
             if (value == -1) return spmv_autotune(h);
             h->A.variant = int(value);
             return CAGMRES_OK;
-        case CAGMRES_OPT_GRAM: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->dev.gram = int(value); return CAGMRES_OK;
+        case CAGMRES_OPT_GRAM: if (value < 0 || value > 2) return CAGMRES_EINVAL; h->dev.gram = int(value); return CAGMRES_OK;
         case CAGMRES_OPT_ARNOLDI: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->dev.arnoldi_ring = int(value); return CAGMRES_OK;
         case CAGMRES_OPT_PANEL_TW: if (value != 16 && value != 32) return CAGMRES_EINVAL; h->dev.panel_tw16 = value == 16; return CAGMRES_OK;
         case CAGMRES_OPT_TRSM: if (value < 0 || value > 4) return CAGMRES_EINVAL; h->dev.trsm_scalar = int(value); return CAGMRES_OK;

@@ -408,7 +408,7 @@ int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const dou
         const XtyWs& ws, cudaStream_t st) {
     if (jx <= 0 || w <= 0 || w > 32 || n < 0) return -1;
     const bool same = (X == Y) && (ldx == ldy) && (jx == w);
-    if (same && d.gram == 1 && size_t(d.sms) * w * w * 2 <= ws.cap) {
+    if (same && d.gram >= 1 && size_t(d.sms) * w * w * 2 <= ws.cap) {
         GramArgs g{n, X, ldx, w, d.panel_pf, ws.part, out, ws.counter, fin_chol ? 1 : 0, R, status};
         if (gram_dfma(d, g, st) == 0) return 0;
     }

@@ -179,7 +179,7 @@ def test_borth_parity(n, j, w):
 @pytest.mark.parametrize("kind,reorth", [("cholqr", False), ("cholqr", True), ("svqr", False),
                                          ("cgs", False), ("mgs", False), ("caqr", False)])
 @pytest.mark.parametrize("n,w", [(100002, 11), (100003, 11), (777, 6), (4096, 1), (20000, 16), (65538, 13)])
-@pytest.mark.parametrize("gram", [0, 1])
+@pytest.mark.parametrize("gram", [0, 1, 2])
 def test_tsqr_parity(kind, reorth, n, w, gram):
     """gram: CAGMRES_OPT_GRAM (0 = DMMA tensor-core Gram, 1 = scalar DFMA ring Gram)."""
     A = G.banded(n=n)
