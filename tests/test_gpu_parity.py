@@ -429,3 +429,26 @@ def test_clear_shifts_reruns_first_cycle_bitwise():
     assert np.array_equal(st3.hist, st1.hist) and torch.equal(x3, x1)
     assert np.array_equal(S.get_shifts()[0], sh1[0])
     assert st2.cycles >= 1
+
+
+def test_distributed_handle_single_rank_nccl_matches_single_gpu():
+    """cagmres_create_dist through a real NCCL communicator (one rank; this box has one GPU):
+    unique-id broadcast, plan, request exchange over NCCL, then a full Newton solve — bitwise
+    equal to the single-GPU handle (the multi-rank host logic is covered by test_dist_gloo)."""
+    import os
+    import torch.distributed as dist
+    os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+    os.environ.setdefault("MASTER_PORT", "29533")
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        A = G.convection_diffusion(40, 3, 7)
+        b = dev(G.rhs(A.n))
+        S1 = Solver(A, s=5, m=30, basis="newton")
+        x1, st1 = S1.solve(b, tol=1e-8, maxit=60)
+        S2 = Solver(A, s=5, m=30, basis="newton", group=dist.group.WORLD,
+                    row_starts=np.array([0, A.n], dtype=np.int64))
+        x2, st2 = S2.solve(b, tol=1e-8, maxit=60)
+        assert st2.status == 0 and st2.cycles == st1.cycles
+        assert np.array_equal(st2.hist, st1.hist) and torch.equal(x2, x1)
+    finally:
+        dist.destroy_process_group()
