@@ -3,7 +3,7 @@ PAPER.md Fig. 10 / Fig. 13: MPK panels W = [q, Aq, ..., A^s q
 s = 10 and s = 15, and the Newton basis), factored by every TSQR variant of the library.
 
 Reports per variant: ||I - Q^T Q||_2, ||W - QR||_F / ||W||_F, cond(W) (from R of CAQR),
-device time, algorithmic GB/s and the paper's "effective Gflop/s" = (4 n w^2 - 4 w^3 / 3) / t
+device time of one call after a warm-up call (includes the call's host synchronisation), algorithmic GB/s and the paper's "effective Gflop/s" = (4 n w^2 - 4 w^3 / 3) / t
 (DGEQRF + DORGQR flops).  Breakdowns are reported, not hidden.
 
     python tools/tsqr_study.py [--n 4194304] > profiles/r1_tsqr_study_C4.json
@@ -23,7 +23,12 @@ from synth import generators as G  # noqa: E402
 
 
 def measure(S, W, w, kind, reorth):
+    try:                                                  # warm-up (first-call set-up, caches)
+        S.tsqr(W.clone(), w, kind, reorth)
+    except L.CagmresError:
+        pass
     P = W.clone()
+    torch.cuda.synchronize()
     st = torch.cuda.current_stream()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(st)
