@@ -299,86 +299,106 @@ void chol(const double* G, int w, double* R, int* status, cudaStream_t st) {
 // SVQR (reading G14): D = diag(G)^{-1/2}; D G D = U S U^T (cyclic
 // Jacobi); s_i <- max(s_i, eps s_max); R_hat = R of qr(S^{1/2} U^T) (Householder, positive
 // diagonal); R = R_hat D^{-1}.  One thread, w <= 32 (a comparator-sized cost).
+// One warp: lane k owns row/column k of the w x w matrices (w <= 32).  Each Jacobi rotation's
+// (c, s) is computed redundantly by every lane from shared memory, then the two columns, the
+// two rows and V are updated lane-parallel; sums (off-diagonal norm, Householder norms and dot
+// products) are warp shuffle reductions.  (The one-thread version took ~0.5 ms at w = 11.)
+__device__ __forceinline__ double warp_sum(double v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
 __global__ void k_svqr(const double* G, int w, double* R, int* status) {
-    __shared__ double A[32 * 32], V[32 * 32], d[32];
-    if (threadIdx.x != 0) return;
-    for (int i = 0; i < w; ++i) {
-        const double g = G[i + w * i];
-        if (!(g > 0.0)) { atomicOr(status, ST_SVQR); d[i] = 1.0; } else d[i] = 1.0 / sqrt(g);
+    __shared__ double A[32 * 33], V[32 * 33], d[32];
+    constexpr int LD = 33;
+    const int k = threadIdx.x;                         // lane
+    pdl_wait();
+    pdl_trigger();
+    if (k < w) {
+        const double g = G[k + w * k];
+        if (!(g > 0.0)) { atomicOr(status, ST_SVQR); d[k] = 1.0; } else d[k] = 1.0 / sqrt(g);
     }
+    __syncwarp();
     for (int j = 0; j < w; ++j)
-        for (int i = 0; i < w; ++i) {
-            const double g = (i <= j) ? G[i + w * j] : G[j + w * i];
-            A[i + 32 * j] = d[i] * g * d[j];
-            V[i + 32 * j] = (i == j) ? 1.0 : 0.0;
+        if (k < w) {
+            const double g = (k <= j) ? G[k + w * j] : G[j + w * k];
+            A[k + LD * j] = d[k] * g * d[j];
+            V[k + LD * j] = (k == j) ? 1.0 : 0.0;
         }
+    __syncwarp();
     for (int sweep = 0; sweep < 60; ++sweep) {
         double off = 0.0, dia = 0.0;
-        for (int j = 0; j < w; ++j) {
-            dia += A[j + 32 * j] * A[j + 32 * j];
-            for (int i = 0; i < j; ++i) off += A[i + 32 * j] * A[i + 32 * j];
+        if (k < w) {
+            dia = A[k + LD * k] * A[k + LD * k];
+            for (int i = 0; i < k; ++i) off += A[i + LD * k] * A[i + LD * k];
         }
+        off = warp_sum(off);
+        dia = warp_sum(dia);
         if (off <= DBL_EPSILON * DBL_EPSILON * dia * 1e-2) break;
         for (int p = 0; p < w - 1; ++p)
             for (int q = p + 1; q < w; ++q) {
-                const double apq = A[p + 32 * q];
-                if (apq == 0.0) continue;
-                const double tau = (A[q + 32 * q] - A[p + 32 * p]) / (2.0 * apq);
+                const double apq = A[p + LD * q];
+                if (apq == 0.0) continue;                  // uniform: every lane read the same value
+                const double tau = (A[q + LD * q] - A[p + LD * p]) / (2.0 * apq);
                 const double t = (tau >= 0.0 ? 1.0 : -1.0) / (fabs(tau) + sqrt(1.0 + tau * tau));
-                const double c = 1.0 / sqrt(1.0 + t * t), s = t * c;
-                for (int k = 0; k < w; ++k) {
-                    const double akp = A[k + 32 * p], akq = A[k + 32 * q];
-                    A[k + 32 * p] = c * akp - s * akq;
-                    A[k + 32 * q] = s * akp + c * akq;
+                const double c = 1.0 / sqrt(1.0 + t * t), sn = t * c;
+                __syncwarp();
+                if (k < w) {                               // columns p, q
+                    const double akp = A[k + LD * p], akq = A[k + LD * q];
+                    A[k + LD * p] = c * akp - sn * akq;
+                    A[k + LD * q] = sn * akp + c * akq;
+                    const double vkp = V[k + LD * p], vkq = V[k + LD * q];
+                    V[k + LD * p] = c * vkp - sn * vkq;
+                    V[k + LD * q] = sn * vkp + c * vkq;
                 }
-                for (int k = 0; k < w; ++k) {
-                    const double apk = A[p + 32 * k], aqk = A[q + 32 * k];
-                    A[p + 32 * k] = c * apk - s * aqk;
-                    A[q + 32 * k] = s * apk + c * aqk;
+                __syncwarp();
+                if (k < w) {                               // rows p, q
+                    const double apk = A[p + LD * k], aqk = A[q + LD * k];
+                    A[p + LD * k] = c * apk - sn * aqk;
+                    A[q + LD * k] = sn * apk + c * aqk;
                 }
-                for (int k = 0; k < w; ++k) {
-                    const double vkp = V[k + 32 * p], vkq = V[k + 32 * q];
-                    V[k + 32 * p] = c * vkp - s * vkq;
-                    V[k + 32 * q] = s * vkp + c * vkq;
-                }
+                __syncwarp();
             }
     }
-    double smax = 0.0;
-    for (int i = 0; i < w; ++i) smax = fmax(smax, A[i + 32 * i]);
-    // M = S^{1/2} U^T  (stored in A)
-    double sq[32];
-    for (int i = 0; i < w; ++i) sq[i] = sqrt(fmax(A[i + 32 * i], DBL_EPSILON * smax));
-    for (int i = 0; i < w; ++i)
-        for (int k = 0; k < w; ++k) A[i + 32 * k] = sq[i] * V[k + 32 * i];
-    // Householder QR of M (w x w), R_hat in the upper triangle of A
-    for (int k = 0; k < w; ++k) {
-        double nrm = 0.0;
-        for (int i = k; i < w; ++i) nrm += A[i + 32 * k] * A[i + 32 * k];
-        nrm = sqrt(nrm);
+    double smax = k < w ? A[k + LD * k] : 0.0;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) smax = fmax(smax, __shfl_xor_sync(0xffffffffu, smax, o));
+    // M = S^{1/2} U^T (stored in A): row i = sq[i] * column i of V
+    const double sqk = k < w ? sqrt(fmax(A[k + LD * k], DBL_EPSILON * smax)) : 0.0;
+    __syncwarp();
+    for (int i = 0; i < w; ++i) {
+        const double sqi = __shfl_sync(0xffffffffu, sqk, i);
+        if (k < w) A[i + LD * k] = sqi * V[k + LD * i];
+    }
+    __syncwarp();
+    // Householder QR of M (w x w); lane = row index
+    for (int kk = 0; kk < w; ++kk) {
+        const double aik = (k >= kk && k < w) ? A[k + LD * kk] : 0.0;
+        const double nrm = sqrt(warp_sum(aik * aik));
         if (nrm == 0.0) continue;
-        const double alpha = -copysign(nrm, A[k + 32 * k]);
-        double v[32];
-        for (int i = k; i < w; ++i) v[i] = A[i + 32 * k];
-        v[k] -= alpha;
-        double vv = 0.0;
-        for (int i = k; i < w; ++i) vv += v[i] * v[i];
+        const double akk = __shfl_sync(0xffffffffu, aik, kk);
+        const double alpha = -copysign(nrm, akk);
+        const double vi = aik - (k == kk ? alpha : 0.0);
+        const double vv = warp_sum(vi * vi);
         if (vv == 0.0) continue;
         const double beta = 2.0 / vv;
-        for (int c = k; c < w; ++c) {
-            double dd = 0.0;
-            for (int i = k; i < w; ++i) dd += v[i] * A[i + 32 * c];
-            dd *= beta;
-            for (int i = k; i < w; ++i) A[i + 32 * c] -= dd * v[i];
+        for (int c = kk; c < w; ++c) {
+            const double aic = (k >= kk && k < w) ? A[k + LD * c] : 0.0;
+            const double dd = warp_sum(vi * aic) * beta;
+            __syncwarp();
+            if (k >= kk && k < w) A[k + LD * c] = aic - dd * vi;
+            __syncwarp();
         }
     }
-    for (int i = 0; i < w; ++i) {
-        const double sg = A[i + 32 * i] < 0.0 ? -1.0 : 1.0;
-        for (int c = 0; c < w; ++c) R[i + w * c] = (c < i) ? 0.0 : sg * A[i + 32 * c] / d[c];
+    if (k < w) {
+        const double sg = A[k + LD * k] < 0.0 ? -1.0 : 1.0;
+        for (int c = 0; c < w; ++c) R[k + w * c] = (c < k) ? 0.0 : sg * A[k + LD * c] / d[c];
     }
 }
 
 void svqr_factor(const double* G, int w, double* R, int* status, cudaStream_t st) {
-    ++g_launches; k_svqr<<<1, 32, 0, st>>>(G, w, R, status);
+    ++g_launches; launch_pdl(k_svqr, dim3(1), dim3(32), 0, st, G, w, R, status);
 }
 
 // ------------------------------------------------------------------------------------
