@@ -40,7 +40,12 @@ CFG = {"C2": dict(build=lambda rows=None: G.convection_diffusion(128, 3, 7, rows
                   workload="C3: G3_circuit-shaped (n=1,585,478), s=5, m=60, Newton, CholQR"),
        "C1": dict(build=lambda rows=None: G.convection_diffusion(32, 2, 5, rows=rows), n=1024, s=5, m=30,
                   basis="newton", tsqr="cholqr", reorth=False,
-                  workload="C1: 2D convection-diffusion 5-pt 32^2 (n=1024), s=5, m=30, Newton, CholQR")}
+                  workload="C1: 2D convection-diffusion 5-pt 32^2 (n=1024), s=5, m=30, Newton, CholQR"),
+       # the metric's large configuration (BASELINE.json configs[4]); fits one B200 (A 21 GB CSR,
+       # V 16 GB); built by the sort-free stencil generator (identical CSR, tests/test_synth.py)
+       "C5": dict(build=lambda rows=None: G.convection_diffusion_stream(400, 3, 27, rows=rows), n=400 ** 3,
+                  s=10, m=30, basis="newton", tsqr="cholqr", reorth=False,
+                  workload="C5: 3D convection-diffusion 27-pt 400^3 (n=64,000,000), s=10, m=30, Newton, CholQR")}
 TOL = 1e-8
 METRIC = "CA-GMRES time-to-solution (rel. residual 1e-8)"
 
@@ -142,6 +147,7 @@ def run_ours(args):
     t0 = time.time()
     if ws == 1:
         A = cfg["build"]()
+        print(f"[bench] A built: n={A.n} nnz={A.nnz} ({time.time() - t0:.1f} s)", file=sys.stderr, flush=True)
         S = Solver(A, cfg["s"], cfg["m"], basis=cfg["basis"], tsqr=cfg["tsqr"], reorth=cfg["reorth"] or args.reorth,
                    onepass=args.onepass)
         b_host = G.rhs(cfg["n"])
@@ -155,6 +161,7 @@ def run_ours(args):
         k_, v_ = kv.split("=")
         S.set_option(k_, int(v_))
     setup_s = time.time() - t0
+    print(f"[bench] setup done ({setup_s:.1f} s)", file=sys.stderr, flush=True)
     stream = torch.cuda.current_stream()
     b = torch.tensor(b_host, device="cuda")
     x = torch.zeros_like(b)

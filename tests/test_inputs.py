@@ -80,3 +80,15 @@ def test_banded_structure():
     assert A[500, 501] == pytest.approx(-wk[0] * 0.7)
     assert A[500, 499] == pytest.approx(-wk[0] * 1.3)
     assert 2 * wk.sum() <= A[500, 500] <= 2 * wk.sum() + 1e-5
+
+
+@pytest.mark.parametrize("N,dim,pts,rows", [(12, 3, 27, None), (9, 3, 7, None), (11, 2, 5, None),
+                                            (13, 3, 27, (100, 1500)), (10, 3, 7, (7, 777))])
+def test_stream_stencil_generator_is_identical(N, dim, pts, rows):
+    """The sort-free generator used for C5 builds the same CSR bit for bit (small chunks so
+    several chunk boundaries are crossed)."""
+    A = G.convection_diffusion(N, dim, pts, rows=rows)
+    B = G.convection_diffusion_stream(N, dim, pts, rows=rows, chunk=97)
+    assert A.row_begin == B.row_begin and A.n == B.n
+    assert np.array_equal(A.rowptr, B.rowptr) and np.array_equal(A.colind, B.colind)
+    assert A.val.tobytes() == B.val.tobytes()
