@@ -305,7 +305,8 @@ def run_ours(args):
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": cfg["workload"], "n": cfg["n"], "s": cfg["s"], "m": cfg["m"],
                        "tol": TOL, "cycles": stats[-1].cycles, "parallelism": f"rows{ws}",
-                       "l2": "inputs larger than L2 (A 175 MB, V 520 MB) + 256 MB flush between steps",
+                       "l2": f"inputs larger than L2 (A {12 * A.nnz / 1e6:.0f} MB as CSR, V {8 * S.ldv * (cfg['m'] + 1) / 1e6:.0f} MB)"
+                             " + 256 MB flush between steps",
                        "setup_s": round(setup_s, 2), "options": args.opt,
                        "orth": ("CholQR" + ("2 (reorth)" if (cfg["reorth"] or args.reorth) else "")
                                 + (", one-pass BOrth+CholQR (NEXT-2)" if args.onepass else ", BOrth CGS")),

@@ -95,17 +95,24 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
         if (W0 == WT && (i0 & 3) == 1) {
             const double* vp = a.val + b0 + lane;
             const double* xr = a.x + r;
-            double v[WT], xv[WT];
-#pragma unroll
-            for (int t = 0; t < WT; ++t) {
-                const int o = __shfl_sync(0xffffffffu, o0, t);
-                v[t] = (CONTIG || PF) ? ldg_stream(vp + 32 * t) : __ldg(vp + 32 * t);
-                xv[t] = __ldg(xr + o);
-            }
             if (MODE >= 1 && live) uu = __ldg(a.u + r);
             if (MODE == 2 && live) ww = __ldg(a.w + r);
+            // 27-point rows: three groups of 9 value / x pairs in flight (all 27 at once spilled
+            // 480 B of stack at the 64-register cap); the FMA order t = 0..WT-1 is unchanged
+            constexpr int GT = WT > 9 ? 9 : WT;
+            static_assert(WT % GT == 0, "DIA width must split into equal groups");
 #pragma unroll
-            for (int t = 0; t < WT; ++t) acc = fma(v[t], xv[t], acc);
+            for (int g0 = 0; g0 < WT; g0 += GT) {
+                double v[GT], xv[GT];
+#pragma unroll
+                for (int t = 0; t < GT; ++t) {
+                    const int o = __shfl_sync(0xffffffffu, o0, g0 + t);
+                    v[t] = (CONTIG || PF) ? ldg_stream(vp + 32 * (g0 + t)) : __ldg(vp + 32 * (g0 + t));
+                    xv[t] = __ldg(xr + o);
+                }
+#pragma unroll
+                for (int t = 0; t < GT; ++t) acc = fma(v[t], xv[t], acc);
+            }
         } else {
             acc = sell_slice_dot<4, true>(r, b0, W0, i0, o0, a.dcol, a.ncols, a.val, a.x, false);
             if (MODE >= 1 && live) uu = __ldg(a.u + r);
