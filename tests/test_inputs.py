@@ -83,7 +83,8 @@ def test_banded_structure():
 
 
 @pytest.mark.parametrize("N,dim,pts,rows", [(12, 3, 27, None), (9, 3, 7, None), (11, 2, 5, None),
-                                            (13, 3, 27, (100, 1500)), (10, 3, 7, (7, 777))])
+                                            (13, 3, 27, (100, 1500)), (10, 3, 7, (7, 777)),
+                                            (2, 3, 27, None), (1, 2, 5, None), (2, 3, 7, (3, 7))])
 def test_stream_stencil_generator_is_identical(N, dim, pts, rows):
     """The sort-free generator used for C5 builds the same CSR bit for bit (small chunks so
     several chunk boundaries are crossed)."""
