@@ -161,6 +161,31 @@ def test_mpk_full_size_C2():
         assert np.max(np.abs(W[:, k] - Wo[:, k])) <= 1e-12 * np.max(np.abs(Wo[:, k]))
 
 
+def test_mpk_full_size_C5_sampled():
+    """Config C5 at full size (400^3 27-pt, n = 64M, 1.72e9 nnz), the launch configuration
+    bench.py times, checked on sampled z-planes.  Step k at a row depends only on rows within k
+    hops, so the oracle runs on the principal sub-block of the planes within s = 10
+    of the sample: its values on the sample plane are exact for every k <= 10."""
+    N, s = 400, 10
+    P = N * N
+    A = G.convection_diffusion_stream(N, 3, 27)
+    S = Solver(A, s=s, m=30, basis="newton")
+    del A
+    S.set_shifts(*SHIFTS)
+    q = G.rhs(N ** 3)
+    q /= np.linalg.norm(q)
+    W = S.mpk(dev(q), s)
+    for z0 in (0, 217, N - 1):                                  # both boundary planes and one inside
+        lo, hi = max(0, z0 - s) * P, min(N, z0 + s + 1) * P
+        sub = G.convection_diffusion_stream(N, 3, 27, rows=(lo, hi)).to_scipy()[:, lo:hi]
+        Wo = O.mpk(sub.tocsr(), q[lo:hi], s, *SHIFTS)
+        a, b = z0 * P - lo, (z0 + 1) * P - lo
+        Wg = W[z0 * P:(z0 + 1) * P].cpu().numpy()
+        for k in range(s + 1):
+            ref = Wo[a:b, k]
+            assert np.max(np.abs(Wg[:, k] - ref)) <= 1e-12 * np.max(np.abs(ref)), (z0, k)
+
+
 # ----------------------------------------------------------------------------- BOrth / TSQR
 @pytest.mark.parametrize("n,j,w", [(5000, 12, 6), (70002, 55, 5), (3000, 1, 1), (40000, 30, 11),
                                    (1000, 70, 3), (70001, 7, 4), (262144, 20, 10)])
