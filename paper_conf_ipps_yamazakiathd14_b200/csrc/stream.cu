@@ -369,7 +369,18 @@ __global__ void __launch_bounds__(256) k_scale1(int64_t n, double* __restrict__ 
     if (al) {
         double2* p2 = reinterpret_cast<double2*>(p);
         const int64_t n2 = n >> 1;
-        for (int64_t i = i0; i < n2; i += stride) {
+        int64_t i = i0;
+        for (; i + 3 * stride < n2; i += 4 * stride) {       // 4 x 16 B in flight per thread
+            double2 v[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) v[u] = __ldcs(p2 + i + u * stride);
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                v[u].x *= inv; v[u].y *= inv;
+                p2[i + u * stride] = v[u];
+            }
+        }
+        for (; i < n2; i += stride) {
             double2 v = __ldcs(p2 + i);
             v.x *= inv; v.y *= inv;
             p2[i] = v;
