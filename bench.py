@@ -42,7 +42,7 @@ CFG = {"C2": dict(build=lambda rows=None: G.convection_diffusion(128, 3, 7, rows
                   basis="newton", tsqr="cholqr", reorth=False,
                   workload="C1: 2D convection-diffusion 5-pt 32^2 (n=1024), s=5, m=30, Newton, CholQR"),
        # the metric's large configuration (BASELINE.json configs[4]); fits one B200 (A 21 GB CSR,
-       # V 16 GB); built by the sort-free stencil generator (identical CSR, tests/test_synth.py)
+       # V 16 GB); built by the sort-free stencil generator (identical CSR, tests/test_inputs.py)
        "C5": dict(build=lambda rows=None: G.convection_diffusion_stream(400, 3, 27, rows=rows), n=400 ** 3,
                   s=10, m=30, basis="newton", tsqr="cholqr", reorth=False,
                   workload="C5: 3D convection-diffusion 27-pt 400^3 (n=64,000,000), s=10, m=30, Newton, CholQR")}
@@ -142,8 +142,12 @@ def run_ours(args):
     group = None
     cfg = CFG[args.config]
     if ws > 1:
+        if torch.cuda.device_count() < ws:
+            raise RuntimeError(f"{ws} ranks but only {torch.cuda.device_count()} CUDA devices on this node")
         dist.init_process_group("nccl", device_id=torch.device("cuda", lrank))
         group = dist.group.WORLD
+        if dist.get_world_size() != args.gpus:
+            raise RuntimeError(f"NCCL world has {dist.get_world_size()} ranks, --gpus {args.gpus}")
     t0 = time.time()
     if ws == 1:
         A = cfg["build"]()
@@ -301,7 +305,7 @@ def run_ours(args):
         out = {
             "metric": METRIC, "value": round(ms_step, 4), "unit": "ms", "n_gpus": ws,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 4),
-            "higher_is_better": False, "scaling": "strong" if ws > 1 else "weak",
+            "higher_is_better": False, "scaling": "strong",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": cfg["workload"], "n": cfg["n"], "s": cfg["s"], "m": cfg["m"],
                        "tol": TOL, "cycles": stats[-1].cycles, "parallelism": f"rows{ws}",
@@ -411,7 +415,7 @@ def run_reference(args):
     cores = _cores()
     out = {"metric": METRIC, "value": round(val, 1), "unit": "ms", "n_gpus": ws, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": round(per * 1e3, 1), "higher_is_better": False,
-           "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
+           "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
            "config": {"workload": cfg["workload"], "n": cfg["n"], "s": cfg["s"], "m": cfg["m"], "tol": TOL,
                       "cycles": cycles, "full_oracle_solve_s": round(t_full, 2)},
            "cpu_baseline": {"value": round(val, 1), "unit": "ms", "cores": cores, "kind": "oracle",
@@ -421,6 +425,30 @@ def run_reference(args):
            "e2e": {"value": round(val, 1), "unit": "ms", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
     return out
+
+
+def _free_port():
+    import socket
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    return port
+
+
+def launch_ranks(args):
+    """--gpus N without a torchrun environment: re-launch this script as N ranks (one process
+    per GPU) under torch.distributed.run.  Refuses (exit 2, one JSON line) when this node has
+    fewer than N GPUs — never a silent 1-GPU number for an N-GPU request."""
+    import torch
+    have = torch.cuda.device_count()
+    if have < args.gpus:
+        print(json.dumps({"metric": METRIC, "error": f"--gpus {args.gpus} requested but this node has {have} "
+                                                     f"CUDA device(s)", "n_gpus": args.gpus}), flush=True)
+        sys.exit(2)
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={_free_port()}", os.path.abspath(__file__)] + sys.argv[1:]
+    sys.exit(subprocess.call(cmd))
 
 
 def main():
@@ -439,6 +467,12 @@ def main():
                          "default: the library's defaults")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
+    ws, _, _ = dist_env()
+    if "WORLD_SIZE" in os.environ and ws != args.gpus:
+        print(json.dumps({"metric": METRIC, "error": f"--gpus {args.gpus} but WORLD_SIZE={ws}"}), flush=True)
+        sys.exit(2)
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        launch_ranks(args)
     if args.impl == "reference":
         run_reference(args)
     else:

@@ -36,7 +36,7 @@ extern "C" {
 #define CAGMRES_NOT_CONVERGED   1   /* solve: maxit cycles done, x holds the last iterate     */
 #define CAGMRES_EINVAL         -1   /* bad argument, shape, leading dimension or alignment    */
 #define CAGMRES_ECUDA          -2   /* a CUDA runtime call failed (no device, launch error)   */
-#define CAGMRES_ENCCL          -3   /* an NCCL call failed                                    */
+#define CAGMRES_ENCCL          -3   /* an NCCL call (or an in-process group collective) failed  */
 #define CAGMRES_EBREAKDOWN     -4   /* Cholesky pivot <= 0, zero norm, singular T     */
 #define CAGMRES_ENOMEM         -5   /* device or host allocation failed                       */
 #define CAGMRES_EGHOST         -6   /* supplied rows do not cover the (s-1)-hop ghost rows    */
@@ -60,6 +60,11 @@ enum { CAGMRES_CHOLQR = 0, CAGMRES_SVQR = 1, CAGMRES_CGS = 2,     /* TSQR, Fig. 
  * four times and needs one reduction instead of two.  CholQR only (else EINVAL); less stable
  * than the two-pass method (use with CAGMRES_REORTH); j + s + 1 <= 64. */
 #define CAGMRES_ONEPASS     0x400
+/* CholQR breakdown (pivot <= 0) -> opt-in SVQR retry of that panel (SURVEY reading G15):
+ * the panel's R is recomputed from the same Gram by SVQR on the device, counted
+ * in cagmres_stats.retried_panels; without it a breakdown returns EBREAKDOWN.  CholQR only
+ * (else EINVAL); two-pass BOrth+TSQR path (not with CAGMRES_ONEPASS / the fused Gram option). */
+#define CAGMRES_SVQR_RETRY  0x800
 
 typedef struct cagmres* cagmres_t;
 
@@ -67,7 +72,10 @@ typedef struct cagmres* cagmres_t;
  *   n                : global dimension (A is n x n, nonsymmetric allowed)
  *   row_begin/row_end: global ids of the rows described by rowptr (nrows = row_end-row_begin)
  *   rowptr           : host, nrows+1 entries, rowptr[0] == 0, int64
- *   colind           : host, global column ids in [0, n), int32
+ *   colind           : host, global column ids in [0, n), int32.  A row's entries may be in
+ *                      any order and may repeat a column: create canonicalises every row
+ *                      (stable sort by column, repeated entries summed in input order), and the
+ *                      device sums each row in increasing global column order
  *   val              : host, fp64 values
  *   own_begin/own_end: the rows this rank owns (block-row distribution);
  *                      must satisfy row_begin <= own_begin <= own_end <= row_end.
@@ -96,6 +104,14 @@ typedef struct {
     int    spmv_launches;   /* SpMV launches timed in ms_spmv                                */
     double ms_spmv;         /* device time of the SpMV launches alone                        */
     double bytes_spmv;      /* algorithmic bytes of those launches                           */
+    int    collect_diag;    /* in: 1 = per-panel numerical diagnostics below (two extra Gram     *
+                             * passes per panel and a host sync per cycle: not for timing)     */
+    double max_orth_err;    /* max over the CA panels of ||I - Q_p^T Q_p||_2, Q_p = [q_j, new     *
+                             * columns] after BOrth+TSQR (0 if none / not collected)    */
+    double max_gram_cond;   /* max over the CA panels of kappa_2(W^T W), W = the MPK output      *
+                             * [q_j, W_1..W_sb] before BOrth (Fig. 12 "cond(B)")   */
+    double ms_setup;        /* host wall time of the create call that built this handle (ms)  */
+    int    retried_panels;  /* CholQR panels re-factored by SVQR (CAGMRES_SVQR_RETRY, G15)      */
 } cagmres_stats;
 
 /* ---- lifetime ---------------------------------------------------------------------- */
@@ -115,6 +131,24 @@ int cagmres_create(cagmres_t* h, const cagmres_csr* A, int s, int m, int basis, 
 int cagmres_create_dist(cagmres_t* h, const cagmres_csr* A, const int64_t* row_starts,
                         int s, int m, int basis, int orth,
                         const void* nccl_unique_id, int rank, int nranks, int cuda_device);
+
+/* In-process group: P ranks of the distributed handle inside ONE process, one host thread
+ * per rank (transport.h).  Rank p runs on devices[p] (NULL: every rank on device 0); ranks on
+ * different devices exchange through peer memory (NVLink), ranks on the same device through
+ * device copies — so the whole multi-rank device path (halo pack -> exchange -> unpack, the
+ * cross-rank sums, the distributed residual) runs on a single GPU.  Sums over ranks are one
+ * fixed-order kernel per rank (bitwise identical on every rank).  Every collective is a host
+ * barrier across the P threads: each rank's calls (create_group, mpk, borth, tsqr, solve,
+ * destroy) must be made from its own thread, concurrently with the other ranks', in the same
+ * order.  A rank that stops calling makes the others fail with ENCCL after 600 s.
+ * nranks in [1, 16].  destroy: EINVAL while a handle created from the group still exists. */
+typedef struct cagmres_group* cagmres_group_t;
+int cagmres_group_create(cagmres_group_t* g, int nranks, const int* devices);
+int cagmres_group_destroy(cagmres_group_t g);
+/* cagmres_create_dist over an in-process group instead of NCCL (same arguments otherwise;
+ * the device is the group's devices[rank]).  Errors: as create_dist; ENCCL = group failure. */
+int cagmres_create_group(cagmres_t* h, const cagmres_csr* A, const int64_t* row_starts,
+                         int s, int m, int basis, int orth, cagmres_group_t g, int rank);
 
 int cagmres_destroy(cagmres_t h);                 /* frees everything create allocated */
 const char* cagmres_strerror(int status);         /* static string, never NULL         */
@@ -249,6 +283,16 @@ int cagmres_plan_set_sends(cagmres_plan_t p, const int64_t* counts, const int64_
 /* Send lists: owned local indices in request order (host, total = sum counts). */
 int cagmres_plan_send_index(cagmres_plan_t p, int64_t* local_idx);
 
+/* SELL-32 device layout of the plan's stored rows, built on the host exactly as create builds
+ * it (lets tests check it without a GPU).  Query the sizes with NULL
+ * arrays first: nslices, ndcol (entries of dcol), nstored (entries of val); then sptr
+ * (nslices+1), sinfo (nslices), dcol, val.  sinfo[sl] = dptr << 2 | clamp << 1 | dia; a DIA
+ * slice stores diagonal t of lane l at val[sptr[sl] + 32 t + l] with column row + dcol[dptr + t],
+ * an explicit slice column dcol[dptr + 32 t + l].  Each row's nonzeros appear in increasing
+ * GLOBAL column order (padding entries are exact zeros). */
+int cagmres_plan_sell(cagmres_plan_t p, int64_t* nslices, int64_t* ndcol, int64_t* nstored,
+                      int64_t* sptr, int64_t* sinfo, int32_t* dcol, double* val);
+
 /* ---- host-only reordering for the row partition ------- */
 /* Reverse Cuthill-McKee order of the symmetrised pattern of A (n x n CSR, host): perm[new] =
  * old.  Each connected component starts at a pseudo-peripheral node (repeated BFS from a
@@ -276,6 +320,9 @@ int cagmres_host_change_of_basis(const double* re, const double* im, int sb, dou
  * H[0:j+sb+1, j:j+sb] = (Rt B - [H[0:j+1,0:j] Rt[0:j,0:sb]; 0]) T^{-1}, T = Rt[j:j+sb,0:sb]. */
 int cagmres_host_hessenberg_update(double* H, int ldh, int j, int sb, const double* Rt,
                                    int ldr, const double* B);
+/* Eigenvalues (ascending) of the symmetric n x n matrix A (ld lda, upper triangle read),
+ * cyclic Jacobi; used for the per-panel diagnostics (kappa_2 of a Gram, ||I - Q^T Q||_2). */
+int cagmres_host_sym_eigvals(const double* A, int lda, int n, double* ev);
 /* y = argmin ||beta e1 - H y|| (H (k+1) x k upper Hessenberg, Givens QR); res[i] =
  * residual estimate after i+1 columns (may be NULL). */
 int cagmres_host_givens_ls(const double* H, int ldh, int k, double beta, double* y,

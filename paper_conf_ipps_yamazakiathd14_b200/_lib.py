@@ -16,7 +16,7 @@ OK, NOT_CONVERGED = 0, 1
 EINVAL, ECUDA, ENCCL, EBREAKDOWN, ENOMEM, EGHOST, ENOTSUP = -1, -2, -3, -4, -5, -6, -7
 MONOMIAL, NEWTON, GMRES = 0, 1, 2
 CHOLQR, SVQR, CGS, MGS, CAQR = 0, 1, 2, 3, 4
-REORTH, BORTH_MGS, ONEPASS = 0x100, 0x200, 0x400
+REORTH, BORTH_MGS, ONEPASS, SVQR_RETRY = 0x100, 0x200, 0x400, 0x800
 OPT_MPK_WAVE, OPT_WAVE_CHUNK, OPT_WAVE_CTAS, OPT_WAVE_LAG, OPT_FUSE, OPT_SPMV = 1, 3, 4, 5, 6, 7
 
 
@@ -35,7 +35,9 @@ class StatsStruct(C.Structure):
                 ("ms_other", C.c_double), ("ms_total", C.c_double),
                 ("bytes_mpk", C.c_double), ("bytes_borth", C.c_double),
                 ("bytes_tsqr", C.c_double), ("bytes_other", C.c_double),
-                ("spmv_launches", C.c_int), ("ms_spmv", C.c_double), ("bytes_spmv", C.c_double)]
+                ("spmv_launches", C.c_int), ("ms_spmv", C.c_double), ("bytes_spmv", C.c_double),
+                ("collect_diag", C.c_int), ("max_orth_err", C.c_double), ("max_gram_cond", C.c_double),
+                ("ms_setup", C.c_double), ("retried_panels", C.c_int)]
 
 
 class CagmresError(RuntimeError):
@@ -59,6 +61,10 @@ SIGNATURES = {
     "cagmres_create_dist": ([C.POINTER(_P), C.POINTER(CSRStruct), _PI64, C.c_int, C.c_int, C.c_int,
                              C.c_int, _P, C.c_int, C.c_int, C.c_int], C.c_int),
     "cagmres_destroy": ([_P], C.c_int),
+    "cagmres_group_create": ([C.POINTER(_P), C.c_int, C.POINTER(C.c_int)], C.c_int),
+    "cagmres_group_destroy": ([_P], C.c_int),
+    "cagmres_create_group": ([C.POINTER(_P), C.POINTER(CSRStruct), _PI64, C.c_int, C.c_int, C.c_int,
+                              C.c_int, _P, C.c_int], C.c_int),
     "cagmres_set_stream": ([_P, _P], C.c_int),
     "cagmres_set_option": ([_P, C.c_int, C.c_int64], C.c_int),
     "cagmres_get_option": ([_P, C.c_int, C.POINTER(C.c_int64)], C.c_int),
@@ -79,6 +85,8 @@ SIGNATURES = {
     "cagmres_plan_recv_index": ([_P, _PI64], C.c_int),
     "cagmres_plan_set_sends": ([_P, _PI64, _PI64, _PI32], C.c_int),
     "cagmres_plan_send_index": ([_P, _PI64], C.c_int),
+    "cagmres_plan_sell": ([_P, _PI64, _PI64, _PI64, _PI64, _PI64, _PI32, _PD], C.c_int),
+    "cagmres_host_sym_eigvals": ([_PD, C.c_int, C.c_int, _PD], C.c_int),
     "cagmres_host_eigvals": ([_PD, C.c_int, C.c_int, _PD, _PD], C.c_int),
     "cagmres_host_rcm": ([_I64, _PI64, _PI32, _PI64], C.c_int),
     "cagmres_host_permute": ([_I64, _PI64, _PI32, _PD, _PI64, _PI64, _PI32, _PD], C.c_int),

@@ -244,6 +244,46 @@ void modified_leja(const double* wr, const double* wi, int cnt, int s,
     }
 }
 
+// Eigenvalues of the symmetric n x n matrix A (ld lda; only the upper triangle is read) by
+// cyclic Jacobi rotations (Golub & Van Loan 8.5); ascending.  For the per-panel diagnostics:
+// kappa_2 of a Gram matrix and ||I - Q^T Q||_2.
+void sym_eigvals(const double* A, int lda, int n, double* ev) {
+    std::vector<double> M(size_t(n) * size_t(n));
+    for (int c = 0; c < n; ++c)
+        for (int i = 0; i < n; ++i)
+            M[size_t(i) + size_t(n) * c] = i <= c ? A[size_t(i) + size_t(lda) * c] : A[size_t(c) + size_t(lda) * i];
+    auto at = [&](int i, int c) -> double& { return M[size_t(i) + size_t(n) * c]; };
+    for (int sweep = 0; sweep < 100; ++sweep) {
+        double off = 0.0, tot = 0.0;
+        for (int c = 0; c < n; ++c)
+            for (int i = 0; i < n; ++i) {
+                tot += at(i, c) * at(i, c);
+                if (i != c) off += at(i, c) * at(i, c);
+            }
+        if (off <= 1e-34 * tot || off == 0.0) break;
+        for (int p = 0; p < n - 1; ++p)
+            for (int q = p + 1; q < n; ++q) {
+                const double apq = at(p, q);
+                if (apq == 0.0) continue;
+                const double theta = (at(q, q) - at(p, p)) / (2.0 * apq);
+                const double t = (theta >= 0.0 ? 1.0 : -1.0) / (std::fabs(theta) + std::sqrt(theta * theta + 1.0));
+                const double cs = 1.0 / std::sqrt(t * t + 1.0), sn = t * cs;
+                for (int k = 0; k < n; ++k) {            // columns p, q
+                    const double akp = at(k, p), akq = at(k, q);
+                    at(k, p) = cs * akp - sn * akq;
+                    at(k, q) = sn * akp + cs * akq;
+                }
+                for (int k = 0; k < n; ++k) {            // rows p, q
+                    const double apk = at(p, k), aqk = at(q, k);
+                    at(p, k) = cs * apk - sn * aqk;
+                    at(q, k) = sn * apk + cs * aqk;
+                }
+            }
+    }
+    for (int i = 0; i < n; ++i) ev[i] = at(i, i);
+    std::sort(ev, ev + n);
+}
+
 }  // namespace host
 
 // ---------------------------------------------------------------------------------------
@@ -279,6 +319,12 @@ int cagmres_host_hessenberg_update(double* H, int ldh, int j, int sb, const doub
     if (!H || !Rt || !B || j < 0 || sb < 1 || ldh < j + sb + 1 || ldr < j + sb + 1)
         return CAGMRES_EINVAL;
     return host::hessenberg_update(H, ldh, j, sb, Rt, ldr, B);
+}
+
+int cagmres_host_sym_eigvals(const double* A, int lda, int n, double* ev) {
+    if (!A || !ev || n < 1 || lda < n) return CAGMRES_EINVAL;
+    host::sym_eigvals(A, lda, n, ev);
+    return CAGMRES_OK;
 }
 
 int cagmres_host_givens_ls(const double* H, int ldh, int k, double beta, double* y, double* res) {

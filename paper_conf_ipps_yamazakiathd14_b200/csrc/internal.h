@@ -32,6 +32,17 @@ struct cagmres_plan {
 int plan_build(cagmres_plan* p, const cagmres_csr* A, const int64_t* row_starts,
                int nranks, int rank, int s);
 
+// Host SELL-32 layout of the plan's stored rows (sell.cpp):
+// sinfo[sl] = dptr << 2 | clamp << 1 | dia; DIA slices: dcol[dptr + t] = offset of diagonal t,
+// else dcol[dptr + 32 t + lane] = column; values val[sptr[sl] + 32 t + lane].
+struct SellHost {
+    int64_t nslices = 0, ndia = 0;
+    std::vector<int64_t> sptr, sinfo;
+    std::vector<int32_t> dcol;
+    std::vector<double> val;
+};
+void sell_build(const cagmres_plan& p, SellHost& out);   // throws std::bad_alloc
+
 // count of entries of the (owner/requester) list `q` whose level <= depth
 int64_t plan_prefix_count(const std::vector<int64_t>& counts, const std::vector<int32_t>& levels,
                           int q, int depth);
@@ -56,4 +67,6 @@ int hessenberg_eigvals(const double* H, int ldh, int m, double* wr, double* wi);
 // modified Leja order (G10); returns >= s shifts (or all available)
 void modified_leja(const double* wr, const double* wi, int cnt, int s,
                    std::vector<double>& ore, std::vector<double>& oim);
+// eigenvalues of a symmetric matrix (upper triangle read), ascending (cyclic Jacobi)
+void sym_eigvals(const double* A, int lda, int n, double* ev);
 }  // namespace host

@@ -309,12 +309,24 @@ __device__ __forceinline__ double warp_sum(double v) {
     return v;
 }
 
-__global__ void k_svqr(const double* G, int w, double* R, int* status) {
+// retry = 1 (G15 opt-in, CAGMRES_SVQR_RETRY): act only if the CholQR of this panel broke down
+// (ST_CHOL set by the Gram/Cholesky launch just before), then clear ST_CHOL and count the retry
+// in status[1]; R is replaced by the SVQR factor of the same Gram G.
+__global__ void k_svqr(const double* G, int w, double* R, int* status, int retry) {
     __shared__ double A[32 * 33], V[32 * 33], d[32];
     constexpr int LD = 33;
     const int k = threadIdx.x;                         // lane
     pdl_wait();
     pdl_trigger();
+    if (retry) {
+        const int st0 = *(volatile int*)status;
+        if (!(st0 & ST_CHOL)) return;
+        __syncwarp();
+        if (k == 0) {
+            atomicAnd(status, ~ST_CHOL);
+            atomicAdd(status + 1, 1);
+        }
+    }
     if (k < w) {
         const double g = G[k + w * k];
         if (!(g > 0.0)) { atomicOr(status, ST_SVQR); d[k] = 1.0; } else d[k] = 1.0 / sqrt(g);
@@ -398,31 +410,41 @@ __global__ void k_svqr(const double* G, int w, double* R, int* status) {
 }
 
 void svqr_factor(const double* G, int w, double* R, int* status, cudaStream_t st) {
-    ++g_launches; launch_pdl(k_svqr, dim3(1), dim3(32), 0, st, G, w, R, status);
+    ++g_launches; launch_pdl(k_svqr, dim3(1), dim3(32), 0, st, G, w, R, status, 0);
+}
+void svqr_retry(const double* G, int w, double* R, int* status, cudaStream_t st) {
+    ++g_launches; launch_pdl(k_svqr, dim3(1), dim3(32), 0, st, G, w, R, status, 1);
 }
 
 // ------------------------------------------------------------------------------------
 // K2: halo pack / unpack
 // ------------------------------------------------------------------------------------
-__global__ void k_gather(const double* __restrict__ src, const int64_t* __restrict__ idx, int64_t cnt,
-                         double* __restrict__ dst) {
-    for (int64_t k = int64_t(blockIdx.x) * NT + threadIdx.x; k < cnt; k += int64_t(gridDim.x) * NT)
-        dst[k] = src[idx[k]];
+template <bool SCATTER>
+__global__ void k_halo_segs(const double* __restrict__ src, const int64_t* __restrict__ idx, Segs sg,
+                            int64_t tot, double* __restrict__ dst) {
+    for (int64_t t = int64_t(blockIdx.x) * NT + threadIdx.x; t < tot; t += int64_t(gridDim.x) * NT) {
+        int i = 0;
+        int64_t k = t;
+        while (k >= sg.cnt[i]) { k -= sg.cnt[i]; ++i; }
+        k += sg.off[i];
+        if (SCATTER) dst[idx[k]] = src[k];
+        else dst[k] = src[idx[k]];
+    }
 }
-__global__ void k_scatter(const double* __restrict__ src, const int64_t* __restrict__ idx, int64_t cnt,
-                          double* __restrict__ dst) {
-    for (int64_t k = int64_t(blockIdx.x) * NT + threadIdx.x; k < cnt; k += int64_t(gridDim.x) * NT)
-        dst[idx[k]] = src[k];
+template <bool SCATTER>
+static void halo_segs(const double* src, const int64_t* idx, const Segs& sg, double* dst, cudaStream_t st) {
+    int64_t tot = 0;
+    for (int i = 0; i < sg.n; ++i) tot += sg.cnt[i];
+    if (tot <= 0) return;
+    const int64_t g = std::min<int64_t>((tot + NT - 1) / NT, 4096);
+    ++g_launches;
+    k_halo_segs<SCATTER><<<unsigned(g), NT, 0, st>>>(src, idx, sg, tot, dst);
 }
-void gather(const double* src, const int64_t* idx, int64_t cnt, double* dst, cudaStream_t st) {
-    if (cnt <= 0) return;
-    const int64_t g = std::min<int64_t>((cnt + NT - 1) / NT, 4096);
-    ++g_launches; k_gather<<<unsigned(g), NT, 0, st>>>(src, idx, cnt, dst);
+void gather_segs(const double* src, const int64_t* idx, const Segs& sg, double* dst, cudaStream_t st) {
+    halo_segs<false>(src, idx, sg, dst, st);
 }
-void scatter(const double* src, const int64_t* idx, int64_t cnt, double* dst, cudaStream_t st) {
-    if (cnt <= 0) return;
-    const int64_t g = std::min<int64_t>((cnt + NT - 1) / NT, 4096);
-    ++g_launches; k_scatter<<<unsigned(g), NT, 0, st>>>(src, idx, cnt, dst);
+void scatter_segs(const double* src, const int64_t* idx, const Segs& sg, double* dst, cudaStream_t st) {
+    halo_segs<true>(src, idx, sg, dst, st);
 }
 
 __global__ void k_add_small(const double* a, const double* b, double* c, int cnt) {

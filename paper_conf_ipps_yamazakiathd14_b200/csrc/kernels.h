@@ -6,7 +6,7 @@
 namespace kern {
 
 // Process-wide count of kernel launches issued by this library (bench.py gpu_launches).
-extern long long g_launches;
+extern long long g_launches;   // (approximate when several host threads launch)
 
 // Programmatic dependent launch (PDL, sm_90+): the hot kernels are launched with
 // programmaticStreamSerializationAllowed, so their CTAs are scheduled while the previous
@@ -283,6 +283,8 @@ int gram_dfma(const Dev& d, const GramArgs& a, cudaStream_t st);
 void chol(const double* G, int w, double* R, int* status, cudaStream_t st);
 // SVQR small factor: R from the Gram G (w x w), one CTA.
 void svqr_factor(const double* G, int w, double* R, int* status, cudaStream_t st);
+// G15 opt-in: if ST_CHOL is set in status[0], R := SVQR factor of G, clear ST_CHOL, ++status[1].
+void svqr_retry(const double* G, int w, double* R, int* status, cudaStream_t st);
 
 // P[:, 0:w] -= X C  (C: jx x w, ld jx)      (BOrth pass 2)
 void update(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, double* P,
@@ -298,9 +300,19 @@ void onepass_finalize(const double* Mx, int j, int w, double* C, double* R, doub
 // P[:, c0:w] = (P R^{-1})[:, c0:w]   (R upper w x w, ld w)
 void trsm(const Dev& d, int64_t n, double* P, int64_t ldp, int w, const double* R, int c0,
           cudaStream_t st);
-// dst[k] = src[idx[k]]  /  dst[idx[k]] = src[k]
-void gather(const double* src, const int64_t* idx, int64_t cnt, double* dst, cudaStream_t st);
-void scatter(const double* src, const int64_t* idx, int64_t cnt, double* dst, cudaStream_t st);
+// Halo pack / unpack over segments [off[i], off[i] + cnt[i]) of an index list (one segment per
+// peer: the depth-limited prefix of that peer's level-sorted list).
+struct Segs {
+    int64_t off[32], cnt[32];
+    int n = 0;
+    void add(int64_t o, int64_t c) {
+        if (c > 0 && n < 32) { off[n] = o; cnt[n] = c; ++n; }
+    }
+};
+// gather_segs: dst[k] = src[idx[k]]   /   scatter_segs: dst[idx[k]] = src[k],   k in the segments.
+// More than 32 segments: one launch per 32.
+void gather_segs(const double* src, const int64_t* idx, const Segs& sg, double* dst, cudaStream_t st);
+void scatter_segs(const double* src, const int64_t* idx, const Segs& sg, double* dst, cudaStream_t st);
 // small device helpers
 void add_small(const double* a, const double* b, double* c, int cnt, cudaStream_t st);
 

@@ -82,28 +82,59 @@ int plan_build(cagmres_plan* p, const cagmres_csr* A, const int64_t* row_starts,
         auto it = ext_of.find(g);
         return it == ext_of.end() ? -1 : it->second;
     };
-    // --- extended local CSR (rows at distance <= s-1), global column order kept ------------
+    // --- extended local CSR (rows at distance <= s-1) ----------------------------------------
+    // Canonical rows: entries sorted by GLOBAL column id, duplicates summed in input order
+    // (the CSR contract allows unsorted rows and repeated entries, include/cagmres.h).  Every
+    // row is summed in global column order by the SpMV whatever the partition.
     p->rowptr.assign(size_t(p->n_mat) + 1, 0);
-    int64_t nnz = 0;
+    p->colind.clear();
+    p->val.clear();
+    {
+        int64_t tot = 0;
+        for (int64_t r = 0; r < p->n_mat; ++r) {
+            const int64_t g = p->ext_gid[r];
+            if (!row_avail(g)) return CAGMRES_EGHOST;
+            tot += A->rowptr[g - rb + 1] - A->rowptr[g - rb];
+        }
+        p->colind.reserve(size_t(tot));
+        p->val.reserve(size_t(tot));
+    }
+    std::vector<std::pair<int64_t, int64_t>> ent;           // (global column, input position)
     for (int64_t r = 0; r < p->n_mat; ++r) {
         const int64_t g = p->ext_gid[r];
-        if (!row_avail(g)) return CAGMRES_EGHOST;
-        nnz += A->rowptr[g - rb + 1] - A->rowptr[g - rb];
-        p->rowptr[r + 1] = nnz;
-    }
-    p->nnz_mat = nnz;
-    p->colind.resize(size_t(nnz));
-    p->val.resize(size_t(nnz));
-    for (int64_t r = 0; r < p->n_mat; ++r) {
-        const int64_t g = p->ext_gid[r], lr = g - rb;
-        int64_t o = p->rowptr[r];
-        for (int64_t e = A->rowptr[lr]; e < A->rowptr[lr + 1]; ++e, ++o) {
-            const int64_t c = ext_id(A->colind[e]);
-            if (c < 0) return CAGMRES_EGHOST;      // cannot happen for distance <= s-1 rows
-            p->colind[size_t(o)] = int32_t(c);
-            p->val[size_t(o)] = A->val[e];
+        const int64_t lr = g - rb;
+        bool canon = true;                                  // already strictly increasing
+        for (int64_t e = A->rowptr[lr] + 1; e < A->rowptr[lr + 1] && canon; ++e)
+            canon = A->colind[e - 1] < A->colind[e];
+        if (canon) {
+            for (int64_t e = A->rowptr[lr]; e < A->rowptr[lr + 1]; ++e) {
+                const int64_t c = ext_id(A->colind[e]);
+                if (c < 0) return CAGMRES_EGHOST;
+                p->colind.push_back(int32_t(c));
+                p->val.push_back(A->val[e]);
+            }
+            p->rowptr[size_t(r) + 1] = int64_t(p->colind.size());
+            continue;
         }
+        ent.clear();
+        for (int64_t e = A->rowptr[lr]; e < A->rowptr[lr + 1]; ++e) ent.push_back({A->colind[e], e});
+        std::stable_sort(ent.begin(), ent.end(),
+                         [](const std::pair<int64_t, int64_t>& a, const std::pair<int64_t, int64_t>& b) {
+                             return a.first < b.first;
+                         });
+        for (size_t k = 0; k < ent.size(); ++k) {
+            if (k > 0 && ent[k].first == ent[k - 1].first) {
+                p->val.back() += A->val[ent[k].second];
+                continue;
+            }
+            const int64_t c = ext_id(ent[k].first);
+            if (c < 0) return CAGMRES_EGHOST;      // cannot happen for distance <= s-1 rows
+            p->colind.push_back(int32_t(c));
+            p->val.push_back(A->val[ent[k].second]);
+        }
+        p->rowptr[size_t(r) + 1] = int64_t(p->colind.size());
     }
+    p->nnz_mat = int64_t(p->colind.size());
     // --- requests to owners, each sorted by (level, gid) -----------------------------------
     p->req_counts.assign(size_t(nranks), 0);
     std::vector<std::vector<int64_t>> byown(static_cast<size_t>(nranks));

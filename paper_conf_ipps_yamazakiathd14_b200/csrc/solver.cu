@@ -11,6 +11,7 @@
 //         block (and of the reorthogonalisation pass); copied to the host once per cycle
 //         for the Hessenberg update and the least-squares solve.
 #include <algorithm>
+#include <chrono>
 #include <climits>
 #include <cmath>
 #include <cstring>
@@ -18,21 +19,18 @@
 #include <string>
 #include <vector>
 
+#include <memory>
+
 #include <cuda_runtime.h>
-#include <nccl.h>
 
 #include "internal.h"
 #include "kernels.h"
+#include "transport.h"
 
 #define CU(x)                                                       \
     do {                                                            \
         cudaError_t e_ = (x);                                       \
         if (e_ != cudaSuccess) { return CAGMRES_ECUDA; }            \
-    } while (0)
-#define NC(x)                                                       \
-    do {                                                            \
-        ncclResult_t r_ = (x);                                      \
-        if (r_ != ncclSuccess) { return CAGMRES_ENCCL; }            \
     } while (0)
 #define TRY(x)                                                      \
     do {                                                            \
@@ -70,7 +68,7 @@ struct cagmres {
     int s = 1, m = 1, basis = CAGMRES_NEWTON, orth = CAGMRES_CHOLQR;
     int64_t n = 0, n_loc = 0, n_ext = 0, ldv = 0;
     int rank = 0, nranks = 1;
-    ncclComm_t comm = nullptr;
+    std::unique_ptr<Transport> tr;         // NCCL or in-process group (transport.h); null on 1 rank
     kern::Dev dev;
     cudaStream_t stream = nullptr, own_stream = nullptr;
     kern::Sell A;
@@ -97,6 +95,12 @@ struct cagmres {
     bool arnoldi_fuse = true;
     bool fuse_borth_gram = false;          // BOrth pass 2 + CholQR Gram in one pass (fused.cu; slower)
     int* status = nullptr;
+    double ms_setup = 0.0;                 // wall time of create
+    // per-panel diagnostics (cagmres_stats.collect_diag): per block [W^T W | Q_p^T Q_p], (s+1)^2 each
+    bool diag_on = false;
+    double* dg = nullptr;
+    double* h_dg = nullptr;
+    size_t dg_cap = 0;
     // halo (distributed)
     std::vector<int64_t> send_off, recv_off;
     std::vector<std::vector<int64_t>> send_pre, recv_pre;   // [rank][depth]
@@ -126,12 +130,13 @@ struct cagmres {
         cudaFree(A.sptr); cudaFree(A.sinfo); cudaFree(A.dcol); cudaFree(A.val);
         cudaFree(V); cudaFree(xe); cudaFree(tab); cudaFree(gbuf); cudaFree(ybuf); cudaFree(caqr_ws); cudaFree(op_M);
         cudaFreeHost(h_tab); cudaFreeHost(h_y); cudaFreeHost(h_beta); cudaFreeHost(h_stat);
+        cudaFree(dg); cudaFreeHost(h_dg);
         if (ev_tab) cudaEventDestroy(ev_tab);
         if (ev_beta) cudaEventDestroy(ev_beta);
         cudaFree(ws.part); cudaFree(ws.counter); cudaFree(status);
         cudaFree(arn_part); cudaFree(arn_counter);
         cudaFree(d_send_idx); cudaFree(d_recv_ext); cudaFree(d_sendbuf); cudaFree(d_recvbuf);
-        if (comm) ncclCommDestroy(comm);
+        tr.reset();
         if (own_stream) cudaStreamDestroy(own_stream);
     }
 };
@@ -157,83 +162,20 @@ struct Scope {
 int64_t round_up(int64_t a, int64_t b) { return (a + b - 1) / b * b; }
 
 // ---- SELL-32 build (host) + upload ------------------------------------------------------
-// SELL-32 with per-slice diagonal-offset column compression.  A slice
-// (32 consecutive rows, one warp) whose rows' column offsets col - row take few distinct
-// values (stencils, banded and most PDE matrices) is stored DIA-style: one int32 offset per
-// stored "diagonal" plus 32 values per diagonal (exact zeros where a row lacks it), so the
-// column stream drops from 4 B to ~4/32 B per stored entry.  Other slices keep explicit
-// column indices.  Entries of a row are visited in increasing column order in both modes.
+// SELL-32 upload of the host layout built by sell_build (sell.cpp).
 int build_sell(cagmres* h, const cagmres_plan& p) {
-    const int64_t nr = p.n_mat;
-    const int64_t ns = (nr + 31) / 32;
-    std::vector<int64_t> sptr(size_t(ns) + 1, 0), sinfo(static_cast<size_t>(ns));
-    std::vector<std::vector<int32_t>> offs(static_cast<size_t>(ns));
-    std::vector<char> dia(static_cast<size_t>(ns), 0);
-    int64_t ndcol = 0, ndia = 0;
-    for (int64_t sl = 0; sl < ns; ++sl) {
-        int64_t wmax = 0;
-        std::vector<int64_t> o;
-        for (int64_t r = sl * 32; r < std::min(nr, sl * 32 + 32); ++r) {
-            wmax = std::max(wmax, p.rowptr[size_t(r) + 1] - p.rowptr[size_t(r)]);
-            for (int64_t e = p.rowptr[size_t(r)]; e < p.rowptr[size_t(r) + 1]; ++e)
-                o.push_back(int64_t(p.colind[size_t(e)]) - r);
-        }
-        std::sort(o.begin(), o.end());
-        o.erase(std::unique(o.begin(), o.end()), o.end());
-        const bool use_dia = int64_t(o.size()) <= wmax + (wmax + 3) / 4 && o.size() <= 32 &&
-                             (o.empty() || (o.front() > INT32_MIN / 2 && o.back() < INT32_MAX / 2));
-        int64_t wdt = wmax;
-        if (use_dia) {
-            dia[size_t(sl)] = 1;
-            ++ndia;
-            wdt = int64_t(o.size());
-            offs[size_t(sl)].assign(o.begin(), o.end());
-            // clamp flag: some row + offset of this slice leaves [0, n_ext)
-            const int64_t r0 = sl * 32, r1 = sl * 32 + 31;
-            const bool clamp = !o.empty() && (r0 + o.front() < 0 || r1 + o.back() >= p.n_ext);
-            sinfo[size_t(sl)] = (ndcol << 2) | (clamp ? 2 : 0) | 1;
-            ndcol += wdt;
-        } else {
-            sinfo[size_t(sl)] = ndcol << 2;
-            ndcol += 32 * wdt;
-        }
-        sptr[size_t(sl) + 1] = sptr[size_t(sl)] + 32 * wdt;
+    SellHost sh;
+    try {
+        sell_build(p, sh);
+    } catch (...) {
+        return CAGMRES_ENOMEM;
     }
-    const int64_t tot = sptr[size_t(ns)];
-    std::vector<int32_t> dcol(static_cast<size_t>(std::max<int64_t>(ndcol, 1)));
-    std::vector<double> val(static_cast<size_t>(std::max<int64_t>(tot, 1)), 0.0);
-    for (int64_t sl = 0; sl < ns; ++sl) {
-        const int64_t wdt = (sptr[size_t(sl) + 1] - sptr[size_t(sl)]) / 32;
-        const int64_t dp = sinfo[size_t(sl)] >> 2;
-        if (dia[size_t(sl)]) {
-            const std::vector<int32_t>& of = offs[size_t(sl)];
-            for (int64_t t = 0; t < wdt; ++t) dcol[size_t(dp + t)] = of[size_t(t)];
-            for (int lane = 0; lane < 32; ++lane) {
-                const int64_t r = sl * 32 + lane;
-                if (r >= nr) continue;
-                int64_t t = 0;
-                for (int64_t e = p.rowptr[size_t(r)]; e < p.rowptr[size_t(r) + 1]; ++e) {
-                    const int64_t off = int64_t(p.colind[size_t(e)]) - r;
-                    while (of[size_t(t)] != off) ++t;          // offsets and columns both ascend
-                    val[size_t(sptr[size_t(sl)] + 32 * t + lane)] = p.val[size_t(e)];
-                }
-            }
-        } else {
-            for (int lane = 0; lane < 32; ++lane) {
-                const int64_t r = sl * 32 + lane;
-                const int64_t b = r < nr ? p.rowptr[size_t(r)] : 0, e = r < nr ? p.rowptr[size_t(r) + 1] : 0;
-                for (int64_t t = 0; t < wdt; ++t) {
-                    const int64_t o = sptr[size_t(sl)] + 32 * t + lane;
-                    if (b + t < e) {
-                        dcol[size_t(dp + 32 * t + lane)] = p.colind[size_t(b + t)];
-                        val[size_t(o)] = p.val[size_t(b + t)];
-                    } else {
-                        dcol[size_t(dp + 32 * t + lane)] = int32_t(r < nr ? r : 0);
-                    }
-                }
-            }
-        }
-    }
+    const int64_t nr = p.n_mat, ns = sh.nslices, tot = sh.sptr[size_t(ns)], ndcol = int64_t(sh.dcol.size());
+    const std::vector<int64_t>& sptr = sh.sptr;
+    const std::vector<int64_t>& sinfo = sh.sinfo;
+    const std::vector<int32_t>& dcol = sh.dcol;
+    const std::vector<double>& val = sh.val;
+    const int64_t ndia = sh.ndia;
     h->A.nrows = nr; h->A.nslices = ns; h->A.nstored = tot; h->A.nnz = p.nnz_mat;
     h->A.ncols = p.n_ext; h->A.ndcol = ndcol; h->A.ndia = ndia;
     {   // most common width among unclamped DIA slices (the specialised SpMV's fast path)
@@ -299,8 +241,8 @@ int common_alloc(cagmres* h) {
     CU(cudaMalloc(&h->arn_part, sizeof(double) * kern::arnoldi_ws_doubles(h->dev)));
     CU(cudaMalloc(&h->arn_counter, sizeof(unsigned int) * kern::XTY_COUNTERS));
     CU(cudaMemset(h->arn_counter, 0, sizeof(unsigned int) * kern::XTY_COUNTERS));
-    CU(cudaMalloc(&h->status, sizeof(int)));
-    CU(cudaMemset(h->status, 0, sizeof(int)));
+    CU(cudaMalloc(&h->status, sizeof(int) * 2));            // [0] breakdown flags, [1] SVQR retries
+    CU(cudaMemset(h->status, 0, sizeof(int) * 2));
     return CAGMRES_OK;
 }
 
@@ -411,13 +353,23 @@ int spmv_autotune(cagmres* h) {
     return CAGMRES_OK;
 }
 
+int init_common_(cagmres* h, const cagmres_csr* A, const int64_t* row_starts, int s, int m,
+                 int basis, int orth);
 int init_common(cagmres* h, const cagmres_csr* A, const int64_t* row_starts, int s, int m,
                 int basis, int orth) {
+    const auto t0 = std::chrono::steady_clock::now();
+    const int st = init_common_(h, A, row_starts, s, m, basis, orth);
+    h->ms_setup = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    return st;
+}
+int init_common_(cagmres* h, const cagmres_csr* A, const int64_t* row_starts, int s, int m,
+                 int basis, int orth) {
     if (s < 1 || m < 1 || s > m || s > 31 || (basis != CAGMRES_MONOMIAL && basis != CAGMRES_NEWTON && basis != CAGMRES_GMRES))
         return CAGMRES_EINVAL;
     const int kind = orth & CAGMRES_TSQR_MASK;
     if (kind > CAGMRES_CAQR) return CAGMRES_EINVAL;
     if ((orth & CAGMRES_ONEPASS) && (kind != CAGMRES_CHOLQR || (orth & CAGMRES_BORTH_MGS))) return CAGMRES_EINVAL;
+    if ((orth & CAGMRES_SVQR_RETRY) && kind != CAGMRES_CHOLQR) return CAGMRES_EINVAL;
     if (kind == CAGMRES_CAQR && h->nranks > 1) return CAGMRES_ENOTSUP;   // single-GPU tree only
     h->s = s; h->m = m; h->basis = basis; h->orth = orth;
     int dv = 0;
@@ -446,7 +398,7 @@ int init_common(cagmres* h, const cagmres_csr* A, const int64_t* row_starts, int
         CU(cudaMalloc(&d_cnt, sizeof(int64_t) * size_t(P)));
         CU(cudaMalloc(&d_all, sizeof(int64_t) * size_t(P) * size_t(P)));
         CU(cudaMemcpy(d_cnt, myc.data(), sizeof(int64_t) * size_t(P), cudaMemcpyHostToDevice));
-        NC(ncclAllGather(d_cnt, d_all, size_t(P), ncclInt64, h->comm, h->stream));
+        TRY(h->tr->allgather(d_cnt, d_all, sizeof(int64_t) * size_t(P), h->stream));
         std::vector<int64_t> all(size_t(P) * size_t(P));
         CU(cudaMemcpyAsync(all.data(), d_all, sizeof(int64_t) * all.size(), cudaMemcpyDeviceToHost, h->stream));
         CU(cudaStreamSynchronize(h->stream));
@@ -464,17 +416,17 @@ int init_common(cagmres* h, const cagmres_csr* A, const int64_t* row_starts, int
             CU(cudaMemcpy(d_og, plan.req_gid.data(), sizeof(int64_t) * size_t(tout), cudaMemcpyHostToDevice));
             CU(cudaMemcpy(d_ol, plan.req_level.data(), sizeof(int32_t) * size_t(tout), cudaMemcpyHostToDevice));
         }
-        NC(ncclGroupStart());
+        std::vector<Msg> sends, recvs;
         int64_t oo = 0, io = 0;
         for (int q = 0; q < P; ++q) {
             const int64_t so = plan.req_counts[size_t(q)], si = inc[size_t(q)];
-            if (so) { NC(ncclSend(d_og + oo, size_t(so), ncclInt64, q, h->comm, h->stream));
-                      NC(ncclSend(d_ol + oo, size_t(so), ncclInt32, q, h->comm, h->stream)); }
-            if (si) { NC(ncclRecv(d_ig + io, size_t(si), ncclInt64, q, h->comm, h->stream));
-                      NC(ncclRecv(d_il + io, size_t(si), ncclInt32, q, h->comm, h->stream)); }
+            if (so) { sends.push_back({q, d_og + oo, sizeof(int64_t) * size_t(so)});
+                      sends.push_back({q, d_ol + oo, sizeof(int32_t) * size_t(so)}); }
+            if (si) { recvs.push_back({q, d_ig + io, sizeof(int64_t) * size_t(si)});
+                      recvs.push_back({q, d_il + io, sizeof(int32_t) * size_t(si)}); }
             oo += so; io += si;
         }
-        NC(ncclGroupEnd());
+        TRY(h->tr->exchange(sends, recvs, h->stream));
         std::vector<int64_t> ig(static_cast<size_t>(tin));
         std::vector<int32_t> il(static_cast<size_t>(tin));
         if (tin) {
@@ -501,33 +453,49 @@ int init_common(cagmres* h, const cagmres_csr* A, const int64_t* row_starts, int
         CU(cudaMalloc(&h->d_recv_ext, sizeof(int64_t) * size_t(std::max<int64_t>(tout, 1))));
         CU(cudaMalloc(&h->d_sendbuf, sizeof(double) * size_t(std::max<int64_t>(tin, 1))));
         CU(cudaMalloc(&h->d_recvbuf, sizeof(double) * size_t(std::max<int64_t>(tout, 1))));
+        CU(cudaMemset(h->d_sendbuf, 0, sizeof(double) * size_t(std::max<int64_t>(tin, 1))));
+        CU(cudaMemset(h->d_recvbuf, 0, sizeof(double) * size_t(std::max<int64_t>(tout, 1))));
         if (tin) CU(cudaMemcpy(h->d_send_idx, plan.send_idx.data(), sizeof(int64_t) * size_t(tin), cudaMemcpyHostToDevice));
         if (tout) CU(cudaMemcpy(h->d_recv_ext, plan.req_ext.data(), sizeof(int64_t) * size_t(tout), cudaMemcpyHostToDevice));
     }
     return CAGMRES_OK;
 }
 
-// ---- collectives ---------------------------------------------------------------------
+// ---- collectives (transport.h: NCCL, or the in-process group) -------------------------
 int allreduce(cagmres* h, double* buf, size_t cnt) {
     if (h->nranks == 1 || cnt == 0) return CAGMRES_OK;
-    NC(ncclAllReduce(buf, buf, cnt, ncclDouble, ncclSum, h->comm, h->stream));
-    return CAGMRES_OK;
+    return h->tr->allreduce_sum(buf, cnt, h->stream);
 }
 
 // Halo exchange of the ghost rows (distance <= depth) of an extended vector (Fig. 4 setup,
-// P:66): pack owned values other ranks need, NCCL send/recv over NVLink, unpack.
+// P:66): pack the owned values the peers need at this depth, grouped send / recv (NVLink),
+// unpack.  Every peer's send / request list is sorted by level, so the depth-limited message
+// to or from a peer is a prefix of its segment; only those prefixes are packed and unpacked.
 int halo(cagmres* h, double* vec, int depth) {
     if (h->nranks == 1 || depth <= 0) return CAGMRES_OK;
-    kern::gather(vec, h->d_send_idx, h->nsend, h->d_sendbuf, h->stream);
-    NC(ncclGroupStart());
+    depth = std::min(depth, h->s);
+    std::vector<std::pair<int64_t, int64_t>> ss, rs;          // (offset, count) per peer
+    std::vector<Msg> sends, recvs;
     for (int q = 0; q < h->nranks; ++q) {
         const int64_t sc = h->send_pre[size_t(q)][size_t(depth)], rc = h->recv_pre[size_t(q)][size_t(depth)];
-        if (sc) NC(ncclSend(h->d_sendbuf + h->send_off[size_t(q)], size_t(sc), ncclDouble, q, h->comm, h->stream));
-        if (rc) NC(ncclRecv(h->d_recvbuf + h->recv_off[size_t(q)], size_t(rc), ncclDouble, q, h->comm, h->stream));
+        if (sc) {
+            ss.push_back({h->send_off[size_t(q)], sc});
+            sends.push_back({q, h->d_sendbuf + h->send_off[size_t(q)], sizeof(double) * size_t(sc)});
+        }
+        if (rc) {
+            rs.push_back({h->recv_off[size_t(q)], rc});
+            recvs.push_back({q, h->d_recvbuf + h->recv_off[size_t(q)], sizeof(double) * size_t(rc)});
+        }
     }
-    NC(ncclGroupEnd());
-    kern::scatter(h->d_recvbuf, h->d_recv_ext, h->nrecv, vec, h->stream);
-    return CAGMRES_OK;
+    auto segs = [](const std::vector<std::pair<int64_t, int64_t>>& v, size_t i0) {
+        kern::Segs sg{};
+        for (size_t i = i0; i < v.size() && i < i0 + 32; ++i) sg.add(v[i].first, v[i].second);
+        return sg;
+    };
+    for (size_t i = 0; i < ss.size(); i += 32) kern::gather_segs(vec, h->d_send_idx, segs(ss, i), h->d_sendbuf, h->stream);
+    TRY(h->tr->exchange(sends, recvs, h->stream));
+    for (size_t i = 0; i < rs.size(); i += 32) kern::scatter_segs(h->d_recvbuf, h->d_recv_ext, segs(rs, i), vec, h->stream);
+    return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
 }
 
 // ---- building blocks ------------------------------------------------------------------
@@ -636,12 +604,13 @@ int borth_panel(cagmres* h, const double* Q, int64_t ldq, int j, double* P, int6
 
 // TSQR of the panel P (n_loc x w, ld ldp), R (device w x w, ld w).  c0 = 1 leaves column 0
 // unwritten (the block's start vector q_j is kept, reading G2).
-int tsqr_panel(cagmres* h, double* P, int64_t ldp, int w, double* R, int kind, int c0) {
+int tsqr_panel(cagmres* h, double* P, int64_t ldp, int w, double* R, int kind, int c0, bool retry = false) {
     Scope sc(h, PH_TSQR);
     const double nl = double(h->n_loc);
     if (kind == CAGMRES_CHOLQR || kind == CAGMRES_SVQR) {
         if (kind == CAGMRES_CHOLQR) {
             TRY(xty_global(h, P, ldp, w, P, ldp, w, h->gbuf, true, R));     // B = V^T V ; R = chol(B)
+            if (retry) kern::svqr_retry(h->gbuf, w, R, h->status, h->stream);   // G15 opt-in
         } else {
             TRY(xty_global(h, P, ldp, w, P, ldp, w, h->gbuf, false, nullptr));
             kern::svqr_factor(h->gbuf, w, R, h->status, h->stream);
@@ -702,16 +671,52 @@ std::vector<Block> schedule(int s, int m) {
     return bl;
 }
 
+int diag_alloc(cagmres* h) {
+    if (h->dg) return CAGMRES_OK;
+    const size_t W = size_t(h->s) + 1;
+    h->dg_cap = 2 * W * W * (size_t(h->m) + 1);
+    CU(cudaMalloc(&h->dg, sizeof(double) * h->dg_cap));
+    CU(cudaMemset(h->dg, 0, sizeof(double) * h->dg_cap));
+    CU(cudaMallocHost(&h->h_dg, sizeof(double) * h->dg_cap));
+    return CAGMRES_OK;
+}
+
+// Per-panel diagnostics of the cycle just copied to h_dg: max kappa_2(W^T W) and max
+// ||I - Q_p^T Q_p||_2 over the blocks (Fig. 12).
+void diag_reduce(cagmres* h, const std::vector<Block>& bl, double& max_orth, double& max_cond) {
+    const size_t W = size_t(h->s) + 1;
+    std::vector<double> ev(W), G(W * W);
+    for (size_t bi = 0; bi < bl.size(); ++bi) {
+        const int w = bl[bi].sb + 1;
+        const double* g0 = h->h_dg + bi * 2 * W * W;
+        host::sym_eigvals(g0, w, w, ev.data());
+        const double cond = ev[0] > 0.0 ? ev[size_t(w - 1)] / ev[0] : INFINITY;
+        max_cond = std::max(max_cond, cond);
+        const double* g1 = g0 + W * W;
+        for (int c = 0; c < w; ++c)
+            for (int i = 0; i < w; ++i) G[size_t(i) + size_t(w) * c] = (i == c ? 1.0 : 0.0) - g1[size_t(i) + size_t(w) * c];
+        host::sym_eigvals(G.data(), w, w, ev.data());
+        max_orth = std::max(max_orth, std::max(std::fabs(ev[0]), std::fabs(ev[size_t(w - 1)])));
+    }
+}
+
 // One CA cycle's GPU work: per block MPK -> BOrth -> TSQR [-> BOrth -> TSQR].
 int ca_cycle(cagmres* h, const std::vector<Block>& bl) {
     const int kind = h->orth & CAGMRES_TSQR_MASK;
     const bool re2 = (h->orth & CAGMRES_REORTH) != 0, mgs = (h->orth & CAGMRES_BORTH_MGS) != 0;
+    const size_t W2 = (size_t(h->s) + 1) * (size_t(h->s) + 1);
+    size_t bi = 0;
     for (const Block& b : bl) {
         const int j = b.j, sb = b.sb, w = sb + 1;
         const std::vector<host::Step> steps = h->basis == CAGMRES_MONOMIAL
             ? host::block_steps({}, {}, sb) : host::block_steps(h->sh_re, h->sh_im, sb);
         TRY(mpk_block(h, j, sb, steps));
         double* Pj = h->V + size_t(h->ldv) * j;                 // panel [q_j | W_1 .. W_sb]
+        double* dgb = h->diag_on ? h->dg + 2 * W2 * bi++ : nullptr;
+        if (dgb) {                                              // diagnostics: W^T W of the MPK output
+            Scope sc(h, PH_OTHER);
+            TRY(xty_global(h, Pj, h->ldv, w, Pj, h->ldv, w, dgb, false, nullptr));
+        }
         for (int pass = 0; pass < (re2 ? 2 : 1); ++pass) {
             double* C = h->tab + (pass ? b.c2 : b.c1);
             double* R = h->tab + (pass ? b.r2 : b.r1);
@@ -755,11 +760,15 @@ int ca_cycle(cagmres* h, const std::vector<Block>& bl) {
                     continue;
                 }
                 h->bytes[PH_BORTH] += 8.0 * nl * (2.0 * j + 3.0 * sb);
-                TRY(tsqr_panel(h, Pj, h->ldv, w, R, kind, 1));
+                TRY(tsqr_panel(h, Pj, h->ldv, w, R, kind, 1, (h->orth & CAGMRES_SVQR_RETRY) != 0));
                 continue;
             }
             TRY(borth_panel(h, h->V, h->ldv, j, Pj + h->ldv, h->ldv, sb, C, mgs));
-            TRY(tsqr_panel(h, Pj, h->ldv, w, R, kind, 1));
+            TRY(tsqr_panel(h, Pj, h->ldv, w, R, kind, 1, (h->orth & CAGMRES_SVQR_RETRY) != 0));
+        }
+        if (dgb) {                                              // ... and Q_p^T Q_p after the passes
+            Scope sc(h, PH_OTHER);
+            TRY(xty_global(h, Pj, h->ldv, w, Pj, h->ldv, w, dgb + W2, false, nullptr));
         }
     }
     return CAGMRES_OK;
@@ -863,7 +872,9 @@ int enqueue_cycle(cagmres* h, bool arnoldi, const std::vector<Block>& bl) {
         TRY(ca_cycle(h, bl));
     }
     CU(cudaMemcpyAsync(h->h_tab, h->tab, sizeof(double) * h->tab_cap, cudaMemcpyDeviceToHost, h->stream));
-    CU(cudaMemcpyAsync(h->h_stat, h->status, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+    if (h->diag_on && !arnoldi)
+        CU(cudaMemcpyAsync(h->h_dg, h->dg, sizeof(double) * h->dg_cap, cudaMemcpyDeviceToHost, h->stream));
+    CU(cudaMemcpyAsync(h->h_stat, h->status, sizeof(int) * 2, cudaMemcpyDeviceToHost, h->stream));
     CU(cudaEventRecord(h->ev_tab, h->stream));
     return CAGMRES_OK;
 }
@@ -893,7 +904,7 @@ const char* cagmres_strerror(int s) {
         case CAGMRES_NOT_CONVERGED: return "not converged within maxit restart cycles";
         case CAGMRES_EINVAL: return "invalid argument";
         case CAGMRES_ECUDA: return "CUDA error";
-        case CAGMRES_ENCCL: return "NCCL error";
+        case CAGMRES_ENCCL: return "communication error (NCCL call or in-process group collective failed)";
         case CAGMRES_EBREAKDOWN: return "numerical breakdown (Cholesky pivot <= 0 / zero norm)";
         case CAGMRES_ENOMEM: return "out of memory";
         case CAGMRES_EGHOST: return "supplied rows do not cover the ghost rows";
@@ -929,9 +940,26 @@ int cagmres_create_dist(cagmres_t* out, const cagmres_csr* A, const int64_t* row
     if (!h) return CAGMRES_ENOMEM;
     h->rank = rank; h->nranks = nranks;
     if (nranks > 1) {
-        ncclUniqueId id;
-        std::memcpy(&id, nccl_unique_id, sizeof(id));
-        if (ncclCommInitRank(&h->comm, nranks, id, rank) != ncclSuccess) { delete h; return CAGMRES_ENCCL; }
+        h->tr.reset(make_nccl_transport(nccl_unique_id, rank, nranks));
+        if (!h->tr) { delete h; return CAGMRES_ENCCL; }
+    }
+    const int st = init_common(h, A, row_starts, s, m, basis, orth);
+    if (st != CAGMRES_OK) { delete h; return st; }
+    *out = h;
+    return CAGMRES_OK;
+}
+
+int cagmres_create_group(cagmres_t* out, const cagmres_csr* A, const int64_t* row_starts,
+                         int s, int m, int basis, int orth, cagmres_group_t g, int rank) {
+    if (!out || !A || !row_starts || !g || rank < 0 || rank >= g->P) return CAGMRES_EINVAL;
+    *out = nullptr;
+    if (cudaSetDevice(g->device[size_t(rank)]) != cudaSuccess) return CAGMRES_ECUDA;
+    cagmres* h = new (std::nothrow) cagmres();
+    if (!h) return CAGMRES_ENOMEM;
+    h->rank = rank; h->nranks = g->P;
+    if (g->P > 1) {
+        h->tr.reset(make_group_transport(g, rank));
+        if (!h->tr) { delete h; return CAGMRES_ENCCL; }
     }
     const int st = init_common(h, A, row_starts, s, m, basis, orth);
     if (st != CAGMRES_OK) { delete h; return st; }
@@ -1060,10 +1088,12 @@ int cagmres_tsqr(cagmres_t h, double* P, int64_t ldp, int w, double* R, int orth
     const int kind = orth & CAGMRES_TSQR_MASK;
     if (kind > CAGMRES_CAQR) return CAGMRES_EINVAL;
     CU(cudaMemsetAsync(h->status, 0, sizeof(int), h->stream));
-    TRY(tsqr_panel(h, P, ldp, w, R, kind, 0));
+    const bool retry = (orth & CAGMRES_SVQR_RETRY) && kind == CAGMRES_CHOLQR;
+    CU(cudaMemsetAsync(h->status, 0, sizeof(int) * 2, h->stream));
+    TRY(tsqr_panel(h, P, ldp, w, R, kind, 0, retry));
     if (orth & CAGMRES_REORTH) {
         double* R2 = h->tab;                        // scratch
-        TRY(tsqr_panel(h, P, ldp, w, R2, kind, 0));
+        TRY(tsqr_panel(h, P, ldp, w, R2, kind, 0, retry));
         std::vector<double> r1(size_t(w) * w), r2(size_t(w) * w), rr(size_t(w) * w, 0.0);
         CU(cudaMemcpyAsync(r1.data(), R, sizeof(double) * r1.size(), cudaMemcpyDeviceToHost, h->stream));
         CU(cudaMemcpyAsync(r2.data(), R2, sizeof(double) * r2.size(), cudaMemcpyDeviceToHost, h->stream));
@@ -1094,7 +1124,11 @@ int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit
     if (st) { st->cycles = 0; st->iters = 0; st->hist_len = 0; }
     cudaEvent_t t0 = nullptr, t1 = nullptr;
     if (h->timer.on) { t0 = h->timer.get(); cudaEventRecord(t0, h->stream); }
-    CU(cudaMemsetAsync(h->status, 0, sizeof(int), h->stream));
+    CU(cudaMemsetAsync(h->status, 0, sizeof(int) * 2, h->stream));
+    h->h_stat[1] = 0;
+    h->diag_on = st && st->collect_diag;
+    double max_orth = 0.0, max_cond = 0.0;
+    if (h->diag_on) TRY(diag_alloc(h));
     double rho0 = 0.0, beta = 0.0;
     TRY(residual_norm_async(h, b, x));
     CU(cudaEventSynchronize(h->ev_beta));
@@ -1117,6 +1151,7 @@ int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit
         pending = false;
         CU(cudaEventSynchronize(h->ev_tab));
         if (*h->h_stat) { rc = CAGMRES_EBREAKDOWN; break; }
+        if (h->diag_on && !arnoldi) diag_reduce(h, bl, max_orth, max_cond);
         // ---- Hessenberg matrix (host) ----
         if (arnoldi) {
             const size_t stride = 2 * size_t(m + 1) + 1;
@@ -1203,6 +1238,10 @@ int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit
         st->bytes_mpk = h->bytes[PH_MPK]; st->bytes_borth = h->bytes[PH_BORTH];
         st->bytes_tsqr = h->bytes[PH_TSQR]; st->bytes_other = h->bytes[PH_OTHER];
         st->bytes_spmv = h->bytes[PH_SPMV]; st->spmv_launches = h->spmv_launches;
+        st->ms_setup = h->ms_setup;
+        st->retried_panels = h->h_stat[1];
+        st->max_orth_err = max_orth;
+        st->max_gram_cond = max_cond;
         st->ms_mpk = st->ms_borth = st->ms_tsqr = st->ms_other = st->ms_total = st->ms_spmv = 0.0;
         if (h->timer.on) {
             float tt = 0.f;
@@ -1213,6 +1252,7 @@ int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit
     }
     h->timer.reset();
     h->timer.on = false;
+    h->diag_on = false;
     return rc;
 }
 

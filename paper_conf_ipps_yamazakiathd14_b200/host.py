@@ -66,10 +66,33 @@ class Plan:
                                                  L.i32ptr(levels)), "set_sends")
         self._send_total = int(counts.sum())
 
+    def sell(self):
+        """The SELL-32 layout create() uploads (cagmres_plan_sell): dict of numpy arrays."""
+        ns, nd, nv = C.c_int64(), C.c_int64(), C.c_int64()
+        L.check(self._lib.cagmres_plan_sell(self._p, C.byref(ns), C.byref(nd), C.byref(nv), None, None, None,
+                                            None), "plan_sell")
+        sptr = np.zeros(ns.value + 1, dtype=np.int64)
+        sinfo = np.zeros(max(ns.value, 1), dtype=np.int64)
+        dcol = np.zeros(max(nd.value, 1), dtype=np.int32)
+        val = np.zeros(max(nv.value, 1), dtype=np.float64)
+        L.check(self._lib.cagmres_plan_sell(self._p, None, None, None, L.i64ptr(sptr), L.i64ptr(sinfo),
+                                            L.i32ptr(dcol), L.dptr(val)), "plan_sell")
+        return dict(sptr=sptr, sinfo=sinfo[:ns.value], dcol=dcol[:nd.value], val=val[:nv.value])
+
     def send_index(self):
         idx = np.zeros(max(self._send_total, 1), dtype=np.int64)
         L.check(self._lib.cagmres_plan_send_index(self._p, L.i64ptr(idx)), "send_index")
         return idx[:self._send_total]
+
+
+def sym_eigvals(A):
+    """Eigenvalues (ascending) of a symmetric matrix by the library's host Jacobi routine."""
+    lib = L.load()
+    Af = np.asfortranarray(A, dtype=np.float64)
+    n = Af.shape[0]
+    ev = np.zeros(n)
+    L.check(lib.cagmres_host_sym_eigvals(Af.ctypes.data_as(L._PD), n, n, L.dptr(ev)), "sym_eigvals")
+    return ev
 
 
 def eigvals(H, m):

@@ -40,6 +40,35 @@ def _csr_struct(A, own_begin=None, own_end=None):
     return s, (rowptr, colind, val)
 
 
+class Group:
+    """In-process group of `nranks` ranks (cagmres_group_create): each rank's Solver is built
+    and driven from its own Python thread (ctypes releases the GIL inside the library), on
+    devices[rank] (default: all on the current device).  Runs the whole multi-rank device
+    path — halo exchange, cross-rank sums — inside one process, e.g. on one GPU."""
+
+    def __init__(self, nranks, devices=None):
+        self._lib = L.load()
+        self.nranks = int(nranks)
+        self._g = C.c_void_p()
+        if devices is None:
+            import torch
+            devices = [torch.cuda.current_device()] * self.nranks
+        self.devices = [int(d) for d in devices]
+        arr = (C.c_int * self.nranks)(*self.devices)
+        L.check(self._lib.cagmres_group_create(C.byref(self._g), self.nranks, arr), "group_create")
+
+    def close(self):
+        if self._g:
+            L.check(self._lib.cagmres_group_destroy(self._g), "group_destroy")
+            self._g = C.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
 @dataclass
 class SolveStats:
     status: int
@@ -49,6 +78,10 @@ class SolveStats:
     ms: dict = field(default_factory=dict)
     bytes: dict = field(default_factory=dict)
     spmv_launches: int = 0
+    max_orth_err: float = 0.0
+    max_gram_cond: float = 0.0
+    ms_setup: float = 0.0
+    retried_panels: int = 0
 
 
 class Solver:
@@ -56,23 +89,33 @@ class Solver:
 
     A: host CSR with attributes n, rowptr (int64), colind (int32, global ids), val (float64)
        and row_begin (first global row described; 0 for the full matrix).
-    group: a torch.distributed process group for the multi-GPU path (one process per GPU);
-       the caller passes this rank's owned rows plus >= (s-1)-hop ghost rows and row_starts.
+    group: a torch.distributed process group for the multi-GPU path (one process per GPU,
+       NCCL), or a `Group` (in-process ranks, one thread each; pass `rank`); the caller
+       passes this rank's owned rows plus >= (s-1)-hop ghost rows and row_starts.
     """
 
     def __init__(self, A, s, m, basis="newton", tsqr="cholqr", reorth=False, borth="cgs",
-                 group=None, row_starts=None, device=None, onepass=False):
+                 group=None, row_starts=None, device=None, onepass=False, rank=None, svqr_retry=False):
         import torch
         self._lib = L.load()
         self.s, self.m = int(s), int(m)
         self.basis = basis
-        self.orth = orth_flags(tsqr, reorth, borth, onepass)
+        self.orth = orth_flags(tsqr, reorth, borth, onepass) | (L.SVQR_RETRY if svqr_retry else 0)
         self._h = C.c_void_p()
+        if isinstance(group, Group):
+            device = group.devices[rank]
         if device is None:
             device = torch.cuda.current_device()
         self.device = torch.device("cuda", device)
         torch.cuda.set_device(self.device)
-        if group is None:
+        if isinstance(group, Group):
+            rs = np.ascontiguousarray(row_starts, dtype=np.int64)
+            st, keep = _csr_struct(A, rs[rank], rs[rank + 1])
+            self._group = group                          # keeps the group alive
+            L.check(self._lib.cagmres_create_group(C.byref(self._h), C.byref(st), L.i64ptr(rs), self.s, self.m,
+                                                   _BASIS[basis], self.orth, group._g, int(rank)),
+                    "cagmres_create_group")
+        elif group is None:
             st, keep = _csr_struct(A)
             L.check(self._lib.cagmres_create(C.byref(self._h), C.byref(st), self.s, self.m,
                                              _BASIS[basis], self.orth), "cagmres_create")
@@ -194,7 +237,7 @@ class Solver:
         L.check(st, "tsqr")
         return R.t()
 
-    def solve(self, b, x=None, tol=1e-8, maxit=200, timing=False):
+    def solve(self, b, x=None, tol=1e-8, maxit=200, timing=False, diag=False):
         """Solve on device tensors b, x (owned rows, float64); x updated in place."""
         import torch
         if x is None:
@@ -204,6 +247,7 @@ class Solver:
         st.hist_cap = len(hist)
         st.rel_resid_hist = L.dptr(hist)
         st.collect_timing = int(timing) if timing else 0       # True/1: all phases, 2: MPK kernel only
+        st.collect_diag = int(bool(diag))
         status = self._lib.cagmres_solve(self._h, C.c_void_p(b.data_ptr()), C.c_void_p(x.data_ptr()),
                                          float(tol), int(maxit), C.byref(st))
         L.check(status, "solve")
@@ -212,5 +256,7 @@ class Solver:
                                    total=st.ms_total, spmv=st.ms_spmv),
                            bytes=dict(mpk=st.bytes_mpk, borth=st.bytes_borth, tsqr=st.bytes_tsqr,
                                       other=st.bytes_other, spmv=st.bytes_spmv),
-                           spmv_launches=st.spmv_launches)
+                           spmv_launches=st.spmv_launches, max_orth_err=st.max_orth_err,
+                           max_gram_cond=st.max_gram_cond, ms_setup=st.ms_setup,
+                           retried_panels=st.retried_panels)
         return x, stats

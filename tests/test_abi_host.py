@@ -148,6 +148,94 @@ def test_plan_levels_match_oracle_boundary_sets(gen, nr, s):
             assert np.array_equal(va[rp[e]:rp[e + 1]], As.data[lo:hi])
 
 
+def _sell_rows(p, ext):
+    """Rows of the SELL-32 layout create() uploads, in stored (= summation) order, as
+    (global columns, values) with padding entries (exact zeros) dropped."""
+    S = p.sell()
+    rows = []
+    for r in range(p.n_mat):
+        sl, lane = divmod(r, 32)
+        info = int(S["sinfo"][sl])
+        W = int(S["sptr"][sl + 1] - S["sptr"][sl]) // 32
+        dp = info >> 2
+        idx = S["sptr"][sl] + 32 * np.arange(W) + lane
+        v = S["val"][idx]
+        if info & 1:
+            c = r + S["dcol"][dp:dp + W].astype(np.int64)
+        else:
+            c = S["dcol"][dp + 32 * np.arange(W) + lane].astype(np.int64)
+        keep = v != 0.0
+        assert np.all((c[keep] >= 0) & (c[keep] < p.n_ext))
+        rows.append((ext[c[keep]], v[keep]))
+    return rows
+
+
+def _scrambled(A, seed):
+    """The same matrix as an unsorted CSR with one entry per row split into two repeats."""
+    from synth.generators import CSR
+    rp, ci, va = [0], [], []
+    rng = np.random.default_rng(seed)
+    for r in range(A.nrows):
+        c = A.colind[A.rowptr[r]:A.rowptr[r + 1]].tolist()
+        v = A.val[A.rowptr[r]:A.rowptr[r + 1]].tolist()
+        k = int(rng.integers(len(c)))
+        c.append(c[k]); v.append(0.25 * v[k]); v[k] = 0.75 * v[k]
+        order = rng.permutation(len(c))
+        ci += [c[i] for i in order]; va += [v[i] for i in order]
+        rp.append(len(ci))
+    return CSR(n=A.n, row_begin=A.row_begin, rowptr=np.array(rp, dtype=np.int64),
+               colind=np.array(ci, dtype=np.int32), val=np.array(va))
+
+
+def _canonical_row(A, g):
+    """Row g of a CSR sorted by column, repeated columns summed in input order."""
+    lo, hi = A.rowptr[g - A.row_begin], A.rowptr[g - A.row_begin + 1]
+    c, v = A.colind[lo:hi].astype(np.int64), A.val[lo:hi]
+    out = {}
+    for k in np.argsort(c, kind="stable"):
+        out[c[k]] = out[c[k]] + v[k] if c[k] in out else v[k]
+    cols = np.array(sorted(out), dtype=np.int64)
+    return cols, np.array([out[k] for k in cols])
+
+
+@pytest.mark.parametrize("gen,nr,s", [("cd7", 2, 3), ("cd7", 4, 4), ("g3", 3, 3), ("band", 3, 2),
+                                      ("cd27", 2, 3), ("cd5_scrambled", 3, 3), ("cd5_scrambled", 1, 3)])
+def test_sell_layout_sums_rows_in_global_column_order(gen, nr, s):
+    """on ranks > 0 the ghost columns that precede the owned ones globally get
+    extended ids >= n_loc, so a DIA slice's diagonals must be ordered by the rows' GLOBAL
+    column order (topological order, sell.cpp), not by local offset.  Every stored row of the
+    uploaded layout, read in summation order, must be the canonical global row (columns
+    ascending, repeats summed in input order) — the premise of multi-rank MPK == single-GPU MPK
+    bit for bit.  Also covers unsorted CSR input with repeated columns."""
+    from paper_conf_ipps_yamazakiathd14_b200.host import Plan
+    A = {"cd7": lambda: G.convection_diffusion(16, 3, 7),
+         "g3": lambda: G.g3_shaped(n=3000, width=60),
+         "band": lambda: G.banded(n=2000),
+         "cd27": lambda: G.convection_diffusion(10, 3, 27),
+         "cd5_scrambled": lambda: _scrambled(G.convection_diffusion(20, 2, 5), 7)}[gen]()
+    rs = O.block_rows(A.n, nr)
+    ndia = 0
+    for r in range(nr):
+        p = Plan(A, rs, r, s)
+        ext = p.ext_rows()
+        ndia += int(np.sum(p.sell()["sinfo"] & 1))
+        for e, (cols, vals) in enumerate(_sell_rows(p, ext)):
+            cref, vref = _canonical_row(A, ext[e])
+            assert np.array_equal(cols, cref), (r, e)
+            assert np.array_equal(vals, vref), (r, e)
+    assert ndia > 0                                     # the DIA path was exercised
+
+
+def test_host_sym_eigvals_matches_numpy():
+    from paper_conf_ipps_yamazakiathd14_b200 import host
+    for n, seed in ((1, 0), (6, 1), (11, 2), (31, 3)):
+        M = G.random_panel(n, n, seed)
+        S = M @ M.T + np.diag(np.logspace(-12, 0, n))
+        ev = host.sym_eigvals(np.triu(S) + np.triu(S, 1).T * 0.0 + np.tril(np.full((n, n), np.nan), -1))
+        ref = np.linalg.eigvalsh(S)
+        assert np.allclose(ev, ref, rtol=0, atol=1e-13 * np.abs(ref).max())
+
+
 def test_plan_reports_missing_ghost_rows():
     from paper_conf_ipps_yamazakiathd14_b200 import _lib as L
     from paper_conf_ipps_yamazakiathd14_b200.host import Plan

@@ -1,0 +1,263 @@
+"""GPU: the multi-rank device path on ONE GPU through the in-process group (cagmres_group,
+transport.h) — P ranks, one host thread each, every rank's handle on device 0.  This runs
+exactly the code the NCCL path runs (setup request exchange, depth-limited halo pack ->
+exchange -> unpack, cross-rank sums followed by the separate Cholesky, distributed residual),
+with peer-to-peer device copies and a fixed-order sum kernel in place of NCCL calls.
+
+Checks (VERDICT r1 "Next round" 1):
+  * MPK: the owned rows of every rank equal the single-GPU MPK BIT FOR BIT (each row is summed
+    in global column order whatever the partition, sell.cpp);
+  * BOrth C and TSQR R of a row-distributed panel match the oracle (relative 1e-10);
+  * solve: per-cycle residuals match the oracle under the DESIGN §8 rule, the cycle count is
+    within +-1, every rank reports bit-identical histories.
+"""
+import threading
+
+import numpy as np
+import pytest
+
+from oracle import cagmres_oracle as O
+from synth import generators as G
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+from test_gpu_parity import SHIFTS, hist_within_envelope, rounding_envelope  # noqa: E402
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _cuda():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_ipps_yamazakiathd14_b200 import _lib
+    _lib.load()
+    torch.cuda.set_device(0)
+
+
+def _mods():
+    from paper_conf_ipps_yamazakiathd14_b200.solver import Group, Solver
+    return Group, Solver
+
+
+GENS = {
+    "cd7_64": lambda: G.convection_diffusion(64, 3, 7),              # 262,144 rows, slabs
+    "g3_40k": lambda: G.g3_shaped(n=40000, width=200),                # long-range edges
+    "band27": lambda: G.banded(n=100003),                             # 27 diagonals, ragged
+}
+
+
+def run_ranks(P, fn, timeout=900):
+    """fn(rank, group) in P threads, each on its own CUDA stream of device 0; returns the
+    per-rank results (re-raises the first exception)."""
+    Group, _ = _mods()
+    grp = Group(P, devices=[0] * P)
+    out, err = [None] * P, [None] * P
+
+    def body(r):
+        try:
+            torch.cuda.set_device(0)
+            st = torch.cuda.Stream()
+            with torch.cuda.stream(st):
+                out[r] = fn(r, grp)
+                st.synchronize()
+        except BaseException as e:  # noqa: BLE001
+            err[r] = e
+
+    th = [threading.Thread(target=body, args=(r,), daemon=True) for r in range(P)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join(timeout)
+    assert not any(t.is_alive() for t in th), "a rank hung"
+    for e in err:
+        if e is not None:
+            raise e
+    return out
+
+
+def dev(x):
+    return torch.tensor(np.ascontiguousarray(x), dtype=torch.float64, device="cuda")
+
+
+def colmajor(M):
+    return dev(np.asarray(M).T).t()
+
+
+# ----------------------------------------------------------------------------- MPK
+@pytest.mark.parametrize("P", [2, 3, 4, 8])
+@pytest.mark.parametrize("gen", sorted(GENS))
+def test_group_mpk_bitwise_equals_single_gpu(P, gen):
+    _, Solver = _mods()
+    A = GENS[gen]()
+    s = 6
+    q = G.u(11, np.arange(A.n))
+    S1 = Solver(A, s=s, m=12, basis="newton")
+    S1.set_shifts(SHIFTS[0][:s], SHIFTS[1][:s])
+    ref = {sb: S1.mpk(dev(q), sb).cpu() for sb in (1, 3, s)}
+    S1.close()
+    rs = O.block_rows(A.n, P)
+
+    def rank(r, grp):
+        S = Solver(A, s=s, m=12, basis="newton", group=grp, row_starts=rs, rank=r)
+        S.set_shifts(SHIFTS[0][:s], SHIFTS[1][:s])
+        lo, hi = rs[r], rs[r + 1]
+        res = {sb: S.mpk(dev(q[lo:hi]), sb).cpu() for sb in (1, 3, s)}
+        S.close()
+        return res
+
+    outs = run_ranks(P, rank)
+    for sb in (1, 3, s):
+        W = torch.cat([o[sb] for o in outs], dim=0)
+        assert torch.equal(W, ref[sb]), (gen, P, sb)
+
+
+def test_group_mpk_monomial_matches_oracle():
+    """Owned rows of a 3-rank monomial MPK vs the oracle's global MPK (Fig. 4)."""
+    _, Solver = _mods()
+    A = G.convection_diffusion(30, 3, 7)
+    As = A.to_scipy()
+    q = G.u(12, np.arange(A.n))
+    rs = O.block_rows(A.n, 3)
+
+    def rank(r, grp):
+        S = Solver(A, s=5, m=10, basis="monomial", group=grp, row_starts=rs, rank=r)
+        W = S.mpk(dev(q[rs[r]:rs[r + 1]]), 5).cpu().numpy()
+        S.close()
+        return W
+
+    W = np.vstack(run_ranks(3, rank))
+    Wo = O.mpk(As, q, 5)
+    for k in range(6):
+        assert np.max(np.abs(W[:, k] - Wo[:, k])) <= 1e-13 * np.max(np.abs(Wo[:, k])), k
+
+
+# ----------------------------------------------------------------------------- BOrth / TSQR
+@pytest.mark.parametrize("P", [2, 3, 8])
+@pytest.mark.parametrize("kind,reorth", [("cholqr", False), ("cholqr", True), ("svqr", False),
+                                         ("cgs", False), ("mgs", False)])
+def test_group_borth_tsqr_match_oracle(P, kind, reorth):
+    """Row-distributed panels: C = Q^T P and R are sums over ranks."""
+    _, Solver = _mods()
+    n, j, w = 60001, 20, 11
+    A = G.banded(n=n)
+    Q, _ = np.linalg.qr(G.random_panel(n, j, 21))
+    Pn = G.random_panel(n, w, 22)
+    Pn[:, 2] += 0.3 * Pn[:, 1]
+    Co, Po = O.borth_cgs(Q, Pn)
+    Qt, Rt = {"cholqr": O.tsqr_cholqr, "svqr": O.tsqr_svqr, "cgs": O.tsqr_cgs,
+              "mgs": O.tsqr_mgs}[kind](Po)
+    if reorth:
+        Qt, R2 = O.tsqr_cholqr(Qt)
+        Rt = R2 @ Rt
+    rs = O.block_rows(n, P)
+
+    def rank(r, grp):
+        lo, hi = rs[r], rs[r + 1]
+        S = Solver(A, s=1, m=max(j, 2), basis="monomial", group=grp, row_starts=rs, rank=r)
+        Qd, Pd = colmajor(Q[lo:hi]), colmajor(Pn[lo:hi])
+        C = S.borth(Qd, j, Pd, w).cpu().numpy()
+        R = S.tsqr(Pd, w, kind, reorth).cpu().numpy()
+        out = (C, R, Pd.cpu().numpy())
+        S.close()
+        return out
+
+    outs = run_ranks(P, rank)
+    for C, R, _ in outs:
+        assert np.allclose(C, Co, rtol=1e-10, atol=1e-12)
+        assert np.allclose(R, Rt, rtol=1e-10, atol=1e-10 * np.abs(Rt).max())
+    assert all(np.array_equal(o[1], outs[0][1]) for o in outs)          # identical R on every rank
+    Qg = np.vstack([o[2] for o in outs])
+    assert O.orth_error(Qg) < 1e-12
+    assert np.allclose(Qg, Qt, rtol=0, atol=1e-10)
+
+
+# ----------------------------------------------------------------------------- solve
+@pytest.mark.parametrize("P,gen,s,m", [(2, "cd7_64", 10, 30), (4, "cd7_64", 10, 30), (8, "cd7_64", 10, 30),
+                                       (3, "g3_40k", 5, 60), (8, "g3_40k", 5, 60), (4, "band27", 10, 30)])
+def test_group_solve_matches_oracle(P, gen, s, m):
+    """Full distributed solve: the Newton first cycle runs on the ranks (GMRES(m) with the
+    1-deep halo and cross-rank CGS sums; Ritz values + Leja order on every rank from identical
+    data), then CA cycles.  Shifts vs the oracle's by value; per-cycle residuals vs the
+    oracle's own solve under the DESIGN §8 rule (its rounding envelope includes the shifts'
+    sensitivity, being measured on permuted reruns of the whole solve)."""
+    _, Solver = _mods()
+    A = GENS[gen]()
+    As = A.to_scipy()
+    b = G.rhs(A.n)
+    rs = O.block_rows(A.n, P)
+    maxit = 200 if gen != "band27" else 4
+
+    def rank(r, grp):
+        S = Solver(A, s=s, m=m, basis="newton", group=grp, row_starts=rs, rank=r)
+        lo, hi = rs[r], rs[r + 1]
+        x, st = S.solve(dev(b[lo:hi]), tol=1e-8, maxit=maxit)
+        sh = S.get_shifts()
+        out = (x.cpu().numpy(), st, sh)
+        S.close()
+        return out
+
+    outs = run_ranks(P, rank)
+    st0 = outs[0][1]
+    for _, st, sh in outs:                                    # every rank: identical bits
+        assert np.array_equal(st.hist, st0.hist) and st.cycles == st0.cycles
+        assert np.array_equal(sh[0], outs[0][2][0])
+    sh = outs[0][2]
+    full, envf = rounding_envelope(As, b, nperm=1, s=s, m=m, basis="newton", tol=1e-8, maxcyc=maxit)
+    shf = O.cagmres(As, b, s, m, basis="newton", tol=1e-8, maxcyc=1)["shifts"]
+    assert np.allclose(sh[0][:s], shf[0][:s], rtol=1e-6)
+    assert abs(st0.cycles - len(full)) <= 1
+    assert hist_within_envelope(st0.hist, full, envf)
+    if gen != "band27":
+        assert st0.status == 0
+        x = np.concatenate([o[0] for o in outs])
+        assert np.linalg.norm(b - As @ x) <= 1.01e-8 * np.linalg.norm(b)
+
+
+@pytest.mark.parametrize("P", [2, 4])
+def test_group_solve_injected_shifts_reorth_and_gmres(P):
+    """CholQR2 (reorth) CA and the GMRES(m) baseline across ranks vs the oracle."""
+    _, Solver = _mods()
+    A = G.convection_diffusion(40, 3, 7)
+    As = A.to_scipy()
+    b = G.rhs(A.n)
+    sh = O.modified_leja(O.ritz_values(O.arnoldi_cgs2(As, b, 30)[1], 30), 10)
+    rs = O.block_rows(A.n, P)
+
+    def rank(r, grp):
+        lo, hi = rs[r], rs[r + 1]
+        S = Solver(A, s=10, m=30, basis="newton", reorth=True, group=grp, row_starts=rs, rank=r)
+        S.set_shifts(*sh)
+        _, st = S.solve(dev(b[lo:hi]), tol=1e-8, maxit=60)
+        S.close()
+        Sg = Solver(A, s=1, m=30, basis="gmres", group=grp, row_starts=rs, rank=r)
+        _, sg = Sg.solve(dev(b[lo:hi]), tol=1e-8, maxit=60)
+        Sg.close()
+        return st, sg
+
+    outs = run_ranks(P, rank)
+    st, sg = outs[0]
+    ref, env = rounding_envelope(As, b, s=10, m=30, basis="newton", reorth=True, tol=1e-8, shifts=sh)
+    assert st.status == 0 and abs(st.cycles - len(ref)) <= 1
+    assert hist_within_envelope(st.hist, ref, env)
+    g = O.gmres(As, b, 30, tol=1e-8)
+    assert sg.status == 0 and abs(sg.cycles - g["cycles"]) <= 1
+    assert np.allclose(sg.hist, g["hist"][:len(sg.hist)], rtol=1e-6)
+
+
+def test_group_single_rank_is_the_single_gpu_handle():
+    """P = 1 through the group API: bitwise the single-GPU solve."""
+    _, Solver = _mods()
+    A = G.convection_diffusion(24, 3, 7)
+    b = G.rhs(A.n)
+    S1 = Solver(A, s=5, m=30, basis="newton")
+    x1, st1 = S1.solve(dev(b), tol=1e-8, maxit=60)
+
+    def rank(r, grp):
+        S = Solver(A, s=5, m=30, basis="newton", group=grp, row_starts=np.array([0, A.n]), rank=0)
+        x, st = S.solve(dev(b), tol=1e-8, maxit=60)
+        S.close()
+        return x.cpu(), st
+
+    x2, st2 = run_ranks(1, rank)[0]
+    assert np.array_equal(st1.hist, st2.hist) and torch.equal(x1.cpu(), x2)
