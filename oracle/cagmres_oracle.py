@@ -225,8 +225,17 @@ def tsqr_caqr(P, row_blocks=1):
     return Q * sg[None, :], sg[:, None] * R
 
 
+def tsqr_cholqr_svqr_retry(P):
+    """CholQR, and on its breakdown (non-positive pivot) the same panel by SVQR
+     — the opt-in retry of reading G15 (no silent fallback without the flag)."""
+    try:
+        return tsqr_cholqr(P)
+    except Breakdown:
+        return tsqr_svqr(P)
+
+
 TSQR = {"cholqr": tsqr_cholqr, "svqr": tsqr_svqr, "mgs": tsqr_mgs, "cgs": tsqr_cgs,
-        "caqr": tsqr_caqr}
+        "caqr": tsqr_caqr, "cholqr_retry": tsqr_cholqr_svqr_retry}
 BORTH = {"cgs": borth_cgs, "mgs": borth_mgs}
 
 

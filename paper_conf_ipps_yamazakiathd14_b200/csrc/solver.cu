@@ -316,7 +316,7 @@ void wave_reset_pairs(cagmres* h) {
 int spmv_autotune(cagmres* h) {
     // 14, 15 (CTA-contiguous) are faster per launch but lose ~1.4 ms per C2 solve in the
     // back-to-back PDL chain (profiles/r1_bench_C2_spmv14.json): options only
-    static const int cand[] = {0, 3, 5, 6, 8, 10, 11, 12, 13, 16, 17, 18};
+    static const int cand[] = {0, 3, 5, 6, 8, 10, 11, 12, 13, 16, 17, 18, 19, 20};
     if (h->m < 1 || h->A.nrows <= 0) return CAGMRES_OK;
     double* x = h->V;
     double* y = h->V + h->ldv;
@@ -985,7 +985,7 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
     switch (opt) {
         case CAGMRES_OPT_MPK_WAVE: h->wave_on = value != 0; h->wave_force = value == 2; return CAGMRES_OK;
         case CAGMRES_OPT_SPMV:
-            if (value < -1 || value > 18) return CAGMRES_EINVAL;
+            if (value < -1 || value > 20) return CAGMRES_EINVAL;
             if (value == -1) return spmv_autotune(h);
             h->A.variant = int(value);
             return CAGMRES_OK;

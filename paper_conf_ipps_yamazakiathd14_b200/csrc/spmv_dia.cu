@@ -46,6 +46,26 @@ __device__ __forceinline__ void prefetch_l2(const void* p) {
     asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
 }
 
+// L2 eviction-priority hints (PF = 3): the value stream is read exactly once per step, so it is
+// loaded / prefetched as evict_first and does not push the basis columns out of the 126 MB L2:
+// the x operand (the column the previous step just wrote) and the y column this step writes
+// (next step's x) stay L2-resident instead of making a DRAM round trip per step.
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ double ldg_stream_hint(const double* p, uint64_t pol) {
+    double v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(p), "l"(pol));
+    return v;
+}
+// one TMA-engine instruction prefetches a whole slice's values (16-B aligned, multiple of 16 B)
+__device__ __forceinline__ void bulk_prefetch_l2(const void* p, uint32_t bytes, uint64_t pol) {
+    asm volatile("cp.async.bulk.prefetch.L2.global.L2::cache_hint [%0], %1, %2;" ::"l"(p), "r"(bytes), "l"(pol)
+                 : "memory");
+}
+
 // PF = 1: while slice i is computed, the value lines of slice i + stride (descriptor already in
 // registers) are prefetched into L2, so next iteration's value loads are L2 hits: one more
 // slice of HBM requests in flight per warp without holding registers.
@@ -55,6 +75,7 @@ __device__ __forceinline__ void prefetch_l2(const void* p) {
 template <int MODE, int WT, int MINB, int CONTIG = 0, int PF = 0>   // MODE 0: Ax  1: + bu u  2: + bw w  3: u - Ax
 __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
     const int lane = threadIdx.x & 31;
+    const uint64_t pol = PF == 3 ? policy_evict_first() : 0;
     const int64_t nsl_all = (a.nrows + 31) >> 5;
     int64_t stride, sl, nsl;
     if (CONTIG) {
@@ -89,6 +110,7 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
         }
         o1 = sell_slice_off(lane, W1, i1, a.dcol);
         if (PF == 1 && lane < 2 * W1) prefetch_l2(a.val + b1 + 16 * lane);     // 128-B lines of slice +1
+        if (PF == 3 && lane == 0 && W1 > 0) bulk_prefetch_l2(a.val + b1, uint32_t(W1) * 256u, pol);
         const int64_t r = sl * 32 + lane;
         const bool live = r < a.nrows;
         double uu = 0.0, ww = 0.0, acc = 0.0;
@@ -107,7 +129,8 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
 #pragma unroll
                 for (int t = 0; t < GT; ++t) {
                     const int o = __shfl_sync(0xffffffffu, o0, g0 + t);
-                    v[t] = (CONTIG || PF) ? ldg_stream(vp + 32 * (g0 + t)) : __ldg(vp + 32 * (g0 + t));
+                    if constexpr (PF == 3) v[t] = ldg_stream_hint(vp + 32 * (g0 + t), pol);
+                    else v[t] = (CONTIG || PF) ? ldg_stream(vp + 32 * (g0 + t)) : __ldg(vp + 32 * (g0 + t));
                     xv[t] = __ldg(xr + o);
                 }
 #pragma unroll
@@ -186,6 +209,8 @@ void spmv_dia(const Dev& d, const Sell& A, int variant, int64_t nrows, const dou
         case 16: go_width<4, 0, 1>(d, a, A.dia_w, st, mode); break;
         case 17: go_width<5, 0, 1>(d, a, A.dia_w, st, mode); break;
         case 18: go_width<4, 0, 2>(d, a, A.dia_w, st, mode); break;
+        case 19: go_width<4, 0, 3>(d, a, A.dia_w, st, mode); break;
+        case 20: go_width<5, 0, 3>(d, a, A.dia_w, st, mode); break;
         default: go_width<6, 0>(d, a, A.dia_w, st, mode); break;
     }
 }

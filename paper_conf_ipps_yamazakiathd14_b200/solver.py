@@ -228,12 +228,12 @@ class Solver:
                                         int(w), C.c_void_p(Cm.data_ptr())), "borth")
         return Cm.t()[:j]
 
-    def tsqr(self, P, w, tsqr="cholqr", reorth=False):
+    def tsqr(self, P, w, tsqr="cholqr", reorth=False, svqr_retry=False):
         import torch
         R = torch.zeros((w, w), dtype=torch.float64, device=self.device)
         pp, ldp = self._col_major(P, self.n_loc)
         st = self._lib.cagmres_tsqr(self._h, C.c_void_p(pp), ldp, int(w), C.c_void_p(R.data_ptr()),
-                                    orth_flags(tsqr, reorth))
+                                    orth_flags(tsqr, reorth) | (L.SVQR_RETRY if svqr_retry else 0))
         L.check(st, "tsqr")
         return R.t()
 

@@ -83,6 +83,19 @@ def test_host_leja_matches_oracle():
     assert np.allclose(r1, r2) and np.allclose(i1, i2)
 
 
+@pytest.mark.parametrize("pts,want_re,want_im", [
+    ([-3.0, 3.0, 1.0], [3.0, -3.0, 1.0], [0.0, 0.0, 0.0]),
+    ([-1.0, 1.0, 5j, -5j], [0.0, 0.0, -1.0, 1.0], [5.0, -5.0, 0.0, 0.0]),
+    ([2.0, 2.0, -1.0], [2.0, -1.0, 2.0], [0.0, 0.0, 0.0]),
+    ([1 + 1j, 1 - 1j, -1 + 1j, -1 - 1j], [1.0, 1.0, -1.0, -1.0], [1.0, -1.0, 1.0, -1.0])])
+def test_host_leja_tie_breaking_by_hand(pts, want_re, want_im):
+    """The library's Leja order on tied candidates = the hand-derived G10 order (the same cases
+    pin the oracle in test_oracle_pins.py)."""
+    from paper_conf_ipps_yamazakiathd14_b200 import host
+    re, im = host.leja(np.array(pts, dtype=np.complex128), len(pts))
+    assert np.array_equal(re[:len(pts)], want_re) and np.array_equal(im[:len(pts)], want_im)
+
+
 @pytest.mark.parametrize("shifts", [([0.0] * 5, [0.0] * 5), ([1.0, 2.0, 2.0, 0.5, 4.0], [0.0, 1.0, -1.0, 0.0, 0.0]),
                                     ([1.0, 2.0, 2.0, 3.0, 3.0], [0.0, 0.0, 0.0, 0.5, -0.5])])
 def test_host_change_of_basis_matches_oracle(shifts):

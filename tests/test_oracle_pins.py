@@ -138,6 +138,25 @@ def test_cholqr_breaks_down_on_rank_deficient_panel():
     assert np.all(np.isfinite(R))
 
 
+def test_cholqr_svqr_retry_factors_the_panel_cholqr_cannot():
+    """G15 opt-in retry: where CholQR breaks down the panel is factored by SVQR —
+    checked against the factorisation itself (P = QR, R upper, diag > 0), not against the
+    oracle's own SVQR; a well-conditioned panel keeps the CholQR factor (Householder R)."""
+    P = G.random_panel(300, 5, 5)
+    P[:, 4] = P[:, 0] - 2.0 * P[:, 1]                          # rank deficient: pivot < 0 here
+    with pytest.raises(O.Breakdown):
+        O.tsqr_cholqr(P)
+    Q, R = O.tsqr_cholqr_svqr_retry(P)
+    assert np.allclose(np.tril(R, -1), 0.0) and np.all(np.diag(R) > 0)
+    assert O.fact_error(P, Q, R) < 1e-12
+    assert np.allclose(Q[:, :4].T @ Q[:, :4], np.eye(4), atol=1e-12)   # the independent part
+    Pw = G.random_panel(3000, 6, 9)
+    Qw, Rw = O.tsqr_cholqr_svqr_retry(Pw)
+    _, Rh = np.linalg.qr(Pw)
+    Rh = np.sign(np.diag(Rh))[:, None] * Rh
+    assert np.allclose(Rw, Rh, rtol=1e-12, atol=1e-12 * np.abs(Rh).max())
+
+
 def test_orthogonality_ordering_fig10():
     """Fig. 10: ||I-Q^TQ|| is O(eps k^2) CholQR/SVQR, O(eps k) MGS, O(eps) CAQR."""
     rng_panel = G.random_panel(4000, 8, 6)
@@ -271,6 +290,49 @@ def test_leja_exhaustive_first_pair_maximises_distance():
     best = max(itertools.permutations(pts, 2),
                key=lambda p: (abs(p[0]) == max(abs(pts))) * 100 + abs(p[0] - p[1]))
     assert (re[0], re[1]) == best
+
+
+@pytest.mark.parametrize("pts,want_re,want_im", [
+    # first point: |3| == |-3| -> the larger real part (G10); then the farther point
+    ([-3.0, 3.0, 1.0], [3.0, -3.0, 1.0], [0.0, 0.0, 0.0]),
+    # max modulus is the pair 0 +- 5i (+im first); then -1 and 1 score log 26 each: tie ->
+    # the first in (re, im) order, i.e. -1
+    ([-1.0, 1.0, 5j, -5j], [0.0, 0.0, -1.0, 1.0], [5.0, -5.0, 0.0, 0.0]),
+    # a repeated value stays a separate candidate with score -inf: it goes last
+    ([2.0, 2.0, -1.0], [2.0, -1.0, 2.0], [0.0, 0.0, 0.0]),
+    # two pairs of equal modulus: larger real part first; the other pair follows its partner
+    ([1 + 1j, 1 - 1j, -1 + 1j, -1 - 1j], [1.0, 1.0, -1.0, -1.0], [1.0, -1.0, 1.0, -1.0]),
+])
+def test_modified_leja_tie_breaking_by_hand(pts, want_re, want_im):
+    """Ties resolved by hand from the G10 reading, not from the oracle: first
+    point max |theta| with ties to the larger real part; then argmax of the log-distance sum with
+    ties to the first candidate in (re, im) order; repeats score -inf."""
+    re, im = O.modified_leja(np.array(pts, dtype=np.complex128), len(pts))
+    assert np.array_equal(re, np.array(want_re)) and np.array_equal(im, np.array(want_im))
+
+
+def test_ritz_values_full_krylov_space_recover_known_spectrum():
+    """Pin of ritz_values (+ the CGS Arnoldi that feeds it): with m = n the Krylov space is the
+    whole space, so the Ritz values of H[0:n,0:n] are the eigenvalues of A.  A is a
+    dense orthogonal similarity of a block-diagonal matrix with KNOWN eigenvalues (real ones
+    and a +- i b pairs from 2x2 rotation-scaling blocks)."""
+    lam_real = [3.0, -1.5, 0.75, 5.0]
+    pairs = [(1.0, 2.0), (-2.0, 0.5)]
+    n = len(lam_real) + 2 * len(pairs)
+    D = np.zeros((n, n))
+    for i, lr in enumerate(lam_real):
+        D[i, i] = lr
+    k = len(lam_real)
+    for a, b in pairs:
+        D[k:k + 2, k:k + 2] = [[a, b], [-b, a]]
+        k += 2
+    Qm, _ = np.linalg.qr(G.random_panel(n, n, 5))
+    A = Qm @ D @ Qm.T
+    import scipy.sparse as sp
+    _, H, _ = O.arnoldi_cgs2(sp.csr_matrix(A), G.u(3, np.arange(n)), n)
+    ritz = np.sort_complex(O.ritz_values(H, n))
+    want = np.sort_complex(np.array(lam_real + [complex(a, s * b) for a, b in pairs for s in (1, -1)]))
+    assert np.allclose(ritz, want, rtol=0, atol=1e-10)
 
 
 # ----------------------------------------------------------------------------- boundary sets (P:60-64)
