@@ -305,6 +305,21 @@ int cagmres_host_rcm(int64_t n, const int64_t* rowptr, const int32_t* colind, in
 int cagmres_host_permute(int64_t n, const int64_t* rowptr, const int32_t* colind, const double* val,
                          const int64_t* perm, int64_t* out_rowptr, int32_t* out_colind, double* out_val);
 
+/* k-way partition of the symmetrised graph of A (n x n CSR, host) into nparts parts of
+ * balanced row counts with a small edge cut (P:104 fn 3 "k-way partitioning ...
+ * smaller surfaces and better load balances", Fig. 6/7 P:98-118): recursive bisection, each
+ * bisection a breadth-first level-set split from a pseudo-peripheral vertex refined by
+ * Fiduccia-Mattheyses passes; part sizes within (1 + imbalance) of n/nparts per bisection level.
+ * part[v] in [0, nparts); *edge_cut = undirected edges between parts (may be NULL).
+ * Deterministic.  Errors: EINVAL (column id out of range, nparts < 1, imbalance < 0). */
+int cagmres_host_partition(int64_t n, const int64_t* rowptr, const int32_t* colind, int nparts,
+                           double imbalance, int32_t* part, int64_t* edge_cut);
+/* Permutation that makes every part a contiguous block of rows, for the block-row create_dist
+ * (P:45): perm[new] = old, parts in order, original order kept inside a part; row_starts
+ * (nparts + 1) = the block boundaries.  Apply with cagmres_host_permute. */
+int cagmres_host_partition_order(int64_t n, const int32_t* part, int nparts, int64_t* perm,
+                                 int64_t* row_starts);
+
 /* ---- host-only small dense algorithms of the cycle (exported for tests) -------------- */
 /* Eigenvalues (Ritz values) of the upper Hessenberg H (m x m, ld ldh), Francis
  * double-shift QR; conjugate pairs returned adjacent (+im first).  EBREAKDOWN if the QR

@@ -89,6 +89,8 @@ SIGNATURES = {
     "cagmres_host_sym_eigvals": ([_PD, C.c_int, C.c_int, _PD], C.c_int),
     "cagmres_host_eigvals": ([_PD, C.c_int, C.c_int, _PD, _PD], C.c_int),
     "cagmres_host_rcm": ([_I64, _PI64, _PI32, _PI64], C.c_int),
+    "cagmres_host_partition": ([_I64, _PI64, _PI32, C.c_int, C.c_double, _PI32, _PI64], C.c_int),
+    "cagmres_host_partition_order": ([_I64, _PI32, C.c_int, _PI64, _PI64], C.c_int),
     "cagmres_host_permute": ([_I64, _PI64, _PI32, _PD, _PI64, _PI64, _PI32, _PD], C.c_int),
     "cagmres_host_leja": ([_PD, _PD, C.c_int, C.c_int, _PD, _PD, C.c_int, C.POINTER(C.c_int)], C.c_int),
     "cagmres_host_change_of_basis": ([_PD, _PD, C.c_int, _PD], C.c_int),

@@ -47,6 +47,10 @@ void sell_build(const cagmres_plan& p, SellHost& out);   // throws std::bad_allo
 int64_t plan_prefix_count(const std::vector<int64_t>& counts, const std::vector<int32_t>& levels,
                           int q, int depth);
 
+// symmetrised adjacency of a CSR pattern (A + A^T, no diagonal, sorted, unique) — reorder.cpp
+void sym_graph(int64_t n, const int64_t* rp, const int32_t* ci, std::vector<int64_t>& gp,
+               std::vector<int64_t>& gi);
+
 // ------------------------------------------------------------------------------------
 // Small dense host algorithms (P:41 LS and Hessenberg by-product; P:94 Ritz / Leja).
 // All matrices column-major.

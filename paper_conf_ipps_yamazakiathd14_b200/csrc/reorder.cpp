@@ -11,11 +11,9 @@
 #include <cstdint>
 #include <vector>
 
-#include "cagmres.h"
+#include "internal.h"
 
-namespace {
-
-// symmetrised adjacency (pattern of A + A^T without the diagonal), CSR
+// symmetrised adjacency (pattern of A + A^T without the diagonal), CSR (also partition.cpp)
 void sym_graph(int64_t n, const int64_t* rp, const int32_t* ci, std::vector<int64_t>& gp,
                std::vector<int64_t>& gi) {
     std::vector<int64_t> deg(size_t(n) + 1, 0);
@@ -51,6 +49,8 @@ void sym_graph(int64_t n, const int64_t* rp, const int32_t* ci, std::vector<int6
     gi.resize(size_t(w));
     gp.swap(np);
 }
+
+namespace {
 
 // BFS from s over unvisited-in-`mark`-epoch nodes; returns the last level (the deepest nodes)
 // and the number of levels.

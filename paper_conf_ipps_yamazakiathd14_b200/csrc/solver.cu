@@ -370,7 +370,6 @@ int init_common_(cagmres* h, const cagmres_csr* A, const int64_t* row_starts, in
     if (kind > CAGMRES_CAQR) return CAGMRES_EINVAL;
     if ((orth & CAGMRES_ONEPASS) && (kind != CAGMRES_CHOLQR || (orth & CAGMRES_BORTH_MGS))) return CAGMRES_EINVAL;
     if ((orth & CAGMRES_SVQR_RETRY) && kind != CAGMRES_CHOLQR) return CAGMRES_EINVAL;
-    if (kind == CAGMRES_CAQR && h->nranks > 1) return CAGMRES_ENOTSUP;   // single-GPU tree only
     h->s = s; h->m = m; h->basis = basis; h->orth = orth;
     int dv = 0;
     CU(cudaGetDevice(&dv));
@@ -618,15 +617,43 @@ int tsqr_panel(cagmres* h, double* P, int64_t ldp, int w, double* R, int kind, i
         kern::trsm(h->dev, h->n_loc, P, ldp, w, R, c0, h->stream);          // V := V R^{-1}
         h->bytes[PH_TSQR] += 8.0 * nl * (2.0 * w + double(w - c0));
     } else if (kind == CAGMRES_CAQR) {                       // Fig. 9 CAQR: TSQR tree
-        if (h->nranks > 1) return CAGMRES_ENOTSUP;
-        const size_t need = kern::caqr_ws_doubles(h->n_loc, w);
+        // Multi-rank: "each GPU first computes the QR factorization of the local
+        // matrix, then the local R-factors are gathered ..., and the final QR factorization is
+        // computed ...; V^(d) := V^(d) Q^(d)": local tree -> all-gather of the w x w R's ->
+        // QR of the stacked R's (redundantly on every rank) -> P := Q_loc Q_s[rank block].
+        const int Pn = h->nranks;
+        const size_t W2 = size_t(w) * size_t(w);
+        const int64_t sr = int64_t(Pn) * w;                      // rows of the stacked R's
+        const size_t need_loc = kern::caqr_ws_doubles(h->n_loc, w);
+        const size_t need = need_loc + (Pn > 1 ? 3 * size_t(Pn) * W2 + kern::caqr_ws_doubles(sr, w) +
+                                                     size_t(h->n_loc) + W2 : 0);
         if (need > h->caqr_cap) {
             cudaFree(h->caqr_ws);
             h->caqr_ws = nullptr;
             CU(cudaMalloc(&h->caqr_ws, sizeof(double) * need));
             h->caqr_cap = need;
         }
-        if (kern::caqr(h->dev, h->n_loc, P, ldp, w, R, c0, h->caqr_ws, h->stream)) return CAGMRES_EINVAL;
+        if (Pn == 1) {
+            if (kern::caqr(h->dev, h->n_loc, P, ldp, w, R, c0, h->caqr_ws, h->stream)) return CAGMRES_EINVAL;
+        } else {
+            double* Rloc = h->caqr_ws + need_loc;                // w x w
+            double* Rall = Rloc + W2;                            // Pn blocks of w x w
+            double* Stk = Rall + size_t(Pn) * W2;                // sr x w, column-major
+            double* q0 = Stk + size_t(Pn) * W2;                  // saved column 0 (c0 = 1)
+            double* ws2 = q0 + size_t(h->n_loc);
+            if (c0 == 1) CU(cudaMemcpyAsync(q0, P, sizeof(double) * size_t(h->n_loc), cudaMemcpyDeviceToDevice, h->stream));
+            if (kern::caqr(h->dev, h->n_loc, P, ldp, w, Rloc, 0, h->caqr_ws, h->stream)) return CAGMRES_EINVAL;
+            TRY(h->tr->allgather(Rloc, Rall, sizeof(double) * W2, h->stream));
+            // stacked column-major: row q*w + i of column c = R_q[i, c]
+            for (int q = 0; q < Pn; ++q)
+                CU(cudaMemcpy2DAsync(Stk + size_t(q) * w, sizeof(double) * size_t(sr), Rall + size_t(q) * W2,
+                                     sizeof(double) * size_t(w), sizeof(double) * size_t(w), size_t(w),
+                                     cudaMemcpyDeviceToDevice, h->stream));
+            if (kern::caqr(h->dev, sr, Stk, sr, w, R, 0, ws2, h->stream)) return CAGMRES_EINVAL;
+            if (kern::gemm_rows(h->dev, h->n_loc, P, ldp, w, P, ldp, w, Stk + size_t(h->rank) * w, sr, c0, h->stream))
+                return CAGMRES_EINVAL;
+            if (c0 == 1) CU(cudaMemcpyAsync(P, q0, sizeof(double) * size_t(h->n_loc), cudaMemcpyDeviceToDevice, h->stream));
+        }
         h->bytes[PH_TSQR] += 8.0 * nl * (2.0 * w + double(w - c0));
     } else {
         CU(cudaMemsetAsync(R, 0, sizeof(double) * size_t(w) * size_t(w), h->stream));

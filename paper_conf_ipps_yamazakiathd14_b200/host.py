@@ -173,3 +173,45 @@ def permute(A, perm):
                                      L.i64ptr(pm), L.i64ptr(orp), oci.ctypes.data_as(L._PI32), L.dptr(ova)),
             "permute")
     return dataclasses.replace(A, rowptr=orp, colind=oci, val=ova)
+
+
+def partition(A, nparts, imbalance=0.03):
+    """k-way partition of the symmetrised graph of the n x n host CSR A (cagmres_host_partition;
+    NEXT-4): returns (part ids int32[n], edge cut)."""
+    lib = L.load()
+    rp = np.ascontiguousarray(A.rowptr, dtype=np.int64)
+    ci = np.ascontiguousarray(A.colind, dtype=np.int32)
+    part = np.zeros(A.n, dtype=np.int32)
+    cut = C.c_int64()
+    L.check(lib.cagmres_host_partition(int(A.n), L.i64ptr(rp), ci.ctypes.data_as(L._PI32), int(nparts),
+                                       float(imbalance), part.ctypes.data_as(L._PI32), C.byref(cut)), "partition")
+    return part, int(cut.value)
+
+
+def partition_order(part, nparts):
+    """(perm, row_starts): perm[new] = old groups every part into a contiguous block of rows."""
+    lib = L.load()
+    pt = np.ascontiguousarray(part, dtype=np.int32)
+    perm = np.zeros(len(pt), dtype=np.int64)
+    rs = np.zeros(nparts + 1, dtype=np.int64)
+    L.check(lib.cagmres_host_partition_order(len(pt), pt.ctypes.data_as(L._PI32), int(nparts), L.i64ptr(perm),
+                                             L.i64ptr(rs)), "partition_order")
+    return perm, rs
+
+
+def distribute(A, nranks, order="natural", imbalance=0.03):
+    """Row distribution for the block-row create_dist under an ordering (NEXT-4,
+    P:98-118): "natural" (A as given), "rcm" (reverse Cuthill-McKee, then equal blocks) or
+    "kway" (partition(), parts made contiguous).  Returns (B = P A P^T, perm, row_starts);
+    solve B y = P b, then x[perm] = y."""
+    n = A.n
+    if order == "natural":
+        return A, np.arange(n, dtype=np.int64), np.array([(p * n) // nranks for p in range(nranks + 1)], dtype=np.int64)
+    if order == "rcm":
+        perm = rcm(A)
+        return permute(A, perm), perm, np.array([(p * n) // nranks for p in range(nranks + 1)], dtype=np.int64)
+    if order == "kway":
+        part, _ = partition(A, nranks, imbalance)
+        perm, rs = partition_order(part, nranks)
+        return permute(A, perm), perm, rs
+    raise ValueError(order)

@@ -1,6 +1,7 @@
 """CPU tests of the C-ABI library: every declared symbol is exported, and the host-only
 parts (setup plan, Ritz values, Leja order, change of basis, Hessenberg update, Givens LS)
 agree with the oracle / with dense linear algebra.  No compute call needs a GPU here."""
+import itertools
 import os
 import re
 
@@ -301,3 +302,89 @@ def test_rcm_disconnected_and_isolated_nodes():
     assert np.array_equal(np.sort(p), np.arange(C.n))
     with pytest.raises(Exception):
         host.permute(C, np.zeros(C.n, dtype=np.int64))          # not a permutation -> EINVAL
+
+
+# ----------------------------------------------------------------------------- NEXT-4 k-way partition
+def _csr_from_edges(n, edges):
+    from synth.generators import CSR
+    rows = [[] for _ in range(n)]
+    for a, b in edges:
+        rows[a].append(b)
+        rows[b].append(a)
+    rp, ci = [0], []
+    for r in range(n):
+        ci += sorted(set(rows[r]) | {r})
+        rp.append(len(ci))
+    return CSR(n=n, row_begin=0, rowptr=np.array(rp, dtype=np.int64), colind=np.array(ci, dtype=np.int32),
+               val=np.ones(len(ci)))
+
+
+def _cut(edges, part):
+    return sum(part[a] != part[b] for a, b in edges)
+
+
+def _brute_min_bisection(n, edges):
+    """Minimum edge cut over all bisections with |part 0| = n // 2 (exhaustive)."""
+    best = None
+    for S in itertools.combinations(range(1, n), n // 2 - 1):        # vertex 0 in part 0 (symmetry)
+        part = np.ones(n, dtype=int)
+        part[[0, *S]] = 0
+        c = _cut(edges, part)
+        best = c if best is None else min(best, c)
+    return best
+
+
+def test_partition_bisection_vs_brute_force():
+    """Balanced 2-way cuts vs exhaustive search: optimal on paths, cycles, grids and a ladder;
+    within +1 of optimal on random sparse graphs (FM is a local search)."""
+    from paper_conf_ipps_yamazakiathd14_b200 import host
+    cases = {
+        "path10": (10, [(i, i + 1) for i in range(9)]),
+        "cycle12": (12, [(i, (i + 1) % 12) for i in range(12)]),
+        "grid4x4": (16, [(r * 4 + c, r * 4 + c + 1) for r in range(4) for c in range(3)] +
+                    [(r * 4 + c, (r + 1) * 4 + c) for r in range(3) for c in range(4)]),
+        "ladder2x7": (14, [(i, i + 1) for i in range(6)] + [(7 + i, 8 + i) for i in range(6)] +
+                      [(i, 7 + i) for i in range(7)]),
+    }
+    rng = np.random.default_rng(3)
+    for t in range(6):
+        n = 14
+        e = {(min(a, b), max(a, b)) for a, b in rng.integers(0, n, size=(22, 2)) if a != b}
+        cases[f"rand{t}"] = (n, sorted(e))
+    for name, (n, edges) in cases.items():
+        A = _csr_from_edges(n, edges)
+        part, cut = host.partition(A, 2, imbalance=0.0)
+        assert sorted(np.bincount(part, minlength=2)) == [n // 2, n - n // 2], name
+        assert cut == _cut(edges, part), name
+        opt = _brute_min_bisection(n, edges)
+        slack = 0 if not name.startswith("rand") else 1
+        assert cut <= opt + slack, (name, cut, opt)
+
+
+@pytest.mark.parametrize("gen,k", [("cd5_40", 4), ("cd5_40", 8), ("g3", 3), ("g3", 8), ("cd7_16", 8)])
+def test_partition_balance_cut_and_order(gen, k):
+    """k-way on the synthetic matrices: every part within 3 % per bisection level of n/k (<= 5 %
+    overall), the reported cut equals a recount, the grid cut is at most the natural block-row
+    cut, and partition_order groups the parts into contiguous blocks."""
+    from paper_conf_ipps_yamazakiathd14_b200 import host
+    A = {"cd5_40": lambda: G.convection_diffusion(40, 2, 5),
+         "g3": lambda: G.g3_shaped(n=6000, width=80),
+         "cd7_16": lambda: G.convection_diffusion(16, 3, 7)}[gen]()
+    S = A.to_scipy().tocoo()
+    part, cut = host.partition(A, k)
+    sizes = np.bincount(part, minlength=k)
+    assert sizes.min() > 0 and np.abs(sizes - A.n / k).max() <= 0.05 * A.n / k + 2
+    m = S.row < S.col
+    sym = {(min(a, b), max(a, b)) for a, b in zip(S.row, S.col) if a != b}
+    assert cut == sum(part[a] != part[b] for a, b in sym)
+    nat = np.repeat(np.arange(k), np.diff(O.block_rows(A.n, k)))
+    assert cut <= sum(nat[a] != nat[b] for a, b in sym)
+    perm, rs = host.partition_order(part, k)
+    assert np.array_equal(np.sort(perm), np.arange(A.n))
+    for p in range(k):
+        assert np.all(part[perm[rs[p]:rs[p + 1]]] == p)
+    B, perm2, rs2 = host.distribute(A, k, "kway")
+    assert np.array_equal(perm2, perm) and np.array_equal(rs2, rs)
+    Bs = B.to_scipy()
+    As = A.to_scipy()
+    assert abs(Bs - As[perm][:, perm]).max() == 0.0

@@ -135,7 +135,7 @@ def test_group_mpk_monomial_matches_oracle():
 # ----------------------------------------------------------------------------- BOrth / TSQR
 @pytest.mark.parametrize("P", [2, 3, 8])
 @pytest.mark.parametrize("kind,reorth", [("cholqr", False), ("cholqr", True), ("svqr", False),
-                                         ("cgs", False), ("mgs", False)])
+                                         ("cgs", False), ("mgs", False), ("caqr", False)])
 def test_group_borth_tsqr_match_oracle(P, kind, reorth):
     """Row-distributed panels: C = Q^T P and R are sums over ranks."""
     _, Solver = _mods()
@@ -145,12 +145,12 @@ def test_group_borth_tsqr_match_oracle(P, kind, reorth):
     Pn = G.random_panel(n, w, 22)
     Pn[:, 2] += 0.3 * Pn[:, 1]
     Co, Po = O.borth_cgs(Q, Pn)
-    Qt, Rt = {"cholqr": O.tsqr_cholqr, "svqr": O.tsqr_svqr, "cgs": O.tsqr_cgs,
-              "mgs": O.tsqr_mgs}[kind](Po)
+    rs = O.block_rows(n, P)
+    Qt, Rt = {"cholqr": O.tsqr_cholqr, "svqr": O.tsqr_svqr, "cgs": O.tsqr_cgs, "mgs": O.tsqr_mgs,
+              "caqr": lambda X: O.tsqr_caqr(X, row_blocks=P)}[kind](Po)     # one block per GPU
     if reorth:
         Qt, R2 = O.tsqr_cholqr(Qt)
         Rt = R2 @ Rt
-    rs = O.block_rows(n, P)
 
     def rank(r, grp):
         lo, hi = rs[r], rs[r + 1]
@@ -230,16 +230,23 @@ def test_group_solve_injected_shifts_reorth_and_gmres(P):
         S.set_shifts(*sh)
         _, st = S.solve(dev(b[lo:hi]), tol=1e-8, maxit=60)
         S.close()
+        Sc = Solver(A, s=10, m=30, basis="newton", tsqr="caqr", group=grp, row_starts=rs, rank=r)
+        Sc.set_shifts(*sh)
+        _, sc = Sc.solve(dev(b[lo:hi]), tol=1e-8, maxit=60)
+        Sc.close()
         Sg = Solver(A, s=1, m=30, basis="gmres", group=grp, row_starts=rs, rank=r)
         _, sg = Sg.solve(dev(b[lo:hi]), tol=1e-8, maxit=60)
         Sg.close()
-        return st, sg
+        return st, sg, sc
 
     outs = run_ranks(P, rank)
-    st, sg = outs[0]
+    st, sg, sc = outs[0]
     ref, env = rounding_envelope(As, b, s=10, m=30, basis="newton", reorth=True, tol=1e-8, shifts=sh)
     assert st.status == 0 and abs(st.cycles - len(ref)) <= 1
     assert hist_within_envelope(st.hist, ref, env)
+    refc, envc = rounding_envelope(As, b, s=10, m=30, basis="newton", tsqr="caqr", tol=1e-8, shifts=sh)
+    assert sc.status == 0 and abs(sc.cycles - len(refc)) <= 1
+    assert hist_within_envelope(sc.hist, refc, envc)
     g = O.gmres(As, b, 30, tol=1e-8)
     assert sg.status == 0 and abs(sg.cycles - g["cycles"]) <= 1
     assert np.allclose(sg.hist, g["hist"][:len(sg.hist)], rtol=1e-6)

@@ -1,9 +1,12 @@
 """GPU parity: the CUDA path (through the C ABI) vs the oracle on identical seeded inputs.
 
-Tolerances (from BASELINE.json north_star + SURVEY §8(c)):
-  MPK columns: |W_gpu - W_orc| <= 1e-12 * max|W_orc[:,k]| (FMA contraction / order only)
+Tolerances (DESIGN.md §8 "Parity tolerances", from BASELINE.json north_star + SURVEY §8(c)):
+  MPK columns: |W_gpu - W_orc| <= 1e-13 * max|W_orc[:,k]| (FMA contraction only; measured
+    <= 8e-15, profiles/r2_parity_margins.json)
   R, C (well conditioned): relative 1e-10
-  per-cycle rho: |rho_gpu - rho_orc| <= 1e-10 * rho_orc + 1e-15 (units of ||r0||)
+  per-cycle rho: |rho_gpu - rho_orc| <= max(1e-10, 10 env_c) rho_orc + 1e-15 (units of ||r0||),
+    env_c = the oracle's own deviation under symmetric permutations (its rounding noise);
+    measured GPU deviation <= 3.1 env_c over six configs (profiles/r2_parity_margins.json)
   restart cycles to 1e-8: +-1
 """
 import numpy as np
@@ -59,7 +62,7 @@ def rounding_envelope(As, b, nperm=2, **kw):
     return ref, np.maximum.accumulate(dev_)
 
 
-def hist_within_envelope(h, ref, env, factor=30.0):
+def hist_within_envelope(h, ref, env, factor=10.0):
     """|rho_gpu - rho_orc| <= max(1e-10, factor * env_c) * rho_orc + 1e-15 per cycle: the
     north-star relative 1e-10 where the problem is well conditioned, else a multiple of the
     oracle's own rounding noise."""
@@ -95,7 +98,7 @@ def test_mpk_parity(basis, gen):
         W = S.mpk(dev(q), sb).cpu().numpy()
         Wo = O.mpk(As, q, sb, re, im)
         for k in range(sb + 1):
-            assert np.max(np.abs(W[:, k] - Wo[:, k])) <= 1e-12 * np.max(np.abs(Wo[:, k])), (sb, k)
+            assert np.max(np.abs(W[:, k] - Wo[:, k])) <= 1e-13 * np.max(np.abs(Wo[:, k])), (sb, k)
 
 
 def test_mpk_newton_zero_shifts_bitwise_equals_monomial():
@@ -158,7 +161,7 @@ def test_mpk_full_size_C2():
     W = S.mpk(dev(q), 10).cpu().numpy()
     Wo = O.mpk(As, q, 10, *SHIFTS)
     for k in range(11):
-        assert np.max(np.abs(W[:, k] - Wo[:, k])) <= 1e-12 * np.max(np.abs(Wo[:, k]))
+        assert np.max(np.abs(W[:, k] - Wo[:, k])) <= 1e-13 * np.max(np.abs(Wo[:, k]))
 
 
 def test_mpk_full_size_C5_sampled():
@@ -183,7 +186,7 @@ def test_mpk_full_size_C5_sampled():
         Wg = W[z0 * P:(z0 + 1) * P].cpu().numpy()
         for k in range(s + 1):
             ref = Wo[a:b, k]
-            assert np.max(np.abs(Wg[:, k] - ref)) <= 1e-12 * np.max(np.abs(ref)), (z0, k)
+            assert np.max(np.abs(Wg[:, k] - ref)) <= 1e-13 * np.max(np.abs(ref)), (z0, k)
 
 
 # ----------------------------------------------------------------------------- BOrth / TSQR
