@@ -217,8 +217,10 @@ void spmv(const Dev& d, const Sell& A, int64_t nrows, const double* x, double* y
     if (nrows <= 0) return;
     ++g_launches;
     if (w && !u) { u = x; bu = 0.0; }             // pair step with a == 0: keep MODE 2 well formed
+    if (A.variant >= 21 && spmv_tma(d, A, A.variant, nrows, x, y, u, bu, w, bw, w ? 2 : (u ? 1 : 0), st) == 0)
+        return;
     if (A.variant >= 10) {
-        spmv_dia(d, A, A.variant, nrows, x, y, u, bu, w, bw, w ? 2 : (u ? 1 : 0), st);
+        spmv_dia(d, A, A.variant >= 21 ? 16 : A.variant, nrows, x, y, u, bu, w, bw, w ? 2 : (u ? 1 : 0), st);
         return;
     }
     if (A.variant >= 4) {
@@ -264,8 +266,9 @@ void residual(const Dev& d, const Sell& A, int64_t nrows, const double* x, const
     (void)d;
     if (nrows <= 0) return;
     ++g_launches;
+    if (A.variant >= 21 && spmv_tma(d, A, A.variant, nrows, x, r, b, 1.0, nullptr, 0.0, 3, st) == 0) return;
     if (A.variant >= 10) {
-        spmv_dia(d, A, A.variant, nrows, x, r, b, 1.0, nullptr, 0.0, 3, st);
+        spmv_dia(d, A, A.variant >= 21 ? 16 : A.variant, nrows, x, r, b, 1.0, nullptr, 0.0, 3, st);
         return;
     }
     if (A.variant >= 4) {

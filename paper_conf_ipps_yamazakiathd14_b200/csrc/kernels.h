@@ -57,6 +57,7 @@ struct Sell {
     int64_t ncols = 0;          // valid x entries (clamp bound for DIA slices)
     int64_t ndcol = 0, ndia = 0;
     int dia_w = 0;              // most common width of the unclamped DIA slices (spmv_dia.cu)
+    uint32_t chunk_bytes = 0;   // largest value block of 8 consecutive slices (spmv_tma.cu stage)
     int64_t* sptr = nullptr;    // nslices+1 value offsets
     int64_t* sinfo = nullptr;   // nslices
     int32_t* dcol = nullptr;    // DIA offsets / explicit column ids
@@ -248,6 +249,9 @@ void spmv(const Dev& d, const Sell& A, int64_t nrows, const double* x, double* y
 // (3 = u - A x).
 void spmv_dia(const Dev& d, const Sell& A, int variant, int64_t nrows, const double* x, double* y,
               const double* u, double bu, const double* w, double bw, int mode, cudaStream_t st);
+// TMA-streamed SpMV (spmv_tma.cu), CAGMRES_OPT_SPMV 21 / 22; -1 if the matrix's chunks do not fit
+int spmv_tma(const Dev& d, const Sell& A, int variant, int64_t nrows, const double* x, double* y,
+             const double* u, double bu, const double* w, double bw, int mode, cudaStream_t st);
 // r[0:nrows) = b - A x
 void residual(const Dev& d, const Sell& A, int64_t nrows, const double* x, const double* b,
               double* r, cudaStream_t st);

@@ -178,6 +178,11 @@ int build_sell(cagmres* h, const cagmres_plan& p) {
     const int64_t ndia = sh.ndia;
     h->A.nrows = nr; h->A.nslices = ns; h->A.nstored = tot; h->A.nnz = p.nnz_mat;
     h->A.ncols = p.n_ext; h->A.ndcol = ndcol; h->A.ndia = ndia;
+    {   // largest value block of 8 consecutive slices (the TMA SpMV's stage size)
+        int64_t mx = 0;
+        for (int64_t c0 = 0; c0 < ns; c0 += 8) mx = std::max(mx, sptr[size_t(std::min(ns, c0 + 8))] - sptr[size_t(c0)]);
+        h->A.chunk_bytes = mx * 8 > int64_t(1) << 30 ? 0u : uint32_t(mx * 8);
+    }
     {   // most common width among unclamped DIA slices (the specialised SpMV's fast path)
         std::vector<int64_t> cnt(33, 0);
         for (int64_t sl = 0; sl < ns; ++sl)
@@ -316,7 +321,7 @@ void wave_reset_pairs(cagmres* h) {
 int spmv_autotune(cagmres* h) {
     // 14, 15 (CTA-contiguous) are faster per launch but lose ~1.4 ms per C2 solve in the
     // back-to-back PDL chain (profiles/r1_bench_C2_spmv14.json): options only
-    static const int cand[] = {0, 3, 5, 6, 8, 10, 11, 12, 13, 16, 17, 18, 19, 20};
+    static const int cand[] = {0, 3, 5, 6, 8, 10, 11, 12, 13, 16, 17, 18, 21, 22};
     if (h->m < 1 || h->A.nrows <= 0) return CAGMRES_OK;
     double* x = h->V;
     double* y = h->V + h->ldv;
@@ -1012,7 +1017,7 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
     switch (opt) {
         case CAGMRES_OPT_MPK_WAVE: h->wave_on = value != 0; h->wave_force = value == 2; return CAGMRES_OK;
         case CAGMRES_OPT_SPMV:
-            if (value < -1 || value > 20) return CAGMRES_EINVAL;
+            if (value < -1 || value > 22) return CAGMRES_EINVAL;
             if (value == -1) return spmv_autotune(h);
             h->A.variant = int(value);
             return CAGMRES_OK;

@@ -142,7 +142,7 @@ def test_spmv_variants_bitwise(gen):
     S = Solver(A, s=6, m=30, basis="newton")
     S.set_shifts(*SHIFTS)
     Ws = []
-    variants = list(range(10)) + [10, 11, 12, 13, 14, 15, 16, 17, 18, 19, 20]
+    variants = list(range(10)) + [10, 11, 12, 13, 14, 15, 16, 17, 18, 19, 20, 21, 22]
     for v in variants:
         S.set_option("spmv", v)
         Ws.append(S.mpk(q, 6))
