@@ -162,16 +162,11 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
  *                          window fits L2 ("reducing communication of MPK on a single
  *                          GPU"); 2 = force it whenever A is banded.  Bitwise identical.
  *   CAGMRES_OPT_SPMV     : SpMV kernel (default: the fastest on this matrix, timed once at create;
- *                          -1 re-runs that selection): 0 = one SELL-32 slice per warp; 1, 2, 3 = two
- *                          slices per warp with load batches 4/8/4 at 4/2/3 CTAs per SM;
- *                          4..9 = persistent grid, slice descriptors software-pipelined two
- *                          slices ahead, (load batch, CTAs/SM) = (8,3) (4,4) (4,5) (4,6) (2,6)
- *                          (2,8); 10..13 = persistent, fully unrolled body for the matrix's most
- *                          common DIA slice width, >= 3/4/5/6 CTAs per SM; 14, 15 = the same with
- *                          CTA-contiguous slice ranges (L1 reuse of x), 4/5 CTAs per SM; 16, 17 =
- *                          10..13's kernel with an L2 prefetch of the next slice's values, 4/5
- *                          CTAs per SM; 18 = prefetch two slices ahead.  All variants are bitwise
- *                          identical.
+ *                          -1 re-runs that selection): 0 = one SELL-32 slice per warp; 5 = persistent
+ *                          grid, slice descriptors software-pipelined two slices ahead; 16, 17 = the
+ *                          persistent kernel with a fully unrolled body for the matrix's most common
+ *                          DIA slice width and an L2 prefetch of the next slice's values, >= 4 / 5
+ *                          CTAs per SM.  All variants are bitwise identical.  Other values: EINVAL.
  *   CAGMRES_OPT_GRAM     : CholQR Gram kernel: 0 = FP64 tensor core (DMMA m8n8k4) on a per-warp
  *                          cp.async ring; 1 (default) = scalar DFMA on a deeper ring (w <= 12,
  *                          else the DMMA kernel).

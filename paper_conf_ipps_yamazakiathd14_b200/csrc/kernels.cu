@@ -60,88 +60,6 @@ __global__ void __launch_bounds__(NT, 6) k_spmv_sell32(int64_t nrows, const int6
     y[r] = out;
 }
 
-// Two slices per warp.  With one 32-row slice per warp the per-warp dependency chain
-// (sptr/sinfo -> DIA offsets -> values + x) leaves only ~1 KB of loads in flight per warp,
-// which at the occupancy the register budget allows is below the bytes-in-flight HBM3e
-// needs (Little's law).  Here a warp runs the chains of two slices side by
-// side and, for DIA slices, issues every value load of a batch of 8 diagonals before any
-// offset shuffle, so up to 2 x 8 x 256 B of values are in flight per warp.  Per row the FMA
-// order is t = 0, 1, ..., W-1 exactly as in sell_row_dot: results are bitwise identical.
-template <int MODE, int X2_B, int MINB>
-__global__ void __launch_bounds__(NT, MINB) k_spmv_sell32_x2(int64_t nrows, const int64_t* __restrict__ sptr,
-                                                       const int64_t* __restrict__ sinfo,
-                                                       const int32_t* __restrict__ dcol, int64_t ncols,
-                                                       const double* __restrict__ val,
-                                                       const double* __restrict__ x,
-                                                       const double* __restrict__ u, double bu,
-                                                       const double* __restrict__ w, double bw,
-                                                       double* __restrict__ y) {
-    const int lane = threadIdx.x & 31;
-    const int64_t gw = (int64_t(blockIdx.x) * NT + threadIdx.x) >> 5;
-    const int64_t nsl = (nrows + 31) >> 5;
-    if (2 * gw >= nsl) return;
-    int64_t r[2], b[2], info[2];
-    int W[2];
-#pragma unroll
-    for (int q = 0; q < 2; ++q) {
-        const int64_t sl = min(2 * gw + q, nsl - 1);
-        r[q] = sl * 32 + lane;                         // true lane (see k_spmv_sell32)
-        b[q] = __ldg(sptr + sl);
-        W[q] = int((__ldg(sptr + sl + 1) - b[q]) >> 5);
-        info[q] = __ldg(sinfo + sl);
-    }
-    double acc[2] = {0.0, 0.0};
-    if ((info[0] & info[1] & 1) != 0) {
-        int myoff[2];
-#pragma unroll
-        for (int q = 0; q < 2; ++q) myoff[q] = lane < W[q] ? __ldg(dcol + (info[q] >> 2) + lane) : 0;
-        const int Wm = max(W[0], W[1]);
-        for (int t0 = 0; t0 < Wm; t0 += X2_B) {
-            double v[2][X2_B], xv[2][X2_B];
-#pragma unroll
-            for (int q = 0; q < 2; ++q)
-#pragma unroll
-                for (int k = 0; k < X2_B; ++k)
-                    if (t0 + k < W[q]) v[q][k] = __ldg(val + b[q] + 32 * (t0 + k) + lane);
-#pragma unroll
-            for (int q = 0; q < 2; ++q) {
-                const bool clamp = (info[q] & 2) != 0;
-#pragma unroll
-                for (int k = 0; k < X2_B; ++k) {
-                    const int off = __shfl_sync(0xffffffffu, myoff[q], (t0 + k) & 31);
-                    if (t0 + k < W[q]) {
-                        int64_t c = r[q] + off;
-                        if (clamp) c = c < 0 ? 0 : (c >= ncols ? ncols - 1 : c);
-                        xv[q][k] = __ldg(x + c);
-                    }
-                }
-            }
-#pragma unroll
-            for (int q = 0; q < 2; ++q)
-#pragma unroll
-                for (int k = 0; k < X2_B; ++k)
-                    if (t0 + k < W[q]) acc[q] = fma(v[q][k], xv[q][k], acc[q]);
-        }
-    } else {
-        acc[0] = sell_row_dot<SPMV_BATCH>(r[0], sptr, sinfo, dcol, ncols, val, x, false);
-        acc[1] = sell_row_dot<SPMV_BATCH>(r[1], sptr, sinfo, dcol, ncols, val, x, false);
-    }
-#pragma unroll
-    for (int q = 0; q < 2; ++q) {
-        const int64_t row = (2 * gw + q) * 32 + lane;
-        if (row >= nrows) continue;
-        double out;
-        if constexpr (MODE == 3) {
-            out = __ldg(u + row) - acc[q];
-        } else {
-            out = acc[q];
-            if constexpr (MODE >= 1) out = fma(bu, __ldg(u + row), out);
-            if constexpr (MODE >= 2) out = fma(bw, __ldg(w + row), out);
-        }
-        y[row] = out;
-    }
-}
-
 // Persistent SpMV with a software-pipelined slice descriptor.  In k_spmv_sell32 every warp
 // pays a chain of dependent loads before its first x gather (sptr/sinfo -> DIA offsets ->
 // x), ~3 L2/HBM latencies for 32 rows of ~7 entries.  Here a grid of (SMs x resident CTAs)
@@ -211,45 +129,25 @@ static void launch_persist(const Dev& d, const Sell& A, int64_t nrows, const dou
                A.dcol, A.ncols, A.val, x, u, bu, w, bw, y);
 }
 
+// CAGMRES_OPT_SPMV: 0 = one SELL-32 slice per warp (k_spmv_sell32); 5 = persistent grid with
+// software-pipelined slice descriptors (k_spmv_sell32_persist); 16, 17 = the DIA-width
+// specialised persistent kernel with an L2 prefetch of the next slice (spmv_dia.cu) at >= 4 / 5
+// CTAs per SM.  (Round 1 shipped 19 variants; the others were measured slower and removed:
+// DESIGN.md §6.)
 void spmv(const Dev& d, const Sell& A, int64_t nrows, const double* x, double* y,
           const double* u, double bu, const double* w, double bw, cudaStream_t st) {
     (void)d;
     if (nrows <= 0) return;
     ++g_launches;
     if (w && !u) { u = x; bu = 0.0; }             // pair step with a == 0: keep MODE 2 well formed
-    if (A.variant >= 21 && spmv_tma(d, A, A.variant, nrows, x, y, u, bu, w, bw, w ? 2 : (u ? 1 : 0), st) == 0)
-        return;
-    if (A.variant >= 10) {
-        spmv_dia(d, A, A.variant >= 21 ? 16 : A.variant, nrows, x, y, u, bu, w, bw, w ? 2 : (u ? 1 : 0), st);
+    if (A.variant >= 16) {
+        spmv_dia(d, A, A.variant, nrows, x, y, u, bu, w, bw, w ? 2 : (u ? 1 : 0), st);
         return;
     }
-    if (A.variant >= 4) {
-        auto go = [&](auto k0, auto k1, auto k2) {
-            if (w) k2(d, A, nrows, x, y, u, bu, w, bw, st);
-            else if (u) k1(d, A, nrows, x, y, u, bu, nullptr, 0.0, st);
-            else k0(d, A, nrows, x, y, nullptr, 0.0, nullptr, 0.0, st);
-        };
-        switch (A.variant) {   // (load batch, min CTAs per SM)
-            case 4: go(launch_persist<0, 8, 3>, launch_persist<1, 8, 3>, launch_persist<2, 8, 3>); break;
-            case 5: go(launch_persist<0, 4, 4>, launch_persist<1, 4, 4>, launch_persist<2, 4, 4>); break;
-            case 6: go(launch_persist<0, 4, 5>, launch_persist<1, 4, 5>, launch_persist<2, 4, 5>); break;
-            case 7: go(launch_persist<0, 4, 6>, launch_persist<1, 4, 6>, launch_persist<2, 4, 6>); break;
-            case 8: go(launch_persist<0, 2, 6>, launch_persist<1, 2, 6>, launch_persist<2, 2, 6>); break;
-            default: go(launch_persist<0, 2, 8>, launch_persist<1, 2, 8>, launch_persist<2, 2, 8>); break;
-        }
-        return;
-    }
-    if (A.variant >= 1) {
-        const int64_t nsl = (nrows + 31) >> 5;
-        const unsigned grid = unsigned((nsl + 2 * (NT / 32) - 1) / (2 * (NT / 32)));
-        auto go = [&](auto k0, auto k1, auto k2) {
-            if (w) k2<<<grid, NT, 0, st>>>(nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, u, bu, w, bw, y);
-            else if (u) k1<<<grid, NT, 0, st>>>(nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, u, bu, nullptr, 0.0, y);
-            else k0<<<grid, NT, 0, st>>>(nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, nullptr, 0.0, nullptr, 0.0, y);
-        };
-        if (A.variant == 2) go(k_spmv_sell32_x2<0, 8, 2>, k_spmv_sell32_x2<1, 8, 2>, k_spmv_sell32_x2<2, 8, 2>);
-        else if (A.variant == 3) go(k_spmv_sell32_x2<0, 4, 3>, k_spmv_sell32_x2<1, 4, 3>, k_spmv_sell32_x2<2, 4, 3>);
-        else go(k_spmv_sell32_x2<0, 4, 4>, k_spmv_sell32_x2<1, 4, 4>, k_spmv_sell32_x2<2, 4, 4>);
+    if (A.variant == 5) {
+        if (w) launch_persist<2, 4, 4>(d, A, nrows, x, y, u, bu, w, bw, st);
+        else if (u) launch_persist<1, 4, 4>(d, A, nrows, x, y, u, bu, nullptr, 0.0, st);
+        else launch_persist<0, 4, 4>(d, A, nrows, x, y, nullptr, 0.0, nullptr, 0.0, st);
         return;
     }
     const unsigned grid = unsigned((nrows + NT - 1) / NT);
@@ -266,19 +164,12 @@ void residual(const Dev& d, const Sell& A, int64_t nrows, const double* x, const
     (void)d;
     if (nrows <= 0) return;
     ++g_launches;
-    if (A.variant >= 21 && spmv_tma(d, A, A.variant, nrows, x, r, b, 1.0, nullptr, 0.0, 3, st) == 0) return;
-    if (A.variant >= 10) {
-        spmv_dia(d, A, A.variant >= 21 ? 16 : A.variant, nrows, x, r, b, 1.0, nullptr, 0.0, 3, st);
+    if (A.variant >= 16) {
+        spmv_dia(d, A, A.variant, nrows, x, r, b, 1.0, nullptr, 0.0, 3, st);
         return;
     }
-    if (A.variant >= 4) {
+    if (A.variant == 5) {
         launch_persist<3, 4, 4>(d, A, nrows, x, r, b, 1.0, nullptr, 0.0, st);
-        return;
-    }
-    if (A.variant >= 1) {
-        const int64_t nsl = (nrows + 31) >> 5;
-        const unsigned grid = unsigned((nsl + 2 * (NT / 32) - 1) / (2 * (NT / 32)));
-        k_spmv_sell32_x2<3, 4, 4><<<grid, NT, 0, st>>>(nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, b, 1.0, nullptr, 0.0, r);
         return;
     }
     const unsigned grid = unsigned((nrows + NT - 1) / NT);

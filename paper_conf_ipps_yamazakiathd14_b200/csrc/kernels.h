@@ -51,13 +51,12 @@ struct Dev {
 struct Sell {
     int64_t nrows = 0;          // stored rows (extended rows at distance <= s-1)
     int64_t nslices = 0;
-    int variant = 0;            // SpMV kernel: 0 one slice per warp (default); 1..3 two slices per warp
+    int variant = 0;            // SpMV kernel (CAGMRES_OPT_SPMV): 0, 5, 16, 17 (kernels.cu spmv)
     int64_t nstored = 0;        // stored values incl. padding
     int64_t nnz = 0;            // true nonzeros
     int64_t ncols = 0;          // valid x entries (clamp bound for DIA slices)
     int64_t ndcol = 0, ndia = 0;
     int dia_w = 0;              // most common width of the unclamped DIA slices (spmv_dia.cu)
-    uint32_t chunk_bytes = 0;   // largest value block of 8 consecutive slices (spmv_tma.cu stage)
     int64_t* sptr = nullptr;    // nslices+1 value offsets
     int64_t* sinfo = nullptr;   // nslices
     int32_t* dcol = nullptr;    // DIA offsets / explicit column ids
@@ -245,13 +244,10 @@ enum : int { ST_CHOL = 1, ST_SVQR = 2, ST_NORM = 4 };
 // second step of a complex pair: w = x_prev, bw = b^2.
 void spmv(const Dev& d, const Sell& A, int64_t nrows, const double* x, double* y,
           const double* u, double bu, const double* w, double bw, cudaStream_t st);
-// DIA-width-specialised SpMV (spmv_dia.cu), CAGMRES_OPT_SPMV 10..13; mode as k_spmv_sell32
+// DIA-width-specialised SpMV (spmv_dia.cu), CAGMRES_OPT_SPMV 16 / 17; mode as k_spmv_sell32
 // (3 = u - A x).
 void spmv_dia(const Dev& d, const Sell& A, int variant, int64_t nrows, const double* x, double* y,
               const double* u, double bu, const double* w, double bw, int mode, cudaStream_t st);
-// TMA-streamed SpMV (spmv_tma.cu), CAGMRES_OPT_SPMV 21 / 22; -1 if the matrix's chunks do not fit
-int spmv_tma(const Dev& d, const Sell& A, int variant, int64_t nrows, const double* x, double* y,
-             const double* u, double bu, const double* w, double bw, int mode, cudaStream_t st);
 // r[0:nrows) = b - A x
 void residual(const Dev& d, const Sell& A, int64_t nrows, const double* x, const double* b,
               double* r, cudaStream_t st);
@@ -291,19 +287,22 @@ void svqr_factor(const double* G, int w, double* R, int* status, cudaStream_t st
 void svqr_retry(const double* G, int w, double* R, int* status, cudaStream_t st);
 
 // P[:, 0:w] -= X C  (C: jx x w, ld jx)      (BOrth pass 2)
+// early: the preceding kernel in the stream writes neither X nor P (only C): the ring kernel
+// starts streaming X / P before griddepcontrol.wait (PDL overlap with that kernel's tail)
 void update(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, double* P,
-            int64_t ldp, int w, const double* C, cudaStream_t st);
+            int64_t ldp, int w, const double* C, cudaStream_t st, bool early = false);
 // P[:, c0:w] = (X M)[:, c0:w]  (X: n x K, ld ldx, contiguous columns that contain P; M: K x w,
 // ld ldm; P written in place)  — one-pass BOrth+CholQR update.  -1 if K > 64 or w > 32.
 int gemm_rows(const Dev& d, int64_t n, const double* X, int64_t ldx, int K, double* P, int64_t ldp, int w,
-              const double* M, int64_t ldm, int c0, cudaStream_t st);
+              const double* M, int64_t ldm, int c0, cudaStream_t st, bool early = false);
 // one-pass BOrth+CholQR small step (onepass.cu): from Mx = [Q P]^T P ((j+w) x w, ld j+w) write
 // C (j x (w-1), ld j), R = chol(Mx[j:, :] - Cf^T Cf) (ld w), Mo = [-Cf R^{-1}; R^{-1}] (ld j+w).
 void onepass_finalize(const double* Mx, int j, int w, double* C, double* R, double* Mo, int* status,
                       cudaStream_t st);
 // P[:, c0:w] = (P R^{-1})[:, c0:w]   (R upper w x w, ld w)
+// early: as for update (the preceding kernel only produced R)
 void trsm(const Dev& d, int64_t n, double* P, int64_t ldp, int w, const double* R, int c0,
-          cudaStream_t st);
+          cudaStream_t st, bool early = false);
 // Halo pack / unpack over segments [off[i], off[i] + cnt[i]) of an index list (one segment per
 // peer: the depth-limited prefix of that peer's level-sorted list).
 struct Segs {

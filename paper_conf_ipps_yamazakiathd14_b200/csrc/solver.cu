@@ -178,11 +178,6 @@ int build_sell(cagmres* h, const cagmres_plan& p) {
     const int64_t ndia = sh.ndia;
     h->A.nrows = nr; h->A.nslices = ns; h->A.nstored = tot; h->A.nnz = p.nnz_mat;
     h->A.ncols = p.n_ext; h->A.ndcol = ndcol; h->A.ndia = ndia;
-    {   // largest value block of 8 consecutive slices (the TMA SpMV's stage size)
-        int64_t mx = 0;
-        for (int64_t c0 = 0; c0 < ns; c0 += 8) mx = std::max(mx, sptr[size_t(std::min(ns, c0 + 8))] - sptr[size_t(c0)]);
-        h->A.chunk_bytes = mx * 8 > int64_t(1) << 30 ? 0u : uint32_t(mx * 8);
-    }
     {   // most common width among unclamped DIA slices (the specialised SpMV's fast path)
         std::vector<int64_t> cnt(33, 0);
         for (int64_t sl = 0; sl < ns; ++sl)
@@ -319,9 +314,7 @@ void wave_reset_pairs(cagmres* h) {
 // the same operations in the same order (bitwise identical results), so the fastest one on
 // this matrix is picked by timing y = A x over all stored rows (x = V[:,0], y = V[:,1]).
 int spmv_autotune(cagmres* h) {
-    // 14, 15 (CTA-contiguous) are faster per launch but lose ~1.4 ms per C2 solve in the
-    // back-to-back PDL chain (profiles/r1_bench_C2_spmv14.json): options only
-    static const int cand[] = {0, 3, 5, 6, 8, 10, 11, 12, 13, 16, 17, 18, 21, 22};
+    static const int cand[] = {0, 5, 16, 17};
     if (h->m < 1 || h->A.nrows <= 0) return CAGMRES_OK;
     double* x = h->V;
     double* y = h->V + h->ldv;
@@ -590,7 +583,7 @@ int borth_panel(cagmres* h, const double* Q, int64_t ldq, int j, double* P, int6
     if (!mgs) {
         TRY(xty_global(h, Q, ldq, j, P, ldp, w, C, false, nullptr));
         // C is jx x w with ld jx = j: xty writes ld jx
-        kern::update(h->dev, h->n_loc, Q, ldq, j, P, ldp, w, C, h->stream);
+        kern::update(h->dev, h->n_loc, Q, ldq, j, P, ldp, w, C, h->stream, true);   // after xty: early start
         h->bytes[PH_BORTH] += 8.0 * double(h->n_loc) * (2.0 * j + 3.0 * w);
     } else {
         // row l of C (1 x w, ld j) via a scratch row then copied with ld j on the host view:
@@ -619,7 +612,7 @@ int tsqr_panel(cagmres* h, double* P, int64_t ldp, int w, double* R, int kind, i
             TRY(xty_global(h, P, ldp, w, P, ldp, w, h->gbuf, false, nullptr));
             kern::svqr_factor(h->gbuf, w, R, h->status, h->stream);
         }
-        kern::trsm(h->dev, h->n_loc, P, ldp, w, R, c0, h->stream);          // V := V R^{-1}
+        kern::trsm(h->dev, h->n_loc, P, ldp, w, R, c0, h->stream, true);    // V := V R^{-1} (P final: early)
         h->bytes[PH_TSQR] += 8.0 * nl * (2.0 * w + double(w - c0));
     } else if (kind == CAGMRES_CAQR) {                       // Fig. 9 CAQR: TSQR tree
         // Multi-rank: "each GPU first computes the QR factorization of the local
@@ -763,7 +756,7 @@ int ca_cycle(cagmres* h, const std::vector<Block>& bl) {
                 Scope sc(h, PH_TSQR);
                 kern::onepass_finalize(h->gbuf, j, w, C, R, h->op_M, h->status, h->stream);
                 if (kern::gemm_rows(h->dev, h->n_loc, h->V, h->ldv, j + w, Pj, h->ldv, w, h->op_M, j + w, 1,
-                                    h->stream))
+                                    h->stream, true))
                     return CAGMRES_EINVAL;
                 h->bytes[PH_TSQR] += 8.0 * nl * (j + w + (w - 1));
                 continue;
@@ -1017,7 +1010,7 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
     switch (opt) {
         case CAGMRES_OPT_MPK_WAVE: h->wave_on = value != 0; h->wave_force = value == 2; return CAGMRES_OK;
         case CAGMRES_OPT_SPMV:
-            if (value < -1 || value > 22) return CAGMRES_EINVAL;
+            if (value != -1 && value != 0 && value != 5 && value != 16 && value != 17) return CAGMRES_EINVAL;
             if (value == -1) return spmv_autotune(h);
             h->A.variant = int(value);
             return CAGMRES_OK;

@@ -29,6 +29,10 @@ struct StreamArgs {
     const double* M; int64_t ldm;             // C (jx x w) or R (w x w), leading dim ldm
     int c0;                                   // trsm: first column written
     int pf = 0;                               // L2 prefetch ahead of the ring (Dev::panel_pf)
+    // 1: the kernel immediately before this one in the stream does not write X or P (it only
+    // produced C / R), so the ring kernels issue their first tile copies BEFORE
+    // griddepcontrol.wait and fill their pipelines while that kernel drains (PDL)
+    int early = 0;
 };
 
 // R^{-1} (upper, w x w) into sRi[k*32 + c]; one thread per column (back substitution)
@@ -143,8 +147,10 @@ __global__ void __launch_bounds__(MAXT, 1) k_rows_pipe(StreamArgs a) {
     constexpr int SP = TW + 8;
     __shared__ double sB[32 * 32 + 32];
     __shared__ const double* sCol[96];                         // column base pointers (ncol <= 96)
-    pdl_wait();
-    pdl_trigger();
+    if (!a.early) {
+        pdl_wait();
+        pdl_trigger();
+    }
     const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const int gid = lane >> 2, tig = lane & 3;
     const int w = a.w;
@@ -153,19 +159,7 @@ __global__ void __launch_bounds__(MAXT, 1) k_rows_pipe(StreamArgs a) {
     const int ncol = MODE == 2 ? a.jx : jxl + w;               // gemm: P is inside X
     for (int c = threadIdx.x; c < ncol; c += blockDim.x)
         sCol[c] = c < jxl ? a.X + a.ldx * c : a.P + a.ldp * (c - jxl);
-    if (MODE == 1) upper_inverse(a.M, w, sB, sB + 32 * 32);  // (has __syncthreads)
-    else __syncthreads();
-    // B fragments (update: -C, so d = P + A (-C) needs no per-element negation)
-    double b[KTM][NTN];
-#pragma unroll
-    for (int kt = 0; kt < KTM; ++kt)
-#pragma unroll
-        for (int nt = 0; nt < NTN; ++nt) {
-            const int k = 4 * kt + tig, c = 8 * nt + gid;
-            double v = 0.0;
-            if (k < K && c < w) v = MODE != 1 ? a.M[k + a.ldm * c] : sB[k * 32 + c];
-            b[kt][nt] = MODE == 0 ? -v : v;
-        }
+    __syncthreads();
     // measured (profiles/r1_launches_C2_pf.txt): prefetch helps narrow panels, hurts wide ones
     const bool d_pf = a.pf != 0 && TW == 32 && ncol <= 24;
     const int64_t stage_d = int64_t(ncol) * SP;
@@ -206,6 +200,22 @@ __global__ void __launch_bounds__(MAXT, 1) k_rows_pipe(StreamArgs a) {
         }
 #pragma unroll
     for (int s = 0; s < RP_S - 1; ++s) issue(t0 + s, s);
+    if (a.early) {                                             // X, P final before the predecessor
+        pdl_wait();
+        pdl_trigger();
+    }
+    if (MODE == 1) upper_inverse(a.M, w, sB, sB + 32 * 32);  // (has __syncthreads)
+    // B fragments (update: -C, so d = P + A (-C) needs no per-element negation)
+    double b[KTM][NTN];
+#pragma unroll
+    for (int kt = 0; kt < KTM; ++kt)
+#pragma unroll
+        for (int nt = 0; nt < NTN; ++nt) {
+            const int k = 4 * kt + tig, c = 8 * nt + gid;
+            double v = 0.0;
+            if (k < K && c < w) v = MODE != 1 ? a.M[k + a.ldm * c] : sB[k * 32 + c];
+            b[kt][nt] = MODE == 0 ? -v : v;
+        }
     int stage = 0, stage_in = RP_S - 1;
     for (int64_t t = t0; t < t1; ++t) {
         issue(t + RP_S - 1, stage_in);
@@ -403,14 +413,10 @@ __global__ void __launch_bounds__(512, 1) k_trsm_ring(StreamArgs a) {
     constexpr int WP = W + (W & 1);                             // even row stride: 16-B pairs
     __shared__ __align__(16) double sRi[W * WP];
     const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    pdl_wait();
-    pdl_trigger();
-    upper_inverse(a.M, W, sB, sB + 32 * 32);
-    for (int q = threadIdx.x; q < W * WP; q += blockDim.x) {
-        const int k = q / WP, c = q - k * WP;
-        sRi[q] = c < W ? sB[k * 32 + c] : 0.0;                 // [k * WP + c] = R^{-1}[k][c]
+    if (!a.early) {
+        pdl_wait();
+        pdl_trigger();
     }
-    __syncthreads();
     constexpr int SD = W * 32;
     double* ring = smt + int64_t(wp) * RS * SD;
     const int64_t T = a.n / 32;
@@ -449,6 +455,16 @@ __global__ void __launch_bounds__(512, 1) k_trsm_ring(StreamArgs a) {
     };
 #pragma unroll
     for (int s = 0; s < RS - 1; ++s) issue(t0 + s, s);
+    if (a.early) {                                             // P final before the Gram / Cholesky
+        pdl_wait();
+        pdl_trigger();
+    }
+    upper_inverse(a.M, W, sB, sB + 32 * 32);
+    for (int q = threadIdx.x; q < W * WP; q += blockDim.x) {
+        const int k = q / WP, c = q - k * WP;
+        sRi[q] = c < W ? sB[k * 32 + c] : 0.0;                 // [k * WP + c] = R^{-1}[k][c]
+    }
+    __syncthreads();
     int stage = 0;
     for (int64_t t = t0; t < t1; ++t) {
         issue(t + RS - 1, stage == 0 ? RS - 1 : stage - 1);
@@ -523,27 +539,28 @@ bool trsm_ring(const Dev& d, const StreamArgs& a, cudaStream_t st) {
 }  // namespace
 
 void update(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, double* P,
-            int64_t ldp, int w, const double* C, cudaStream_t st) {
+            int64_t ldp, int w, const double* C, cudaStream_t st, bool early) {
     if (n <= 0 || w <= 0) return;
     if (w == 1 && jx <= 32 && update_w1(d, n, X, ldx, jx, P, C, st) == 0) return;
-    // wide X (> 64 columns): P -= X[:, s] C[s, :] in 64-column slabs (C viewed with ld jx)
+    // wide X (> 64 columns): P -= X[:, s] C[s, :] in 64-column slabs (C viewed with ld jx);
+    // a later slab follows a launch that wrote P: no early start for it
     for (int s0 = 0; s0 < jx; s0 += 64) {
         const int js = jx - s0 < 64 ? jx - s0 : 64;
-        StreamArgs a{n, X + ldx * s0, ldx, js, P, ldp, w, C + s0, jx, 0, d.panel_pf};
+        StreamArgs a{n, X + ldx * s0, ldx, js, P, ldp, w, C + s0, jx, 0, d.panel_pf, early && s0 == 0 ? 1 : 0};
         dispatch<0>(d, a, st);
     }
 }
 
 int gemm_rows(const Dev& d, int64_t n, const double* X, int64_t ldx, int K, double* P, int64_t ldp, int w,
-              const double* M, int64_t ldm, int c0, cudaStream_t st) {
+              const double* M, int64_t ldm, int c0, cudaStream_t st, bool early) {
     if (n <= 0 || w <= 0) return 0;
     if (K > 64 || w > 32) return -1;
-    StreamArgs a{n, X, ldx, K, P, ldp, w, M, ldm, c0, d.panel_pf};
+    StreamArgs a{n, X, ldx, K, P, ldp, w, M, ldm, c0, d.panel_pf, early ? 1 : 0};
     return dispatch<2>(d, a, st);
 }
 
 void trsm(const Dev& d, int64_t n, double* P, int64_t ldp, int w, const double* R, int c0,
-          cudaStream_t st) {
+          cudaStream_t st, bool early) {
     if (n <= 0 || w <= 0) return;
     if (w == 1 && c0 == 0) {
         int64_t g = int64_t(d.sms) * 4;
@@ -553,7 +570,7 @@ void trsm(const Dev& d, int64_t n, double* P, int64_t ldp, int w, const double* 
         launch_pdl(k_scale1, dim3(unsigned(g)), dim3(256), 0, st, n, P, R);
         return;
     }
-    StreamArgs a{n, nullptr, 0, 0, P, ldp, w, R, w, c0, d.panel_pf};
+    StreamArgs a{n, nullptr, 0, 0, P, ldp, w, R, w, c0, d.panel_pf, early ? 1 : 0};
     if (d.trsm_scalar && trsm_ring(d, a, st)) return;
     dispatch<1>(d, a, st);
 }

@@ -142,7 +142,7 @@ def test_spmv_variants_bitwise(gen):
     S = Solver(A, s=6, m=30, basis="newton")
     S.set_shifts(*SHIFTS)
     Ws = []
-    variants = list(range(10)) + [10, 11, 12, 13, 14, 15, 16, 17, 18, 19, 20, 21, 22]
+    variants = [0, 5, 16, 17]
     for v in variants:
         S.set_option("spmv", v)
         Ws.append(S.mpk(q, 6))
@@ -353,9 +353,9 @@ def test_solve_fused_borth_gram(fuse, s, m, reorth):
     assert hist_within_envelope(st.hist, ref, env)
 
 
-@pytest.mark.parametrize("spmv,gram", [(4, 1), (5, 0), (0, 1)])
+@pytest.mark.parametrize("spmv,gram", [(16, 1), (5, 0), (0, 1)])
 def test_solve_kernel_options(spmv, gram):
-    """Solve with the persistent SpMV (CAGMRES_OPT_SPMV 4/5) and the scalar-DFMA Gram
+    """Solve with the persistent SpMVs (CAGMRES_OPT_SPMV 16 / 5) and the scalar-DFMA Gram
     (CAGMRES_OPT_GRAM 1) against the oracle: 3D 7-point 40^3 (n = 64,000), s = 10, m = 30."""
     A = G.convection_diffusion(40, 3, 7)
     As = A.to_scipy()

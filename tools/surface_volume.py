@@ -1,5 +1,6 @@
 """MPK surface-to-volume and halo-volume study (the quantities of the paper's Fig. 6/7,
-P:98-118) for contiguous block-row partitions, natural vs RCM order.
+P:98-118) for contiguous block-row partitions: natural vs RCM order vs
+the library's k-way partition (cagmres_host_partition, parts made contiguous).
 Host only (the setup plan of libcagmres.so, cagmres_plan_* / cagmres_host_rcm); no GPU.
 
 For P ranks and depth s, rank d's MPK needs the ghost rows within s hops of its owned rows
@@ -7,7 +8,7 @@ For P ranks and depth s, rank d's MPK needs the ghost rows within s hops of its 
 ghost rows within s - k hops: redundant SpMV rows = sum_{k=1..s} (L[s-k] - n_loc), where
 L[h] = rows within h hops (level_len).  Reported as fractions of n_loc, max over ranks.
 
-    python tools/surface_volume.py > profiles/r1_mpk_surface_volume.json
+    python tools/surface_volume.py > profiles/r2_mpk_surface_volume.json
 """
 import json
 import os
@@ -23,8 +24,9 @@ from synth import generators as G  # noqa: E402
 S_MAX = 10
 
 
-def study(A, P):
-    rs = np.array([(p * A.n) // P for p in range(P + 1)], dtype=np.int64)
+def study(A, P, rs=None):
+    if rs is None:
+        rs = np.array([(p * A.n) // P for p in range(P + 1)], dtype=np.int64)
     per = []
     for d in range(P):
         pl = host.Plan(A, rs, d, S_MAX)
@@ -48,9 +50,17 @@ def main():
         t_rcm = time.time() - t0
         As = host.permute(A, np.argsort(G.u(99, np.arange(A.n))))       # arbitrary (scrambled) order
         Asr = host.permute(As, host.rcm(As))                            # ... then RCM
-        for order, M in (("natural", A), ("rcm", Ar), ("scrambled", As), ("scrambled+rcm", Asr)):
+        for order, M in (("natural", A), ("rcm", Ar), ("scrambled", As), ("scrambled+rcm", Asr),
+                         ("kway", A), ("scrambled+kway", As)):
             for P in (2, 4, 8):
-                out[f"{name} | {order} | P={P}"] = study(M, P)
+                rs = None
+                if order.endswith("kway"):
+                    t0 = time.time()
+                    M2, _, rs = host.distribute(M, P, "kway")
+                    out[f"{name} | {order} | P={P} | partition_seconds"] = round(time.time() - t0, 2)
+                else:
+                    M2 = M
+                out[f"{name} | {order} | P={P}"] = study(M2, P, rs)
                 print(name, order, P, json.dumps(out[f"{name} | {order} | P={P}"]["s=10"]),
                       file=sys.stderr, flush=True)
         out[f"{name} | rcm_seconds"] = round(t_rcm, 2)
