@@ -185,7 +185,9 @@ struct WaveArgs {
     int64_t n; int64_t bw; int CH, nC;    // rows, half-bandwidth, rows per chunk, chunks
     const int2* pairs; int npairs;        // (chunk, step) items in wavefront order
     int* done;                            // (s+1) x nC epoch-stamped completion flags
+    int* queue;                           // item ticket counter (zeroed before each launch)
     int epoch;
+    int dia_w;                            // the matrix's dominant DIA width (fast row body)
     double theta[32], b2[32];
     int kind[32];
 };

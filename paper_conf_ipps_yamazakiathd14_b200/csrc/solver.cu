@@ -284,8 +284,8 @@ int wave_pairs(cagmres* h, int sb) {
         h->npairs.assign(size_t(h->s) + 1, 0);
         cudaFree(h->d_done);
         h->d_done = nullptr;
-        CU(cudaMalloc(&h->d_done, sizeof(int) * size_t(nC) * size_t(h->s + 1)));
-        CU(cudaMemset(h->d_done, 0, sizeof(int) * size_t(nC) * size_t(h->s + 1)));
+        CU(cudaMalloc(&h->d_done, sizeof(int) * (size_t(nC) * size_t(h->s + 1) + 1)));
+        CU(cudaMemset(h->d_done, 0, sizeof(int) * (size_t(nC) * size_t(h->s + 1) + 1)));
         h->wave_nC = nC;
         h->wave_epoch = 0;
     }
@@ -533,10 +533,13 @@ int mpk_block(cagmres* h, int j, int sb, const std::vector<host::Step>& steps) {
         a.n = h->n_loc; a.bw = h->wave_bw; a.CH = h->wave_CH; a.nC = h->wave_nC;
         a.pairs = h->d_pairs[size_t(sb)]; a.npairs = h->npairs[size_t(sb)];
         a.done = h->d_done;
+        a.queue = h->d_done + size_t(h->wave_nC) * size_t(h->s + 1);
+        a.dia_w = h->A.dia_w;
         if (++h->wave_epoch == 0x7fffffff) {                 // epoch wrap: clear the flags
             CU(cudaMemsetAsync(h->d_done, 0, sizeof(int) * size_t(h->wave_nC) * size_t(h->s + 1), h->stream));
             h->wave_epoch = 1;
         }
+        CU(cudaMemsetAsync(a.queue, 0, sizeof(int), h->stream));
         a.epoch = h->wave_epoch;
         for (int k = 1; k <= sb; ++k) {
             a.theta[k - 1] = steps[size_t(k - 1)].a;

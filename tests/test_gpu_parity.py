@@ -127,6 +127,11 @@ def test_mpk_wave_bitwise_equals_stepwise(gen):
     for sb in (10, 4, 2):
         W1, W2 = S1.mpk(q, sb), S2.mpk(q, sb)
         assert torch.equal(W1, W2), (gen, sb)
+    if gen == "cd27_40":                          # and directly against the oracle (Fig. 4)
+        Wo = O.mpk(A.to_scipy(), q.cpu().numpy(), 10, *SHIFTS)
+        W1 = S1.mpk(q, 10).cpu().numpy()
+        for k in range(11):
+            assert np.max(np.abs(W1[:, k] - Wo[:, k])) <= 1e-13 * np.max(np.abs(Wo[:, k])), k
 
 
 @pytest.mark.parametrize("gen", ["cd27_ragged", "g3_small", "banded", "cd7_ragged"])
