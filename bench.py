@@ -155,12 +155,20 @@ def run_ours(args):
         S = Solver(A, cfg["s"], cfg["m"], basis=cfg["basis"], tsqr=cfg["tsqr"], reorth=cfg["reorth"] or args.reorth,
                    onepass=args.onepass)
         b_host = G.rhs(cfg["n"])
-    else:
+    elif args.order == "natural":
         rs = np.array([(p * cfg["n"]) // ws for p in range(ws + 1)], dtype=np.int64)
         A = ghost_rows(cfg, rs, rank, cfg["s"])
         S = Solver(A, cfg["s"], cfg["m"], basis=cfg["basis"], tsqr=cfg["tsqr"], reorth=cfg["reorth"] or args.reorth,
                    group=group, row_starts=rs, onepass=args.onepass)
         b_host = G.rhs(cfg["n"], rows=(rs[rank], rs[rank + 1]))
+    else:
+        # NEXT-4 row distribution: every rank builds the same permutation of the whole
+        # matrix (k-way partition or RCM, host library, deterministic) and owns a block of B = P A P^T
+        from paper_conf_ipps_yamazakiathd14_b200 import host
+        A, perm, rs = host.distribute(cfg["build"](), ws, args.order)
+        S = Solver(A, cfg["s"], cfg["m"], basis=cfg["basis"], tsqr=cfg["tsqr"], reorth=cfg["reorth"] or args.reorth,
+                   group=group, row_starts=rs, onepass=args.onepass)
+        b_host = G.rhs(cfg["n"])[perm][rs[rank]:rs[rank + 1]]
     for kv in args.opt:
         k_, v_ = kv.split("=")
         S.set_option(k_, int(v_))
@@ -309,6 +317,7 @@ def run_ours(args):
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": cfg["workload"], "n": cfg["n"], "s": cfg["s"], "m": cfg["m"],
                        "tol": TOL, "cycles": stats[-1].cycles, "parallelism": f"rows{ws}",
+                       "row_order": args.order if ws > 1 else "natural",
                        "l2": f"inputs larger than L2 (A {12 * A.nnz / 1e6:.0f} MB as CSR, V {8 * S.ldv * (cfg['m'] + 1) / 1e6:.0f} MB)"
                              " + 256 MB flush between steps",
                        "setup_s": round(setup_s, 2), "options": args.opt,
@@ -462,6 +471,9 @@ def main():
     ap.add_argument("--no-gmres", action="store_true", help="skip the GPU GMRES(m) comparator")
     ap.add_argument("--reorth", action="store_true", help="2x BOrth+TSQR (CholQR2)")
     ap.add_argument("--onepass", action="store_true", help="one-pass BOrth+CholQR (CAGMRES_ONEPASS, NEXT-2)")
+    ap.add_argument("--order", default="natural", choices=["natural", "rcm", "kway"],
+                    help="row distribution for --gpus N > 1 (NEXT-4): natural block rows, RCM, or the "
+                         "library's k-way partition made contiguous")
     ap.add_argument("--opt", action="append", default=[],
                     help="solver option NAME=VALUE (CAGMRES_OPT_*: spmv, gram, fuse, mpk_wave, ...); "
                          "default: the library's defaults")

@@ -51,12 +51,21 @@ def hist_close(h, ref, rtol=1e-10, atol=1e-15):
 def rounding_envelope(As, b, nperm=2, **kw):
     """The oracle's own sensitivity to summation order: rerun it on symmetric permutations
     P A P^T, P b (identical in exact arithmetic, different rounding) and return
-    (reference history, running max of the relative deviation per cycle)."""
+    (reference history, running max of the relative deviation per cycle).
+    SVQR additionally: its R is the Cholesky factor of the Gram in exact arithmetic,
+    computed through a symmetric eigendecomposition whose algorithm differs between the sides
+    (LAPACK dsyevd vs the device's Jacobi sweeps); the oracle's own SVQR-vs-CholQR difference
+    measures that algorithm noise and joins the envelope."""
     ref = O.cagmres(As, b, **kw)["hist"]
     dev_ = np.zeros(len(ref))
+    alts = [dict(kw, tsqr="cholqr")] if kw.get("tsqr") == "svqr" else []
     for s in range(nperm):
         p = np.argsort(G.u(1000 + s, np.arange(As.shape[0])))
         hp = O.cagmres(As[p][:, p], b[p], **kw)["hist"]
+        k = min(len(hp), len(ref))
+        dev_[:k] = np.maximum(dev_[:k], np.abs(hp[:k] - ref[:k]) / ref[:k])
+    for kw2 in alts:
+        hp = O.cagmres(As, b, **kw2)["hist"]
         k = min(len(hp), len(ref))
         dev_[:k] = np.maximum(dev_[:k], np.abs(hp[:k] - ref[:k]) / ref[:k])
     return ref, np.maximum.accumulate(dev_)

@@ -64,7 +64,15 @@ def solve_margins():
         "cd7_40_s10": (lambda: G.convection_diffusion(40, 3, 7), dict(s=10, m=30, basis="newton"), True),
         "g3_40k": (lambda: G.g3_shaped(n=40000, width=200), dict(s=5, m=60, basis="newton"), False),
         "C2_full": (lambda: G.convection_diffusion(128, 3, 7), dict(s=10, m=30, basis="newton"), False),
+        "C1_svqr": (lambda: G.convection_diffusion(32, 2, 5), dict(s=5, m=30, basis="newton", tsqr="svqr"), True),
+        "C1_cholqr2": (lambda: G.convection_diffusion(32, 2, 5), dict(s=5, m=30, basis="newton", reorth=True), True),
+        "C1_cgs2": (lambda: G.convection_diffusion(32, 2, 5), dict(s=5, m=30, basis="newton", tsqr="cgs", reorth=True), True),
+        "C1_mgs": (lambda: G.convection_diffusion(32, 2, 5), dict(s=5, m=30, basis="newton", tsqr="mgs", borth="mgs"), True),
+        "C1_caqr": (lambda: G.convection_diffusion(32, 2, 5), dict(s=5, m=30, basis="newton", tsqr="caqr"), True),
     }
+    only = os.environ.get("MARGINS_ONLY")
+    if only:
+        cases = {k: v for k, v in cases.items() if k in only.split(",")}
     out = {}
     for name, (f, kw, inject) in cases.items():
         A = f()
@@ -91,4 +99,7 @@ def solve_margins():
 
 if __name__ == "__main__":
     torch.cuda.set_device(0)
-    print(json.dumps({"mpk": mpk_margins(), "solve": solve_margins()}, indent=1))
+    out = {"solve": solve_margins()}
+    if not os.environ.get("MARGINS_ONLY"):
+        out["mpk"] = mpk_margins()
+    print(json.dumps(out, indent=1))
