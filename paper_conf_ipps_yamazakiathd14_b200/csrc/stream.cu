@@ -144,7 +144,9 @@ constexpr int RP_S = 3;
 template <int MODE, int KTM, int NTN, int TW, int MAXT = 512>   // MAXT 256: up to 255 registers
 __global__ void __launch_bounds__(MAXT, 1) k_rows_pipe(StreamArgs a) {
     extern __shared__ __align__(16) double smp[];
-    constexpr int SP = TW + 8;
+    constexpr int SP = TW + 4;     // == 4 mod 16 doubles: A (8 rows x 4 cols) and P (8 rows x cols
+                                   // 2 tig + h) fragment reads both take the 2 ideal wavefronts
+                                   // (TW + 8 put the 4 P columns of a lane quad on the same banks)
     __shared__ double sB[32 * 32 + 32];
     __shared__ const double* sCol[96];                         // column base pointers (ncol <= 96)
     if (!a.early) {
@@ -301,7 +303,7 @@ bool run_pipe_tw(const Dev& d, const StreamArgs& a, cudaStream_t st) {
                          (a.ldp % 2 == 0) && (MODE == 1 || a.ldx % 2 == 0);
     if (!aligned || a.n < 64 * TW) return false;
     const int ncol = MODE == 2 ? a.jx : (MODE == 0 ? a.jx : 0) + a.w;
-    const size_t ring_w = size_t(RP_S) * ncol * (TW + 8) * sizeof(double);
+    const size_t ring_w = size_t(RP_S) * ncol * (TW + 4) * sizeof(double);
     int nw = int((200 * 1024) / ring_w);
     nw = nw < 2 ? 2 : (nw > 16 ? 16 : nw);
     const size_t smem = size_t(nw) * ring_w;
@@ -407,7 +409,7 @@ __global__ void __launch_bounds__(256) k_scale1(int64_t n, double* __restrict__ 
 // out[c] = sum_{k <= c} p[k] Ri[k][c] for c >= c0 with R^{-1} broadcast from shared memory:
 // w(w+1)/2 DFMAs per row, no padding.
 template <int W, int RS>
-__global__ void __launch_bounds__(512, 1) k_trsm_ring(StreamArgs a) {
+__global__ void __launch_bounds__(256, 1) k_trsm_ring(StreamArgs a) {
     extern __shared__ __align__(16) double smt[];
     __shared__ double sB[32 * 32 + 32];
     constexpr int WP = W + (W & 1);                             // even row stride: 16-B pairs
@@ -417,28 +419,46 @@ __global__ void __launch_bounds__(512, 1) k_trsm_ring(StreamArgs a) {
         pdl_wait();
         pdl_trigger();
     }
-    constexpr int SD = W * 32;
+    // 64-row tiles, two rows per lane (rows 2 lane, 2 lane + 1: one 16-B shared load per column):
+    // every broadcast load of two R^{-1} entries feeds four FMAs (ncu, 32-row tiles with one row
+    // per lane: MIO-throttle / short-scoreboard bound on the R^{-1} loads)
+    constexpr int TR = 64;
+    constexpr int SD = W * TR;
     double* ring = smt + int64_t(wp) * RS * SD;
-    const int64_t T = a.n / 32;
+    const int64_t T = a.n / TR;
     const int64_t Wn = int64_t(gridDim.x) * nw;
     const int64_t g = int64_t(blockIdx.x) * nw + wp;
     const int64_t t0 = g * T / Wn, t1 = (g + 1) * T / Wn;
     const int c0 = a.c0;
-    const int part2 = 2 * (lane & 15), cfirst = lane >> 4;
-    const double* srcl = a.P + a.ldp * cfirst + part2;         // this lane's copy slots: columns
-    const int64_t cstride = 2 * a.ldp;                          // cfirst, cfirst + 2, ...
     auto issue = [&](int64_t t, int stage) {
         if (t < t1) {
-            double* dst = ring + stage * SD + cfirst * 32 + part2;
-            const double* src = srcl + t * 32;
+            double* dst = ring + stage * SD + 2 * lane;
+            const double* src = a.P + t * TR + 2 * lane;
 #pragma unroll
-            for (int c = cfirst; c < W; c += 2, dst += 64, src += cstride) ptx::cp_async16(dst, src);
+            for (int c = 0; c < W; ++c) ptx::cp_async16(dst + c * TR, src + a.ldp * c);
         }
         ptx::cp_async_commit();
     };
     // two output columns per 16-B broadcast load of R^{-1}: out[c], out[c+1] = sum_k p[k] Ri[k][.]
-    // (Ri[c+1][c] = 0: the extra term adds an exact zero)
-    auto rowout = [&](const double (&v)[W], double* out) {
+    // (Ri[c+1][c] = 0: the extra term adds an exact zero); per output the FMAs run k = 0..c+1
+    auto rowout2 = [&](const double (&v0)[W], const double (&v1)[W], double* out) {
+#pragma unroll
+        for (int c = 0; c < W; c += 2) {
+            if (c + 1 < c0) continue;
+            double a00 = 0.0, a01 = 0.0, a10 = 0.0, a11 = 0.0;
+#pragma unroll
+            for (int k = 0; k <= c + 1 && k < W; ++k) {
+                const double2 r2 = *reinterpret_cast<const double2*>(&sRi[k * WP + c]);
+                a00 = fma(v0[k], r2.x, a00);
+                a01 = fma(v0[k], r2.y, a01);
+                a10 = fma(v1[k], r2.x, a10);
+                a11 = fma(v1[k], r2.y, a11);
+            }
+            if (c >= c0) *reinterpret_cast<double2*>(out + a.ldp * c) = make_double2(a00, a10);
+            if (c + 1 < W) *reinterpret_cast<double2*>(out + a.ldp * (c + 1)) = make_double2(a01, a11);
+        }
+    };
+    auto rowout = [&](const double (&v)[W], double* out) {           // one row (ragged tail)
 #pragma unroll
         for (int c = 0; c < W; c += 2) {
             if (c + 1 < c0) continue;
@@ -468,22 +488,23 @@ __global__ void __launch_bounds__(512, 1) k_trsm_ring(StreamArgs a) {
     int stage = 0;
     for (int64_t t = t0; t < t1; ++t) {
         issue(t + RS - 1, stage == 0 ? RS - 1 : stage - 1);
-        if (a.pf && t + RS - 1 + ptx::PF_DIST < t1 && lane < 2 * W)
-            ptx::prefetch_l2(a.P + a.ldp * (lane >> 1) + (t + RS - 1 + ptx::PF_DIST) * 32 + 16 * (lane & 1));
         ptx::cp_async_wait<RS - 1>();
         __syncwarp();
-        const double* sl = ring + stage * SD + lane;
-        double v[W];
+        const double* sl = ring + stage * SD + 2 * lane;
+        double v0[W], v1[W];
 #pragma unroll
-        for (int k = 0; k < W; ++k) v[k] = sl[k * 32];
-        rowout(v, a.P + t * 32 + lane);
+        for (int k = 0; k < W; ++k) {
+            const double2 p2 = *reinterpret_cast<const double2*>(sl + k * TR);
+            v0[k] = p2.x;
+            v1[k] = p2.y;
+        }
+        rowout2(v0, v1, a.P + t * TR + 2 * lane);
         __syncwarp();
         stage = stage == RS - 1 ? 0 : stage + 1;
     }
     ptx::cp_async_wait<0>();
-    if (blockIdx.x == 0 && wp == 0) {                          // ragged tail rows [32 T, n)
-        const int64_t r = T * 32 + lane;
-        if (r < a.n) {
+    if (blockIdx.x == 0 && wp == 0) {                          // ragged tail rows [64 T, n)
+        for (int64_t r = T * TR + lane; r < a.n; r += 32) {
             double v[W];
 #pragma unroll
             for (int k = 0; k < W; ++k) v[k] = a.P[a.ldp * k + r];
@@ -494,9 +515,9 @@ __global__ void __launch_bounds__(512, 1) k_trsm_ring(StreamArgs a) {
 
 template <int W, int RS>
 bool go_trsm_rs(const Dev& d, const StreamArgs& a, cudaStream_t st) {
-    const size_t ring_w = size_t(RS) * W * 32 * sizeof(double);
+    const size_t ring_w = size_t(RS) * W * 64 * sizeof(double);
     int nw = int((200 * 1024) / ring_w);
-    nw = nw < 2 ? 2 : (nw > 16 ? 16 : nw);
+    nw = nw < 2 ? 2 : (nw > 8 ? 8 : nw);              // <= 256 threads: R^{-1} stays in registers
     const size_t smem = size_t(nw) * ring_w;
     cudaFuncSetAttribute(k_trsm_ring<W, RS>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
     ++g_launches;
