@@ -173,7 +173,10 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
  *   CAGMRES_OPT_ARNOLDI  : width-1 Arnoldi passes (first Newton cycle, GMRES baseline): 0 = one
  *                          thread per row, register loads; 1 (default) = per-warp cp.async ring.
  *   CAGMRES_OPT_FUSE     : bit 0 (default 0) = BOrth pass 2 fused with the CholQR Gram;
- *                          bit 1 (default 1) = fused first-cycle Arnoldi passes.
+ *                          bit 1 (default 1) = fused first-cycle Arnoldi passes;
+ *                          bit 2 (default 1) = the normalisations q = w / ||w|| (restart vector,
+ *                          Arnoldi vectors) fused into the SpMV that consumes q (DIA SpMV variants;
+ *                          bitwise identical to the separate scaling pass).
  *   CAGMRES_OPT_WAVE_CHUNK / _WAVE_CTAS / _WAVE_LAG : temporal-blocking tuning (rows per
  *                          chunk, multiple of 256; resident CTAs per SM; wavefront lag in
  *                          chunks, 0 = automatic). */

@@ -42,7 +42,7 @@ __global__ void __launch_bounds__(NT) k_arnoldi_fused(ArnoldiArgs a) {
         if constexpr (MODE != 0) {
 #pragma unroll
             for (int i = 0; i < JX; ++i) v = fma(-q[i], sc[i], v);
-            if (jx > 0) a.v[r] = v;
+            if (jx > 0) (a.vout ? a.vout : a.v)[r] = v;
         }
         if constexpr (MODE != 2) {
 #pragma unroll
@@ -125,7 +125,7 @@ __global__ void __launch_bounds__(512, 1) k_arnoldi_ring(ArnoldiArgs a) {
 #pragma unroll
             for (int i = 0; i < JX; ++i)
                 if (i < jx) vv = fma(-sq[i * 32], sc[i], vv);
-            if (jx > 0) a.v[r] = vv;
+            if (jx > 0) (a.vout ? a.vout : a.v)[r] = vv;
         }
         if constexpr (MODE == 0 || MODE == 1) {
 #pragma unroll
@@ -217,7 +217,7 @@ bool ring_dispatch(const Dev& d, const ArnoldiArgs& a, cudaStream_t st) {
 int update_w1(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, double* p, const double* c,
               cudaStream_t st) {
     if (!d.arnoldi_ring || jx < 1 || jx > 32) return -1;
-    ArnoldiArgs a{d.panel_pf, n, X, ldx, jx, p, c, nullptr, nullptr, nullptr, nullptr, 0};
+    ArnoldiArgs a{d.panel_pf, n, X, ldx, jx, p, c, nullptr, nullptr, nullptr, nullptr, 0, nullptr};
     const bool ok = ring_dispatch<3>(d, a, st);
     return ok ? 0 : -1;
 }

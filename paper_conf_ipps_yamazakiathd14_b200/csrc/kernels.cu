@@ -159,6 +159,31 @@ void spmv(const Dev& d, const Sell& A, int64_t nrows, const double* x, double* y
         k_spmv_sell32<0><<<grid, NT, 0, st>>>(nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, nullptr, 0.0, nullptr, 0.0, y);
 }
 
+int spmv_scaled(const Dev& d, const Sell& A, int64_t nrows, const double* w, const double* wnrm, double* xs,
+                double* y, double bu, bool shift, cudaStream_t st) {
+    if (A.variant < 16) return -1;
+    if (nrows <= 0) return 0;
+    ++g_launches;
+    spmv_dia(d, A, A.variant, nrows, w, y, nullptr, bu, nullptr, 0.0, shift ? 5 : 4, st, wnrm, xs);
+    return 0;
+}
+
+__global__ void __launch_bounds__(256) k_scale_copy(int64_t n, const double* __restrict__ w,
+                                                    const double* __restrict__ wnrm, double* __restrict__ xs) {
+    pdl_wait();
+    pdl_trigger();
+    const double inv = 1.0 / __ldg(wnrm);                  // the product k_scale1 forms
+    for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x)
+        xs[i] = __ldg(w + i) * inv;
+}
+
+void scale_copy(int64_t n, const double* w, const double* wnrm, double* xs, cudaStream_t st) {
+    if (n <= 0) return;
+    const int64_t g = std::min<int64_t>((n + 255) / 256, 148 * 8);
+    ++g_launches;
+    launch_pdl(k_scale_copy, dim3(unsigned(g)), dim3(256), 0, st, n, w, wnrm, xs);
+}
+
 void residual(const Dev& d, const Sell& A, int64_t nrows, const double* x, const double* b,
               double* r, cudaStream_t st) {
     (void)d;

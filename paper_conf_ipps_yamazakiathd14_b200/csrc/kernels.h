@@ -69,15 +69,21 @@ struct Sell {
 // Loads of BATCH entries are issued before their FMAs; DIA offsets are loaded once per slice (lane
 // t holds offset t) and broadcast with shuffles, so no column index is loaded per entry.
 // SEL: load with selects (arrays always assigned) instead of guarded assignments; same FMAs.
-template <int BATCH, bool SEL = false>
+// SCALE: every x operand is multiplied by xscale after its load (the fused q = w / ||w|| of the
+// SX SpMV, spmv_dia.cu); otherwise xscale is ignored.
+template <int BATCH, bool SEL = false, bool SCALE = false>
 __device__ __forceinline__ double sell_slice_dot(int64_t r, int64_t b, int W, int64_t info, int myoff,
                                                  const int32_t* __restrict__ dcol, int64_t ncols,
                                                  const double* __restrict__ val,
-                                                 const double* __restrict__ x, bool coherent) {
+                                                 const double* __restrict__ x, bool coherent,
+                                                 double xscale = 1.0) {
     const int lane = int(r & 31);
     const int64_t dp = info >> 2;
     double acc = 0.0;
-    auto ldx = [&](const double* p) { return coherent ? __ldca(p) : __ldg(p); };
+    auto ldx = [&](const double* p) {
+        const double v = coherent ? __ldca(p) : __ldg(p);
+        return SCALE ? v * xscale : v;
+    };
     const double* vp = val + b + lane;              // entry t of this row: vp[32 t]
     if (info & 1) {
         if (!(info & 2)) {                          // no clamping: x address = x + r + offset
@@ -207,6 +213,7 @@ struct ArnoldiArgs {
     unsigned int* counter;
     int* status;
     int sqrt_out;
+    double* vout = nullptr;     // modes 1 / 2: write the updated v here instead of in place
 };
 int arnoldi_fused(const Dev& d, const ArnoldiArgs& a, int mode, cudaStream_t st);
 // p -= X c, p a single column (n), X n x jx (jx <= 32), c device jx-vector; -1 if not applicable
@@ -248,8 +255,18 @@ void spmv(const Dev& d, const Sell& A, int64_t nrows, const double* x, double* y
           const double* u, double bu, const double* w, double bw, cudaStream_t st);
 // DIA-width-specialised SpMV (spmv_dia.cu), CAGMRES_OPT_SPMV 16 / 17; mode as k_spmv_sell32
 // (3 = u - A x).
+// mode 4 / 5 = modes 0 / 1 with the fused normalisation (SX): x is an unnormalised w with
+// ||w|| = *xnrm (device), the operand is w * (1 / ||w||), and rows [0, nrows) of that normalised
+// vector are also stored to xs (u is ignored: the shift operand is the normalised x).
 void spmv_dia(const Dev& d, const Sell& A, int variant, int64_t nrows, const double* x, double* y,
-              const double* u, double bu, const double* w, double bw, int mode, cudaStream_t st);
+              const double* u, double bu, const double* w, double bw, int mode, cudaStream_t st,
+              const double* xnrm = nullptr, double* xs = nullptr);
+// y = A (w / ||w||) [- theta (w / ||w||)] and xs = w / ||w|| on rows [0, nrows) in one launch
+// (DIA variants 16 / 17 only; returns -1 otherwise and does nothing).
+int spmv_scaled(const Dev& d, const Sell& A, int64_t nrows, const double* w, const double* wnrm, double* xs,
+                double* y, double bu, bool shift, cudaStream_t st);
+// xs[0:n) = w[0:n) * (1 / *wnrm)   (the same product as k_scale1)
+void scale_copy(int64_t n, const double* w, const double* wnrm, double* xs, cudaStream_t st);
 // r[0:nrows) = b - A x
 void residual(const Dev& d, const Sell& A, int64_t nrows, const double* x, const double* b,
               double* r, cudaStream_t st);

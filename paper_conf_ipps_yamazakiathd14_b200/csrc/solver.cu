@@ -77,6 +77,15 @@ struct cagmres {
     std::vector<int64_t> nnz_prefix;       // nnz of stored rows with distance <= h (h <= s-1)
     double* V = nullptr;
     double* xe = nullptr;                  // ext scratch for the residual (distributed)
+    // Fused normalisation (CAGMRES_OPT_FUSE bit 2, default on): the residual r and each Arnoldi
+    // vector w are left unnormalised in S (ext length) with their norm on the device; the SpMV
+    // that consumes them forms q = w * (1/||w||) on the fly and stores q into V[:, pend_col]
+    // (kern::spmv_scaled) — bitwise the separate scaling pass, one launch and one vector pass less.
+    double* S = nullptr;
+    bool fuse_scale = true;
+    bool pend = false;                     // V[:, pend_col] = S / *pend_nrm still to be formed
+    const double* pend_nrm = nullptr;
+    int pend_col = 0;
     double* tab = nullptr; size_t tab_cap = 0;
     double* gbuf = nullptr;                // Gram / small scratch
     double* ybuf = nullptr;                // LS solution (m)
@@ -128,7 +137,7 @@ struct cagmres {
         cudaFree(d_done);
         for (int2* p : d_pairs) cudaFree(p);
         cudaFree(A.sptr); cudaFree(A.sinfo); cudaFree(A.dcol); cudaFree(A.val);
-        cudaFree(V); cudaFree(xe); cudaFree(tab); cudaFree(gbuf); cudaFree(ybuf); cudaFree(caqr_ws); cudaFree(op_M);
+        cudaFree(V); cudaFree(xe); cudaFree(S); cudaFree(tab); cudaFree(gbuf); cudaFree(ybuf); cudaFree(caqr_ws); cudaFree(op_M);
         cudaFreeHost(h_tab); cudaFreeHost(h_y); cudaFreeHost(h_beta); cudaFreeHost(h_stat);
         cudaFree(dg); cudaFreeHost(h_dg);
         if (ev_tab) cudaEventDestroy(ev_tab);
@@ -214,6 +223,8 @@ int common_alloc(cagmres* h) {
     const size_t vbytes = sizeof(double) * size_t(h->ldv) * size_t(h->m + 1);
     if (cudaMalloc(&h->V, vbytes) != cudaSuccess) return CAGMRES_ENOMEM;
     CU(cudaMemset(h->V, 0, vbytes));
+    if (cudaMalloc(&h->S, sizeof(double) * size_t(h->ldv)) != cudaSuccess) return CAGMRES_ENOMEM;
+    CU(cudaMemset(h->S, 0, sizeof(double) * size_t(h->ldv)));
     if (h->nranks > 1) {
         if (cudaMalloc(&h->xe, sizeof(double) * size_t(h->ldv)) != cudaSuccess) return CAGMRES_ENOMEM;
         CU(cudaMemset(h->xe, 0, sizeof(double) * size_t(h->ldv)));
@@ -521,10 +532,23 @@ double spmv_bytes(cagmres* h, int64_t rows_out, int depth_in, bool pair2) {
     return 12.0 * nnz + 4.0 * double(r + 1) + 8.0 * rin + 8.0 * double(r) + (pair2 ? 8.0 * double(r) : 0.0);
 }
 
+// Forms a pending normalised vector V[:, pend_col] = S / ||S|| (owned rows) for a consumer that
+// cannot fuse it (generic SpMV variants, the temporally blocked MPK, the unfused Arnoldi path).
+int materialize(cagmres* h) {
+    if (!h->pend) return CAGMRES_OK;
+    kern::scale_copy(h->n_loc, h->S, h->pend_nrm, h->V + size_t(h->ldv) * h->pend_col, h->stream);
+    h->pend = false;
+    h->bytes[PH_OTHER] += 16.0 * double(h->n_loc);
+    return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
+}
+
 // MPK of one block (Fig. 4): V[:, j+1 .. j+sb] from V[:, j].  Step k computes the rows at
 // distance <= sb-k (a prefix of the extended numbering) from the rows at distance <= sb-k+1.
 int mpk_block(cagmres* h, int j, int sb, const std::vector<host::Step>& steps) {
     Scope sc(h, PH_MPK);
+    const bool fused_q = h->pend && h->pend_col == j && h->A.variant >= 16 &&
+                         !(h->wave_on && h->nranks == 1 && sb >= 2 && wave_fits(h));
+    if (!fused_q) TRY(materialize(h));
     if (h->wave_on && h->nranks == 1 && sb >= 2 && wave_fits(h)) {
         TRY(wave_pairs(h, sb));
         kern::WaveArgs a{};
@@ -557,7 +581,7 @@ int mpk_block(cagmres* h, int j, int sb, const std::vector<host::Step>& steps) {
         h->spmv_launches++;
         return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
     }
-    TRY(halo(h, h->V + size_t(h->ldv) * j, sb));
+    TRY(halo(h, fused_q ? h->S : h->V + size_t(h->ldv) * j, sb));
     for (int k = 1; k <= sb; ++k) {
         const host::Step& stp = steps[size_t(k - 1)];
         const double* x = h->V + size_t(h->ldv) * (j + k - 1);
@@ -566,8 +590,15 @@ int mpk_block(cagmres* h, int j, int sb, const std::vector<host::Step>& steps) {
         const bool pair2 = stp.kind == 2;
         {
             Scope sv(h, PH_SPMV);
-            kern::spmv(h->dev, h->A, rows, x, y, (stp.a != 0.0 || pair2) ? x : nullptr, -stp.a,
-                       pair2 ? h->V + size_t(h->ldv) * (j + k - 2) : nullptr, stp.b2, h->stream);
+            if (k == 1 && fused_q) {       // q_j = S / ||S|| formed inside the first step (stored to V[:, j])
+                if (kern::spmv_scaled(h->dev, h->A, rows, h->S, h->pend_nrm, h->V + size_t(h->ldv) * j, y, -stp.a,
+                                      stp.a != 0.0, h->stream))
+                    return CAGMRES_EINVAL;
+                h->pend = false;
+            } else {
+                kern::spmv(h->dev, h->A, rows, x, y, (stp.a != 0.0 || pair2) ? x : nullptr, -stp.a,
+                           pair2 ? h->V + size_t(h->ldv) * (j + k - 2) : nullptr, stp.b2, h->stream);
+            }
         }
         const double by = spmv_bytes(h, rows, sb - k + 1, pair2);
         h->bytes[PH_MPK] += by;
@@ -816,9 +847,17 @@ int arnoldi_cycle(cagmres* h, bool cgs2) {
         double* r = c2 + (m + 1);
         {
             Scope sc(h, PH_MPK);
-            TRY(halo(h, vk, 1));
+            const bool fused_q = h->pend && h->pend_col == k && h->A.variant >= 16;
+            if (!fused_q) TRY(materialize(h));
+            TRY(halo(h, fused_q ? h->S : vk, 1));
             Scope sv(h, PH_SPMV);
-            kern::spmv(h->dev, h->A, h->n_loc, vk, v, nullptr, 0.0, nullptr, 0.0, h->stream);
+            if (fused_q) {                 // v_k = S / ||S|| formed inside the SpMV (stored to V[:, k])
+                if (kern::spmv_scaled(h->dev, h->A, h->n_loc, h->S, h->pend_nrm, vk, v, 0.0, false, h->stream))
+                    return CAGMRES_EINVAL;
+                h->pend = false;
+            } else {
+                kern::spmv(h->dev, h->A, h->n_loc, vk, v, nullptr, 0.0, nullptr, 0.0, h->stream);
+            }
             const double by = spmv_bytes(h, h->n_loc, 1, false);
             h->bytes[PH_MPK] += by; h->bytes[PH_SPMV] += by; h->spmv_launches++;
         }
@@ -844,13 +883,20 @@ int arnoldi_cycle(cagmres* h, bool cgs2) {
             {
                 Scope sc(h, PH_TSQR);
                 aa.c_in = cgs2 ? c2 : c1; aa.c_out = r;
+                aa.vout = h->fuse_scale ? h->S : nullptr;          // w -> S, normalised by the next SpMV
                 if (kern::arnoldi_fused(h->dev, aa, 2, h->stream)) return CAGMRES_EINVAL;
+                aa.vout = nullptr;
                 if (h->nranks > 1) {
                     TRY(allreduce(h, r, 1));
                     kern::chol(r, 1, r, h->status, h->stream);     // r = sqrt(r)
                 }
-                kern::trsm(h->dev, h->n_loc, v, h->ldv, 1, r, 0, h->stream);
-                h->bytes[PH_TSQR] += 8.0 * nl * ((k + 1) + 2.0 + 2.0);
+                if (h->fuse_scale) {
+                    h->pend = true; h->pend_nrm = r; h->pend_col = k + 1;
+                    h->bytes[PH_TSQR] += 8.0 * nl * ((k + 1) + 2.0);
+                } else {
+                    kern::trsm(h->dev, h->n_loc, v, h->ldv, 1, r, 0, h->stream);
+                    h->bytes[PH_TSQR] += 8.0 * nl * ((k + 1) + 2.0 + 2.0);
+                }
             }
             continue;
         }
@@ -858,6 +904,7 @@ int arnoldi_cycle(cagmres* h, bool cgs2) {
         if (cgs2) TRY(borth_panel(h, h->V, h->ldv, k + 1, v, h->ldv, 1, c2, false));
         TRY(tsqr_panel(h, v, h->ldv, 1, r, CAGMRES_CHOLQR, 0));
     }
+    h->pend = false;                       // V[:, m] (unnormalised, in S) is never read
     return CAGMRES_OK;
 }
 
@@ -872,10 +919,11 @@ int residual_norm_async(cagmres* h, const double* b, const double* x) {
         TRY(halo(h, h->xe, 1));
         xx = h->xe;
     }
-    kern::residual(h->dev, h->A, h->n_loc, xx, b, h->V, h->stream);
+    double* rv = h->fuse_scale ? h->S : h->V;          // r: unnormalised in S (fused) or in V[:, 0]
+    kern::residual(h->dev, h->A, h->n_loc, xx, b, rv, h->stream);
     double* rr = h->gbuf + 8;
     {   // ||r|| by the scalar reduction kernel (mode 2 with no Q columns)
-        kern::ArnoldiArgs aa{h->dev.panel_pf, h->n_loc, h->V, h->ldv, 0, h->V, nullptr, rr, h->arn_part, h->arn_counter,
+        kern::ArnoldiArgs aa{h->dev.panel_pf, h->n_loc, h->V, h->ldv, 0, rv, nullptr, rr, h->arn_part, h->arn_counter,
                              h->status, h->nranks == 1 ? 1 : 0};
         if (kern::arnoldi_fused(h->dev, aa, 2, h->stream)) return CAGMRES_EINVAL;
         if (h->nranks > 1) {
@@ -885,8 +933,13 @@ int residual_norm_async(cagmres* h, const double* b, const double* x) {
     }
     CU(cudaMemcpyAsync(h->h_beta, rr, sizeof(double), cudaMemcpyDeviceToHost, h->stream));
     CU(cudaEventRecord(h->ev_beta, h->stream));
-    kern::trsm(h->dev, h->n_loc, h->V, h->ldv, 1, rr, 0, h->stream);     // q_0 = r / beta
-    h->bytes[PH_OTHER] += spmv_bytes(h, h->n_loc, 1, false) + 8.0 * double(h->n_loc) * 3.0;
+    if (h->fuse_scale) {                                   // q_0 = r / beta formed by the next SpMV
+        h->pend = true; h->pend_nrm = rr; h->pend_col = 0;
+        h->bytes[PH_OTHER] += spmv_bytes(h, h->n_loc, 1, false) + 8.0 * double(h->n_loc);
+    } else {
+        kern::trsm(h->dev, h->n_loc, h->V, h->ldv, 1, rr, 0, h->stream);     // q_0 = r / beta
+        h->bytes[PH_OTHER] += spmv_bytes(h, h->n_loc, 1, false) + 8.0 * double(h->n_loc) * 3.0;
+    }
     return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
 }
 
@@ -1023,7 +1076,9 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
         case CAGMRES_OPT_TRSM: if (value < 0 || value > 4) return CAGMRES_EINVAL; h->dev.trsm_scalar = int(value); return CAGMRES_OK;
         case CAGMRES_OPT_PDL: if (value < 0 || value > 1) return CAGMRES_EINVAL; kern::g_pdl = int(value); return CAGMRES_OK;
         case CAGMRES_OPT_PANEL_PF: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->dev.panel_pf = int(value); return CAGMRES_OK;
-        case CAGMRES_OPT_FUSE: h->fuse_borth_gram = (value & 1) != 0; h->arnoldi_fuse = (value & 2) != 0; return CAGMRES_OK;
+        case CAGMRES_OPT_FUSE:
+            h->fuse_borth_gram = (value & 1) != 0; h->arnoldi_fuse = (value & 2) != 0; h->fuse_scale = (value & 4) != 0;
+            return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK:
             if (value < 256 || value % 256) return CAGMRES_EINVAL;
             h->wave_CH = int(value); wave_reset_pairs(h); return CAGMRES_OK;
@@ -1044,7 +1099,9 @@ int cagmres_get_option(cagmres_t h, int opt, int64_t* value) {
         case CAGMRES_OPT_TRSM: *value = h->dev.trsm_scalar; return CAGMRES_OK;
         case CAGMRES_OPT_PDL: *value = kern::g_pdl; return CAGMRES_OK;
         case CAGMRES_OPT_PANEL_PF: *value = h->dev.panel_pf; return CAGMRES_OK;
-        case CAGMRES_OPT_FUSE: *value = (h->fuse_borth_gram ? 1 : 0) | (h->arnoldi_fuse ? 2 : 0); return CAGMRES_OK;
+        case CAGMRES_OPT_FUSE:
+            *value = (h->fuse_borth_gram ? 1 : 0) | (h->arnoldi_fuse ? 2 : 0) | (h->fuse_scale ? 4 : 0);
+            return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK: *value = h->wave_CH; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CTAS: *value = h->wave_ctas; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_LAG: *value = h->wave_lag; return CAGMRES_OK;
@@ -1089,6 +1146,7 @@ int cagmres_get_shifts(cagmres_t h, double* re, double* im, int cap, int* count)
 int cagmres_mpk(cagmres_t h, const double* q, double* W, int64_t ldw, int sb) {
     if (!h || !q || !W || sb < 1 || sb > h->s || ldw < h->n_loc || sb > h->m) return CAGMRES_EINVAL;
     if (h->basis == CAGMRES_NEWTON && !h->have_shifts) return CAGMRES_EINVAL;
+    h->pend = false;
     CU(cudaMemcpyAsync(h->V, q, sizeof(double) * size_t(h->n_loc), cudaMemcpyDeviceToDevice, h->stream));
     const std::vector<host::Step> steps = h->basis != CAGMRES_NEWTON
         ? host::block_steps({}, {}, sb) : host::block_steps(h->sh_re, h->sh_im, sb);

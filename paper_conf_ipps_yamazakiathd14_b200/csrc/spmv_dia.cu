@@ -32,6 +32,8 @@ struct DiaArgs {
     const double* u; double bu;
     const double* w; double bw;
     double* y;
+    const double* xnrm;     // SX: x is an unnormalised w, the operand is w * (1 / *xnrm)
+    double* xs;             // SX: the normalised operand's rows [0, nrows) are stored here
 };
 }  // namespace
 
@@ -50,7 +52,12 @@ __device__ __forceinline__ void prefetch_l2(const void* p) {
 // registers) are prefetched into L2, so next iteration's value loads are L2 hits: one more
 // slice of HBM requests in flight per warp without holding registers.  Slices are grid-strided
 // over all warps of the persistent grid.
-template <int MODE, int WT, int MINB>   // MODE 0: Ax  1: + bu u  2: + bw w  3: u - Ax
+// SX (fused normalisation, MODE 0 / 1 only): the input vector is w with ||w|| = *xnrm on the
+// device (the Arnoldi / residual norm just computed); every x operand is w[c] * (1 / ||w||) —
+// exactly the product the separate scaling kernel k_scale1 forms — and each thread also stores
+// its row of the normalised vector to xs.  So the q = w / ||w|| pass (a read and a write of the
+// vector, one launch) disappears and the results are bitwise those of scale-then-SpMV.
+template <int MODE, int WT, int MINB, bool SX = false>   // MODE 0: Ax  1: + bu u  2: + bw w  3: u - Ax
 __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
     const int lane = threadIdx.x & 31;
     const int64_t nsl = (a.nrows + 31) >> 5;
@@ -65,6 +72,7 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
     o0 = sell_slice_off(lane, W0, i0, a.dcol);
     pdl_wait();
     pdl_trigger();
+    const double inv = SX ? 1.0 / __ldg(a.xnrm) : 1.0;
 #pragma unroll 1
     for (; sl < nsl; sl += stride) {
         b2 = 0; W2 = 0; i2 = 1;
@@ -74,10 +82,14 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
         const int64_t r = sl * 32 + lane;
         const bool live = r < a.nrows;
         double uu = 0.0, ww = 0.0, acc = 0.0;
+        if (SX && live) {                                               // own row of q = w / ||w||
+            uu = __ldg(a.x + r) * inv;
+            a.xs[r] = uu;
+        }
         if (W0 == WT && (i0 & 3) == 1) {
             const double* vp = a.val + b0 + lane;
             const double* xr = a.x + r;
-            if (MODE >= 1 && live) uu = __ldg(a.u + r);
+            if (!SX && MODE >= 1 && live) uu = __ldg(a.u + r);
             if (MODE == 2 && live) ww = __ldg(a.w + r);
             // 27-point rows: three groups of 9 value / x pairs in flight (all 27 at once spilled
             // 480 B of stack at the 64-register cap); the FMA order t = 0..WT-1 is unchanged
@@ -92,12 +104,16 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
                     v[t] = ldg_stream(vp + 32 * (g0 + t));
                     xv[t] = __ldg(xr + o);
                 }
+                if (SX) {
+#pragma unroll
+                    for (int t = 0; t < GT; ++t) xv[t] *= inv;
+                }
 #pragma unroll
                 for (int t = 0; t < GT; ++t) acc = fma(v[t], xv[t], acc);
             }
         } else {
-            acc = sell_slice_dot<4, true>(r, b0, W0, i0, o0, a.dcol, a.ncols, a.val, a.x, false);
-            if (MODE >= 1 && live) uu = __ldg(a.u + r);
+            acc = sell_slice_dot<4, true, SX>(r, b0, W0, i0, o0, a.dcol, a.ncols, a.val, a.x, false, inv);
+            if (!SX && MODE >= 1 && live) uu = __ldg(a.u + r);
             if (MODE == 2 && live) ww = __ldg(a.w + r);
         }
         if (live) {
@@ -117,18 +133,18 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
 }
 
 namespace {
-template <int MODE, int WT, int MINB>
+template <int MODE, int WT, int MINB, bool SX = false>
 void go_dia(const Dev& d, const DiaArgs& a, cudaStream_t st) {
     static int occ = 0;
     if (occ == 0) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_spmv_dia<MODE, WT, MINB>, DT_NT, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_spmv_dia<MODE, WT, MINB, SX>, DT_NT, 0);
         if (occ < 1) occ = 1;
     }
     const int64_t nsl = (a.nrows + 31) >> 5;
     int64_t g = int64_t(d.sms) * occ;
     const int64_t need = (nsl + DT_NT / 32 - 1) / (DT_NT / 32);
     if (g > need) g = need;
-    launch_pdl(k_spmv_dia<MODE, WT, MINB>, dim3(unsigned(g)), dim3(DT_NT), 0, st, a);
+    launch_pdl(k_spmv_dia<MODE, WT, MINB, SX>, dim3(unsigned(g)), dim3(DT_NT), 0, st, a);
 }
 
 template <int WT, int MINB>
@@ -137,6 +153,8 @@ void go_modes(const Dev& d, const DiaArgs& a, cudaStream_t st, int mode) {
         case 0: go_dia<0, WT, MINB>(d, a, st); break;
         case 1: go_dia<1, WT, MINB>(d, a, st); break;
         case 2: go_dia<2, WT, MINB>(d, a, st); break;
+        case 4: go_dia<0, WT, MINB, true>(d, a, st); break;      // 4 / 5: modes 0 / 1 with SX
+        case 5: go_dia<1, WT, MINB, true>(d, a, st); break;
         default: go_dia<3, WT, MINB>(d, a, st); break;
     }
 }
@@ -156,8 +174,9 @@ void go_width(const Dev& d, const DiaArgs& a, int wt, cudaStream_t st, int mode)
 // CTA-contiguous slice ranges, a two-slice-deep prefetch — and round 2's L2 evict-first hints
 // and TMA-streamed value rings measured slower: DESIGN.md §6.)
 void spmv_dia(const Dev& d, const Sell& A, int variant, int64_t nrows, const double* x, double* y,
-              const double* u, double bu, const double* w, double bw, int mode, cudaStream_t st) {
-    DiaArgs a{nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, u, bu, w, bw, y};
+              const double* u, double bu, const double* w, double bw, int mode, cudaStream_t st,
+              const double* xnrm, double* xs) {
+    DiaArgs a{nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, u, bu, w, bw, y, xnrm, xs};
     if (variant == 17) go_width<5>(d, a, A.dia_w, st, mode);
     else go_width<4>(d, a, A.dia_w, st, mode);
 }

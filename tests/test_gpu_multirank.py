@@ -252,6 +252,27 @@ def test_group_solve_injected_shifts_reorth_and_gmres(P):
     assert np.allclose(sg.hist, g["hist"][:len(sg.hist)], rtol=1e-6)
 
 
+def test_group_solve_fused_normalisation_halo_on_S():
+    """The fused normalisation across ranks: the halo exchanges the unnormalised vector S and
+    every rank forms q = S / ||S|| (global norm) inside its SpMV; both settings give the same
+    bits (P = 3, 3-D 40^3, s = 10, m = 30)."""
+    _, Solver = _mods()
+    A = G.convection_diffusion(40, 3, 7)
+    b = G.rhs(A.n)
+    rs = O.block_rows(A.n, 3)
+    res = {}
+    for f in (6, 2):
+        def rank(r, grp, f=f):
+            S = Solver(A, s=10, m=30, basis="newton", group=grp, row_starts=rs, rank=r)
+            S.set_option("fuse", f)
+            x, st = S.solve(dev(b[rs[r]:rs[r + 1]]), tol=1e-8, maxit=60)
+            S.close()
+            return x.cpu(), st
+        res[f] = run_ranks(3, rank)
+    for (xa, sa), (xb, sb) in zip(res[6], res[2]):
+        assert np.array_equal(sa.hist, sb.hist) and torch.equal(xa, xb)
+
+
 def test_group_single_rank_is_the_single_gpu_handle():
     """P = 1 through the group API: bitwise the single-GPU solve."""
     _, Solver = _mods()

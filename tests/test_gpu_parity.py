@@ -457,6 +457,24 @@ def test_onepass_cycle_basis_matches_two_pass():
     assert np.allclose(out[0], out[1], rtol=1e-8)
 
 
+@pytest.mark.parametrize("gen,basis", [("C1", "newton"), ("cd7_40", "newton"), ("cd7_40", "gmres"),
+                                       ("cd27_ragged", "monomial")])
+def test_fused_normalisation_is_bitwise_the_separate_scaling(gen, basis):
+    """CAGMRES_OPT_FUSE bit 2: q = w / ||w|| formed inside the consuming SpMV (restart vector and
+    Arnoldi vectors) gives bit-for-bit the histories and solution of the separate scaling pass."""
+    A = {"C1": lambda: G.convection_diffusion(32, 2, 5), "cd7_40": lambda: G.convection_diffusion(40, 3, 7),
+         "cd27_ragged": lambda: G.convection_diffusion(13, 3, 27)}[gen]()
+    b = dev(G.rhs(A.n))
+    out = []
+    for fuse in (6, 2):
+        S = Solver(A, s=5 if basis != "gmres" else 1, m=30, basis=basis)
+        S.set_option("fuse", fuse)
+        assert S.get_option("fuse") == fuse
+        x, st = S.solve(b, tol=1e-10, maxit=60)
+        out.append((x, st))
+    assert np.array_equal(out[0][1].hist, out[1][1].hist) and torch.equal(out[0][0], out[1][0])
+
+
 def test_clear_shifts_reruns_first_cycle_bitwise():
     """set_shifts(count = 0): the next Newton solve runs its own GMRES shift cycle again
     and, the reductions being deterministic, reproduces the first solve bit for bit."""
