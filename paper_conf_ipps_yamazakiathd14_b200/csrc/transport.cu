@@ -84,6 +84,10 @@ struct GroupTransport final : Transport {
     cagmres_group* g = nullptr;
     int r = 0;
     ~GroupTransport() override {
+        // destroy is collective: after the last collective's second barrier a peer may still be
+        // enqueueing its waits on our `done` event — no rank destroys its events before every
+        // rank has returned from that collective and reached its own destroy
+        if (!g->aborted) g->barrier();
         cagmres_group::Post& me = g->post[size_t(r)];
         if (me.ready) cudaEventDestroy(me.ready);
         if (me.done) cudaEventDestroy(me.done);

@@ -156,7 +156,7 @@ def test_spmv_variants_bitwise(gen):
     S = Solver(A, s=6, m=30, basis="newton")
     S.set_shifts(*SHIFTS)
     Ws = []
-    variants = [0, 5, 16, 17]
+    variants = [0, 5, 16, 17, 18, 19]
     for v in variants:
         S.set_option("spmv", v)
         Ws.append(S.mpk(q, 6))
