@@ -166,9 +166,7 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
  *                          grid, slice descriptors software-pipelined two slices ahead; 16, 17 = the
  *                          persistent kernel with a fully unrolled body for the matrix's most common
  *                          DIA slice width and an L2 prefetch of the next slice's values, >= 4 / 5
- *                          CTAs per SM; 18, 19 = the same body on two slices per warp iteration
- *                          (DIA widths <= 9), >= 2 / 3 CTAs per SM.  All variants are bitwise
- *                          identical.  Other values: EINVAL.
+ *                          CTAs per SM.  All variants are bitwise identical.  Other values: EINVAL.
  *   CAGMRES_OPT_GRAM     : CholQR Gram kernel: 0 = FP64 tensor core (DMMA m8n8k4) on a per-warp
  *                          cp.async ring; 1 (default) = scalar DFMA on a deeper ring (w <= 12,
  *                          else the DMMA kernel).

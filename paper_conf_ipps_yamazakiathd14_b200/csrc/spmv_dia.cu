@@ -133,143 +133,6 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
 }
 
 namespace {
-// Two slices per warp per iteration (variants 18, 19: >= 2 / 3 CTAs per SM; DIA widths <= 9): the slice body is
-// latency-bound (descriptor -> offset -> value / x loads -> FMAs -> store, ~2 us per slice per
-// warp at 32 warps per SM), so here each warp issues the value and x loads of slices sl and
-// sl + stride together before the FMAs of either: twice the loads in flight per warp for the
-// same occupancy.  Per row the FMA order and epilogue are those of k_spmv_dia: bitwise identical.
-template <int MODE, int WT, int MINB, bool SX = false>
-__global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia2(DiaArgs a) {
-    static_assert(WT <= 9, "two-slice body for narrow DIA widths");
-    const int lane = threadIdx.x & 31;
-    const int64_t nsl = (a.nrows + 31) >> 5;
-    const int64_t stride = int64_t(gridDim.x) * (DT_NT / 32);
-    int64_t sl = (int64_t(blockIdx.x) * DT_NT + threadIdx.x) >> 5;
-    if (sl >= nsl) { pdl_wait(); pdl_trigger(); return; }
-    int64_t b[2], in[2], bn[2], inn[2];
-    int W[2], o[2], Wn[2];
-    auto meta = [&](int64_t s, int64_t& bb, int& ww, int64_t& ii) {
-        if (s < nsl) sell_slice_meta(s, a.sptr, a.sinfo, bb, ww, ii);
-        else { bb = 0; ww = 0; ii = 1; }
-    };
-#pragma unroll
-    for (int u = 0; u < 2; ++u) {
-        meta(sl + u * stride, b[u], W[u], in[u]);
-        o[u] = sell_slice_off(lane, W[u], in[u], a.dcol);
-        meta(sl + (2 + u) * stride, bn[u], Wn[u], inn[u]);
-    }
-    pdl_wait();
-    pdl_trigger();
-    const double inv = SX ? 1.0 / __ldg(a.xnrm) : 1.0;
-#pragma unroll 1
-    for (; sl < nsl; sl += 2 * stride) {
-        int on[2];
-#pragma unroll
-        for (int u = 0; u < 2; ++u) {
-            on[u] = sell_slice_off(lane, Wn[u], inn[u], a.dcol);
-            if (lane < 2 * Wn[u]) prefetch_l2(a.val + bn[u] + 16 * lane);   // 128-B lines of the next pair
-        }
-        int64_t bnn[2], innn[2];
-        int Wnn[2];
-#pragma unroll
-        for (int u = 0; u < 2; ++u) meta(sl + (4 + u) * stride, bnn[u], Wnn[u], innn[u]);
-        int64_t r[2];
-        bool live[2];
-        double uu[2] = {0.0, 0.0}, ww[2] = {0.0, 0.0}, acc[2] = {0.0, 0.0};
-#pragma unroll
-        for (int u = 0; u < 2; ++u) {
-            r[u] = (sl + u * stride) * 32 + lane;
-            live[u] = sl + u * stride < nsl && r[u] < a.nrows;
-            if (SX && live[u]) {
-                uu[u] = __ldg(a.x + r[u]) * inv;
-                a.xs[r[u]] = uu[u];
-            }
-        }
-        const bool fast0 = W[0] == WT && (in[0] & 3) == 1;
-        const bool fast1 = (W[1] == WT && (in[1] & 3) == 1) || sl + stride >= nsl;
-        if (fast0 && fast1) {
-            const bool has1 = sl + stride < nsl;
-            double v[2][WT], xv[2][WT];
-#pragma unroll
-            for (int u = 0; u < 2; ++u) {
-                if (u == 1 && !has1) break;
-                const double* vp = a.val + b[u] + lane;
-                const double* xr = a.x + r[u];
-#pragma unroll
-                for (int t = 0; t < WT; ++t) {
-                    const int off = __shfl_sync(0xffffffffu, o[u], t);
-                    v[u][t] = ldg_stream(vp + 32 * t);
-                    xv[u][t] = __ldg(xr + off);
-                }
-                if (!SX && MODE >= 1 && live[u]) uu[u] = __ldg(a.u + r[u]);
-                if (MODE == 2 && live[u]) ww[u] = __ldg(a.w + r[u]);
-            }
-#pragma unroll
-            for (int u = 0; u < 2; ++u) {
-                if (u == 1 && !has1) break;
-#pragma unroll
-                for (int t = 0; t < WT; ++t) {
-                    const double xx = SX ? xv[u][t] * inv : xv[u][t];
-                    acc[u] = fma(v[u][t], xx, acc[u]);
-                }
-            }
-        } else {
-#pragma unroll
-            for (int u = 0; u < 2; ++u) {
-                if (sl + u * stride >= nsl) break;
-                if (W[u] == WT && (in[u] & 3) == 1) {
-                    const double* vp = a.val + b[u] + lane;
-                    const double* xr = a.x + r[u];
-#pragma unroll
-                    for (int t = 0; t < WT; ++t) {
-                        const int off = __shfl_sync(0xffffffffu, o[u], t);
-                        const double xx = SX ? __ldg(xr + off) * inv : __ldg(xr + off);
-                        acc[u] = fma(ldg_stream(vp + 32 * t), xx, acc[u]);
-                    }
-                } else {
-                    acc[u] = sell_slice_dot<4, true, SX>(r[u], b[u], W[u], in[u], o[u], a.dcol, a.ncols, a.val, a.x,
-                                                         false, inv);
-                }
-                if (!SX && MODE >= 1 && live[u]) uu[u] = __ldg(a.u + r[u]);
-                if (MODE == 2 && live[u]) ww[u] = __ldg(a.w + r[u]);
-            }
-        }
-#pragma unroll
-        for (int u = 0; u < 2; ++u) {
-            if (!live[u]) continue;
-            double out;
-            if constexpr (MODE == 3) {
-                out = uu[u] - acc[u];
-            } else {
-                out = acc[u];
-                if constexpr (MODE >= 1) out = fma(a.bu, uu[u], out);
-                if constexpr (MODE >= 2) out = fma(a.bw, ww[u], out);
-            }
-            a.y[r[u]] = out;
-        }
-#pragma unroll
-        for (int u = 0; u < 2; ++u) {
-            b[u] = bn[u]; W[u] = Wn[u]; in[u] = inn[u]; o[u] = on[u];
-            bn[u] = bnn[u]; Wn[u] = Wnn[u]; inn[u] = innn[u];
-        }
-    }
-}
-
-template <int MODE, int WT, int MINB, bool SX = false>
-void go_dia2(const Dev& d, const DiaArgs& a, cudaStream_t st) {
-    static int occ = 0;
-    if (occ == 0) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_spmv_dia2<MODE, WT, MINB, SX>, DT_NT, 0);
-        if (occ < 1) occ = 1;
-    }
-    const int64_t nsl = (a.nrows + 31) >> 5;
-    int64_t g = int64_t(d.sms) * occ;
-    const int64_t need = (nsl + 2 * (DT_NT / 32) - 1) / (2 * (DT_NT / 32));
-    if (g > need) g = need;
-    if (g < 1) g = 1;
-    launch_pdl(k_spmv_dia2<MODE, WT, MINB, SX>, dim3(unsigned(g)), dim3(DT_NT), 0, st, a);
-}
-
 template <int MODE, int WT, int MINB, bool SX = false>
 void go_dia(const Dev& d, const DiaArgs& a, cudaStream_t st) {
     static int occ = 0;
@@ -296,18 +159,6 @@ void go_modes(const Dev& d, const DiaArgs& a, cudaStream_t st, int mode) {
     }
 }
 
-template <int WT, int MINB>
-void go_modes2(const Dev& d, const DiaArgs& a, cudaStream_t st, int mode) {
-    switch (mode) {
-        case 0: go_dia2<0, WT, MINB>(d, a, st); break;
-        case 1: go_dia2<1, WT, MINB>(d, a, st); break;
-        case 2: go_dia2<2, WT, MINB>(d, a, st); break;
-        case 4: go_dia2<0, WT, MINB, true>(d, a, st); break;
-        case 5: go_dia2<1, WT, MINB, true>(d, a, st); break;
-        default: go_dia2<3, WT, MINB>(d, a, st); break;
-    }
-}
-
 template <int MINB>
 void go_width(const Dev& d, const DiaArgs& a, int wt, cudaStream_t st, int mode) {
     switch (wt) {
@@ -326,17 +177,6 @@ void spmv_dia(const Dev& d, const Sell& A, int variant, int64_t nrows, const dou
               const double* u, double bu, const double* w, double bw, int mode, cudaStream_t st,
               const double* xnrm, double* xs) {
     DiaArgs a{nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, u, bu, w, bw, y, xnrm, xs};
-    if (variant == 18 || variant == 19) {                   // two slices per warp (widths 5, 7)
-        if (A.dia_w == 5) {
-            if (variant == 18) go_modes2<5, 2>(d, a, st, mode); else go_modes2<5, 3>(d, a, st, mode);
-            return;
-        }
-        if (A.dia_w != 27) {
-            if (variant == 18) go_modes2<7, 2>(d, a, st, mode); else go_modes2<7, 3>(d, a, st, mode);
-            return;
-        }
-        variant = 16;                                        // 27-wide rows: the one-slice body
-    }
     if (variant == 17) go_width<5>(d, a, A.dia_w, st, mode);
     else go_width<4>(d, a, A.dia_w, st, mode);
 }

@@ -273,6 +273,28 @@ def test_group_solve_fused_normalisation_halo_on_S():
         assert np.array_equal(sa.hist, sb.hist) and torch.equal(xa, xb)
 
 
+@pytest.mark.parametrize("P", [3, 8])
+def test_group_solve_bitwise_independent_of_per_rank_spmv_variant(P):
+    """Every SpMV variant sums each row identically, so a distributed solve whose ranks use
+    DIFFERENT variants (fused normalisation on some, separate scaling on others) gives the
+    same bits as one where all ranks use the default."""
+    _, Solver = _mods()
+    A = G.g3_shaped(n=40000, width=200)
+    b = G.rhs(A.n)
+    rs = O.block_rows(A.n, P)
+    res = {}
+    for mix in (False, True):
+        def rank(r, grp, mix=mix):
+            S = Solver(A, s=5, m=60, basis="newton", group=grp, row_starts=rs, rank=r)
+            S.set_option("spmv", (16, 0, 17, 5)[r % 4] if mix else 16)
+            x, st = S.solve(dev(b[rs[r]:rs[r + 1]]), tol=1e-8, maxit=200)
+            S.close()
+            return x.cpu(), st
+        res[mix] = run_ranks(P, rank)
+    for (xa, sa), (xb, sb) in zip(res[False], res[True]):
+        assert np.array_equal(sa.hist, sb.hist) and torch.equal(xa, xb)
+
+
 def test_group_single_rank_is_the_single_gpu_handle():
     """P = 1 through the group API: bitwise the single-GPU solve."""
     _, Solver = _mods()
