@@ -532,24 +532,38 @@ double spmv_bytes(cagmres* h, int64_t rows_out, int depth_in, bool pair2) {
     return 12.0 * nnz + 4.0 * double(r + 1) + 8.0 * rin + 8.0 * double(r) + (pair2 ? 8.0 * double(r) : 0.0);
 }
 
-// Forms a pending normalised vector V[:, pend_col] = S / ||S|| (owned rows) for a consumer that
-// cannot fuse it (generic SpMV variants, the temporally blocked MPK, the unfused Arnoldi path).
-int materialize(cagmres* h) {
+// Forms a pending normalised vector V[:, pend_col] = S / ||S|| on its first `rows` extended rows
+// for a consumer that cannot fuse it (generic SpMV variants, the temporally blocked MPK).
+int materialize(cagmres* h, int64_t rows) {
     if (!h->pend) return CAGMRES_OK;
-    kern::scale_copy(h->n_loc, h->S, h->pend_nrm, h->V + size_t(h->ldv) * h->pend_col, h->stream);
+    kern::scale_copy(rows, h->S, h->pend_nrm, h->V + size_t(h->ldv) * h->pend_col, h->stream);
     h->pend = false;
-    h->bytes[PH_OTHER] += 16.0 * double(h->n_loc);
+    h->bytes[PH_OTHER] += 16.0 * double(rows);
     return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
+}
+
+// Halo of the start vector of an SpMV chain at column col, depth `depth`.  With a pending
+// normalisation the UNNORMALISED S is exchanged on every rank (the pending state is the same on
+// all ranks; the SpMV variant — fused or not — may differ per rank, so the exchanged
+// representation must not depend on it); a rank that cannot fuse then forms V[:, col] = S/||S||
+// on its owned AND ghost rows.  Returns true when the caller's first SpMV must fuse (read S).
+int start_halo(cagmres* h, int col, int depth, bool& fuse) {
+    fuse = false;
+    if (!(h->pend && h->pend_col == col)) {
+        TRY(materialize(h, h->n_loc));
+        return halo(h, h->V + size_t(h->ldv) * col, depth);
+    }
+    TRY(halo(h, h->S, depth));
+    if (h->A.variant >= 16) { fuse = true; return CAGMRES_OK; }
+    return materialize(h, h->level_len[size_t(std::min(depth, h->s))]);
 }
 
 // MPK of one block (Fig. 4): V[:, j+1 .. j+sb] from V[:, j].  Step k computes the rows at
 // distance <= sb-k (a prefix of the extended numbering) from the rows at distance <= sb-k+1.
 int mpk_block(cagmres* h, int j, int sb, const std::vector<host::Step>& steps) {
     Scope sc(h, PH_MPK);
-    const bool fused_q = h->pend && h->pend_col == j && h->A.variant >= 16 &&
-                         !(h->wave_on && h->nranks == 1 && sb >= 2 && wave_fits(h));
-    if (!fused_q) TRY(materialize(h));
     if (h->wave_on && h->nranks == 1 && sb >= 2 && wave_fits(h)) {
+        TRY(materialize(h, h->n_loc));
         TRY(wave_pairs(h, sb));
         kern::WaveArgs a{};
         a.sptr = h->A.sptr; a.sinfo = h->A.sinfo; a.dcol = h->A.dcol; a.val = h->A.val; a.ncols = h->A.ncols;
@@ -581,7 +595,8 @@ int mpk_block(cagmres* h, int j, int sb, const std::vector<host::Step>& steps) {
         h->spmv_launches++;
         return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
     }
-    TRY(halo(h, fused_q ? h->S : h->V + size_t(h->ldv) * j, sb));
+    bool fused_q = false;
+    TRY(start_halo(h, j, sb, fused_q));
     for (int k = 1; k <= sb; ++k) {
         const host::Step& stp = steps[size_t(k - 1)];
         const double* x = h->V + size_t(h->ldv) * (j + k - 1);
@@ -847,9 +862,8 @@ int arnoldi_cycle(cagmres* h, bool cgs2) {
         double* r = c2 + (m + 1);
         {
             Scope sc(h, PH_MPK);
-            const bool fused_q = h->pend && h->pend_col == k && h->A.variant >= 16;
-            if (!fused_q) TRY(materialize(h));
-            TRY(halo(h, fused_q ? h->S : vk, 1));
+            bool fused_q = false;
+            TRY(start_halo(h, k, 1, fused_q));
             Scope sv(h, PH_SPMV);
             if (fused_q) {                 // v_k = S / ||S|| formed inside the SpMV (stored to V[:, k])
                 if (kern::spmv_scaled(h->dev, h->A, h->n_loc, h->S, h->pend_nrm, vk, v, 0.0, false, h->stream))
