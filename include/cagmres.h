@@ -195,6 +195,11 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
                                        previous one drains), 0 = plain stream order */
 #define CAGMRES_OPT_PANEL_PF   13   /* 1 (default) = panel ring kernels also prefetch tiles beyond
                                        their cp.async window into L2; 0 = off */
+#define CAGMRES_OPT_PEER       14   /* in-process group handles: 1 (default) = one-sided peer access —
+                                       the MPK halo is ONE pull kernel reading the owners' vectors
+                                       directly, and the cross-rank Gram sum + Cholesky is one
+                                       launch; 0 = pack / peer copies / unpack and a separate sum.
+                                       Must be set identically on every rank.  get: 1 if in use. */
 #define CAGMRES_OPT_TRSM       11   /* CholQR/SVQR panel update V R^{-1}: 1 (default) = scalar
                                        FP64 on a cp.async ring (w <= 16), 0 = FP64 tensor core */
 int cagmres_set_option(cagmres_t h, int opt, int64_t value);

@@ -116,6 +116,10 @@ struct cagmres {
     int64_t nsend = 0, nrecv = 0;
     int64_t* d_send_idx = nullptr;
     int64_t* d_recv_ext = nullptr;
+    int64_t* d_recv_src = nullptr;         // owner-local row of each requested value (peer pull)
+    bool peer_ok = false;                  // transport offers one-sided peer access (in-process group)
+    bool peer_pull = true;                 // CAGMRES_OPT_PEER: use it (1, default) or the copies (0)
+    double* gsum = nullptr;                // fused cross-rank Gram sum (32 x 32)
     double* d_sendbuf = nullptr;
     double* d_recvbuf = nullptr;
     // shifts
@@ -144,7 +148,8 @@ struct cagmres {
         if (ev_beta) cudaEventDestroy(ev_beta);
         cudaFree(ws.part); cudaFree(ws.counter); cudaFree(status);
         cudaFree(arn_part); cudaFree(arn_counter);
-        cudaFree(d_send_idx); cudaFree(d_recv_ext); cudaFree(d_sendbuf); cudaFree(d_recvbuf);
+        cudaFree(d_send_idx); cudaFree(d_recv_ext); cudaFree(d_recv_src); cudaFree(d_sendbuf); cudaFree(d_recvbuf);
+        cudaFree(gsum);
         tr.reset();
         if (own_stream) cudaStreamDestroy(own_stream);
     }
@@ -465,6 +470,17 @@ int init_common_(cagmres* h, const cagmres_csr* A, const int64_t* row_starts, in
         CU(cudaMemset(h->d_recvbuf, 0, sizeof(double) * size_t(std::max<int64_t>(tout, 1))));
         if (tin) CU(cudaMemcpy(h->d_send_idx, plan.send_idx.data(), sizeof(int64_t) * size_t(tin), cudaMemcpyHostToDevice));
         if (tout) CU(cudaMemcpy(h->d_recv_ext, plan.req_ext.data(), sizeof(int64_t) * size_t(tout), cudaMemcpyHostToDevice));
+        {   // owner-local rows of the requested values, for the one-sided halo pull
+            std::vector<int64_t> src(static_cast<size_t>(std::max<int64_t>(tout, 1)), 0);
+            int64_t k = 0;
+            for (int q = 0; q < P; ++q)
+                for (int64_t e = 0; e < plan.req_counts[size_t(q)]; ++e, ++k)
+                    src[size_t(k)] = plan.req_gid[size_t(k)] - row_starts[q];
+            CU(cudaMalloc(&h->d_recv_src, sizeof(int64_t) * src.size()));
+            CU(cudaMemcpy(h->d_recv_src, src.data(), sizeof(int64_t) * src.size(), cudaMemcpyHostToDevice));
+        }
+        CU(cudaMalloc(&h->gsum, sizeof(double) * 32 * 32));
+        h->peer_ok = h->tr->peer_capable() && h->peer_pull;
     }
     return CAGMRES_OK;
 }
@@ -482,6 +498,24 @@ int allreduce(cagmres* h, double* buf, size_t cnt) {
 int halo(cagmres* h, double* vec, int depth) {
     if (h->nranks == 1 || depth <= 0) return CAGMRES_OK;
     depth = std::min(depth, h->s);
+    if (h->peer_ok && h->nranks <= 16) {
+        // one-sided: every rank posts its vector, then ONE kernel pulls the depth-limited
+        // prefix of each owner's list straight from the owner's owned rows (peer memory)
+        std::vector<const void*> peers;
+        TRY(h->tr->peer_acquire(vec, peers, h->stream));
+        kern::PullSegs sg{};
+        for (int q = 0; q < h->nranks; ++q) {
+            const int64_t rc = h->recv_pre[size_t(q)][size_t(depth)];
+            if (!rc) continue;
+            sg.src[sg.n] = static_cast<const double*>(peers[size_t(q)]);
+            sg.off[sg.n] = h->recv_off[size_t(q)];
+            sg.cnt[sg.n] = rc;
+            ++sg.n;
+        }
+        kern::halo_pull(sg, h->d_recv_src, h->d_recv_ext, vec, h->stream);
+        TRY(h->tr->peer_release(h->stream));
+        return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
+    }
     std::vector<std::pair<int64_t, int64_t>> ss, rs;          // (offset, count) per peer
     std::vector<Msg> sends, recvs;
     for (int q = 0; q < h->nranks; ++q) {
@@ -517,6 +551,18 @@ int xty_global(cagmres* h, const double* X, int64_t ldx, int jx, const double* Y
     }
     if (kern::xty(h->dev, h->n_loc, X, ldx, jx, Y, ldy, w, out, false, nullptr, h->status, h->ws, h->stream))
         return CAGMRES_EINVAL;
+    if (chol && h->peer_ok && w <= 32) {
+        // one-sided: the cross-rank sum of the Gram and its Cholesky in one launch reading the
+        // peers' partial Grams directly; the sum then replaces this rank's partial
+        std::vector<const void*> peers;
+        TRY(h->tr->peer_acquire(out, peers, h->stream));
+        std::vector<const double*> src(peers.size());
+        for (size_t q = 0; q < peers.size(); ++q) src[q] = static_cast<const double*>(peers[q]);
+        kern::sum_chol(src.data(), h->nranks, w, h->gsum, R, h->status, h->stream);
+        TRY(h->tr->peer_release(h->stream));
+        CU(cudaMemcpyAsync(out, h->gsum, sizeof(double) * size_t(w) * size_t(w), cudaMemcpyDeviceToDevice, h->stream));
+        return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
+    }
     TRY(allreduce(h, out, size_t(jx) * size_t(w)));
     if (chol) kern::chol(out, w, R, h->status, h->stream);
     return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
@@ -1090,6 +1136,11 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
         case CAGMRES_OPT_TRSM: if (value < 0 || value > 4) return CAGMRES_EINVAL; h->dev.trsm_scalar = int(value); return CAGMRES_OK;
         case CAGMRES_OPT_PDL: if (value < 0 || value > 1) return CAGMRES_EINVAL; kern::g_pdl = int(value); return CAGMRES_OK;
         case CAGMRES_OPT_PANEL_PF: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->dev.panel_pf = int(value); return CAGMRES_OK;
+        case CAGMRES_OPT_PEER:
+            if (value < 0 || value > 1) return CAGMRES_EINVAL;
+            h->peer_pull = value != 0;
+            h->peer_ok = h->tr && h->tr->peer_capable() && h->peer_pull;
+            return CAGMRES_OK;
         case CAGMRES_OPT_FUSE:
             h->fuse_borth_gram = (value & 1) != 0; h->arnoldi_fuse = (value & 2) != 0; h->fuse_scale = (value & 4) != 0;
             return CAGMRES_OK;
@@ -1113,6 +1164,7 @@ int cagmres_get_option(cagmres_t h, int opt, int64_t* value) {
         case CAGMRES_OPT_TRSM: *value = h->dev.trsm_scalar; return CAGMRES_OK;
         case CAGMRES_OPT_PDL: *value = kern::g_pdl; return CAGMRES_OK;
         case CAGMRES_OPT_PANEL_PF: *value = h->dev.panel_pf; return CAGMRES_OK;
+        case CAGMRES_OPT_PEER: *value = h->peer_ok ? 1 : 0; return CAGMRES_OK;
         case CAGMRES_OPT_FUSE:
             *value = (h->fuse_borth_gram ? 1 : 0) | (h->arnoldi_fuse ? 2 : 0) | (h->fuse_scale ? 4 : 0);
             return CAGMRES_OK;

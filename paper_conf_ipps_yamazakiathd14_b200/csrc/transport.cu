@@ -5,6 +5,7 @@
 
 #include <nccl.h>
 
+#include "dense_dev.cuh"
 #include "internal.h"
 #include "kernels.h"
 #include "transport.h"
@@ -109,6 +110,21 @@ struct GroupTransport final : Transport {
             if (q != r && cudaStreamWaitEvent(st, g->post[size_t(q)].done, 0) != cudaSuccess) return CAGMRES_ECUDA;
         return CAGMRES_OK;
     }
+    int peer_acquire(const void* mine, std::vector<const void*>& all, cudaStream_t st) override {
+        cagmres_group::Post& me = g->post[size_t(r)];
+        me.ptr = mine;
+        me.bytes = 0;
+        if (cudaEventRecord(me.ready, st) != cudaSuccess) return CAGMRES_ECUDA;
+        if (int e = sync_point()) return e;
+        all.assign(size_t(g->P), nullptr);
+        for (int q = 0; q < g->P; ++q) {
+            if (q != r && cudaStreamWaitEvent(st, g->post[size_t(q)].ready, 0) != cudaSuccess) return CAGMRES_ECUDA;
+            all[size_t(q)] = g->post[size_t(q)].ptr;
+        }
+        return CAGMRES_OK;
+    }
+    int peer_release(cudaStream_t st) override { return finish(st); }
+    bool peer_capable() const override { return true; }
     int allreduce_sum(double* buf, size_t cnt, cudaStream_t st) override {
         cagmres_group::Post& me = g->post[size_t(r)];
         if (cnt > me.tmp_cap) {
@@ -220,6 +236,47 @@ __global__ void k_sum_ranks(SumSrc s, int P, size_t cnt, double* __restrict__ ou
         for (int q = 1; q < P; ++q) a += s.p[q][i];
         out[i] = a;
     }
+}
+
+__global__ void k_sum_chol(SumSrc s, int P, int w, double* __restrict__ G, double* __restrict__ R, int* status) {
+    __shared__ double sm[32 * 32];
+    pdl_wait();
+    pdl_trigger();
+    for (int i = threadIdx.x; i < w * w; i += blockDim.x) {
+        double a = s.p[0][i];
+        for (int q = 1; q < P; ++q) a += s.p[q][i];
+        G[i] = a;
+    }
+    __syncwarp();
+    __threadfence_block();
+    chol_upper_warp(G, w, w, R, status, sm);
+}
+
+void sum_chol(const double* const* src, int P, int w, double* G, double* R, int* status, cudaStream_t st) {
+    SumSrc s{};
+    for (int q = 0; q < P && q < 16; ++q) s.p[q] = src[q];
+    ++g_launches;
+    launch_pdl(k_sum_chol, dim3(1), dim3(32), 0, st, s, P, w, G, R, status);
+}
+
+__global__ void k_halo_pull(PullSegs sg, int64_t tot, const int64_t* __restrict__ loc,
+                            const int64_t* __restrict__ ext, double* __restrict__ dst) {
+    for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < tot; t += int64_t(gridDim.x) * blockDim.x) {
+        int i = 0;
+        int64_t k = t;
+        while (k >= sg.cnt[i]) { k -= sg.cnt[i]; ++i; }
+        k += sg.off[i];
+        dst[ext[k]] = sg.src[i][loc[k]];
+    }
+}
+
+void halo_pull(const PullSegs& sg, const int64_t* loc, const int64_t* ext, double* dst, cudaStream_t st) {
+    int64_t tot = 0;
+    for (int i = 0; i < sg.n; ++i) tot += sg.cnt[i];
+    if (tot <= 0) return;
+    const int64_t g = std::min<int64_t>((tot + 255) / 256, 4096);
+    ++g_launches;
+    k_halo_pull<<<unsigned(g), 256, 0, st>>>(sg, tot, loc, ext, dst);
 }
 
 void sum_ranks(const double* const* src, int P, size_t cnt, double* out, cudaStream_t st) {

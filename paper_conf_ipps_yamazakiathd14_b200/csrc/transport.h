@@ -38,6 +38,18 @@ struct Transport {
     virtual int allgather(const void* send, void* recv, size_t bytes, cudaStream_t st) = 0;
     // grouped send / recv; the k-th send to a peer matches that peer's k-th recv from us
     virtual int exchange(const std::vector<Msg>& sends, const std::vector<Msg>& recvs, cudaStream_t st) = 0;
+    // One-sided peer access (in-process group only; NCCL: ENOTSUP).  peer_acquire posts `mine`,
+    // makes the stream wait until every rank's buffer is complete and returns all ranks'
+    // pointers (device-loadable: same device or peer access enabled); the caller then launches
+    // ONE kernel that reads the peers' buffers directly (the halo pull, the fused cross-rank
+    // sum + Cholesky) and calls peer_release, after which no rank reuses its buffer before
+    // every reader is done.  Same calling contract as the collectives.
+    virtual int peer_acquire(const void* mine, std::vector<const void*>& all, cudaStream_t st) {
+        (void)mine; (void)all; (void)st;
+        return -7;   // CAGMRES_ENOTSUP
+    }
+    virtual int peer_release(cudaStream_t st) { (void)st; return -7; }
+    virtual bool peer_capable() const { return false; }
 };
 
 // NCCL communicator from a 128-byte ncclUniqueId; nullptr on failure.
@@ -72,4 +84,16 @@ Transport* make_group_transport(cagmres_group* g, int rank);
 namespace kern {
 // out[0:cnt) = src[0][.] + src[1][.] + ... + src[P-1][.] in this order (P <= 16)
 void sum_ranks(const double* const* src, int P, size_t cnt, double* out, cudaStream_t st);
+// G = sum over ranks of the w x w Grams src[q] (rank order), R = chol(G) (upper, ld w) in ONE
+// launch (one warp); breakdown sets ST_CHOL in *status
+void sum_chol(const double* const* src, int P, int w, double* G, double* R, int* status, cudaStream_t st);
+// Halo pull over peer memory: for each segment i (one per owner rank) and k in
+// [off[i], off[i] + cnt[i]): dst[ext[k]] = src_i[loc[k]] — owner-local index loc, extended
+// row ext.  One launch replaces pack -> P-1 copies -> unpack.
+struct PullSegs {
+    const double* src[16];
+    int64_t off[16], cnt[16];
+    int n = 0;
+};
+void halo_pull(const PullSegs& sg, const int64_t* loc, const int64_t* ext, double* dst, cudaStream_t st);
 }

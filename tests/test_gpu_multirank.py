@@ -295,6 +295,30 @@ def test_group_solve_bitwise_independent_of_per_rank_spmv_variant(P):
         assert np.array_equal(sa.hist, sb.hist) and torch.equal(xa, xb)
 
 
+@pytest.mark.parametrize("P", [2, 5])
+def test_group_peer_access_path_is_bitwise_the_copy_path(P):
+    """CAGMRES_OPT_PEER: the one-sided halo pull (one kernel reading the owners' rows) and the
+    fused cross-rank Gram sum + Cholesky give the same bits as pack / copy / unpack and the
+    separate sum + Cholesky (rank-order sums both ways)."""
+    _, Solver = _mods()
+    A = G.convection_diffusion(40, 3, 7)
+    b = G.rhs(A.n)
+    rs = O.block_rows(A.n, P)
+    res = {}
+    for peer in (1, 0):
+        def rank(r, grp, peer=peer):
+            S = Solver(A, s=10, m=30, basis="newton", group=grp, row_starts=rs, rank=r)
+            S.set_option("peer", peer)
+            assert S.get_option("peer") == peer
+            x, st = S.solve(dev(b[rs[r]:rs[r + 1]]), tol=1e-8, maxit=60)
+            W = S.mpk(dev(G.u(4, np.arange(rs[r], rs[r + 1]))), 10).cpu()
+            S.close()
+            return x.cpu(), st, W
+        res[peer] = run_ranks(P, rank)
+    for (xa, sa, wa), (xb, sb, wb) in zip(res[1], res[0]):
+        assert np.array_equal(sa.hist, sb.hist) and torch.equal(xa, xb) and torch.equal(wa, wb)
+
+
 def test_group_single_rank_is_the_single_gpu_handle():
     """P = 1 through the group API: bitwise the single-GPU solve."""
     _, Solver = _mods()

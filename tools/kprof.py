@@ -15,6 +15,7 @@ from synth import generators as G  # noqa: E402
 ap = argparse.ArgumentParser()
 ap.add_argument("--opt", action="append", default=[])
 ap.add_argument("--config", default="C2")
+ap.add_argument("--mpk-only", action="store_true", help="three MPK blocks instead of a solve")
 args = ap.parse_args()
 torch.cuda.set_device(0)
 if args.config == "C2":
@@ -26,6 +27,15 @@ for kv in args.opt:
     k, v = kv.split("=")
     S.set_option(k, int(v))
 b = torch.tensor(G.rhs(A.n), device="cuda")
-x, st = S.solve(b, tol=1e-8, maxit=200)
-torch.cuda.synchronize()
-print("cycles", st.cycles, "spmv variant", S.get_option("spmv"))
+if args.mpk_only:
+    import numpy as np
+    S.set_shifts(np.linspace(0.5, 3.0, s), np.zeros(s))
+    q = b / b.norm()
+    for _ in range(3):
+        S.mpk(q, s)
+    torch.cuda.synchronize()
+    print("mpk done, spmv variant", S.get_option("spmv"))
+else:
+    x, st = S.solve(b, tol=1e-8, maxit=200)
+    torch.cuda.synchronize()
+    print("cycles", st.cycles, "spmv variant", S.get_option("spmv"))
