@@ -203,11 +203,13 @@ __global__ void __launch_bounds__(NT, 1) k_xty_pipe(XtyArgs a) {
         }
         ptx::cp_async_commit();
     };
-    double acc[MT][NTN][2];
+    // two accumulator sets, even / odd 4-row k-steps: twice the independent DMMA chains per warp
+    // (ncu: the single set stalled on the DMMA dependency, "wait"); summed in a fixed order at the end
+    double acc[MT][NTN][2], acc2[MT][NTN][2];
 #pragma unroll
     for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
-        for (int nt = 0; nt < NTN; ++nt) acc[mt][nt][0] = acc[mt][nt][1] = 0.0;
+        for (int nt = 0; nt < NTN; ++nt) acc[mt][nt][0] = acc[mt][nt][1] = acc2[mt][nt][0] = acc2[mt][nt][1] = 0.0;
     // slot column of each fragment lane (clamped: padded lanes feed discarded entries)
     int ycol[NTN], xcol[SYM ? 1 : MT];
 #pragma unroll
@@ -243,17 +245,19 @@ __global__ void __launch_bounds__(NT, 1) k_xty_pipe(XtyArgs a) {
             double bn[NTN];
 #pragma unroll
             for (int nt = 0; nt < NTN; ++nt) bn[nt] = sy[nt][4 * u];
+            constexpr bool SPLIT = MT * NTN <= 8;                    // (wider tiles: registers)
+            auto& A = (SPLIT && (u & 1)) ? acc2 : acc;
             if constexpr (SYM) {
 #pragma unroll
                 for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
-                    for (int nt = mt; nt < NTN; ++nt) ptx::dmma(acc[mt][nt][0], acc[mt][nt][1], bn[mt], bn[nt]);
+                    for (int nt = mt; nt < NTN; ++nt) ptx::dmma(A[mt][nt][0], A[mt][nt][1], bn[mt], bn[nt]);
             } else {
 #pragma unroll
                 for (int mt = 0; mt < MT; ++mt) {
                     const double am = sx[mt][4 * u];
 #pragma unroll
-                    for (int nt = 0; nt < NTN; ++nt) ptx::dmma(acc[mt][nt][0], acc[mt][nt][1], am, bn[nt]);
+                    for (int nt = 0; nt < NTN; ++nt) ptx::dmma(A[mt][nt][0], A[mt][nt][1], am, bn[nt]);
                 }
             }
         }
@@ -261,6 +265,13 @@ __global__ void __launch_bounds__(NT, 1) k_xty_pipe(XtyArgs a) {
         stage = (stage + 1) % PIPE_S;
     }
     ptx::cp_async_wait<0>();
+#pragma unroll
+    for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < NTN; ++nt) {
+            acc[mt][nt][0] += acc2[mt][nt][0];
+            acc[mt][nt][1] += acc2[mt][nt][1];
+        }
     // ragged tail rows [T*TW, n): warp 0 of CTA 0, direct zero-padded loads
     if (blockIdx.x == 0 && wp == 0) {
         for (int64_t kr = T * TW; kr < a.n; kr += 4) {
