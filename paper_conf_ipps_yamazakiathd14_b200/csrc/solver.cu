@@ -105,6 +105,15 @@ struct cagmres {
     bool fuse_borth_gram = false;          // BOrth pass 2 + CholQR Gram in one pass (fused.cu; slower)
     int* status = nullptr;
     double ms_setup = 0.0;                 // wall time of create
+    // CUDA graph of one CA cycle (single rank, untimed solves): captured once per configuration
+    // (shifts, options) on a private stream and replayed every cycle
+    cudaStream_t cap_stream = nullptr;
+    cudaGraphExec_t cyc_exec = nullptr;
+    uint64_t cfg_version = 1, cyc_version = 0;
+    double cyc_bytes[PH_N] = {0, 0, 0, 0, 0};
+    int cyc_spmv = 0;
+    long long cyc_launches = 0;
+    bool use_graphs = true;                // CAGMRES_OPT_GRAPH
     // per-panel diagnostics (cagmres_stats.collect_diag): per block [W^T W | Q_p^T Q_p], (s+1)^2 each
     bool diag_on = false;
     double* dg = nullptr;
@@ -152,6 +161,8 @@ struct cagmres {
         cudaFree(gsum);
         tr.reset();
         if (own_stream) cudaStreamDestroy(own_stream);
+        if (cyc_exec) cudaGraphExecDestroy(cyc_exec);
+        if (cap_stream) cudaStreamDestroy(cap_stream);
     }
 };
 
@@ -1020,6 +1031,54 @@ int enqueue_cycle(cagmres* h, bool arnoldi, const std::vector<Block>& bl) {
     return CAGMRES_OK;
 }
 
+// One CA cycle through a CUDA graph (single rank; no timing events, diagnostics or temporally
+// blocked MPK — their host-side state changes per launch): the cycle's ~45 launches, table
+// copies and ev_tab record are captured on a private stream once per configuration and the
+// executable graph is replayed on the handle's stream.  Programmatic dependent launch edges are
+// kept by the capture.  Host-side accounting (algorithmic bytes, launch counts, the pending
+// normalisation) is replayed from the capture's deltas.
+bool graph_ok(const cagmres* h) {
+    return h->use_graphs && h->nranks == 1 && !h->timer.on && !h->diag_on && !h->wave_on &&
+           (!h->pend || (h->pend_col == 0 && h->pend_nrm == h->gbuf + 8));
+}
+
+int enqueue_ca_cycle(cagmres* h, const std::vector<Block>& bl) {
+    if (!graph_ok(h)) return enqueue_cycle(h, false, bl);
+    const uint64_t key = h->cfg_version * 2 + (h->pend ? 1 : 0);   // the entry state is part of the graph
+    if (h->cyc_exec == nullptr || h->cyc_version != key) {
+        if (h->cyc_exec) { cudaGraphExecDestroy(h->cyc_exec); h->cyc_exec = nullptr; }
+        if (!h->cap_stream) CU(cudaStreamCreateWithFlags(&h->cap_stream, cudaStreamNonBlocking));
+        double b0[PH_N];
+        std::memcpy(b0, h->bytes, sizeof(b0));
+        const int s0 = h->spmv_launches;
+        const long long l0 = kern::g_launches;
+        cudaStream_t saved = h->stream;
+        h->stream = h->cap_stream;
+        CU(cudaStreamBeginCapture(h->cap_stream, cudaStreamCaptureModeThreadLocal));
+        const int rc = enqueue_cycle(h, false, bl);
+        cudaGraph_t g = nullptr;
+        const cudaError_t ce = cudaStreamEndCapture(h->cap_stream, &g);
+        h->stream = saved;
+        if (rc != CAGMRES_OK) { if (g) cudaGraphDestroy(g); return rc; }
+        if (ce != cudaSuccess) return CAGMRES_ECUDA;
+        const cudaError_t ie = cudaGraphInstantiate(&h->cyc_exec, g, 0);
+        cudaGraphDestroy(g);
+        if (ie != cudaSuccess) { h->cyc_exec = nullptr; return CAGMRES_ECUDA; }
+        for (int p = 0; p < PH_N; ++p) { h->cyc_bytes[p] = h->bytes[p] - b0[p]; h->bytes[p] = b0[p]; }
+        h->cyc_spmv = h->spmv_launches - s0;
+        h->spmv_launches = s0;
+        h->cyc_launches = kern::g_launches - l0;
+        kern::g_launches = l0;
+        h->cyc_version = key;
+    }
+    CU(cudaGraphLaunch(h->cyc_exec, h->stream));
+    for (int p = 0; p < PH_N; ++p) h->bytes[p] += h->cyc_bytes[p];
+    h->spmv_launches += h->cyc_spmv;
+    kern::g_launches += h->cyc_launches;
+    h->pend = false;                       // consumed by the cycle's first SpMV
+    return CAGMRES_OK;
+}
+
 void collect_timing(cagmres* h, cagmres_stats* st) {
     double ms[PH_N] = {0, 0, 0, 0, 0};
     for (auto& r : h->timer.rec) {
@@ -1123,6 +1182,7 @@ int cagmres_set_stream(cagmres_t h, void* s) {
 
 int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
     if (!h) return CAGMRES_EINVAL;
+    ++h->cfg_version;                      // any option may change the captured cycle
     switch (opt) {
         case CAGMRES_OPT_MPK_WAVE: h->wave_on = value != 0; h->wave_force = value == 2; return CAGMRES_OK;
         case CAGMRES_OPT_SPMV:
@@ -1136,6 +1196,10 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
         case CAGMRES_OPT_TRSM: if (value < 0 || value > 4) return CAGMRES_EINVAL; h->dev.trsm_scalar = int(value); return CAGMRES_OK;
         case CAGMRES_OPT_PDL: if (value < 0 || value > 1) return CAGMRES_EINVAL; kern::g_pdl = int(value); return CAGMRES_OK;
         case CAGMRES_OPT_PANEL_PF: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->dev.panel_pf = int(value); return CAGMRES_OK;
+        case CAGMRES_OPT_GRAPH:
+            if (value < 0 || value > 1) return CAGMRES_EINVAL;
+            h->use_graphs = value != 0;
+            return CAGMRES_OK;
         case CAGMRES_OPT_PEER:
             if (value < 0 || value > 1) return CAGMRES_EINVAL;
             h->peer_pull = value != 0;
@@ -1165,6 +1229,7 @@ int cagmres_get_option(cagmres_t h, int opt, int64_t* value) {
         case CAGMRES_OPT_PDL: *value = kern::g_pdl; return CAGMRES_OK;
         case CAGMRES_OPT_PANEL_PF: *value = h->dev.panel_pf; return CAGMRES_OK;
         case CAGMRES_OPT_PEER: *value = h->peer_ok ? 1 : 0; return CAGMRES_OK;
+        case CAGMRES_OPT_GRAPH: *value = h->use_graphs ? 1 : 0; return CAGMRES_OK;
         case CAGMRES_OPT_FUSE:
             *value = (h->fuse_borth_gram ? 1 : 0) | (h->arnoldi_fuse ? 2 : 0) | (h->fuse_scale ? 4 : 0);
             return CAGMRES_OK;
@@ -1189,6 +1254,7 @@ int cagmres_set_shifts(cagmres_t h, const double* re, const double* im, int coun
         h->sh_re.clear();                    // with the GMRES cycle again
         h->sh_im.clear();
         h->have_shifts = false;
+        ++h->cfg_version;
         return CAGMRES_OK;
     }
     if (!re || !im) return CAGMRES_EINVAL;
@@ -1199,6 +1265,7 @@ int cagmres_set_shifts(cagmres_t h, const double* re, const double* im, int coun
     h->sh_re.assign(re, re + count);
     h->sh_im.assign(im, im + count);
     h->have_shifts = true;
+    ++h->cfg_version;
     return CAGMRES_OK;
 }
 
@@ -1299,7 +1366,7 @@ int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit
         const bool arnoldi = first_newton || h->basis == CAGMRES_GMRES;
         const bool cgs2 = (h->orth & CAGMRES_REORTH) != 0;
         std::fill(H.begin(), H.end(), 0.0);
-        if (!pending) TRY(enqueue_cycle(h, arnoldi, bl));
+        if (!pending) TRY(arnoldi ? enqueue_cycle(h, true, bl) : enqueue_ca_cycle(h, bl));
         pending = false;
         CU(cudaEventSynchronize(h->ev_tab));
         if (*h->h_stat) { rc = CAGMRES_EBREAKDOWN; break; }
@@ -1367,12 +1434,13 @@ int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit
             if (host::hessenberg_eigvals(H.data(), m + 1, m, wr.data(), wi.data()) != CAGMRES_OK) { rc = CAGMRES_EBREAKDOWN; break; }
             host::modified_leja(wr.data(), wi.data(), m, h->s, h->sh_re, h->sh_im);
             h->have_shifts = true;
+            ++h->cfg_version;
         }
         // Speculate: the next cycle needs only the device-resident q_0, so enqueue it before
         // waiting for beta unless the least-squares residual estimate says this cycle has
         // (almost) converged — hides the host round trip of the convergence test.
         if (cyc + 1 < maxit && res[size_t(m - 1)] > 2.0 * tol * rho0) {
-            TRY(enqueue_cycle(h, h->basis == CAGMRES_GMRES, bl));
+            TRY(h->basis == CAGMRES_GMRES ? enqueue_cycle(h, true, bl) : enqueue_ca_cycle(h, bl));
             pending = true;
         }
         CU(cudaEventSynchronize(h->ev_beta));

@@ -478,6 +478,33 @@ def test_fused_normalisation_is_bitwise_the_separate_scaling(gen, basis):
         assert np.array_equal(out[0][1].hist, st.hist) and torch.equal(out[0][0], x)
 
 
+@pytest.mark.parametrize("gen,kw", [("cd7_40", dict(basis="newton")), ("C1", dict(basis="monomial", reorth=True)),
+                                    ("cd7_40", dict(basis="newton", onepass=True)),
+                                    ("g3_small", dict(basis="newton", tsqr="svqr"))])
+def test_cuda_graph_cycles_are_bitwise_the_stream_launches(gen, kw):
+    """CAGMRES_OPT_GRAPH: every CA cycle replayed from one captured CUDA graph gives the bits of
+    the stream-launched cycles; re-capture after new shifts (second solve with cleared shifts)
+    and after an option change; also with the separate normalisation (different entry state)."""
+    A = {"C1": lambda: G.convection_diffusion(32, 2, 5), "cd7_40": lambda: G.convection_diffusion(40, 3, 7),
+         "g3_small": lambda: G.g3_shaped(n=40000, width=200)}[gen]()
+    b = dev(G.rhs(A.n))
+    out = {}
+    for graph in (1, 0):
+        S = Solver(A, s=5, m=30 if gen != "g3_small" else 60, **kw)
+        S.set_option("graph", graph)
+        res = []
+        for fuse in (6, 2):
+            S.set_option("fuse", fuse)
+            S.clear_shifts()
+            x, st = S.solve(b, tol=1e-10, maxit=80)
+            res.append((x.clone(), st))
+        out[graph] = res
+    for (xa, sa), (xb, sb) in zip(out[1], out[0]):
+        assert sa.status == 0 and sa.cycles == sb.cycles
+        assert np.array_equal(sa.hist, sb.hist) and torch.equal(xa, xb)
+        assert sa.spmv_launches == sb.spmv_launches and sa.bytes == sb.bytes
+
+
 def test_clear_shifts_reruns_first_cycle_bitwise():
     """set_shifts(count = 0): the next Newton solve runs its own GMRES shift cycle again
     and, the reductions being deterministic, reproduces the first solve bit for bit."""
