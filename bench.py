@@ -323,7 +323,7 @@ def run_ours(args):
                        "setup_s": round(setup_s, 2), "options": args.opt,
                        "orth": ("CholQR" + ("2 (reorth)" if (cfg["reorth"] or args.reorth) else "")
                                 + (", one-pass BOrth+CholQR (NEXT-2)" if args.onepass else ", BOrth CGS")),
-                       "kernels": {k_: S.get_option(k_) for k_ in ("spmv", "gram", "fuse", "mpk_wave")}},
+                       "kernels": {k_: S.get_option(k_) for k_ in ("spmv", "gram", "fuse", "mpk_wave", "graph")}},
             "e2e": {"value": round(e2e, 4), "unit": "ms", "stat": "median of K", "h2d_bytes_per_step": 8 * len(b_host),
                     "d2h_bytes_per_step": 8 * len(b_host), "each_ms": [round(v, 3) for v in e2e_ms]},
             "value_each_ms": [round(float(v), 3) for v in ms],

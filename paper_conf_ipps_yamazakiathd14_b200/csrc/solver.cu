@@ -114,6 +114,8 @@ struct cagmres {
     int cyc_spmv = 0;
     long long cyc_launches = 0;
     bool use_graphs = true;                // CAGMRES_OPT_GRAPH
+    bool capturing = false;
+    int graph_err = 0;                     // cudaError_t of a failed capture (graphs then off)
     // per-panel diagnostics (cagmres_stats.collect_diag): per block [W^T W | Q_p^T Q_p], (s+1)^2 each
     bool diag_on = false;
     double* dg = nullptr;
@@ -1027,7 +1029,10 @@ int enqueue_cycle(cagmres* h, bool arnoldi, const std::vector<Block>& bl) {
     if (h->diag_on && !arnoldi)
         CU(cudaMemcpyAsync(h->h_dg, h->dg, sizeof(double) * h->dg_cap, cudaMemcpyDeviceToHost, h->stream));
     CU(cudaMemcpyAsync(h->h_stat, h->status, sizeof(int) * 2, cudaMemcpyDeviceToHost, h->stream));
-    CU(cudaEventRecord(h->ev_tab, h->stream));
+    // under stream capture the record must become an external event node of the graph, so the
+    // host can wait on it after each replay (a plain record is a capture-internal dependency)
+    if (h->capturing) CU(cudaEventRecordWithFlags(h->ev_tab, h->stream, cudaEventRecordExternal));
+    else CU(cudaEventRecord(h->ev_tab, h->stream));
     return CAGMRES_OK;
 }
 
@@ -1053,17 +1058,31 @@ int enqueue_ca_cycle(cagmres* h, const std::vector<Block>& bl) {
         const int s0 = h->spmv_launches;
         const long long l0 = kern::g_launches;
         cudaStream_t saved = h->stream;
+        const bool pend0 = h->pend;
         h->stream = h->cap_stream;
-        CU(cudaStreamBeginCapture(h->cap_stream, cudaStreamCaptureModeThreadLocal));
-        const int rc = enqueue_cycle(h, false, bl);
+        h->capturing = true;
+        cudaError_t ce = cudaStreamBeginCapture(h->cap_stream, cudaStreamCaptureModeThreadLocal);
+        int rc = ce == cudaSuccess ? enqueue_cycle(h, false, bl) : CAGMRES_ECUDA;
         cudaGraph_t g = nullptr;
-        const cudaError_t ce = cudaStreamEndCapture(h->cap_stream, &g);
+        if (ce == cudaSuccess) ce = cudaStreamEndCapture(h->cap_stream, &g);
+        h->capturing = false;
         h->stream = saved;
-        if (rc != CAGMRES_OK) { if (g) cudaGraphDestroy(g); return rc; }
-        if (ce != cudaSuccess) return CAGMRES_ECUDA;
-        const cudaError_t ie = cudaGraphInstantiate(&h->cyc_exec, g, 0);
-        cudaGraphDestroy(g);
-        if (ie != cudaSuccess) { h->cyc_exec = nullptr; return CAGMRES_ECUDA; }
+        if (rc == CAGMRES_OK && ce == cudaSuccess) {
+            ce = cudaGraphInstantiate(&h->cyc_exec, g, 0);
+            if (ce != cudaSuccess) h->cyc_exec = nullptr;
+        }
+        if (g) cudaGraphDestroy(g);
+        if (rc != CAGMRES_OK || ce != cudaSuccess) {
+            // capture not possible here: remember why, restore the host state, launch eagerly
+            h->graph_err = ce != cudaSuccess ? int(ce) : -1;
+            cudaGetLastError();
+            std::memcpy(h->bytes, b0, sizeof(b0));
+            h->spmv_launches = s0;
+            kern::g_launches = l0;
+            h->pend = pend0;
+            h->use_graphs = false;
+            return enqueue_cycle(h, false, bl);
+        }
         for (int p = 0; p < PH_N; ++p) { h->cyc_bytes[p] = h->bytes[p] - b0[p]; h->bytes[p] = b0[p]; }
         h->cyc_spmv = h->spmv_launches - s0;
         h->spmv_launches = s0;
@@ -1229,7 +1248,7 @@ int cagmres_get_option(cagmres_t h, int opt, int64_t* value) {
         case CAGMRES_OPT_PDL: *value = kern::g_pdl; return CAGMRES_OK;
         case CAGMRES_OPT_PANEL_PF: *value = h->dev.panel_pf; return CAGMRES_OK;
         case CAGMRES_OPT_PEER: *value = h->peer_ok ? 1 : 0; return CAGMRES_OK;
-        case CAGMRES_OPT_GRAPH: *value = h->use_graphs ? 1 : 0; return CAGMRES_OK;
+        case CAGMRES_OPT_GRAPH: *value = h->graph_err ? -int64_t(h->graph_err) : (h->use_graphs ? 1 : 0); return CAGMRES_OK;
         case CAGMRES_OPT_FUSE:
             *value = (h->fuse_borth_gram ? 1 : 0) | (h->arnoldi_fuse ? 2 : 0) | (h->fuse_scale ? 4 : 0);
             return CAGMRES_OK;

@@ -498,6 +498,7 @@ def test_cuda_graph_cycles_are_bitwise_the_stream_launches(gen, kw):
             S.clear_shifts()
             x, st = S.solve(b, tol=1e-10, maxit=80)
             res.append((x.clone(), st))
+        assert S.get_option("graph") == graph            # (negative: the capture failed)
         out[graph] = res
     for (xa, sa), (xb, sb) in zip(out[1], out[0]):
         assert sa.status == 0 and sa.cycles == sb.cycles
