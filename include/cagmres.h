@@ -200,9 +200,11 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
                                        directly, and the cross-rank Gram sum + Cholesky is one
                                        launch; 0 = pack / peer copies / unpack and a separate sum.
                                        Must be set identically on every rank.  get: 1 if in use. */
-#define CAGMRES_OPT_GRAPH      15   /* 1 (default) = single-rank untimed solves replay each CA
-                                       restart cycle as one captured CUDA graph (re-captured when
-                                       the shifts or an option change); 0 = stream launches */
+#define CAGMRES_OPT_GRAPH      15   /* 1 = single-rank untimed solves replay each CA restart
+                                       cycle as one captured CUDA graph (re-captured when the
+                                       shifts or an option change); 0 (default: measured neutral,
+                                       the host already runs ahead of the GPU) = stream launches.
+                                       get: a negative value = the cudaError of a failed capture */
 #define CAGMRES_OPT_TRSM       11   /* CholQR/SVQR panel update V R^{-1}: 1 (default) = scalar
                                        FP64 on a cp.async ring (w <= 16), 0 = FP64 tensor core */
 int cagmres_set_option(cagmres_t h, int opt, int64_t value);

@@ -113,7 +113,7 @@ struct cagmres {
     double cyc_bytes[PH_N] = {0, 0, 0, 0, 0};
     int cyc_spmv = 0;
     long long cyc_launches = 0;
-    bool use_graphs = true;                // CAGMRES_OPT_GRAPH
+    bool use_graphs = false;               // CAGMRES_OPT_GRAPH (measured neutral on C2: off)
     bool capturing = false;
     int graph_err = 0;                     // cudaError_t of a failed capture (graphs then off)
     // per-panel diagnostics (cagmres_stats.collect_diag): per block [W^T W | Q_p^T Q_p], (s+1)^2 each
@@ -350,15 +350,20 @@ int spmv_autotune(cagmres* h) {
     cudaEvent_t e0, e1;
     CU(cudaEventCreate(&e0));
     CU(cudaEventCreate(&e1));
-    float best = 1e30f;
-    int pick = 0;
+    constexpr int NC = int(sizeof(cand) / sizeof(cand[0]));
     constexpr int CHAIN = 8;                 // an MPK-like chain of dependent launches
-    for (int v : cand) {
-        h->A.variant = v;
-        for (int k = 0; k < 2; ++k)          // warm-up
+    float tmin[NC];
+    for (int i = 0; i < NC; ++i) {
+        tmin[i] = 1e30f;
+        h->A.variant = cand[i];
+        for (int k = 0; k < 2; ++k)          // warm-up (and the clock ramp) for every candidate
             kern::spmv(h->dev, h->A, h->A.nrows, k ? y : x, k ? x : y, nullptr, 0.0, nullptr, 0.0, h->stream);
-        float tmin = 1e30f;
-        for (int r = 0; r < 3; ++r) {
+    }
+    // round-robin over the candidates (5 rounds, best of each): clock ramp or drift does not
+    // favour a candidate by its position in the list
+    for (int r = 0; r < 5; ++r)
+        for (int i = 0; i < NC; ++i) {
+            h->A.variant = cand[i];
             CU(cudaEventRecord(e0, h->stream));
             for (int k = 0; k < CHAIN; ++k)
                 kern::spmv(h->dev, h->A, h->A.nrows, (k & 1) ? y : x, (k & 1) ? x : y, nullptr, 0.0, nullptr, 0.0,
@@ -367,10 +372,18 @@ int spmv_autotune(cagmres* h) {
             CU(cudaEventSynchronize(e1));
             float ms = 0.f;
             CU(cudaEventElapsedTime(&ms, e0, e1));
-            tmin = std::min(tmin, ms / CHAIN);
+            tmin[i] = std::min(tmin[i], ms / CHAIN);
         }
-        if (tmin < best) { best = tmin; pick = v; }
-    }
+    int bi = 0;
+    for (int i = 1; i < NC; ++i)
+        if (tmin[i] < tmin[bi]) bi = i;
+    // the DIA kernels also fuse the q = w / ||w|| normalisations: prefer them within 3 %
+    int bd = -1;
+    for (int i = 0; i < NC; ++i)
+        if (cand[i] >= 16 && (bd < 0 || tmin[i] < tmin[bd])) bd = i;
+    if (cand[bi] < 16 && bd >= 0 && tmin[bd] <= 1.03f * tmin[bi]) bi = bd;
+    const float best = tmin[bi];
+    const int pick = cand[bi];
     cudaEventDestroy(e0);
     cudaEventDestroy(e1);
     h->A.variant = pick;

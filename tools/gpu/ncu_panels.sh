@@ -10,6 +10,6 @@ for k in gram_ring trsm_ring xty_pipe rows_pipe; do
   ncu -i /tmp/ncu/$k.ncu-rep --page details > gpurun_out/${TAG}_ncu_${k}.txt 2>&1
   ncu -i /tmp/ncu/$k.ncu-rep --page raw --csv > gpurun_out/${TAG}_ncu_${k}_raw.csv 2>&1
 done
-timeout 300 ncu --set full --clock-control none --import-source on -k regex:spmv_dia -s 150 -c 1 -o /tmp/ncu/spmv_C3 python tools/kprof.py --config C3 > /dev/null 2>&1
+timeout 300 ncu --set full --clock-control none --import-source on -k regex:spmv -s 175 -c 1 -o /tmp/ncu/spmv_C3 python tools/kprof.py --config C3 --mpk-only > /dev/null 2>&1
 ncu -i /tmp/ncu/spmv_C3.ncu-rep --page details > gpurun_out/${TAG}_ncu_spmv_C3.txt 2>&1
 ncu -i /tmp/ncu/spmv_C3.ncu-rep --page raw --csv > gpurun_out/${TAG}_ncu_spmv_C3_raw.csv 2>&1

@@ -31,7 +31,7 @@ if args.mpk_only:
     import numpy as np
     S.set_shifts(np.linspace(0.5, 3.0, s), np.zeros(s))
     q = b / b.norm()
-    for _ in range(3):
+    for _ in range(6):
         S.mpk(q, s)
     torch.cuda.synchronize()
     print("mpk done, spmv variant", S.get_option("spmv"))
