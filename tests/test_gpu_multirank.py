@@ -319,6 +319,48 @@ def test_group_peer_access_path_is_bitwise_the_copy_path(P):
         assert np.array_equal(sa.hist, sb.hist) and torch.equal(xa, xb) and torch.equal(wa, wb)
 
 
+@pytest.mark.parametrize("order", ["natural", "kway", "rcm"])
+def test_group_solve_with_bench_row_distribution(order):
+    """The row distributions bench.py uses for --gpus N (natural block rows with the ghost-row
+    band of bench.ghost_rows, or host.distribute's k-way / RCM permutations) through the
+    group at P = 4: the solve converges like the oracle's on the permuted system, and x maps back."""
+    import importlib.util
+    import os
+    from paper_conf_ipps_yamazakiathd14_b200 import host
+    _, Solver = _mods()
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    spec = importlib.util.spec_from_file_location("bench_mod", os.path.join(root, "bench.py"))
+    bench = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(bench)
+    N, P = 48, 4
+    cfg = dict(build=lambda rows=None: G.convection_diffusion(N, 3, 7, rows=rows), n=N ** 3)
+    b = G.rhs(cfg["n"])
+    if order == "natural":
+        rs = np.array([(p * cfg["n"]) // P for p in range(P + 1)], dtype=np.int64)
+        parts = [bench.ghost_rows(cfg, rs, r, 10) for r in range(P)]
+        perm = np.arange(cfg["n"])
+    else:
+        B, perm, rs = host.distribute(cfg["build"](), P, order)
+        parts = [B] * P
+    bp = b[perm]
+
+    def rank(r, grp):
+        S = Solver(parts[r], s=10, m=30, basis="newton", group=grp, row_starts=rs, rank=r)
+        x, st = S.solve(dev(bp[rs[r]:rs[r + 1]]), tol=1e-8, maxit=60)
+        S.close()
+        return x.cpu().numpy(), st
+
+    outs = run_ranks(P, rank)
+    xp = np.concatenate([o[0] for o in outs])
+    x = np.empty_like(xp)
+    x[perm] = xp
+    As = cfg["build"]().to_scipy()
+    assert outs[0][1].status == 0
+    assert np.linalg.norm(b - As @ x) <= 1.01e-8 * np.linalg.norm(b)
+    ref = O.cagmres(As, b, 10, 30, basis="newton", tol=1e-8, maxcyc=60)
+    assert abs(outs[0][1].cycles - ref["cycles"]) <= 1
+
+
 def test_group_single_rank_is_the_single_gpu_handle():
     """P = 1 through the group API: bitwise the single-GPU solve."""
     _, Solver = _mods()
