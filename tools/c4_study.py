@@ -40,7 +40,7 @@ def main():
     # bytes per variant (DESIGN.md §6 algorithmic model): Gram read + TRSM read/write per pass;
     # column passes of MGS / CGS as the solver counts them; CAQR reads twice, writes once
     nb = 8.0 * n
-    model = {"cholqr": nb * (3 * w - 1), "svqr": nb * (3 * w - 1), "cholqr2": 2 * nb * (3 * w - 1),
+    model = {"cholqr": nb * 3 * w, "svqr": nb * 3 * w, "cholqr2": 2 * nb * 3 * w,      # (the API writes all w columns)
              "mgs": nb * sum(5 * k + 3 for k in range(w)), "cgs": nb * sum((2 * k + 3 if k else 0) + 3 for k in range(w)),
              "caqr": nb * 3 * w}
     out = {"config": "C4 banded-27, n = 4,194,304, monomial MPK panel s = 10 (w = 11)", "kappa_W": kappa, "variants": {}}
