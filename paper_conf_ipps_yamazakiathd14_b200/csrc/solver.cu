@@ -343,7 +343,7 @@ void wave_reset_pairs(cagmres* h) {
 // the same operations in the same order (bitwise identical results), so the fastest one on
 // this matrix is picked by timing y = A x over all stored rows (x = V[:,0], y = V[:,1]).
 int spmv_autotune(cagmres* h) {
-    static const int cand[] = {0, 5, 16, 17, 18, 19};
+    static const int cand[] = {0, 5, 16, 17};
     if (h->m < 1 || h->A.nrows <= 0) return CAGMRES_OK;
     double* x = h->V;
     double* y = h->V + h->ldv;
@@ -1218,7 +1218,7 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
     switch (opt) {
         case CAGMRES_OPT_MPK_WAVE: h->wave_on = value != 0; h->wave_force = value == 2; return CAGMRES_OK;
         case CAGMRES_OPT_SPMV:
-            if (value != -1 && value != 0 && value != 5 && (value < 16 || value > 19)) return CAGMRES_EINVAL;
+            if (value != -1 && value != 0 && value != 5 && value != 16 && value != 17) return CAGMRES_EINVAL;
             if (value == -1) return spmv_autotune(h);
             h->A.variant = int(value);
             return CAGMRES_OK;

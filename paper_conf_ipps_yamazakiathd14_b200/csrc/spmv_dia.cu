@@ -133,159 +133,6 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
 }
 
 namespace {
-// Two rows per lane (variant 18; DIA widths <= 16).  A warp takes a PAIR of consecutive SELL-32
-// slices; lane l handles rows 2 (l & 15), 2 (l & 15) + 1 of slice 2p + (l >> 4), so every value
-// load is a 16-B double2 (the two rows are adjacent in the slice's column-major layout) and so is
-// every x gather whose offset is even (the row pair starts at an even row); odd offsets take two
-// 8-B loads.  Half the load instructions per row and twice the bytes in flight per warp for the
-// same register budget as two independent slices.  Per row the FMA order (t = 0..W-1) and the
-// epilogue are those of k_spmv_dia: bitwise identical.  A pair that is not uniformly "width WT,
-// no clamping" is done slice by slice with the generic body.
-template <int MODE, int WT, int MINB, bool SX = false>
-__global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia64(DiaArgs a) {
-    static_assert(WT <= 16, "two rows per lane: <= 16 diagonals per half warp");
-    const int lane = threadIdx.x & 31, hl = lane >> 4, li = lane & 15;
-    const int64_t nsl = (a.nrows + 31) >> 5;
-    const int64_t npr = (nsl + 1) >> 1;
-    const int64_t stride = int64_t(gridDim.x) * (DT_NT / 32);
-    int64_t pr = (int64_t(blockIdx.x) * DT_NT + threadIdx.x) >> 5;
-    if (pr >= npr) { pdl_wait(); pdl_trigger(); return; }
-    // this lane's slice descriptor (its half's slice) for the current and the next pair
-    auto meta = [&](int64_t p, int64_t& b, int& W, int64_t& in, int& off) {
-        const int64_t sl = 2 * p + hl;
-        if (p < npr && sl < nsl) {
-            sell_slice_meta(sl, a.sptr, a.sinfo, b, W, in);
-            off = ((in & 1) && li < W) ? __ldg(a.dcol + (in >> 2) + li) : 0;
-        } else {
-            b = 0; W = 0; in = 1; off = 0;
-        }
-    };
-    int64_t b0, i0, b1, i1;
-    int W0, W1, o0, o1;
-    meta(pr, b0, W0, i0, o0);
-    meta(pr + stride, b1, W1, i1, o1);
-    pdl_wait();
-    pdl_trigger();
-    const double inv = SX ? 1.0 / __ldg(a.xnrm) : 1.0;
-#pragma unroll 1
-    for (; pr < npr; pr += stride) {
-        if (li < W1) prefetch_l2(a.val + b1 + 16 * li);          // next pair: 2 x 128-B lines / diag
-        const int64_t sl = 2 * pr + hl;
-        const bool have = sl < nsl;
-        const int64_t r = sl * 32 + 2 * li;                       // even: rows r, r + 1
-        const bool live0 = have && r < a.nrows, live1 = have && r + 1 < a.nrows;
-        const bool fast = __all_sync(0xffffffffu, !have || (W0 == WT && (i0 & 3) == 1));
-        double acc0 = 0.0, acc1 = 0.0, u0 = 0.0, u1 = 0.0, w0 = 0.0, w1 = 0.0;
-        if (fast) {
-            if (have) {
-                const double* vp = a.val + b0 + 2 * li;
-                double2 v[WT];
-                double x0[WT], x1[WT];
-#pragma unroll
-                for (int t = 0; t < WT; ++t) {
-                    const int o = __shfl_sync(0xffffffffu, o0, (lane & 16) + t);
-                    v[t] = __ldg(reinterpret_cast<const double2*>(vp + 32 * t));
-                    const int64_t c = r + o;
-                    if ((o & 1) == 0) {
-                        const double2 xx = __ldg(reinterpret_cast<const double2*>(a.x + c));
-                        x0[t] = xx.x; x1[t] = xx.y;
-                    } else {
-                        x0[t] = __ldg(a.x + c);
-                        x1[t] = __ldg(a.x + c + 1);
-                    }
-                }
-                if (SX) {
-                    const double2 xx = __ldg(reinterpret_cast<const double2*>(a.x + r));
-                    u0 = xx.x * inv; u1 = xx.y * inv;
-                    if (live0) a.xs[r] = u0;
-                    if (live1) a.xs[r + 1] = u1;
-                } else if (MODE >= 1) {
-                    if (live0) u0 = __ldg(a.u + r);
-                    if (live1) u1 = __ldg(a.u + r + 1);
-                }
-                if (MODE == 2) {
-                    if (live0) w0 = __ldg(a.w + r);
-                    if (live1) w1 = __ldg(a.w + r + 1);
-                }
-#pragma unroll
-                for (int t = 0; t < WT; ++t) {
-                    acc0 = fma(v[t].x, SX ? x0[t] * inv : x0[t], acc0);
-                    acc1 = fma(v[t].y, SX ? x1[t] * inv : x1[t], acc1);
-                }
-            }
-        } else {
-            // slice by slice, one row per lane, with the generic body
-#pragma unroll 1
-            for (int hh = 0; hh < 2; ++hh) {
-                const int64_t s2 = 2 * pr + hh;
-                if (s2 >= nsl) break;
-                int64_t bb, ii;
-                int WW;
-                sell_slice_meta(s2, a.sptr, a.sinfo, bb, WW, ii);
-                const int oo = sell_slice_off(lane, WW, ii, a.dcol);
-                const int64_t rr = s2 * 32 + lane;
-                const double acc = sell_slice_dot<4, true, SX>(rr, bb, WW, ii, oo, a.dcol, a.ncols, a.val, a.x, false, inv);
-                if (rr < a.nrows) {
-                    double uu = 0.0, ww = 0.0;
-                    if (SX) { uu = __ldg(a.x + rr) * inv; a.xs[rr] = uu; }
-                    else if (MODE >= 1) uu = __ldg(a.u + rr);
-                    if (MODE == 2) ww = __ldg(a.w + rr);
-                    double out;
-                    if constexpr (MODE == 3) {
-                        out = uu - acc;
-                    } else {
-                        out = acc;
-                        if constexpr (MODE >= 1) out = fma(a.bu, uu, out);
-                        if constexpr (MODE >= 2) out = fma(a.bw, ww, out);
-                    }
-                    a.y[rr] = out;
-                }
-            }
-        }
-        if (fast && have) {
-            double out0, out1;
-            if constexpr (MODE == 3) {
-                out0 = u0 - acc0; out1 = u1 - acc1;
-            } else {
-                out0 = acc0; out1 = acc1;
-                if constexpr (MODE >= 1) { out0 = fma(a.bu, u0, out0); out1 = fma(a.bu, u1, out1); }
-                if constexpr (MODE >= 2) { out0 = fma(a.bw, w0, out0); out1 = fma(a.bw, w1, out1); }
-            }
-            if (live1) *reinterpret_cast<double2*>(a.y + r) = make_double2(out0, out1);
-            else if (live0) a.y[r] = out0;
-        }
-        b0 = b1; W0 = W1; i0 = i1; o0 = o1;
-        meta(pr + 2 * stride, b1, W1, i1, o1);
-    }
-}
-
-template <int MODE, int WT, int MINB, bool SX = false>
-void go_dia64(const Dev& d, const DiaArgs& a, cudaStream_t st) {
-    static int occ = 0;
-    if (occ == 0) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_spmv_dia64<MODE, WT, MINB, SX>, DT_NT, 0);
-        if (occ < 1) occ = 1;
-    }
-    const int64_t npr = (((a.nrows + 31) >> 5) + 1) >> 1;
-    int64_t g = int64_t(d.sms) * occ;
-    const int64_t need = (npr + DT_NT / 32 - 1) / (DT_NT / 32);
-    if (g > need) g = need;
-    if (g < 1) g = 1;
-    launch_pdl(k_spmv_dia64<MODE, WT, MINB, SX>, dim3(unsigned(g)), dim3(DT_NT), 0, st, a);
-}
-
-template <int WT, int MINB>
-void go_modes64(const Dev& d, const DiaArgs& a, cudaStream_t st, int mode) {
-    switch (mode) {
-        case 0: go_dia64<0, WT, MINB>(d, a, st); break;
-        case 1: go_dia64<1, WT, MINB>(d, a, st); break;
-        case 2: go_dia64<2, WT, MINB>(d, a, st); break;
-        case 4: go_dia64<0, WT, MINB, true>(d, a, st); break;
-        case 5: go_dia64<1, WT, MINB, true>(d, a, st); break;
-        default: go_dia64<3, WT, MINB>(d, a, st); break;
-    }
-}
-
 template <int MODE, int WT, int MINB, bool SX = false>
 void go_dia(const Dev& d, const DiaArgs& a, cudaStream_t st) {
     static int occ = 0;
@@ -330,11 +177,6 @@ void spmv_dia(const Dev& d, const Sell& A, int variant, int64_t nrows, const dou
               const double* u, double bu, const double* w, double bw, int mode, cudaStream_t st,
               const double* xnrm, double* xs) {
     DiaArgs a{nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, u, bu, w, bw, y, xnrm, xs};
-    if ((variant == 18 || variant == 19) && A.dia_w != 27) { // two rows per lane (widths <= 16)
-        if (A.dia_w == 5) { if (variant == 18) go_modes64<5, 3>(d, a, st, mode); else go_modes64<5, 2>(d, a, st, mode); }
-        else { if (variant == 18) go_modes64<7, 3>(d, a, st, mode); else go_modes64<7, 2>(d, a, st, mode); }
-        return;
-    }
     if (variant == 17) go_width<5>(d, a, A.dia_w, st, mode);
     else go_width<4>(d, a, A.dia_w, st, mode);
 }

@@ -47,7 +47,7 @@ def main():
         S = Solver(A, s=args.s, m=30, basis="monomial")
         res = {}
         W0 = None
-        for v in (0, 5, 16, 17, 18, 19):
+        for v in (0, 5, 16, 17):
             S.set_option("spmv", v)
             W = S.mpk(q, args.s)
             if W0 is None:
