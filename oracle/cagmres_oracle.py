@@ -11,9 +11,12 @@ Citations: "P:n" = /root/reference/PAPER.md line n.  Readings of garbled / silen
 Pinning (tests/test_oracle_pins.py): every function below is pinned by something other
 than itself — dense direct solve, dense matrix powers, numpy Householder QR, brute-force
 Krylov least squares, Arnoldi relation, brute-force BFS.  Exception noted inline:
-  * modified_leja: pinned only by brute-force greedy-product check on <= 8 points and by
-    the conjugate-adjacency invariant; tie-breaking beyond that is "parity unpinned"
-    (GPU parity tests inject shifts, G19).
+  * modified_leja: pinned by the brute-force greedy-product check on <= 8 points, the
+    conjugate-adjacency invariant and hand-derived tie cases of the G10 reading (equal moduli,
+    equal log-distance sums, repeated values); GPU solve parity tests still inject shifts
+    where near-ties of computed Ritz values could reorder them (G19).
+  * ritz_values: pinned with the CGS Arnoldi by recovering a known spectrum from a full Krylov
+    space (m = n).
 """
 from __future__ import annotations
 
