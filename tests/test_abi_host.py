@@ -51,6 +51,26 @@ def test_create_rejects_bad_arguments(lib):
     assert lib.cagmres_create(None, C.byref(st), 2, 4, L.NEWTON, L.CHOLQR) == L.EINVAL
 
 
+def test_group_api_argument_checks(lib):
+    """cagmres_group_create / _destroy / create_group argument errors (host-side, no GPU work)."""
+    import ctypes as C
+    from paper_conf_ipps_yamazakiathd14_b200 import _lib as L
+    g = C.c_void_p()
+    assert lib.cagmres_group_create(C.byref(g), 0, None) == L.EINVAL
+    assert lib.cagmres_group_create(C.byref(g), 17, None) == L.EINVAL
+    assert lib.cagmres_group_create(None, 2, None) == L.EINVAL
+    assert lib.cagmres_group_create(C.byref(g), 2, None) == L.OK and g.value
+    h = C.c_void_p()
+    rs = np.array([0, 10, 20], dtype=np.int64)
+    from paper_conf_ipps_yamazakiathd14_b200.solver import _csr_struct
+    A = G.convection_diffusion(5, 2, 5)
+    st, keep = _csr_struct(A, 0, 10)
+    assert lib.cagmres_create_group(C.byref(h), C.byref(st), L.i64ptr(rs), 2, 4, L.NEWTON, L.CHOLQR, g, 2) == L.EINVAL
+    assert lib.cagmres_create_group(C.byref(h), C.byref(st), L.i64ptr(rs), 2, 4, L.NEWTON, L.CHOLQR, None, 0) == L.EINVAL
+    assert lib.cagmres_group_destroy(g) == L.OK
+    assert lib.cagmres_group_destroy(None) == L.OK
+
+
 def test_host_eigvals_match_numpy():
     from paper_conf_ipps_yamazakiathd14_b200 import host
     A = G.convection_diffusion(16, 2, 5).to_scipy()
