@@ -207,6 +207,18 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
                                        get: a negative value = the cudaError of a failed capture */
 #define CAGMRES_OPT_TRSM       11   /* CholQR/SVQR panel update V R^{-1}: 1 (default) = scalar
                                        FP64 on a cp.async ring (w <= 16), 0 = FP64 tensor core */
+#define CAGMRES_OPT_FOLD       16   /* 1 (default) = the last block's final panel update of a CA
+                                       cycle (V := P R^{-1}; one-pass: P := [Q P] M) is not
+                                       formed: those columns are read only by the solution update
+                                       x += V y, and Q_new y = P (R^{-1} [0; y]), so the host
+                                       folds R^{-1} (and -C R^{-1}) into the coefficients and one
+                                       pass over V[:, 0:m+1] updates x.  Equal in exact arithmetic;
+                                       off with collect_diag (it needs the final Q).  0 = form it. */
+#define CAGMRES_OPT_SERP       17   /* serpentine row order (bit mask of kernels that traverse their
+                                       row ranges in reverse, so the tiles their predecessor read
+                                       last are L2 hits): bit 0 = CholQR/SVQR panel update (after
+                                       the Gram); bit 1 = every second MPK step (DIA SpMV).
+                                       Default 3.  Row-wise kernels: results identical. */
 int cagmres_set_option(cagmres_t h, int opt, int64_t value);
 /* Current value of an option (e.g. the SpMV variant the create-time selection picked).
  * EINVAL for a null handle / pointer or an unknown option. */

@@ -40,7 +40,9 @@ struct Dev {
     int arnoldi_ring = 1;       // first-cycle / GMRES Arnoldi passes: 1 = cp.async ring kernels
     int trsm_scalar = 1;        // CholQR/SVQR update: 1 = scalar DFMA ring (w <= 16), 0 = DMMA
     int panel_tw16 = 1;
-    int panel_pf = 1;           // panel rings: L2 prefetch PF_DIST tiles beyond the cp.async window         // panel ring kernels: 16-row tiles when >= 24 columns are streamed
+    int panel_pf = 1;           // panel rings: L2 prefetch PF_DIST tiles beyond the cp.async window
+    int serp = 3;               // CAGMRES_OPT_SERP bits: kernels that run their row ranges in reverse
+                                // (serpentine order with the predecessor: its last tiles are L2 hits)
 };
 
 // Sliced ELLPACK, slice height 32 (one warp), column-major inside a slice, with per-slice
@@ -57,6 +59,7 @@ struct Sell {
     int64_t ncols = 0;          // valid x entries (clamp bound for DIA slices)
     int64_t ndcol = 0, ndia = 0;
     int dia_w = 0;              // most common width of the unclamped DIA slices (spmv_dia.cu)
+    int rev = 0;                // next DIA SpMV launch visits the slices in descending order (serpentine)
     int64_t* sptr = nullptr;    // nslices+1 value offsets
     int64_t* sinfo = nullptr;   // nslices
     int32_t* dcol = nullptr;    // DIA offsets / explicit column ids

@@ -103,6 +103,13 @@ struct cagmres {
     unsigned int* arn_counter = nullptr;
     bool arnoldi_fuse = true;
     bool fuse_borth_gram = false;          // BOrth pass 2 + CholQR Gram in one pass (fused.cu; slower)
+    // CAGMRES_OPT_FOLD (default on): the last block's final panel update (P R^{-1}, or the
+    // one-pass [Q P] M) is never formed — the restart only needs x += V y, and
+    // Q_new y_new = P (R^{-1} [0; y_new]) — so it is folded into the solution update.
+    // fold_kind of the cycle just enqueued: 0 = none, 1 = P R^{-1}, 2 = one-pass; fold_pass = the
+    // pass whose R (and C) the host applies.
+    bool fold = true;
+    int fold_kind = 0, fold_pass = 0;
     int* status = nullptr;
     double ms_setup = 0.0;                 // wall time of create
     // CUDA graph of one CA cycle (single rank, untimed solves): captured once per configuration
@@ -675,6 +682,7 @@ int mpk_block(cagmres* h, int j, int sb, const std::vector<host::Step>& steps) {
         double* y = h->V + size_t(h->ldv) * (j + k);
         const int64_t rows = h->level_len[size_t(sb - k)];
         const bool pair2 = stp.kind == 2;
+        h->A.rev = (h->dev.serp & 2) && (k & 1) == 0 ? 1 : 0;   // OPT_SERP bit 1: even steps reversed
         {
             Scope sv(h, PH_SPMV);
             if (k == 1 && fused_q) {       // q_j = S / ||S|| formed inside the first step (stored to V[:, j])
@@ -687,6 +695,7 @@ int mpk_block(cagmres* h, int j, int sb, const std::vector<host::Step>& steps) {
                            pair2 ? h->V + size_t(h->ldv) * (j + k - 2) : nullptr, stp.b2, h->stream);
             }
         }
+        h->A.rev = 0;
         const double by = spmv_bytes(h, rows, sb - k + 1, pair2);
         h->bytes[PH_MPK] += by;
         h->bytes[PH_SPMV] += by;
@@ -722,7 +731,9 @@ int borth_panel(cagmres* h, const double* Q, int64_t ldq, int j, double* P, int6
 
 // TSQR of the panel P (n_loc x w, ld ldp), R (device w x w, ld w).  c0 = 1 leaves column 0
 // unwritten (the block's start vector q_j is kept, reading G2).
-int tsqr_panel(cagmres* h, double* P, int64_t ldp, int w, double* R, int kind, int c0, bool retry = false) {
+// skip_update (CholQR / SVQR only): R is formed but P is left as is (OPT_FOLD).
+int tsqr_panel(cagmres* h, double* P, int64_t ldp, int w, double* R, int kind, int c0, bool retry = false,
+               bool skip_update = false) {
     Scope sc(h, PH_TSQR);
     const double nl = double(h->n_loc);
     if (kind == CAGMRES_CHOLQR || kind == CAGMRES_SVQR) {
@@ -733,8 +744,12 @@ int tsqr_panel(cagmres* h, double* P, int64_t ldp, int w, double* R, int kind, i
             TRY(xty_global(h, P, ldp, w, P, ldp, w, h->gbuf, false, nullptr));
             kern::svqr_factor(h->gbuf, w, R, h->status, h->stream);
         }
-        kern::trsm(h->dev, h->n_loc, P, ldp, w, R, c0, h->stream, true);    // V := V R^{-1} (P final: early)
-        h->bytes[PH_TSQR] += 8.0 * nl * (2.0 * w + double(w - c0));
+        if (skip_update) {
+            h->bytes[PH_TSQR] += 8.0 * nl * w;
+        } else {
+            kern::trsm(h->dev, h->n_loc, P, ldp, w, R, c0, h->stream, true);    // V := V R^{-1} (P final: early)
+            h->bytes[PH_TSQR] += 8.0 * nl * (2.0 * w + double(w - c0));
+        }
     } else if (kind == CAGMRES_CAQR) {                       // Fig. 9 CAQR: TSQR tree
         // Multi-rank: "each GPU first computes the QR factorization of the local
         // matrix, then the local R-factors are gathered ..., and the final QR factorization is
@@ -852,8 +867,10 @@ int ca_cycle(cagmres* h, const std::vector<Block>& bl) {
     const bool re2 = (h->orth & CAGMRES_REORTH) != 0, mgs = (h->orth & CAGMRES_BORTH_MGS) != 0;
     const size_t W2 = (size_t(h->s) + 1) * (size_t(h->s) + 1);
     size_t bi = 0;
+    h->fold_kind = 0;
     for (const Block& b : bl) {
         const int j = b.j, sb = b.sb, w = sb + 1;
+        const bool last_block = &b == &bl.back();
         const std::vector<host::Step> steps = h->basis == CAGMRES_MONOMIAL
             ? host::block_steps({}, {}, sb) : host::block_steps(h->sh_re, h->sh_im, sb);
         TRY(mpk_block(h, j, sb, steps));
@@ -866,6 +883,8 @@ int ca_cycle(cagmres* h, const std::vector<Block>& bl) {
         for (int pass = 0; pass < (re2 ? 2 : 1); ++pass) {
             double* C = h->tab + (pass ? b.c2 : b.c1);
             double* R = h->tab + (pass ? b.r2 : b.r1);
+            // fold this pass's panel update into x += V y (OPT_FOLD): last block, final pass
+            const bool fold = h->fold && !h->diag_on && last_block && pass == (re2 ? 1 : 0);
             if (j > 0 && (h->orth & CAGMRES_ONEPASS) && j + w <= 64) {
                 // one-pass BOrth + CholQR (NEXT-2): [Q P]^T P ; small step ; P := [Q P] M
                 const double nl = double(h->n_loc);
@@ -876,6 +895,7 @@ int ca_cycle(cagmres* h, const std::vector<Block>& bl) {
                 }
                 Scope sc(h, PH_TSQR);
                 kern::onepass_finalize(h->gbuf, j, w, C, R, h->op_M, h->status, h->stream);
+                if (fold) { h->fold_kind = 2; h->fold_pass = pass; continue; }
                 if (kern::gemm_rows(h->dev, h->n_loc, h->V, h->ldv, j + w, Pj, h->ldv, w, h->op_M, j + w, 1,
                                     h->stream, true))
                     return CAGMRES_EINVAL;
@@ -901,16 +921,20 @@ int ca_cycle(cagmres* h, const std::vector<Block>& bl) {
                         TRY(allreduce(h, h->gbuf, size_t(w) * size_t(w)));
                         kern::chol(h->gbuf, w, R, h->status, h->stream);
                     }
+                    if (fold) { h->fold_kind = 1; h->fold_pass = pass; continue; }
                     kern::trsm(h->dev, h->n_loc, Pj, h->ldv, w, R, 1, h->stream);
                     h->bytes[PH_TSQR] += 8.0 * nl * (2.0 * w + double(w - 1));   // Gram bytes as if unfused
                     continue;
                 }
                 h->bytes[PH_BORTH] += 8.0 * nl * (2.0 * j + 3.0 * sb);
-                TRY(tsqr_panel(h, Pj, h->ldv, w, R, kind, 1, (h->orth & CAGMRES_SVQR_RETRY) != 0));
+                TRY(tsqr_panel(h, Pj, h->ldv, w, R, kind, 1, (h->orth & CAGMRES_SVQR_RETRY) != 0, fold));
+                if (fold) { h->fold_kind = 1; h->fold_pass = pass; }
                 continue;
             }
             TRY(borth_panel(h, h->V, h->ldv, j, Pj + h->ldv, h->ldv, sb, C, mgs));
-            TRY(tsqr_panel(h, Pj, h->ldv, w, R, kind, 1, (h->orth & CAGMRES_SVQR_RETRY) != 0));
+            const bool fold_tsqr = fold && (kind == CAGMRES_CHOLQR || kind == CAGMRES_SVQR);
+            TRY(tsqr_panel(h, Pj, h->ldv, w, R, kind, 1, (h->orth & CAGMRES_SVQR_RETRY) != 0, fold_tsqr));
+            if (fold_tsqr) { h->fold_kind = 1; h->fold_pass = pass; }
         }
         if (dgb) {                                              // ... and Q_p^T Q_p after the passes
             Scope sc(h, PH_OTHER);
@@ -1240,6 +1264,8 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
         case CAGMRES_OPT_FUSE:
             h->fuse_borth_gram = (value & 1) != 0; h->arnoldi_fuse = (value & 2) != 0; h->fuse_scale = (value & 4) != 0;
             return CAGMRES_OK;
+        case CAGMRES_OPT_FOLD: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->fold = value != 0; return CAGMRES_OK;
+        case CAGMRES_OPT_SERP: if (value < 0 || value > 255) return CAGMRES_EINVAL; h->dev.serp = int(value); return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK:
             if (value < 256 || value % 256) return CAGMRES_EINVAL;
             h->wave_CH = int(value); wave_reset_pairs(h); return CAGMRES_OK;
@@ -1265,6 +1291,8 @@ int cagmres_get_option(cagmres_t h, int opt, int64_t* value) {
         case CAGMRES_OPT_FUSE:
             *value = (h->fuse_borth_gram ? 1 : 0) | (h->arnoldi_fuse ? 2 : 0) | (h->fuse_scale ? 4 : 0);
             return CAGMRES_OK;
+        case CAGMRES_OPT_FOLD: *value = h->fold ? 1 : 0; return CAGMRES_OK;
+        case CAGMRES_OPT_SERP: *value = h->dev.serp; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK: *value = h->wave_CH; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CTAS: *value = h->wave_ctas; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_LAG: *value = h->wave_lag; return CAGMRES_OK;
@@ -1453,12 +1481,39 @@ int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit
         }
         // ---- least squares + solution update ----
         if (host::givens_ls(H.data(), m + 1, m, beta, y.data(), res.data()) != CAGMRES_OK) { rc = CAGMRES_EBREAKDOWN; break; }
+        int ncoef = m;
         for (int i = 0; i < m; ++i) h->h_y[i] = -y[size_t(i)];    // update() subtracts X C
+        if (!arnoldi && h->fold_kind) {
+            // OPT_FOLD: the last block's columns j+1..j+sb of V still hold the panel P (BOrth-
+            // updated); Q_new[:, c] = (P R^{-1})[:, c] (c >= 1), or ([Q P] Mo)[:, c] with
+            // Mo = [-Cf R^{-1}; R^{-1}] for one-pass.  So Q_new y_new = P z (- Q Cf z), with
+            // z = R^{-1} [0; y_{j+1..j+sb}] (y_m := 0: the last column is not in the LS).
+            const Block& b0 = bl.back();
+            const int j = b0.j, sb = b0.sb, w = sb + 1;
+            const double* Rf = htab + (h->fold_pass ? b0.r2 : b0.r1);
+            std::vector<double> z(size_t(w), 0.0);
+            for (int c = 1; c < w; ++c) z[size_t(c)] = j + c < m ? y[size_t(j + c)] : 0.0;
+            for (int k = w - 1; k >= 0; --k) {                  // back substitution R z = [0; y]
+                double a = z[size_t(k)];
+                for (int l = k + 1; l < w; ++l) a -= Rf[size_t(k) + size_t(w) * l] * z[size_t(l)];
+                z[size_t(k)] = a / Rf[size_t(k) + size_t(w) * k];
+            }
+            for (int k = 0; k < w; ++k) h->h_y[j + k] = (k == 0 ? -y[size_t(j)] : 0.0) - z[size_t(k)];
+            if (h->fold_kind == 2) {
+                const double* Cf = htab + (h->fold_pass ? b0.c2 : b0.c1);   // C[i, c-1], ld j
+                for (int i = 0; i < j; ++i) {
+                    double a = 0.0;
+                    for (int c = 1; c < w; ++c) a += Cf[size_t(i) + size_t(j) * (c - 1)] * z[size_t(c)];
+                    h->h_y[i] += a;
+                }
+            }
+            ncoef = j + w;                                       // = m + 1
+        }
         {
             Scope sc(h, PH_OTHER);
-            CU(cudaMemcpyAsync(h->ybuf, h->h_y, sizeof(double) * size_t(m), cudaMemcpyHostToDevice, h->stream));
-            kern::update(h->dev, h->n_loc, h->V, h->ldv, m, x, h->n_loc, 1, h->ybuf, h->stream);
-            h->bytes[PH_OTHER] += 8.0 * double(h->n_loc) * (m + 2.0);
+            CU(cudaMemcpyAsync(h->ybuf, h->h_y, sizeof(double) * size_t(ncoef), cudaMemcpyHostToDevice, h->stream));
+            kern::update(h->dev, h->n_loc, h->V, h->ldv, ncoef, x, h->n_loc, 1, h->ybuf, h->stream);
+            h->bytes[PH_OTHER] += 8.0 * double(h->n_loc) * (ncoef + 2.0);
         }
         TRY(residual_norm_async(h, b, x));                        // r, beta, q_0 for the next cycle
         if (first_newton) {                                      // Ritz values -> Leja shifts

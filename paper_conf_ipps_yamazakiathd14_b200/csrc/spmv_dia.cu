@@ -34,6 +34,7 @@ struct DiaArgs {
     double* y;
     const double* xnrm;     // SX: x is an unnormalised w, the operand is w * (1 / *xnrm)
     double* xs;             // SX: the normalised operand's rows [0, nrows) are stored here
+    int rev;                // 1: slices visited in descending order (serpentine MPK steps)
 };
 }  // namespace
 
@@ -64,11 +65,14 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
     const int64_t stride = int64_t(gridDim.x) * (DT_NT / 32);
     int64_t sl = (int64_t(blockIdx.x) * DT_NT + threadIdx.x) >> 5;
     if (sl >= nsl) { pdl_wait(); pdl_trigger(); return; }
+    // serpentine order (rev): the grid walks the slices from the end, so the first slices read
+    // are the ones the previous MPK step read last — their A values and x lines are L2 hits
+    const int64_t rx = a.rev ? nsl - 1 : 0, rs = a.rev ? -1 : 1;     // slice = rx + rs * sl
     int64_t b0, i0, b1 = 0, i1 = 1, b2 = 0, i2 = 1;
     int W0, W1 = 0, W2 = 0, o0, o1;
     // slice descriptors (static during a solve) are loaded before the PDL wait
-    sell_slice_meta(sl, a.sptr, a.sinfo, b0, W0, i0);
-    if (sl + stride < nsl) sell_slice_meta(sl + stride, a.sptr, a.sinfo, b1, W1, i1);
+    sell_slice_meta(rx + rs * sl, a.sptr, a.sinfo, b0, W0, i0);
+    if (sl + stride < nsl) sell_slice_meta(rx + rs * (sl + stride), a.sptr, a.sinfo, b1, W1, i1);
     o0 = sell_slice_off(lane, W0, i0, a.dcol);
     pdl_wait();
     pdl_trigger();
@@ -76,10 +80,10 @@ __global__ void __launch_bounds__(DT_NT, MINB) k_spmv_dia(DiaArgs a) {
 #pragma unroll 1
     for (; sl < nsl; sl += stride) {
         b2 = 0; W2 = 0; i2 = 1;
-        if (sl + 2 * stride < nsl) sell_slice_meta(sl + 2 * stride, a.sptr, a.sinfo, b2, W2, i2);
+        if (sl + 2 * stride < nsl) sell_slice_meta(rx + rs * (sl + 2 * stride), a.sptr, a.sinfo, b2, W2, i2);
         o1 = sell_slice_off(lane, W1, i1, a.dcol);
         if (lane < 2 * W1) prefetch_l2(a.val + b1 + 16 * lane);        // 128-B lines of slice +1
-        const int64_t r = sl * 32 + lane;
+        const int64_t r = (rx + rs * sl) * 32 + lane;
         const bool live = r < a.nrows;
         double uu = 0.0, ww = 0.0, acc = 0.0;
         if (SX && live) {                                               // own row of q = w / ||w||
@@ -176,7 +180,7 @@ void go_width(const Dev& d, const DiaArgs& a, int wt, cudaStream_t st, int mode)
 void spmv_dia(const Dev& d, const Sell& A, int variant, int64_t nrows, const double* x, double* y,
               const double* u, double bu, const double* w, double bw, int mode, cudaStream_t st,
               const double* xnrm, double* xs) {
-    DiaArgs a{nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, u, bu, w, bw, y, xnrm, xs};
+    DiaArgs a{nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, u, bu, w, bw, y, xnrm, xs, A.rev};
     if (variant == 17) go_width<5>(d, a, A.dia_w, st, mode);
     else go_width<4>(d, a, A.dia_w, st, mode);
 }

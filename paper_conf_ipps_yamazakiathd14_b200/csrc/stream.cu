@@ -33,6 +33,10 @@ struct StreamArgs {
     // produced C / R), so the ring kernels issue their first tile copies BEFORE
     // griddepcontrol.wait and fill their pipelines while that kernel drains (PDL)
     int early = 0;
+    // 1: run every warp's tile range in descending order — the reverse of the predecessor's
+    // temporal order, so the first tiles read are the ones the predecessor touched last (still
+    // in L2).  Row-wise kernels only (no reduction): results are identical either way.
+    int rev = 0;
 };
 
 // R^{-1} (upper, w x w) into sRi[k*32 + c]; one thread per column (back substitution)
@@ -432,6 +436,7 @@ __global__ void __launch_bounds__(256, 1) k_trsm_ring(StreamArgs a) {
     const int c0 = a.c0;
     auto issue = [&](int64_t t, int stage) {
         if (t < t1) {
+            if (a.rev) t = t0 + t1 - 1 - t;
             double* dst = ring + stage * SD + 2 * lane;
             const double* src = a.P + t * TR + 2 * lane;
 #pragma unroll
@@ -498,7 +503,7 @@ __global__ void __launch_bounds__(256, 1) k_trsm_ring(StreamArgs a) {
             v0[k] = p2.x;
             v1[k] = p2.y;
         }
-        rowout2(v0, v1, a.P + t * TR + 2 * lane);
+        rowout2(v0, v1, a.P + (a.rev ? t0 + t1 - 1 - t : t) * TR + 2 * lane);
         __syncwarp();
         stage = stage == RS - 1 ? 0 : stage + 1;
     }
@@ -591,7 +596,7 @@ void trsm(const Dev& d, int64_t n, double* P, int64_t ldp, int w, const double* 
         launch_pdl(k_scale1, dim3(unsigned(g)), dim3(256), 0, st, n, P, R);
         return;
     }
-    StreamArgs a{n, nullptr, 0, 0, P, ldp, w, R, w, c0, d.panel_pf, early ? 1 : 0};
+    StreamArgs a{n, nullptr, 0, 0, P, ldp, w, R, w, c0, d.panel_pf, early ? 1 : 0, (d.serp & 1) ? 1 : 0};
     if (d.trsm_scalar && trsm_ring(d, a, st)) return;
     dispatch<1>(d, a, st);
 }

@@ -443,6 +443,42 @@ def test_solve_onepass(s, m, reorth, gen):
     assert np.linalg.norm(r) <= 1.01e-8 * np.linalg.norm(b)
 
 
+@pytest.mark.parametrize("kw", [dict(), dict(reorth=True), dict(onepass=True), dict(onepass=True, reorth=True),
+                                dict(tsqr="svqr"), dict(basis="monomial")])
+def test_fold_last_panel_update_into_solution_update(kw):
+    """CAGMRES_OPT_FOLD: the last block's final panel update is not formed and x += V y uses
+    the panel P with coefficients R^{-1}[0; y] (and -C R^{-1}[0; y] for one-pass).  Equal in exact
+    arithmetic: both settings must match the oracle (same rule as every solve test) and each
+    other to rounding; the folded cycle launches one panel kernel less."""
+    A = G.convection_diffusion(40, 3, 7)
+    As = A.to_scipy()
+    b = G.rhs(A.n)
+    kw = dict(kw)
+    basis = kw.pop("basis", "newton")
+    sv = 10 if basis == "newton" else 5
+    sh = O.modified_leja(O.ritz_values(O.arnoldi_cgs2(As, b, 30)[1], 30), sv) if basis == "newton" else None
+    ref, env = rounding_envelope(As, b, nperm=1, s=sv, m=30, basis=basis, tol=1e-8, maxcyc=60, shifts=sh,
+                                 reorth=kw.get("reorth", False), onepass=kw.get("onepass", False),
+                                 tsqr=kw.get("tsqr", "cholqr"))
+    out = {}
+    for fold in (0, 1):
+        S = Solver(A, s=sv, m=30, basis=basis, **kw)
+        S.set_option("fold", fold)
+        assert S.get_option("fold") == fold
+        if sh is not None:
+            S.set_shifts(*sh)
+        x, st = S.solve(dev(b), tol=1e-8, maxit=60)
+        assert st.status == 0 and abs(st.cycles - len(ref)) <= 1
+        assert hist_within_envelope(st.hist, ref, env)
+        r = b - As @ x.cpu().numpy()
+        assert np.linalg.norm(r) <= 1.01e-8 * np.linalg.norm(b)
+        out[fold] = (x.cpu().numpy(), st)
+    (x0, s0), (x1, s1) = out[0], out[1]
+    assert s0.cycles == s1.cycles
+    assert np.allclose(s0.hist, s1.hist, rtol=1e-6, atol=1e-15)
+    assert np.linalg.norm(x0 - x1) <= 1e-9 * np.linalg.norm(x0)
+
+
 def test_onepass_cycle_basis_matches_two_pass():
     """One cycle, same shifts: the one-pass basis spans the same space as the two-pass one —
     residual histories agree to rounding (Pythagoras exact when Q^T Q = I)."""
