@@ -214,11 +214,13 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
                                        folds R^{-1} (and -C R^{-1}) into the coefficients and one
                                        pass over V[:, 0:m+1] updates x.  Equal in exact arithmetic;
                                        off with collect_diag (it needs the final Q).  0 = form it. */
-#define CAGMRES_OPT_SERP       17   /* serpentine row order (bit mask of kernels that traverse their
-                                       row ranges in reverse, so the tiles their predecessor read
-                                       last are L2 hits): bit 0 = CholQR/SVQR panel update (after
-                                       the Gram); bit 1 = every second MPK step (DIA SpMV).
-                                       Default 3.  Row-wise kernels: results identical. */
+#define CAGMRES_OPT_SERP       17   /* 1 (default) = serpentine row order: every streaming kernel
+                                       (SpMV, BOrth / Gram / TRSM / Arnoldi panel kernels) sweeps the
+                                       rows opposite to the launch before it, so the rows that
+                                       launch touched last — still in the 126 MB L2 — are read
+                                       first; 0 = every launch sweeps forward.  Row-wise kernels
+                                       give identical results either way; the reductions (xTy, Gram,
+                                       norms) sum in another fixed order (deterministic). */
 int cagmres_set_option(cagmres_t h, int opt, int64_t value);
 /* Current value of an option (e.g. the SpMV variant the create-time selection picked).
  * EINVAL for a null handle / pointer or an unknown option. */

@@ -105,13 +105,13 @@ __global__ void __launch_bounds__(512, 1) k_arnoldi_ring(ArnoldiArgs a) {
     const int64_t T = a.n / 32;
     const int64_t Wn = int64_t(gridDim.x) * nw;
     const int64_t g = int64_t(blockIdx.x) * nw + wp;
-    const int64_t t0 = g * T / Wn, t1 = (g + 1) * T / Wn;
+    const int64_t cnt = band_count(T, Wn, g);                     // tiles of this warp (band order)
     const int part2 = 2 * (lane & 15), cfirst = lane >> 4;
     const int64_t cstride = 2 * a.ldq;
-    auto issue = [&](int64_t t, int stage) {
-        if (t < t1) {
+    auto issue = [&](int64_t i, int stage) {
+        if (i < cnt) {
             double* dst = ring + stage * stage_d + cfirst * 32 + part2;
-            const int64_t r0 = t * 32 + part2;
+            const int64_t r0 = band_tile(T, Wn, g, i, a.rev) * 32 + part2;
             const double* src = a.Q + a.ldq * cfirst + r0;
             int c = cfirst;
 #pragma unroll 4
@@ -136,19 +136,19 @@ __global__ void __launch_bounds__(512, 1) k_arnoldi_ring(ArnoldiArgs a) {
         }
     };
 #pragma unroll
-    for (int s = 0; s < AR_S - 1; ++s) issue(t0 + s, s);
+    for (int s = 0; s < AR_S - 1; ++s) issue(s, s);
     int stage = 0;
-    for (int64_t t = t0; t < t1; ++t) {
-        issue(t + AR_S - 1, (stage + AR_S - 1) % AR_S);
-        if (a.pf && t + AR_S - 1 + ptx::PF_DIST < t1) {
-            const int64_t rp = (t + AR_S - 1 + ptx::PF_DIST) * 32;
+    for (int64_t i = 0; i < cnt; ++i) {
+        issue(i + AR_S - 1, (stage + AR_S - 1) % AR_S);
+        if (a.pf && i + AR_S - 1 + ptx::PF_DIST < cnt) {
+            const int64_t rp = band_tile(T, Wn, g, i + AR_S - 1 + ptx::PF_DIST, a.rev) * 32;
             for (int q = lane; q < ncol * 2; q += 32)
                 ptx::prefetch_l2((q >> 1 < jx ? a.Q + a.ldq * (q >> 1) : a.v) + rp + 16 * (q & 1));
         }
         ptx::cp_async_wait<AR_S - 1>();
         __syncwarp();
         const double* sl = ring + stage * stage_d + lane;
-        row(sl, sl[jx * 32], t * 32 + lane);
+        row(sl, sl[jx * 32], band_tile(T, Wn, g, i, a.rev) * 32 + lane);
         __syncwarp();
         stage = (stage + 1) % AR_S;
     }
@@ -188,7 +188,9 @@ __global__ void __launch_bounds__(512, 1) k_arnoldi_ring(ArnoldiArgs a) {
 
 namespace {
 template <int JX, int MODE>
-bool go_ring(const Dev& d, const ArnoldiArgs& a, cudaStream_t st) {
+bool go_ring(const Dev& d, const ArnoldiArgs& a0, cudaStream_t st) {
+    ArnoldiArgs a = a0;
+    a.rev = d.rev;
     const bool aligned = ((reinterpret_cast<uintptr_t>(a.v) | reinterpret_cast<uintptr_t>(a.Q)) % 16 == 0) &&
                          (a.ldq % 2 == 0 || a.jx == 0);
     if (!aligned || a.n < 64 * 32) return false;

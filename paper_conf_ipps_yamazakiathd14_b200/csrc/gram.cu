@@ -33,7 +33,6 @@ namespace {
 constexpr int GR_NT = 512;               // 16 warps = 8 pairs, one CTA per SM
 constexpr int GR_TW = 64;                // rows per tile (2 per lane: one LDS.128 per column)
 constexpr int GR_NP = GR_NT / 64;        // warp pairs
-constexpr bool GR_PF = false;            // L2 prefetch beyond the ring: measured no gain (50.8 vs 50.2 us)
 
 template <int W>
 __host__ __device__ constexpr int gram_stages() { return W <= 6 ? 6 : (W <= 8 ? 5 : 4); }
@@ -75,7 +74,7 @@ __device__ __forceinline__ void gram_pair_body(const GramArgs& a, double* smg, d
     const int64_t T = a.n / GR_TW;                                 // full tiles
     const int64_t NPg = int64_t(gridDim.x) * GR_NP;
     const int64_t g = int64_t(blockIdx.x) * GR_NP + pair;
-    const int64_t t0 = g * T / NPg, t1 = (g + 1) * T / NPg;
+    const int64_t cnt = band_count(T, NPg, g);                    // tiles of this pair (band order)
     // this thread's 16-B chunks of a tile (pair-thread q = 64 k + pt): fixed offsets
     constexpr int CPC = GR_TW * 8 / 16;                            // 16-B chunks per column tile
     constexpr int NCH = W * CPC;
@@ -90,9 +89,9 @@ __device__ __forceinline__ void gram_pair_body(const GramArgs& a, double* smg, d
         gof[k] = q < NCH ? a.ldp * c + part * 2 : -1;
         sof[k] = c * GR_TW + part * 2;
     }
-    auto issue = [&](int64_t t, double* slot) {
-        if (t < t1) {
-            const double* src = a.P + t * GR_TW;
+    auto issue = [&](int64_t i, double* slot) {
+        if (i < cnt) {
+            const double* src = a.P + band_tile(T, NPg, g, i, a.rev) * GR_TW;
 #pragma unroll
             for (int k = 0; k < KC; ++k)
                 if (k * 64 + 63 < NCH || gof[k] >= 0) ptx::cp_async16(slot + sof[k], src + gof[k]);
@@ -103,17 +102,14 @@ __device__ __forceinline__ void gram_pair_body(const GramArgs& a, double* smg, d
 #pragma unroll
     for (int e = 0; e < NA; ++e) acc[e] = 0.0;
 #pragma unroll
-    for (int s = 0; s < S - 1; ++s) issue(t0 + s, ring + s * stage_d);
+    for (int s = 0; s < S - 1; ++s) issue(s, ring + s * stage_d);
     double* cur = ring;                                            // slot of tile t
     double* nxt = ring + (S - 1) * stage_d;                        // slot refilled at step t
     double* const rend = ring + S * stage_d;
-    for (int64_t t = t0; t < t1; ++t) {
-        ptx::cp_async_wait<S - 2>();                               // my copies of tile t landed
+    for (int64_t i = 0; i < cnt; ++i) {
+        ptx::cp_async_wait<S - 2>();                               // my copies of tile i landed
         pair_sync(pair);                                           // ... and my partner's; slot
-        issue(t + S - 1, nxt);                                     //  of step t-1 is free
-        if (GR_PF && a.pf && t + S - 1 + ptx::PF_DIST < t1 && pt < W * (GR_TW / 16))   // 128-B lines, tile +PF
-            ptx::prefetch_l2(a.P + a.ldp * (pt / (GR_TW / 16)) + (t + S - 1 + ptx::PF_DIST) * GR_TW +
-                             16 * (pt % (GR_TW / 16)));
+        issue(i + S - 1, nxt);                                     //  of step i-1 is free
         if (HI > LO) rank1_part<W, LO, (HI > LO ? HI : LO + 1)>(cur, lane, acc);
         cur += stage_d; if (cur == rend) cur = ring;
         nxt += stage_d; if (nxt == rend) nxt = ring;
@@ -186,14 +182,14 @@ __global__ void __launch_bounds__(GW_NW * 32, 1) k_gram_warp(GramArgs a) {
     const int64_t T = a.n / 32;
     const int64_t Wn = int64_t(gridDim.x) * GW_NW;
     const int64_t g = int64_t(blockIdx.x) * GW_NW + wp;
-    const int64_t t0 = g * T / Wn, t1 = (g + 1) * T / Wn;
+    const int64_t cnt = band_count(T, Wn, g);
     const int part2 = 2 * (lane & 15), cfirst = lane >> 4;
     const double* srcl = a.P + a.ldp * cfirst + part2;
     const int64_t cstride = 2 * a.ldp;
-    auto issue = [&](int64_t t, int stage) {
-        if (t < t1) {
+    auto issue = [&](int64_t i, int stage) {
+        if (i < cnt) {
             double* dst = ring + stage * SD + cfirst * 32 + part2;
-            const double* src = srcl + t * 32;
+            const double* src = srcl + band_tile(T, Wn, g, i, a.rev) * 32;
 #pragma unroll
             for (int c = cfirst; c < W; c += 2, dst += 64, src += cstride) ptx::cp_async16(dst, src);
         }
@@ -213,10 +209,10 @@ __global__ void __launch_bounds__(GW_NW * 32, 1) k_gram_warp(GramArgs a) {
             for (int k = i; k < W; ++k, ++e) acc[e] = fma(v[i], v[k], acc[e]);
     };
 #pragma unroll
-    for (int s = 0; s < GW_S - 1; ++s) issue(t0 + s, s);
+    for (int s = 0; s < GW_S - 1; ++s) issue(s, s);
     int stage = 0;
-    for (int64_t t = t0; t < t1; ++t) {
-        issue(t + GW_S - 1, stage == 0 ? GW_S - 1 : stage - 1);
+    for (int64_t i = 0; i < cnt; ++i) {
+        issue(i + GW_S - 1, stage == 0 ? GW_S - 1 : stage - 1);
         ptx::cp_async_wait<GW_S - 1>();
         __syncwarp();
         rank1(ring + stage * SD + lane);
@@ -257,7 +253,9 @@ __global__ void __launch_bounds__(GW_NW * 32, 1) k_gram_warp(GramArgs a) {
     }
 }
 
-int gram_warp(const Dev& d, const GramArgs& a, cudaStream_t st) {
+int gram_warp(const Dev& d, const GramArgs& a0, cudaStream_t st) {
+    GramArgs a = a0;
+    a.rev = d.rev;
     auto go = [&](auto kfn) {
         size_t smem = size_t(GW_NW) * GW_S * a.w * 32 * sizeof(double);
         const size_t need = size_t(32 * 32) * sizeof(double);
@@ -279,7 +277,9 @@ int gram_warp(const Dev& d, const GramArgs& a, cudaStream_t st) {
     return 0;
 }
 
-int gram_dfma(const Dev& d, const GramArgs& a, cudaStream_t st) {
+int gram_dfma(const Dev& d, const GramArgs& a0, cudaStream_t st) {
+    GramArgs a = a0;
+    a.rev = d.rev;
     const bool aligned = (reinterpret_cast<uintptr_t>(a.P) % 16 == 0) && a.ldp % 2 == 0;
     if (!aligned || a.w < 1 || a.w > 12 || a.n < 64 * GR_TW) return -1;
     if (d.gram == 2 && gram_warp(d, a, st) == 0) return 0;

@@ -41,9 +41,21 @@ struct Dev {
     int trsm_scalar = 1;        // CholQR/SVQR update: 1 = scalar DFMA ring (w <= 16), 0 = DMMA
     int panel_tw16 = 1;
     int panel_pf = 1;           // panel rings: L2 prefetch PF_DIST tiles beyond the cp.async window
-    int serp = 3;               // CAGMRES_OPT_SERP bits: kernels that run their row ranges in reverse
-                                // (serpentine order with the predecessor: its last tiles are L2 hits)
+    int rev = 0;                // direction of the next streaming launch (serpentine order, solver.cu)
 };
+
+// Tile order of the streaming kernels (DESIGN.md §6 "serpentine order").  Unit g of NU (a warp,
+// or a warp pair) handles the tiles g, g + NU, g + 2 NU, ... of the T full tiles, so a band of NU
+// consecutive tiles sweeps the panel and the temporal order is global, independent of the grid
+// geometry; rev = 1 sweeps from the last tile down.  A kernel launched opposite to its
+// predecessor first reads the rows the predecessor touched last — still in the 126 MB L2.
+__host__ __device__ __forceinline__ int64_t band_count(int64_t T, int64_t NU, int64_t g) {
+    return g < T ? (T - 1 - g) / NU + 1 : 0;
+}
+__host__ __device__ __forceinline__ int64_t band_tile(int64_t T, int64_t NU, int64_t g, int64_t i, int rev) {
+    const int64_t t = g + i * NU;
+    return rev ? T - 1 - t : t;
+}
 
 // Sliced ELLPACK, slice height 32 (one warp), column-major inside a slice, with per-slice
 // diagonal-offset column compression: sinfo[sl] = dptr << 2 | clamp << 1 | dia.
@@ -59,7 +71,6 @@ struct Sell {
     int64_t ncols = 0;          // valid x entries (clamp bound for DIA slices)
     int64_t ndcol = 0, ndia = 0;
     int dia_w = 0;              // most common width of the unclamped DIA slices (spmv_dia.cu)
-    int rev = 0;                // next DIA SpMV launch visits the slices in descending order (serpentine)
     int64_t* sptr = nullptr;    // nslices+1 value offsets
     int64_t* sinfo = nullptr;   // nslices
     int32_t* dcol = nullptr;    // DIA offsets / explicit column ids
@@ -217,6 +228,7 @@ struct ArnoldiArgs {
     int* status;
     int sqrt_out;
     double* vout = nullptr;     // modes 1 / 2: write the updated v here instead of in place
+    int rev = 0;                // tile order (band_tile); set from Dev::rev by the launcher
 };
 int arnoldi_fused(const Dev& d, const ArnoldiArgs& a, int mode, cudaStream_t st);
 // p -= X c, p a single column (n), X n x jx (jx <= 32), c device jx-vector; -1 if not applicable
@@ -298,6 +310,7 @@ struct GramArgs {
     int fin_chol;
     double* R;
     int* status;
+    int rev = 0;                // tile order (band_tile); set from Dev::rev by the launcher
 };
 int gram_dfma(const Dev& d, const GramArgs& a, cudaStream_t st);
 

@@ -110,6 +110,10 @@ struct cagmres {
     // pass whose R (and C) the host applies.
     bool fold = true;
     int fold_kind = 0, fold_pass = 0;
+    // CAGMRES_OPT_SERP (default on): serpentine order — every streaming launch (SpMV, panel ring
+    // kernels) sweeps the rows opposite to the previous one (kern::band_tile), so it first reads
+    // what its predecessor touched last, still in L2.  Reset at the start of every cycle.
+    bool serp = true;
     int* status = nullptr;
     double ms_setup = 0.0;                 // wall time of create
     // CUDA graph of one CA cycle (single rank, untimed solves): captured once per configuration
@@ -120,6 +124,7 @@ struct cagmres {
     double cyc_bytes[PH_N] = {0, 0, 0, 0, 0};
     int cyc_spmv = 0;
     long long cyc_launches = 0;
+    int cyc_rev_end = 0;
     bool use_graphs = false;               // CAGMRES_OPT_GRAPH (measured neutral on C2: off)
     bool capturing = false;
     int graph_err = 0;                     // cudaError_t of a failed capture (graphs then off)
@@ -194,6 +199,12 @@ struct Scope {
 };
 
 int64_t round_up(int64_t a, int64_t b) { return (a + b - 1) / b * b; }
+
+// Device descriptor for the next streaming launch: flips the sweep direction (OPT_SERP).
+kern::Dev& sdev(cagmres* h) {
+    h->dev.rev = h->serp ? (h->dev.rev ^ 1) : 0;
+    return h->dev;
+}
 
 // ---- SELL-32 build (host) + upload ------------------------------------------------------
 // SELL-32 upload of the host layout built by sell_build (sell.cpp).
@@ -578,11 +589,11 @@ int halo(cagmres* h, double* vec, int depth) {
 int xty_global(cagmres* h, const double* X, int64_t ldx, int jx, const double* Y, int64_t ldy,
                int w, double* out, bool chol, double* R) {
     if (h->nranks == 1) {
-        if (kern::xty(h->dev, h->n_loc, X, ldx, jx, Y, ldy, w, out, chol, R, h->status, h->ws, h->stream))
+        if (kern::xty(sdev(h), h->n_loc, X, ldx, jx, Y, ldy, w, out, chol, R, h->status, h->ws, h->stream))
             return CAGMRES_EINVAL;
         return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
     }
-    if (kern::xty(h->dev, h->n_loc, X, ldx, jx, Y, ldy, w, out, false, nullptr, h->status, h->ws, h->stream))
+    if (kern::xty(sdev(h), h->n_loc, X, ldx, jx, Y, ldy, w, out, false, nullptr, h->status, h->ws, h->stream))
         return CAGMRES_EINVAL;
     if (chol && h->peer_ok && w <= 32) {
         // one-sided: the cross-rank sum of the Gram and its Cholesky in one launch reading the
@@ -682,20 +693,18 @@ int mpk_block(cagmres* h, int j, int sb, const std::vector<host::Step>& steps) {
         double* y = h->V + size_t(h->ldv) * (j + k);
         const int64_t rows = h->level_len[size_t(sb - k)];
         const bool pair2 = stp.kind == 2;
-        h->A.rev = (h->dev.serp & 2) && (k & 1) == 0 ? 1 : 0;   // OPT_SERP bit 1: even steps reversed
         {
             Scope sv(h, PH_SPMV);
             if (k == 1 && fused_q) {       // q_j = S / ||S|| formed inside the first step (stored to V[:, j])
-                if (kern::spmv_scaled(h->dev, h->A, rows, h->S, h->pend_nrm, h->V + size_t(h->ldv) * j, y, -stp.a,
+                if (kern::spmv_scaled(sdev(h), h->A, rows, h->S, h->pend_nrm, h->V + size_t(h->ldv) * j, y, -stp.a,
                                       stp.a != 0.0, h->stream))
                     return CAGMRES_EINVAL;
                 h->pend = false;
             } else {
-                kern::spmv(h->dev, h->A, rows, x, y, (stp.a != 0.0 || pair2) ? x : nullptr, -stp.a,
+                kern::spmv(sdev(h), h->A, rows, x, y, (stp.a != 0.0 || pair2) ? x : nullptr, -stp.a,
                            pair2 ? h->V + size_t(h->ldv) * (j + k - 2) : nullptr, stp.b2, h->stream);
             }
         }
-        h->A.rev = 0;
         const double by = spmv_bytes(h, rows, sb - k + 1, pair2);
         h->bytes[PH_MPK] += by;
         h->bytes[PH_SPMV] += by;
@@ -713,14 +722,14 @@ int borth_panel(cagmres* h, const double* Q, int64_t ldq, int j, double* P, int6
     if (!mgs) {
         TRY(xty_global(h, Q, ldq, j, P, ldp, w, C, false, nullptr));
         // C is jx x w with ld jx = j: xty writes ld jx
-        kern::update(h->dev, h->n_loc, Q, ldq, j, P, ldp, w, C, h->stream, true);   // after xty: early start
+        kern::update(sdev(h), h->n_loc, Q, ldq, j, P, ldp, w, C, h->stream, true);   // after xty: early start
         h->bytes[PH_BORTH] += 8.0 * double(h->n_loc) * (2.0 * j + 3.0 * w);
     } else {
         // row l of C (1 x w, ld j) via a scratch row then copied with ld j on the host view:
         for (int l = 0; l < j; ++l) {
             double* row = h->gbuf;
             TRY(xty_global(h, Q + size_t(ldq) * l, ldq, 1, P, ldp, w, row, false, nullptr));
-            kern::update(h->dev, h->n_loc, Q + size_t(ldq) * l, ldq, 1, P, ldp, w, row, h->stream);
+            kern::update(sdev(h), h->n_loc, Q + size_t(ldq) * l, ldq, 1, P, ldp, w, row, h->stream);
             CU(cudaMemcpy2DAsync(C + l, sizeof(double) * size_t(j), row, sizeof(double), sizeof(double),
                                  size_t(w), cudaMemcpyDeviceToDevice, h->stream));
             h->bytes[PH_BORTH] += 8.0 * double(h->n_loc) * (2.0 + 3.0 * w);
@@ -747,7 +756,7 @@ int tsqr_panel(cagmres* h, double* P, int64_t ldp, int w, double* R, int kind, i
         if (skip_update) {
             h->bytes[PH_TSQR] += 8.0 * nl * w;
         } else {
-            kern::trsm(h->dev, h->n_loc, P, ldp, w, R, c0, h->stream, true);    // V := V R^{-1} (P final: early)
+            kern::trsm(sdev(h), h->n_loc, P, ldp, w, R, c0, h->stream, true);    // V := V R^{-1} (P final: early)
             h->bytes[PH_TSQR] += 8.0 * nl * (2.0 * w + double(w - c0));
         }
     } else if (kind == CAGMRES_CAQR) {                       // Fig. 9 CAQR: TSQR tree
@@ -784,7 +793,7 @@ int tsqr_panel(cagmres* h, double* P, int64_t ldp, int w, double* R, int kind, i
                                      sizeof(double) * size_t(w), sizeof(double) * size_t(w), size_t(w),
                                      cudaMemcpyDeviceToDevice, h->stream));
             if (kern::caqr(h->dev, sr, Stk, sr, w, R, 0, ws2, h->stream)) return CAGMRES_EINVAL;
-            if (kern::gemm_rows(h->dev, h->n_loc, P, ldp, w, P, ldp, w, Stk + size_t(h->rank) * w, sr, c0, h->stream))
+            if (kern::gemm_rows(sdev(h), h->n_loc, P, ldp, w, P, ldp, w, Stk + size_t(h->rank) * w, sr, c0, h->stream))
                 return CAGMRES_EINVAL;
             if (c0 == 1) CU(cudaMemcpyAsync(P, q0, sizeof(double) * size_t(h->n_loc), cudaMemcpyDeviceToDevice, h->stream));
         }
@@ -796,20 +805,20 @@ int tsqr_panel(cagmres* h, double* P, int64_t ldp, int w, double* R, int kind, i
             if (k > 0) {
                 if (kind == CAGMRES_CGS) {          // Fig. 9 right: r = V_{1:k-1}^T v_k
                     TRY(xty_global(h, P, ldp, k, pk, ldp, 1, R + size_t(w) * k, false, nullptr));
-                    kern::update(h->dev, h->n_loc, P, ldp, k, pk, ldp, 1, R + size_t(w) * k, h->stream);
+                    kern::update(sdev(h), h->n_loc, P, ldp, k, pk, ldp, 1, R + size_t(w) * k, h->stream);
                     h->bytes[PH_TSQR] += 8.0 * nl * (2.0 * k + 3.0);
                 } else {                             // Fig. 9 left: one dot at a time
                     for (int l = 0; l < k; ++l) {
                         double* rl = R + l + size_t(w) * k;
                         TRY(xty_global(h, P + size_t(ldp) * l, ldp, 1, pk, ldp, 1, rl, false, nullptr));
-                        kern::update(h->dev, h->n_loc, P + size_t(ldp) * l, ldp, 1, pk, ldp, 1, rl, h->stream);
+                        kern::update(sdev(h), h->n_loc, P + size_t(ldp) * l, ldp, 1, pk, ldp, 1, rl, h->stream);
                         h->bytes[PH_TSQR] += 8.0 * nl * 5.0;
                     }
                 }
             }
             double* rkk = R + k + size_t(w) * k;
             TRY(xty_global(h, pk, ldp, 1, pk, ldp, 1, h->gbuf, true, rkk));   // r_kk = ||v_k||
-            if (k >= c0) kern::trsm(h->dev, h->n_loc, pk, ldp, 1, rkk, 0, h->stream);
+            if (k >= c0) kern::trsm(sdev(h), h->n_loc, pk, ldp, 1, rkk, 0, h->stream);
             h->bytes[PH_TSQR] += 8.0 * nl * (k >= c0 ? 3.0 : 1.0);
         }
     }
@@ -896,7 +905,7 @@ int ca_cycle(cagmres* h, const std::vector<Block>& bl) {
                 Scope sc(h, PH_TSQR);
                 kern::onepass_finalize(h->gbuf, j, w, C, R, h->op_M, h->status, h->stream);
                 if (fold) { h->fold_kind = 2; h->fold_pass = pass; continue; }
-                if (kern::gemm_rows(h->dev, h->n_loc, h->V, h->ldv, j + w, Pj, h->ldv, w, h->op_M, j + w, 1,
+                if (kern::gemm_rows(sdev(h), h->n_loc, h->V, h->ldv, j + w, Pj, h->ldv, w, h->op_M, j + w, 1,
                                     h->stream, true))
                     return CAGMRES_EINVAL;
                 h->bytes[PH_TSQR] += 8.0 * nl * (j + w + (w - 1));
@@ -911,9 +920,9 @@ int ca_cycle(cagmres* h, const std::vector<Block>& bl) {
                     TRY(xty_global(h, h->V, h->ldv, j, Pj + h->ldv, h->ldv, sb, C, false, nullptr));
                     kern::UpdGramArgs ua{h->n_loc, h->V, h->ldv, j, Pj + h->ldv, h->ldv, sb, Pj, C, h->ws.part,
                                          h->gbuf, h->ws.counter, h->nranks == 1 ? 1 : 0, R, h->status};
-                    fused = kern::update_gram(h->dev, ua, h->stream);
+                    fused = kern::update_gram(sdev(h), ua, h->stream);
                     if (fused == 0) h->bytes[PH_BORTH] += 8.0 * nl * (2.0 * j + 3.0 * sb);
-                    else kern::update(h->dev, h->n_loc, h->V, h->ldv, j, Pj + h->ldv, h->ldv, sb, C, h->stream);
+                    else kern::update(sdev(h), h->n_loc, h->V, h->ldv, j, Pj + h->ldv, h->ldv, sb, C, h->stream);
                 }
                 if (fused == 0) {
                     Scope sc(h, PH_TSQR);
@@ -922,7 +931,7 @@ int ca_cycle(cagmres* h, const std::vector<Block>& bl) {
                         kern::chol(h->gbuf, w, R, h->status, h->stream);
                     }
                     if (fold) { h->fold_kind = 1; h->fold_pass = pass; continue; }
-                    kern::trsm(h->dev, h->n_loc, Pj, h->ldv, w, R, 1, h->stream);
+                    kern::trsm(sdev(h), h->n_loc, Pj, h->ldv, w, R, 1, h->stream);
                     h->bytes[PH_TSQR] += 8.0 * nl * (2.0 * w + double(w - 1));   // Gram bytes as if unfused
                     continue;
                 }
@@ -962,11 +971,11 @@ int arnoldi_cycle(cagmres* h, bool cgs2) {
             TRY(start_halo(h, k, 1, fused_q));
             Scope sv(h, PH_SPMV);
             if (fused_q) {                 // v_k = S / ||S|| formed inside the SpMV (stored to V[:, k])
-                if (kern::spmv_scaled(h->dev, h->A, h->n_loc, h->S, h->pend_nrm, vk, v, 0.0, false, h->stream))
+                if (kern::spmv_scaled(sdev(h), h->A, h->n_loc, h->S, h->pend_nrm, vk, v, 0.0, false, h->stream))
                     return CAGMRES_EINVAL;
                 h->pend = false;
             } else {
-                kern::spmv(h->dev, h->A, h->n_loc, vk, v, nullptr, 0.0, nullptr, 0.0, h->stream);
+                kern::spmv(sdev(h), h->A, h->n_loc, vk, v, nullptr, 0.0, nullptr, 0.0, h->stream);
             }
             const double by = spmv_bytes(h, h->n_loc, 1, false);
             h->bytes[PH_MPK] += by; h->bytes[PH_SPMV] += by; h->spmv_launches++;
@@ -979,11 +988,11 @@ int arnoldi_cycle(cagmres* h, bool cgs2) {
             {
                 Scope sc(h, PH_BORTH);
                 aa.c_out = c1;
-                if (kern::arnoldi_fused(h->dev, aa, 0, h->stream)) return CAGMRES_EINVAL;
+                if (kern::arnoldi_fused(sdev(h), aa, 0, h->stream)) return CAGMRES_EINVAL;
                 TRY(allreduce(h, c1, size_t(k + 1)));
                 if (cgs2) {
                     aa.c_in = c1; aa.c_out = c2;
-                    if (kern::arnoldi_fused(h->dev, aa, 1, h->stream)) return CAGMRES_EINVAL;
+                    if (kern::arnoldi_fused(sdev(h), aa, 1, h->stream)) return CAGMRES_EINVAL;
                     TRY(allreduce(h, c2, size_t(k + 1)));
                     h->bytes[PH_BORTH] += 8.0 * nl * (3.0 * (k + 1) + 4.0);
                 } else {
@@ -994,7 +1003,7 @@ int arnoldi_cycle(cagmres* h, bool cgs2) {
                 Scope sc(h, PH_TSQR);
                 aa.c_in = cgs2 ? c2 : c1; aa.c_out = r;
                 aa.vout = h->fuse_scale ? h->S : nullptr;          // w -> S, normalised by the next SpMV
-                if (kern::arnoldi_fused(h->dev, aa, 2, h->stream)) return CAGMRES_EINVAL;
+                if (kern::arnoldi_fused(sdev(h), aa, 2, h->stream)) return CAGMRES_EINVAL;
                 aa.vout = nullptr;
                 if (h->nranks > 1) {
                     TRY(allreduce(h, r, 1));
@@ -1004,7 +1013,7 @@ int arnoldi_cycle(cagmres* h, bool cgs2) {
                     h->pend = true; h->pend_nrm = r; h->pend_col = k + 1;
                     h->bytes[PH_TSQR] += 8.0 * nl * ((k + 1) + 2.0);
                 } else {
-                    kern::trsm(h->dev, h->n_loc, v, h->ldv, 1, r, 0, h->stream);
+                    kern::trsm(h->dev, h->n_loc, v, h->ldv, 1, r, 0, h->stream);   // (w = 1: no sweep order)
                     h->bytes[PH_TSQR] += 8.0 * nl * ((k + 1) + 2.0 + 2.0);
                 }
             }
@@ -1030,12 +1039,12 @@ int residual_norm_async(cagmres* h, const double* b, const double* x) {
         xx = h->xe;
     }
     double* rv = h->fuse_scale ? h->S : h->V;          // r: unnormalised in S (fused) or in V[:, 0]
-    kern::residual(h->dev, h->A, h->n_loc, xx, b, rv, h->stream);
+    kern::residual(sdev(h), h->A, h->n_loc, xx, b, rv, h->stream);
     double* rr = h->gbuf + 8;
     {   // ||r|| by the scalar reduction kernel (mode 2 with no Q columns)
         kern::ArnoldiArgs aa{h->dev.panel_pf, h->n_loc, h->V, h->ldv, 0, rv, nullptr, rr, h->arn_part, h->arn_counter,
                              h->status, h->nranks == 1 ? 1 : 0};
-        if (kern::arnoldi_fused(h->dev, aa, 2, h->stream)) return CAGMRES_EINVAL;
+        if (kern::arnoldi_fused(sdev(h), aa, 2, h->stream)) return CAGMRES_EINVAL;
         if (h->nranks > 1) {
             TRY(allreduce(h, rr, 1));
             kern::chol(rr, 1, rr, h->status, h->stream);
@@ -1047,7 +1056,7 @@ int residual_norm_async(cagmres* h, const double* b, const double* x) {
         h->pend = true; h->pend_nrm = rr; h->pend_col = 0;
         h->bytes[PH_OTHER] += spmv_bytes(h, h->n_loc, 1, false) + 8.0 * double(h->n_loc);
     } else {
-        kern::trsm(h->dev, h->n_loc, h->V, h->ldv, 1, rr, 0, h->stream);     // q_0 = r / beta
+        kern::trsm(h->dev, h->n_loc, h->V, h->ldv, 1, rr, 0, h->stream);     // q_0 = r / beta (w = 1)
         h->bytes[PH_OTHER] += spmv_bytes(h, h->n_loc, 1, false) + 8.0 * double(h->n_loc) * 3.0;
     }
     return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
@@ -1055,6 +1064,7 @@ int residual_norm_async(cagmres* h, const double* b, const double* x) {
 
 // One restart cycle's GPU work plus the async copy of its coefficient table and status.
 int enqueue_cycle(cagmres* h, bool arnoldi, const std::vector<Block>& bl) {
+    h->dev.rev = 1;                        // the cycle's first streaming launch sweeps forward
     if (arnoldi) {
         // standard GMRES as the paper runs it: CGS Arnoldi (Fig. 14 "GMRES ... CGS" rows), CGS2
         // with CAGMRES_REORTH — for the shift-finding Newton cycle (G12) and the baseline
@@ -1125,9 +1135,11 @@ int enqueue_ca_cycle(cagmres* h, const std::vector<Block>& bl) {
         h->spmv_launches = s0;
         h->cyc_launches = kern::g_launches - l0;
         kern::g_launches = l0;
+        h->cyc_rev_end = h->dev.rev;
         h->cyc_version = key;
     }
     CU(cudaGraphLaunch(h->cyc_exec, h->stream));
+    h->dev.rev = h->cyc_rev_end;           // the sweep state a stream-launched cycle ends in
     for (int p = 0; p < PH_N; ++p) h->bytes[p] += h->cyc_bytes[p];
     h->spmv_launches += h->cyc_spmv;
     kern::g_launches += h->cyc_launches;
@@ -1265,7 +1277,7 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
             h->fuse_borth_gram = (value & 1) != 0; h->arnoldi_fuse = (value & 2) != 0; h->fuse_scale = (value & 4) != 0;
             return CAGMRES_OK;
         case CAGMRES_OPT_FOLD: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->fold = value != 0; return CAGMRES_OK;
-        case CAGMRES_OPT_SERP: if (value < 0 || value > 255) return CAGMRES_EINVAL; h->dev.serp = int(value); return CAGMRES_OK;
+        case CAGMRES_OPT_SERP: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->serp = value != 0; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK:
             if (value < 256 || value % 256) return CAGMRES_EINVAL;
             h->wave_CH = int(value); wave_reset_pairs(h); return CAGMRES_OK;
@@ -1292,7 +1304,7 @@ int cagmres_get_option(cagmres_t h, int opt, int64_t* value) {
             *value = (h->fuse_borth_gram ? 1 : 0) | (h->arnoldi_fuse ? 2 : 0) | (h->fuse_scale ? 4 : 0);
             return CAGMRES_OK;
         case CAGMRES_OPT_FOLD: *value = h->fold ? 1 : 0; return CAGMRES_OK;
-        case CAGMRES_OPT_SERP: *value = h->dev.serp; return CAGMRES_OK;
+        case CAGMRES_OPT_SERP: *value = h->serp ? 1 : 0; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK: *value = h->wave_CH; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CTAS: *value = h->wave_ctas; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_LAG: *value = h->wave_lag; return CAGMRES_OK;
@@ -1340,6 +1352,7 @@ int cagmres_mpk(cagmres_t h, const double* q, double* W, int64_t ldw, int sb) {
     if (!h || !q || !W || sb < 1 || sb > h->s || ldw < h->n_loc || sb > h->m) return CAGMRES_EINVAL;
     if (h->basis == CAGMRES_NEWTON && !h->have_shifts) return CAGMRES_EINVAL;
     h->pend = false;
+    h->dev.rev = 1;                        // sweep order restarts with every call (deterministic)
     CU(cudaMemcpyAsync(h->V, q, sizeof(double) * size_t(h->n_loc), cudaMemcpyDeviceToDevice, h->stream));
     const std::vector<host::Step> steps = h->basis != CAGMRES_NEWTON
         ? host::block_steps({}, {}, sb) : host::block_steps(h->sh_re, h->sh_im, sb);
@@ -1356,6 +1369,7 @@ int cagmres_borth(cagmres_t h, const double* Q, int64_t ldq, int j, double* P, i
     if (!h || j < 0 || w < 1 || w > 32 || ldq < h->n_loc || ldp < h->n_loc) return CAGMRES_EINVAL;
     if (j == 0) return CAGMRES_OK;
     if (!Q || !P || !C || j > int(h->tab_cap)) return CAGMRES_EINVAL;
+    h->dev.rev = 1;
     TRY(borth_panel(h, Q, ldq, j, P, ldp, w, C, (h->orth & CAGMRES_BORTH_MGS) != 0));
     CU(cudaStreamSynchronize(h->stream));
     h->timer.reset();
@@ -1369,6 +1383,7 @@ int cagmres_tsqr(cagmres_t h, double* P, int64_t ldp, int w, double* R, int orth
     CU(cudaMemsetAsync(h->status, 0, sizeof(int), h->stream));
     const bool retry = (orth & CAGMRES_SVQR_RETRY) && kind == CAGMRES_CHOLQR;
     CU(cudaMemsetAsync(h->status, 0, sizeof(int) * 2, h->stream));
+    h->dev.rev = 1;
     TRY(tsqr_panel(h, P, ldp, w, R, kind, 0, retry));
     if (orth & CAGMRES_REORTH) {
         double* R2 = h->tab;                        // scratch
@@ -1409,6 +1424,7 @@ int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit
     double max_orth = 0.0, max_cond = 0.0;
     if (h->diag_on) TRY(diag_alloc(h));
     double rho0 = 0.0, beta = 0.0;
+    h->dev.rev = 1;                        // sweep order: every solve starts the same way
     TRY(residual_norm_async(h, b, x));
     CU(cudaEventSynchronize(h->ev_beta));
     rho0 = *h->h_beta;
@@ -1512,7 +1528,7 @@ int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit
         {
             Scope sc(h, PH_OTHER);
             CU(cudaMemcpyAsync(h->ybuf, h->h_y, sizeof(double) * size_t(ncoef), cudaMemcpyHostToDevice, h->stream));
-            kern::update(h->dev, h->n_loc, h->V, h->ldv, ncoef, x, h->n_loc, 1, h->ybuf, h->stream);
+            kern::update(sdev(h), h->n_loc, h->V, h->ldv, ncoef, x, h->n_loc, 1, h->ybuf, h->stream);
             h->bytes[PH_OTHER] += 8.0 * double(h->n_loc) * (ncoef + 2.0);
         }
         TRY(residual_norm_async(h, b, x));                        // r, beta, q_0 for the next cycle

@@ -34,7 +34,7 @@ struct DiaArgs {
     double* y;
     const double* xnrm;     // SX: x is an unnormalised w, the operand is w * (1 / *xnrm)
     double* xs;             // SX: the normalised operand's rows [0, nrows) are stored here
-    int rev;                // 1: slices visited in descending order (serpentine MPK steps)
+    int rev;                // 1: slices visited in descending order (serpentine order, Dev::rev)
 };
 }  // namespace
 
@@ -180,7 +180,7 @@ void go_width(const Dev& d, const DiaArgs& a, int wt, cudaStream_t st, int mode)
 void spmv_dia(const Dev& d, const Sell& A, int variant, int64_t nrows, const double* x, double* y,
               const double* u, double bu, const double* w, double bw, int mode, cudaStream_t st,
               const double* xnrm, double* xs) {
-    DiaArgs a{nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, u, bu, w, bw, y, xnrm, xs, A.rev};
+    DiaArgs a{nrows, A.sptr, A.sinfo, A.dcol, A.ncols, A.val, x, u, bu, w, bw, y, xnrm, xs, d.rev};
     if (variant == 17) go_width<5>(d, a, A.dia_w, st, mode);
     else go_width<4>(d, a, A.dia_w, st, mode);
 }

@@ -33,10 +33,7 @@ struct StreamArgs {
     // produced C / R), so the ring kernels issue their first tile copies BEFORE
     // griddepcontrol.wait and fill their pipelines while that kernel drains (PDL)
     int early = 0;
-    // 1: run every warp's tile range in descending order — the reverse of the predecessor's
-    // temporal order, so the first tiles read are the ones the predecessor touched last (still
-    // in L2).  Row-wise kernels only (no reduction): results are identical either way.
-    int rev = 0;
+    int rev = 0;                              // tile order (band_tile), from Dev::rev
 };
 
 // R^{-1} (upper, w x w) into sRi[k*32 + c]; one thread per column (back substitution)
@@ -173,16 +170,16 @@ __global__ void __launch_bounds__(MAXT, 1) k_rows_pipe(StreamArgs a) {
     const int64_t T = a.n / TW;
     const int64_t W = int64_t(gridDim.x) * nw;
     const int64_t g = int64_t(blockIdx.x) * nw + wp;
-    const int64_t t0 = g * T / W, t1 = (g + 1) * T / W;
+    const int64_t cnt = band_count(T, W, g);                  // tiles of this warp (band order)
     auto colptr = [&](int c) -> const double* { return sCol[c]; };
     // copy slots: lane covers 16-B part (lane % CPC) of columns lane / CPC, + 32 / CPC, ...
     constexpr int CPC = TW * 8 / 16;
     constexpr int CSTEP = 32 / CPC;
     const int part2 = 2 * (lane % CPC), cfirst = lane / CPC;
-    auto issue = [&](int64_t t, int stage) {
-        if (t < t1) {
+    auto issue = [&](int64_t i, int stage) {
+        if (i < cnt) {
             double* dst = ring + stage * stage_d + part2;
-            const int64_t r0 = t * TW + part2;
+            const int64_t r0 = band_tile(T, W, g, i, a.rev) * TW + part2;
 #pragma unroll 4
             for (int c = cfirst; c < ncol; c += CSTEP) ptx::cp_async16(dst + c * SP, sCol[c] + r0);
         }
@@ -202,10 +199,10 @@ __global__ void __launch_bounds__(MAXT, 1) k_rows_pipe(StreamArgs a) {
             const int c = 8 * nt + 2 * tig + h;
             pcol[nt][h] = (jxl + min(c, w - 1)) * SP;
             wcol[nt][h] = c < w && (MODE == 0 || c >= a.c0);
-            pst[nt][h] = a.P + a.ldp * min(c, w - 1) + gid + t0 * TW;
+            pst[nt][h] = a.P + a.ldp * min(c, w - 1) + gid;
         }
 #pragma unroll
-    for (int s = 0; s < RP_S - 1; ++s) issue(t0 + s, s);
+    for (int s = 0; s < RP_S - 1; ++s) issue(s, s);
     if (a.early) {                                             // X, P final before the predecessor
         pdl_wait();
         pdl_trigger();
@@ -223,16 +220,17 @@ __global__ void __launch_bounds__(MAXT, 1) k_rows_pipe(StreamArgs a) {
             b[kt][nt] = MODE == 0 ? -v : v;
         }
     int stage = 0, stage_in = RP_S - 1;
-    for (int64_t t = t0; t < t1; ++t) {
-        issue(t + RP_S - 1, stage_in);
-        if (d_pf && t + RP_S - 1 + ptx::PF_DIST < t1) {
-            const int64_t rp = (t + RP_S - 1 + ptx::PF_DIST) * TW;
+    for (int64_t i = 0; i < cnt; ++i) {
+        issue(i + RP_S - 1, stage_in);
+        if (d_pf && i + RP_S - 1 + ptx::PF_DIST < cnt) {
+            const int64_t rp = band_tile(T, W, g, i + RP_S - 1 + ptx::PF_DIST, a.rev) * TW;
             constexpr int LPC = TW / 16;                        // 128-B lines per column tile
             for (int q = lane; q < ncol * LPC; q += 32) ptx::prefetch_l2(colptr(q / LPC) + rp + 16 * (q % LPC));
         }
         ptx::cp_async_wait<RP_S - 1>();
         __syncwarp();
         const double* sl = ring + stage * stage_d + gid;
+        const int64_t toff = band_tile(T, W, g, i, a.rev) * TW;
         // per-tile operand pointers; the 8-row groups below are unrolled, so every shared load
         // and global store is [register + immediate]
         const double* sa[KTM];
@@ -261,12 +259,8 @@ __global__ void __launch_bounds__(MAXT, 1) k_rows_pipe(StreamArgs a) {
             for (int nt = 0; nt < NTN; ++nt)
 #pragma unroll
                 for (int h = 0; h < 2; ++h)
-                    if (wcol[nt][h]) __stcs(pst[nt][h] + 8 * g8, d[nt][h]);
-        }
-#pragma unroll
-        for (int nt = 0; nt < NTN; ++nt)
-#pragma unroll
-            for (int h = 0; h < 2; ++h) pst[nt][h] += TW;
+                    if (wcol[nt][h]) pst[nt][h][toff + 8 * g8] = d[nt][h];   // (L2-normal: the next
+        }                                                             //  kernel reads it, serpentine)
         __syncwarp();
         stage = stage == RP_S - 1 ? 0 : stage + 1;
         stage_in = stage_in == RP_S - 1 ? 0 : stage_in + 1;
@@ -432,13 +426,12 @@ __global__ void __launch_bounds__(256, 1) k_trsm_ring(StreamArgs a) {
     const int64_t T = a.n / TR;
     const int64_t Wn = int64_t(gridDim.x) * nw;
     const int64_t g = int64_t(blockIdx.x) * nw + wp;
-    const int64_t t0 = g * T / Wn, t1 = (g + 1) * T / Wn;
+    const int64_t cnt = band_count(T, Wn, g);
     const int c0 = a.c0;
-    auto issue = [&](int64_t t, int stage) {
-        if (t < t1) {
-            if (a.rev) t = t0 + t1 - 1 - t;
+    auto issue = [&](int64_t i, int stage) {
+        if (i < cnt) {
             double* dst = ring + stage * SD + 2 * lane;
-            const double* src = a.P + t * TR + 2 * lane;
+            const double* src = a.P + band_tile(T, Wn, g, i, a.rev) * TR + 2 * lane;
 #pragma unroll
             for (int c = 0; c < W; ++c) ptx::cp_async16(dst + c * TR, src + a.ldp * c);
         }
@@ -479,7 +472,7 @@ __global__ void __launch_bounds__(256, 1) k_trsm_ring(StreamArgs a) {
         }
     };
 #pragma unroll
-    for (int s = 0; s < RS - 1; ++s) issue(t0 + s, s);
+    for (int s = 0; s < RS - 1; ++s) issue(s, s);
     if (a.early) {                                             // P final before the Gram / Cholesky
         pdl_wait();
         pdl_trigger();
@@ -491,8 +484,8 @@ __global__ void __launch_bounds__(256, 1) k_trsm_ring(StreamArgs a) {
     }
     __syncthreads();
     int stage = 0;
-    for (int64_t t = t0; t < t1; ++t) {
-        issue(t + RS - 1, stage == 0 ? RS - 1 : stage - 1);
+    for (int64_t i = 0; i < cnt; ++i) {
+        issue(i + RS - 1, stage == 0 ? RS - 1 : stage - 1);
         ptx::cp_async_wait<RS - 1>();
         __syncwarp();
         const double* sl = ring + stage * SD + 2 * lane;
@@ -503,7 +496,7 @@ __global__ void __launch_bounds__(256, 1) k_trsm_ring(StreamArgs a) {
             v0[k] = p2.x;
             v1[k] = p2.y;
         }
-        rowout2(v0, v1, a.P + (a.rev ? t0 + t1 - 1 - t : t) * TR + 2 * lane);
+        rowout2(v0, v1, a.P + band_tile(T, Wn, g, i, a.rev) * TR + 2 * lane);
         __syncwarp();
         stage = stage == RS - 1 ? 0 : stage + 1;
     }
@@ -572,7 +565,7 @@ void update(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, doubl
     // a later slab follows a launch that wrote P: no early start for it
     for (int s0 = 0; s0 < jx; s0 += 64) {
         const int js = jx - s0 < 64 ? jx - s0 : 64;
-        StreamArgs a{n, X + ldx * s0, ldx, js, P, ldp, w, C + s0, jx, 0, d.panel_pf, early && s0 == 0 ? 1 : 0};
+        StreamArgs a{n, X + ldx * s0, ldx, js, P, ldp, w, C + s0, jx, 0, d.panel_pf, early && s0 == 0 ? 1 : 0, d.rev};
         dispatch<0>(d, a, st);
     }
 }
@@ -581,7 +574,7 @@ int gemm_rows(const Dev& d, int64_t n, const double* X, int64_t ldx, int K, doub
               const double* M, int64_t ldm, int c0, cudaStream_t st, bool early) {
     if (n <= 0 || w <= 0) return 0;
     if (K > 64 || w > 32) return -1;
-    StreamArgs a{n, X, ldx, K, P, ldp, w, M, ldm, c0, d.panel_pf, early ? 1 : 0};
+    StreamArgs a{n, X, ldx, K, P, ldp, w, M, ldm, c0, d.panel_pf, early ? 1 : 0, d.rev};
     return dispatch<2>(d, a, st);
 }
 
@@ -596,7 +589,7 @@ void trsm(const Dev& d, int64_t n, double* P, int64_t ldp, int w, const double* 
         launch_pdl(k_scale1, dim3(unsigned(g)), dim3(256), 0, st, n, P, R);
         return;
     }
-    StreamArgs a{n, nullptr, 0, 0, P, ldp, w, R, w, c0, d.panel_pf, early ? 1 : 0, (d.serp & 1) ? 1 : 0};
+    StreamArgs a{n, nullptr, 0, 0, P, ldp, w, R, w, c0, d.panel_pf, early ? 1 : 0, d.rev};
     if (d.trsm_scalar && trsm_ring(d, a, st)) return;
     dispatch<1>(d, a, st);
 }

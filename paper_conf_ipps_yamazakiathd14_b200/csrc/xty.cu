@@ -40,6 +40,7 @@ struct XtyArgs {
     double* R;
     int* status;
     int pf = 0;                 // L2 prefetch ahead of the ring (Dev::panel_pf)
+    int rev = 0;                // tile order (band_tile), from Dev::rev
 };
 
 // ---- CTA partial -> two-level fixed-order total (+ Cholesky) ---------------------------
@@ -184,7 +185,7 @@ __global__ void __launch_bounds__(NT, 1) k_xty_pipe(XtyArgs a) {
     const int64_t T = a.n / TW;                                    // full tiles
     const int64_t W = int64_t(gridDim.x) * nw;
     const int64_t g = int64_t(blockIdx.x) * nw + wp;
-    const int64_t t0 = g * T / W, t1 = (g + 1) * T / W;
+    const int64_t cnt = band_count(T, W, g);                      // tiles of this warp (band order)
     // columns: Y cols 0..w-1 at slot cols 0..w-1; X cols (if streamed) at w..w+nx-1
     const double* xbase = a.X == a.Y && !SYM ? a.Y + a.ldy * colbase : a.X + a.ldx * colbase;
     __shared__ const double* sCol[96];                             // column base pointers
@@ -194,10 +195,10 @@ __global__ void __launch_bounds__(NT, 1) k_xty_pipe(XtyArgs a) {
     constexpr int CPC = TW * 8 / 16;                               // 16-B chunks per column
     constexpr int CSTEP = 32 / CPC;
     const int part2 = 2 * (lane % CPC), cfirst = lane / CPC;
-    auto issue = [&](int64_t t, int stage) {
-        if (t < t1) {
+    auto issue = [&](int64_t i, int stage) {
+        if (i < cnt) {
             double* dst = ring + stage * stage_d + part2;
-            const int64_t r0 = t * TW + part2;
+            const int64_t r0 = band_tile(T, W, g, i, a.rev) * TW + part2;
 #pragma unroll 4
             for (int c = cfirst; c < ncol; c += CSTEP) ptx::cp_async16(dst + c * SP, sCol[c] + r0);
         }
@@ -219,12 +220,12 @@ __global__ void __launch_bounds__(NT, 1) k_xty_pipe(XtyArgs a) {
         for (int mt = 0; mt < MT; ++mt) xcol[mt] = (nx ? w : 0) + min(8 * mt + gid, nxc - 1);
     }
 #pragma unroll
-    for (int s = 0; s < PIPE_S - 1; ++s) issue(t0 + s, s);
+    for (int s = 0; s < PIPE_S - 1; ++s) issue(s, s);
     int stage = 0;
-    for (int64_t t = t0; t < t1; ++t) {
-        issue(t + PIPE_S - 1, (stage + PIPE_S - 1) % PIPE_S);
-        if (a.pf && TW == 32 && ncol <= 24 && t + PIPE_S - 1 + ptx::PF_DIST < t1) {   // narrow panels only
-            const int64_t rp = (t + PIPE_S - 1 + ptx::PF_DIST) * TW;
+    for (int64_t i = 0; i < cnt; ++i) {
+        issue(i + PIPE_S - 1, (stage + PIPE_S - 1) % PIPE_S);
+        if (a.pf && TW == 32 && ncol <= 24 && i + PIPE_S - 1 + ptx::PF_DIST < cnt) {   // narrow panels only
+            const int64_t rp = band_tile(T, W, g, i + PIPE_S - 1 + ptx::PF_DIST, a.rev) * TW;
             constexpr int LPC = TW / 16;
             for (int q = lane; q < ncol * LPC; q += 32) ptx::prefetch_l2(colptr(q / LPC) + rp + 16 * (q % LPC));
         }
@@ -425,7 +426,7 @@ int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const dou
     }
     Geo o = geometry(d, n, jx, w, same);
     if (size_t(o.gx) * o.gy * o.chunk * w * 2 > ws.cap || o.gy * TR_CNT > XTY_COUNTERS) return -1;
-    XtyArgs a{n, X, ldx, jx, Y, ldy, w, o.chunk, ws.part, out, ws.counter, fin_chol ? 1 : 0, R, status, d.panel_pf};
+    XtyArgs a{n, X, ldx, jx, Y, ldy, w, o.chunk, ws.part, out, ws.counter, fin_chol ? 1 : 0, R, status, d.panel_pf, d.rev};
     const bool aligned = ((reinterpret_cast<uintptr_t>(X) | reinterpret_cast<uintptr_t>(Y)) % 16 == 0) &&
                          (ldx % 2 == 0) && (ldy % 2 == 0);
     if (aligned && n >= 32 * 64) {

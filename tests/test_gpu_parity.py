@@ -164,6 +164,57 @@ def test_spmv_variants_bitwise(gen):
         assert torch.equal(Ws[i], Ws[0]), v
 
 
+@pytest.mark.parametrize("gen", ["cd7_ragged", "g3_small"])
+def test_serpentine_order(gen):
+    """CAGMRES_OPT_SERP: every streaming kernel sweeps the rows opposite to its
+    predecessor (band order, kern::band_tile).  Row-wise kernels are unchanged: the MPK basis is
+    bitwise that of the all-forward order for every SpMV variant.  The reductions (Gram, xTy,
+    norms) sum the same products in another fixed order: R and Q agree to rounding, and the
+    solve matches the oracle under the §8 rule either way (and reproduces itself bit for bit)."""
+    A = {"g3_small": lambda: G.g3_shaped(n=40000, width=200),
+         "cd7_ragged": lambda: G.convection_diffusion(45, 3, 7)}[gen]()
+    As = A.to_scipy()
+    q = dev(G.u(6, np.arange(A.n)))
+    W = {}
+    for serp in (0, 1):
+        for v in (16, 0):
+            S = Solver(A, s=6, m=30, basis="newton")
+            S.set_option("serp", serp)
+            assert S.get_option("serp") == serp
+            S.set_option("spmv", v)
+            S.set_shifts(*SHIFTS)
+            W[serp, v] = S.mpk(q, 6)
+    for key in W:
+        assert torch.equal(W[key], W[0, 16]), key
+    P = G.random_panel(A.n, 11, 31)
+    QR = {}
+    for serp in (0, 1):
+        S = Solver(A, s=6, m=30, basis="newton")
+        S.set_option("serp", serp)
+        Q = colmajor(P)
+        R = S.tsqr(Q, 11, "cholqr")
+        QR[serp] = (Q.cpu().numpy(), R.cpu().numpy())
+    (Q0, R0), (Q1, R1) = QR[0], QR[1]
+    assert np.max(np.abs(R1 - R0)) <= 1e-13 * np.max(np.abs(R0))
+    assert np.max(np.abs(Q1 - Q0)) <= 1e-13 * np.max(np.abs(Q0))
+    assert O.fact_error(P, Q1, R1) < 1e-13 and O.orth_error(Q1) < 1e-12
+    b = G.rhs(A.n)
+    m = 60 if gen == "g3_small" else 30
+    sh = O.modified_leja(O.ritz_values(O.arnoldi_cgs2(As, b, m)[1], m), 5)
+    ref, env = rounding_envelope(As, b, nperm=1, s=5, m=m, basis="newton", tol=1e-8, maxcyc=100, shifts=sh)
+    hist = {}
+    for serp in (0, 1, 1):
+        S = Solver(A, s=5, m=m, basis="newton")
+        S.set_option("serp", serp)
+        S.set_shifts(*sh)
+        x, st = S.solve(dev(b), tol=1e-8, maxit=100)
+        assert st.status == 0 and abs(st.cycles - len(ref)) <= 1
+        assert hist_within_envelope(st.hist, ref, env)
+        if serp in hist:
+            assert np.array_equal(hist[serp][0], st.hist) and torch.equal(hist[serp][1], x)
+        hist[serp] = (st.hist, x)
+
+
 def test_mpk_full_size_C2():
     """Config C2 at full size (n = 2,097,152) in the launch configuration bench.py times."""
     A = G.convection_diffusion(128, 3, 7)
