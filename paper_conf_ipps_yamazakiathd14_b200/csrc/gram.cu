@@ -6,8 +6,8 @@
 // tensor pipe sustains (tools/fp64_probe.cu).  The scalar form needs W(W+1)/2 = 66 DFMAs
 // per row, a fraction of the DFMA pipe.
 //
-// Data movement: the warps of a CTA work in pairs; each pair streams its own contiguous
-// range of 64-row tiles of the W columns through an S-stage shared-memory ring with 16-B
+// Data movement: the warps of a CTA work in pairs; each pair streams its band-order share
+// (kern::band_tile: tiles g, g + 8 x 148, ...; descending in serpentine order) of the 64-row tiles of the W columns through an S-stage shared-memory ring with 16-B
 // cp.async copies (both warps issue half of every tile's copies), so the bytes in flight
 // (~150 KB per SM) live in shared memory, not in registers.  Lane l of both warps owns rows
 // 2l, 2l+1 of a tile (one 16-B shared load per column; 32-row tiles with one row per lane

@@ -42,6 +42,7 @@ struct Dev {
     int panel_tw16 = 1;
     int panel_pf = 1;           // panel rings: L2 prefetch PF_DIST tiles beyond the cp.async window
     int rev = 0;                // direction of the next streaming launch (serpentine order, solver.cu)
+    int exp = 0;                // CAGMRES_OPT_EXPERIMENT bits (A/B of kernel changes under evaluation)
 };
 
 // Tile order of the streaming kernels (DESIGN.md §6 "serpentine order").  Unit g of NU (a warp,

@@ -1278,6 +1278,7 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
             return CAGMRES_OK;
         case CAGMRES_OPT_FOLD: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->fold = value != 0; return CAGMRES_OK;
         case CAGMRES_OPT_SERP: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->serp = value != 0; return CAGMRES_OK;
+        case CAGMRES_OPT_EXPERIMENT: h->dev.exp = int(value); return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK:
             if (value < 256 || value % 256) return CAGMRES_EINVAL;
             h->wave_CH = int(value); wave_reset_pairs(h); return CAGMRES_OK;
@@ -1305,6 +1306,7 @@ int cagmres_get_option(cagmres_t h, int opt, int64_t* value) {
             return CAGMRES_OK;
         case CAGMRES_OPT_FOLD: *value = h->fold ? 1 : 0; return CAGMRES_OK;
         case CAGMRES_OPT_SERP: *value = h->serp ? 1 : 0; return CAGMRES_OK;
+        case CAGMRES_OPT_EXPERIMENT: *value = h->dev.exp; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK: *value = h->wave_CH; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CTAS: *value = h->wave_ctas; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_LAG: *value = h->wave_lag; return CAGMRES_OK;

@@ -136,7 +136,7 @@ __global__ void __launch_bounds__(NT) k_rows_mma(StreamArgs a) {
     }
 }
 
-// Per-warp cp.async pipeline (aligned panels): each warp streams contiguous TW-row tiles of
+// Per-warp cp.async pipeline (aligned panels): each warp streams its band-order share (kern::band_tile) of the TW-row tiles of
 // the input columns (X then P for the update, P for TRSM) through its own S-stage shared
 // ring; 8-row groups read A fragments (8 rows x 4 cols) from the ring with a column stride
 // of TW+8 doubles (== 8 mod 16: conflict free for that pattern) and store results directly.

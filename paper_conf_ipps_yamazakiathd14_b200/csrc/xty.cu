@@ -158,8 +158,8 @@ __global__ void __launch_bounds__(NT, 1) k_xty_mma(XtyArgs a) {
 }
 
 // ======================================================================================
-// Per-warp cp.async pipeline (aligned panels).  Each warp streams a contiguous range of
-// TW-row tiles of all ncol needed columns through its own S-stage shared-memory ring
+// Per-warp cp.async pipeline (aligned panels).  Each warp streams its band-order share
+// (kern::band_tile) of the TW-row tiles of all ncol needed columns through its own S-stage shared-memory ring
 // (LDGSTS 16-B copies, commit/wait groups, __syncwarp only — no CTA barrier), so the bytes
 // in flight (~(S-1) stages per warp) live in shared memory instead of registers; the
 // register-load kernel above was latency-bound (ncu: long_scoreboard, 16 warps/SM).

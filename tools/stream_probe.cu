@@ -1,0 +1,91 @@
+// stream_probe.cu — what one kernel launch can move on this B200, cold L2, as a function of
+// size: read-only (sum) and copy (read + write) of a flat buffer with 16-B loads, grid-strided,
+// (clean L2: evicted by reading another 512 MB before every timed launch)
+// U independent loads in flight per thread.  Calibrates the per-kernel roofline fractions of the
+// panel kernels: a 185 MB panel read is not a 2 GB copy.
+// nvcc -O3 -gencode arch=compute_100a,code=sm_100a -o /tmp/sp tools/stream_probe.cu
+#include <cstdio>
+#include <cuda_runtime.h>
+
+template <int U>
+__global__ void __launch_bounds__(256) k_read(const double2* __restrict__ p, long n2, double* sink) {
+    double acc = 0.0;
+    const long stride = long(gridDim.x) * blockDim.x;
+    long i = long(blockIdx.x) * blockDim.x + threadIdx.x;
+    for (; i + (U - 1) * stride < n2; i += U * stride) {
+        double2 v[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) v[u] = __ldcg(p + i + u * stride);
+#pragma unroll
+        for (int u = 0; u < U; ++u) acc += v[u].x + v[u].y;
+    }
+    for (; i < n2; i += stride) acc += p[i].x;
+    if (acc == 1.2345) *sink = acc;
+}
+
+template <int U>
+__global__ void __launch_bounds__(256) k_copy(const double2* __restrict__ p, double2* __restrict__ q, long n2) {
+    const long stride = long(gridDim.x) * blockDim.x;
+    long i = long(blockIdx.x) * blockDim.x + threadIdx.x;
+    for (; i + (U - 1) * stride < n2; i += U * stride) {
+        double2 v[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) v[u] = __ldcg(p + i + u * stride);
+#pragma unroll
+        for (int u = 0; u < U; ++u) q[i + u * stride] = v[u];
+    }
+    for (; i < n2; i += stride) q[i] = p[i];
+}
+
+// L2 eviction by READING another 512 MB: the timed kernel starts with clean lines (a write
+// flush would leave ~126 MB of dirty lines whose write-back the timed kernel would pay for)
+__global__ void k_flush(const double* f, long m, double* sink) {
+    double acc = 0.0;
+    for (long i = long(blockIdx.x) * blockDim.x + threadIdx.x; i < m; i += long(gridDim.x) * blockDim.x) acc += f[i];
+    if (acc == 1.2345) *sink = acc;
+}
+
+int main() {
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
+    const long maxb = 2048L << 20;
+    double2 *P, *Q;
+    double *F, *sink;
+    const long fm = 512L << 17;
+    cudaMalloc(&P, maxb);
+    cudaMalloc(&Q, maxb);
+    cudaMalloc(&F, sizeof(double) * fm);
+    cudaMalloc(&sink, 8);
+    cudaMemset(P, 0, maxb);
+    cudaMemset(Q, 0, maxb);
+    cudaMemset(F, 0, sizeof(double) * fm);
+    cudaEvent_t a, b;
+    cudaEventCreate(&a);
+    cudaEventCreate(&b);
+    const long sizes_mb[] = {17, 64, 138, 185, 350, 520, 1024, 2048};
+    for (long mb : sizes_mb) {
+        const long n2 = (mb << 20) / 16;
+        for (int kind = 0; kind < 2; ++kind) {
+            for (int cpsm : {4, 8}) {
+                float best = 1e9f;
+                for (int rep = 0; rep < 5; ++rep) {
+                    k_flush<<<sms * 4, 512>>>(F, fm, sink);
+                    cudaEventRecord(a);
+                    if (kind == 0) k_read<8><<<sms * cpsm, 256>>>(P, n2, sink);
+                    else k_copy<4><<<sms * cpsm, 256>>>(P, Q, n2 / 2);
+                    cudaEventRecord(b);
+                    cudaEventSynchronize(b);
+                    float t = 0.f;
+                    cudaEventElapsedTime(&t, a, b);
+                    if (t < best) best = t;
+                }
+                const double bytes = kind == 0 ? double(mb << 20) : double(mb << 20);   // copy: mb/2 read + mb/2 written
+                printf("%-5s %5ld MB  ctas/SM %d  %9.1f us  %7.0f GB/s\n", kind ? "copy" : "read", mb, cpsm, best * 1e3,
+                       bytes / (best * 1e-3) / 1e9);
+            }
+        }
+    }
+    cudaError_t e = cudaDeviceSynchronize();
+    printf("status: %s\n", cudaGetErrorString(e));
+    return e == cudaSuccess ? 0 : 1;
+}
