@@ -222,8 +222,7 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
                                        give identical results either way; the reductions (xTy, Gram,
                                        norms) sum in another fixed order (deterministic). */
 #define CAGMRES_OPT_EXPERIMENT 18   /* bit mask of kernel changes under evaluation (A/B runs on the
-                                       GPU box; default 0): bit 3 = 3-stage rings for the 1-4
-                                       column Arnoldi / norm passes. */
+                                       GPU box; default 0; no bit is assigned in this build). */
 int cagmres_set_option(cagmres_t h, int opt, int64_t value);
 /* Current value of an option (e.g. the SpMV variant the create-time selection picked).
  * EINVAL for a null handle / pointer or an unknown option. */

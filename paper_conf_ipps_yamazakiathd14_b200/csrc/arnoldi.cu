@@ -83,10 +83,8 @@ __global__ void __launch_bounds__(NT) k_arnoldi_fused(ArnoldiArgs a) {
 // of [Q | v] through an AR_S-stage shared-memory ring with 16-B cp.async (no registers held),
 // lane l owns row l of a tile and reads its Q row from the ring (column c at c*32 + l:
 // conflict-free).  Same per-row operations as k_arnoldi_fused; partials reduced in a fixed order.
-// AR_S ring stages: 3 for wide [Q | v] tiles; narrow ones (the residual norm, the first Arnoldi
-// steps: 1-4 columns, 256 B per column tile) need more stages for enough bytes in flight per SM
-// (2 x 256 B per warp at 3 stages: ~1 TB/s on the norm of one column)
-template <int JX, int MODE, int AR_S = 3>
+constexpr int AR_S = 3;
+template <int JX, int MODE>
 __global__ void __launch_bounds__(512, 1) k_arnoldi_ring(ArnoldiArgs a) {
     extern __shared__ __align__(16) double sma[];
     __shared__ double sc[JX > 0 ? JX : 1];
@@ -189,8 +187,8 @@ __global__ void __launch_bounds__(512, 1) k_arnoldi_ring(ArnoldiArgs a) {
 }
 
 namespace {
-template <int JX, int MODE, int AR_S>
-bool go_ring_s(const Dev& d, const ArnoldiArgs& a0, cudaStream_t st) {
+template <int JX, int MODE>
+bool go_ring(const Dev& d, const ArnoldiArgs& a0, cudaStream_t st) {
     ArnoldiArgs a = a0;
     a.rev = d.rev;
     const bool aligned = ((reinterpret_cast<uintptr_t>(a.v) | reinterpret_cast<uintptr_t>(a.Q)) % 16 == 0) &&
@@ -200,20 +198,10 @@ bool go_ring_s(const Dev& d, const ArnoldiArgs& a0, cudaStream_t st) {
     int nw = int((200 * 1024) / ring_w);
     nw = nw < 2 ? 2 : (nw > 16 ? 16 : nw);
     const size_t smem = size_t(nw) * ring_w;
-    cudaFuncSetAttribute(k_arnoldi_ring<JX, MODE, AR_S>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    cudaFuncSetAttribute(k_arnoldi_ring<JX, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
     ++g_launches;
-    launch_pdl(k_arnoldi_ring<JX, MODE, AR_S>, dim3(unsigned(d.sms)), dim3(32 * nw), smem, st, a);
+    launch_pdl(k_arnoldi_ring<JX, MODE>, dim3(unsigned(d.sms)), dim3(32 * nw), smem, st, a);
     return true;
-}
-
-template <int JX, int MODE>
-bool go_ring(const Dev& d, const ArnoldiArgs& a, cudaStream_t st) {
-    const int ncol = a.jx + 1;
-    if (JX == 8 && !(d.exp & 8)) {
-        if (ncol <= 2) return go_ring_s<JX, MODE, 8>(d, a, st);
-        if (ncol <= 4) return go_ring_s<JX, MODE, 5>(d, a, st);
-    }
-    return go_ring_s<JX, MODE, 3>(d, a, st);
 }
 }  // namespace
 
