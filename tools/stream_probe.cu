@@ -37,6 +37,39 @@ __global__ void __launch_bounds__(256) k_copy(const double2* __restrict__ p, dou
     for (; i < n2; i += stride) q[i] = p[i];
 }
 
+// Same read with DYNAMIC work distribution: every warp takes 64 KB chunks (16 sub-steps of 8 x
+// 16 B per lane) from a global atomic counter, fetching the next chunk index while it reads the
+// current one, until the buffer is done — SMs that see more bandwidth do more chunks (static
+// shares finish when the slowest SM does).
+template <int CH>
+__global__ void __launch_bounds__(256) k_read_dyn(const double2* __restrict__ p, long n2, double* sink,
+                                                  unsigned long long* ctr) {
+    const int lane = threadIdx.x & 31;
+    constexpr int SUB = 16;
+    const long per = 32L * CH * SUB;
+    double acc = 0.0;
+    long c = 0;
+    if (lane == 0) c = long(atomicAdd(ctr, 1ull));
+    c = __shfl_sync(0xffffffffu, c, 0);
+    while (c * per < n2) {
+        long nx = 0;
+        if (lane == 0) nx = long(atomicAdd(ctr, 1ull));                  // next chunk, in flight
+        const long c0 = c * per;
+        for (int sb = 0; sb < SUB; ++sb) {
+            double2 v[CH];
+#pragma unroll
+            for (int u = 0; u < CH; ++u) {
+                const long i = c0 + (long(sb) * CH + u) * 32 + lane;
+                v[u] = i < n2 ? __ldcg(p + i) : make_double2(0.0, 0.0);
+            }
+#pragma unroll
+            for (int u = 0; u < CH; ++u) acc += v[u].x + v[u].y;
+        }
+        c = __shfl_sync(0xffffffffu, nx, 0);
+    }
+    if (acc == 1.2345) *sink = acc;
+}
+
 // L2 eviction by READING another 512 MB: the timed kernel starts with clean lines (a write
 // flush would leave ~126 MB of dirty lines whose write-back the timed kernel would pay for)
 __global__ void k_flush(const double* f, long m, double* sink) {
@@ -56,6 +89,8 @@ int main() {
     cudaMalloc(&Q, maxb);
     cudaMalloc(&F, sizeof(double) * fm);
     cudaMalloc(&sink, 8);
+    unsigned long long* ctr;
+    cudaMalloc(&ctr, 8);
     cudaMemset(P, 0, maxb);
     cudaMemset(Q, 0, maxb);
     cudaMemset(F, 0, sizeof(double) * fm);
@@ -65,14 +100,16 @@ int main() {
     const long sizes_mb[] = {17, 64, 138, 185, 350, 520, 1024, 2048};
     for (long mb : sizes_mb) {
         const long n2 = (mb << 20) / 16;
-        for (int kind = 0; kind < 2; ++kind) {
+        for (int kind = 0; kind < 3; ++kind) {
             for (int cpsm : {4, 8}) {
                 float best = 1e9f;
                 for (int rep = 0; rep < 5; ++rep) {
                     k_flush<<<sms * 4, 512>>>(F, fm, sink);
+                    cudaMemsetAsync(ctr, 0, 8);
                     cudaEventRecord(a);
                     if (kind == 0) k_read<8><<<sms * cpsm, 256>>>(P, n2, sink);
-                    else k_copy<4><<<sms * cpsm, 256>>>(P, Q, n2 / 2);
+                    else if (kind == 1) k_copy<4><<<sms * cpsm, 256>>>(P, Q, n2 / 2);
+                    else k_read_dyn<8><<<sms * cpsm, 256>>>(P, n2, sink, ctr);
                     cudaEventRecord(b);
                     cudaEventSynchronize(b);
                     float t = 0.f;
@@ -80,7 +117,7 @@ int main() {
                     if (t < best) best = t;
                 }
                 const double bytes = kind == 0 ? double(mb << 20) : double(mb << 20);   // copy: mb/2 read + mb/2 written
-                printf("%-5s %5ld MB  ctas/SM %d  %9.1f us  %7.0f GB/s\n", kind ? "copy" : "read", mb, cpsm, best * 1e3,
+                printf("%-8s %5ld MB  ctas/SM %d  %9.1f us  %7.0f GB/s\n", kind == 0 ? "read" : (kind == 1 ? "copy" : "read-dyn"), mb, cpsm, best * 1e3,
                        bytes / (best * 1e-3) / 1e9);
             }
         }
