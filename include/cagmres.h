@@ -160,7 +160,10 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
  *   CAGMRES_OPT_MPK_WAVE : 0 (default) = one SpMV launch per MPK step; 1 = single-GPU
  *                          temporally blocked MPK when A is banded enough and the reuse
  *                          window fits L2 ("reducing communication of MPK on a single
- *                          GPU"); 2 = force it whenever A is banded.  Bitwise identical.
+ *                          GPU"); 2 = force it whenever A is banded; 3 = every MPK block in
+ *                          ONE persistent launch (DIA SpMV variants, one rank): the steps are
+ *                          separated by grid barriers instead of kernel boundaries.  All
+ *                          settings give the same bits.  EINVAL for other values.
  *   CAGMRES_OPT_SPMV     : SpMV kernel (default: the fastest on this matrix, timed once at create;
  *                          -1 re-runs that selection): 0 = one SELL-32 slice per warp; 5 = persistent
  *                          grid, slice descriptors software-pipelined two slices ahead; 16, 17 = the

@@ -214,6 +214,21 @@ struct WaveArgs {
 };
 void mpk_wave(const Dev& d, const WaveArgs& a, int ctas_per_sm, cudaStream_t st);
 
+// Single-GPU MPK block in one persistent launch with grid barriers between the steps
+// (mpk_sweep.cu, CAGMRES_OPT_MPK_WAVE = 3).  bar: a device counter that only grows; bar_base
+// its value before this launch, *next_base its value after.  Returns -1 if not applicable.
+struct SweepArgs {
+    const int64_t* sptr; const int64_t* sinfo; const int32_t* dcol; const double* val; int64_t ncols;
+    double* V; int64_t ldv; int j; int sb;
+    int64_t n;
+    int dia_w;
+    int rev0;                             // sweep direction of step 1 (then alternating)
+    unsigned* bar; unsigned bar_base;
+    double theta[32], b2[32];
+    int kind[32];
+};
+int mpk_sweep(const Dev& d, const SweepArgs& a, cudaStream_t st, unsigned* next_base);
+
 // Fused Arnoldi passes of the first (GMRES) cycle (arnoldi.cu).  mode 1: v -= Q c_in and
 // c_out = Q^T v; mode 2: v -= Q c_in and c_out[0] = v^T v (sqrt if sqrt_out).  jx <= 32
 // (returns -1 otherwise).  part: >= arnoldi_ws_doubles() doubles; counter: zeroed uint.

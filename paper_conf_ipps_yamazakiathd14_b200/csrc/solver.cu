@@ -154,6 +154,9 @@ struct cagmres {
     // single-GPU temporally blocked MPK (mpk_wave.cu)
     bool wave_ok = false, wave_on = false;   // off until it beats the stepwise MPK
     bool wave_force = false;               // option value 2: skip the L2-fit heuristic
+    bool sweep_on = false;                 // option value 3: one persistent launch per MPK block
+    unsigned* sweep_bar = nullptr;         // its grid-barrier counter (only grows)
+    unsigned sweep_base = 0;
     int64_t wave_bw = 0;
     int wave_CH = 1024, wave_ctas = 4, wave_lag = 0, wave_nC = 0, wave_epoch = 0;
     int* d_done = nullptr;
@@ -164,6 +167,7 @@ struct cagmres {
         cudaFree(d_done);
         for (int2* p : d_pairs) cudaFree(p);
         cudaFree(A.sptr); cudaFree(A.sinfo); cudaFree(A.dcol); cudaFree(A.val);
+        cudaFree(sweep_bar);
         cudaFree(V); cudaFree(xe); cudaFree(S); cudaFree(tab); cudaFree(gbuf); cudaFree(ybuf); cudaFree(caqr_ws); cudaFree(op_M);
         cudaFreeHost(h_tab); cudaFreeHost(h_y); cudaFreeHost(h_beta); cudaFreeHost(h_stat);
         cudaFree(dg); cudaFreeHost(h_dg);
@@ -652,6 +656,31 @@ int start_halo(cagmres* h, int col, int depth, bool& fuse) {
 // distance <= sb-k (a prefix of the extended numbering) from the rows at distance <= sb-k+1.
 int mpk_block(cagmres* h, int j, int sb, const std::vector<host::Step>& steps) {
     Scope sc(h, PH_MPK);
+    if (h->sweep_on && h->nranks == 1 && sb >= 2 && h->A.variant >= 16 && h->sweep_bar) {
+        TRY(materialize(h, h->n_loc));
+        kern::SweepArgs a{};
+        a.sptr = h->A.sptr; a.sinfo = h->A.sinfo; a.dcol = h->A.dcol; a.val = h->A.val; a.ncols = h->A.ncols;
+        a.V = h->V; a.ldv = h->ldv; a.j = j; a.sb = sb; a.n = h->n_loc; a.dia_w = h->A.dia_w;
+        a.bar = h->sweep_bar; a.bar_base = h->sweep_base;
+        for (int k = 1; k <= sb; ++k) {
+            a.theta[k - 1] = steps[size_t(k - 1)].a;
+            a.b2[k - 1] = steps[size_t(k - 1)].b2;
+            a.kind[k - 1] = steps[size_t(k - 1)].kind;
+        }
+        kern::Dev& d = sdev(h);
+        a.rev0 = d.rev;
+        {
+            Scope sv(h, PH_SPMV);
+            if (kern::mpk_sweep(d, a, h->stream, &h->sweep_base)) return CAGMRES_EINVAL;
+        }
+        h->dev.rev = a.rev0 ^ ((sb - 1) & 1);            // direction of the block's last step
+        double by = 0.0;
+        for (int k = 1; k <= sb; ++k) by += spmv_bytes(h, h->n_loc, 1, steps[size_t(k - 1)].kind == 2);
+        h->bytes[PH_MPK] += by;
+        h->bytes[PH_SPMV] += by;
+        h->spmv_launches++;
+        return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
+    }
     if (h->wave_on && h->nranks == 1 && sb >= 2 && wave_fits(h)) {
         TRY(materialize(h, h->n_loc));
         TRY(wave_pairs(h, sb));
@@ -1090,7 +1119,7 @@ int enqueue_cycle(cagmres* h, bool arnoldi, const std::vector<Block>& bl) {
 // kept by the capture.  Host-side accounting (algorithmic bytes, launch counts, the pending
 // normalisation) is replayed from the capture's deltas.
 bool graph_ok(const cagmres* h) {
-    return h->use_graphs && h->nranks == 1 && !h->timer.on && !h->diag_on && !h->wave_on &&
+    return h->use_graphs && h->nranks == 1 && !h->timer.on && !h->diag_on && !h->wave_on && !h->sweep_on &&
            (!h->pend || (h->pend_col == 0 && h->pend_nrm == h->gbuf + 8));
 }
 
@@ -1252,7 +1281,15 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
     if (!h) return CAGMRES_EINVAL;
     ++h->cfg_version;                      // any option may change the captured cycle
     switch (opt) {
-        case CAGMRES_OPT_MPK_WAVE: h->wave_on = value != 0; h->wave_force = value == 2; return CAGMRES_OK;
+        case CAGMRES_OPT_MPK_WAVE:
+            if (value < 0 || value > 3) return CAGMRES_EINVAL;
+            h->wave_on = value == 1 || value == 2; h->wave_force = value == 2; h->sweep_on = value == 3;
+            if (h->sweep_on && !h->sweep_bar) {
+                CU(cudaMalloc(&h->sweep_bar, sizeof(unsigned)));
+                CU(cudaMemset(h->sweep_bar, 0, sizeof(unsigned)));
+                h->sweep_base = 0;
+            }
+            return CAGMRES_OK;
         case CAGMRES_OPT_SPMV:
             if (value != -1 && value != 0 && value != 5 && value != 16 && value != 17) return CAGMRES_EINVAL;
             if (value == -1) return spmv_autotune(h);
@@ -1291,7 +1328,7 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
 int cagmres_get_option(cagmres_t h, int opt, int64_t* value) {
     if (!h || !value) return CAGMRES_EINVAL;
     switch (opt) {
-        case CAGMRES_OPT_MPK_WAVE: *value = h->wave_on ? (h->wave_force ? 2 : 1) : 0; return CAGMRES_OK;
+        case CAGMRES_OPT_MPK_WAVE: *value = h->sweep_on ? 3 : (h->wave_on ? (h->wave_force ? 2 : 1) : 0); return CAGMRES_OK;
         case CAGMRES_OPT_SPMV: *value = h->A.variant; return CAGMRES_OK;
         case CAGMRES_OPT_GRAM: *value = h->dev.gram; return CAGMRES_OK;
         case CAGMRES_OPT_ARNOLDI: *value = h->dev.arnoldi_ring; return CAGMRES_OK;

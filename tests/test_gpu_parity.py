@@ -143,6 +143,49 @@ def test_mpk_wave_bitwise_equals_stepwise(gen):
             assert np.max(np.abs(W1[:, k] - Wo[:, k])) <= 1e-13 * np.max(np.abs(Wo[:, k])), k
 
 
+@pytest.mark.parametrize("gen", ["C2", "cd27_ragged", "g3_small", "banded", "cd7_ragged"])
+def test_mpk_sweep_bitwise_equals_stepwise(gen):
+    """CAGMRES_OPT_MPK_WAVE = 3: the whole MPK block in one persistent launch (grid barriers
+    between the steps, alternating sweep direction) computes every row as the stepwise MPK —
+    bitwise identical bases for every block size, including complex-conjugate pairs (SHIFTS
+    has two) and a block ending inside a pair; then whole solves, bit for bit, and directly
+    against the oracle's MPK."""
+    A = {"C2": lambda: G.convection_diffusion(128, 3, 7),
+         "cd27_ragged": lambda: G.convection_diffusion(17, 3, 27),
+         "g3_small": lambda: G.g3_shaped(n=40000, width=200),
+         "banded": lambda: G.banded(n=300001),
+         "cd7_ragged": lambda: G.convection_diffusion(45, 3, 7)}[gen]()
+    q = dev(G.u(5, np.arange(A.n)))
+    S1 = Solver(A, s=10, m=30, basis="newton")
+    S2 = Solver(A, s=10, m=30, basis="newton")
+    S1.set_option("mpk_wave", 3)
+    assert S1.get_option("mpk_wave") == 3
+    S2.set_option("mpk_wave", 0)
+    for S in (S1, S2):
+        S.set_option("spmv", 16)
+        S.set_shifts(*SHIFTS)
+    for sb in (10, 7, 4, 2, 1):
+        W1, W2 = S1.mpk(q, sb), S2.mpk(q, sb)
+        assert torch.equal(W1, W2), (gen, sb)
+    if gen in ("cd27_ragged", "g3_small"):
+        Wo = O.mpk(A.to_scipy(), q.cpu().numpy(), 10, *SHIFTS)
+        W1 = S1.mpk(q, 10).cpu().numpy()
+        for k in range(11):
+            assert np.max(np.abs(W1[:, k] - Wo[:, k])) <= 1e-13 * np.max(np.abs(Wo[:, k])), k
+    if gen in ("cd7_ragged", "g3_small"):
+        b = dev(G.rhs(A.n))
+        m = 60 if gen == "g3_small" else 30
+        out = []
+        for wave in (3, 0):
+            S = Solver(A, s=5, m=m, basis="newton")
+            S.set_option("spmv", 16)
+            S.set_option("mpk_wave", wave)
+            x, st = S.solve(b, tol=1e-8, maxit=100)
+            assert st.status == 0
+            out.append((x, st))
+        assert np.array_equal(out[0][1].hist, out[1][1].hist) and torch.equal(out[0][0], out[1][0])
+
+
 @pytest.mark.parametrize("gen", ["cd27_ragged", "g3_small", "banded", "cd7_ragged"])
 def test_spmv_variants_bitwise(gen):
     """Every SpMV kernel variant (CAGMRES_OPT_SPMV: one or two SELL-32 slices per warp, load
