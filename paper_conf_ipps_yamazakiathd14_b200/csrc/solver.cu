@@ -22,6 +22,7 @@
 #include <memory>
 
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include "internal.h"
 #include "kernels.h"
@@ -187,13 +188,23 @@ struct cagmres {
 namespace {
 
 // ---- timing helpers --------------------------------------------------------------------
+// A phase of the cycle (SURVEY §5 tracing): an NVTX range on the host thread that enqueues it
+// (visible to Nsight Systems / any NVTX tool; a no-op without one) and, with collect_timing, a
+// pair of CUDA events on the handle's stream.
+const char* const kPhaseName[] = {"MPK", "BOrth", "TSQR", "other", "SpMV"};
+struct NvtxRange {
+    explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
 struct Scope {
     cagmres* h; int ph; cudaEvent_t e0 = nullptr;
     bool act;
     Scope(cagmres* hh, int p) : h(hh), ph(p), act(hh->timer.on && (!hh->timer.light || p == PH_SPMV)) {
+        nvtxRangePushA(kPhaseName[p]);
         if (act) { e0 = h->timer.get(); cudaEventRecord(e0, h->stream); }
     }
     ~Scope() {
+        nvtxRangePop();
         if (act) {
             cudaEvent_t e1 = h->timer.get();
             cudaEventRecord(e1, h->stream);
@@ -1448,6 +1459,7 @@ int cagmres_tsqr(cagmres_t h, double* P, int64_t ldp, int w, double* R, int orth
 
 int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit, cagmres_stats* st) {
     if (!h || !b || !x || maxit < 0 || !(tol >= 0.0)) return CAGMRES_EINVAL;
+    const NvtxRange solve_range("cagmres_solve");
     const int m = h->m;
     h->timer.reset();
     h->timer.on = st && st->collect_timing;
@@ -1479,6 +1491,9 @@ int cagmres_solve(cagmres_t h, const double* b, double* x, double tol, int maxit
     for (; cyc < maxit && rc != CAGMRES_OK; ++cyc) {
         const bool first_newton = h->basis == CAGMRES_NEWTON && !h->have_shifts;
         const bool arnoldi = first_newton || h->basis == CAGMRES_GMRES;
+        char rname[48];
+        snprintf(rname, sizeof rname, "restart cycle %d (%s)", cyc + 1, arnoldi ? "GMRES" : "CA");
+        const NvtxRange cycle_range(rname);
         const bool cgs2 = (h->orth & CAGMRES_REORTH) != 0;
         std::fill(H.begin(), H.end(), 0.0);
         if (!pending) TRY(arnoldi ? enqueue_cycle(h, true, bl) : enqueue_ca_cycle(h, bl));
