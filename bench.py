@@ -139,6 +139,10 @@ def run_ours(args):
 
     ws, rank, lrank = dist_env()
     torch.cuda.set_device(lrank)
+    # one ordinary (non-default) stream for everything: the solver binds torch's current stream,
+    # so the copies of b / x and the flush are ordered with its kernels, and programmatic
+    # dependent launch applies (it is not used on the legacy default stream)
+    torch.cuda.set_stream(torch.cuda.Stream())
     group = None
     cfg = CFG[args.config]
     if ws > 1:
@@ -245,7 +249,7 @@ def run_ours(args):
         S.solve(bd, torch.zeros_like(bd), tol=TOL, maxit=200)
         x_pin.copy_(bd, non_blocking=True)
     torch.cuda.synchronize()
-    e2e_ms = []
+    e2e_ms, e2e_cycles = [], []
     for k in range(args.steps):
         flush.fill_(float(k))
         if group is not None:
@@ -256,11 +260,12 @@ def run_ours(args):
         S.clear_shifts()
         bd = b_pin.to("cuda", non_blocking=True)
         xd = torch.zeros_like(bd)
-        S.solve(bd, xd, tol=TOL, maxit=200)
+        _, st_e = S.solve(bd, xd, tol=TOL, maxit=200)
         x_pin.copy_(xd, non_blocking=True)
         e1.record(stream)
         torch.cuda.synchronize()
         e2e_ms.append(e0.elapsed_time(e1))
+        e2e_cycles.append(st_e.cycles)
     e2e = float(np.median(e2e_ms))          # median: robust to a rare host-side stall (each_ms kept)
     if group is not None:
         t = torch.tensor([e2e], device="cuda")
@@ -325,7 +330,8 @@ def run_ours(args):
                                 + (", one-pass BOrth+CholQR (NEXT-2)" if args.onepass else ", BOrth CGS")),
                        "kernels": {k_: S.get_option(k_) for k_ in ("spmv", "gram", "fuse", "mpk_wave", "graph")}},
             "e2e": {"value": round(e2e, 4), "unit": "ms", "stat": "median of K", "h2d_bytes_per_step": 8 * len(b_host),
-                    "d2h_bytes_per_step": 8 * len(b_host), "each_ms": [round(v, 3) for v in e2e_ms]},
+                    "d2h_bytes_per_step": 8 * len(b_host), "each_ms": [round(v, 3) for v in e2e_ms],
+                    "cycles": sorted(set(e2e_cycles))},
             "value_each_ms": [round(float(v), 3) for v in ms],
             "gpu_launches": int(launches_total),
             "gpu_launches_per_step": round(launches_total / args.steps, 1),

@@ -153,7 +153,10 @@ int cagmres_create_group(cagmres_t* h, const cagmres_csr* A, const int64_t* row_
 int cagmres_destroy(cagmres_t h);                 /* frees everything create allocated */
 const char* cagmres_strerror(int status);         /* static string, never NULL         */
 
-/* cudaStream_t to enqueue on (NULL = the handle's own stream).  Not owned. */
+/* cudaStream_t to enqueue on (NULL = the handle's own non-blocking stream; cudaStreamLegacy for
+ * the legacy default stream — the handle's work is then ordered with everything the caller
+ * queues there, e.g. the copy of b).  Programmatic dependent launch is used on ordinary streams
+ * only.  Not owned. */
 int cagmres_set_stream(cagmres_t h, void* cuda_stream);
 
 /* Tuning options (value semantics per option); EINVAL for an unknown option.
@@ -226,6 +229,12 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
                                        norms) sum in another fixed order (deterministic). */
 #define CAGMRES_OPT_EXPERIMENT 18   /* bit mask of kernel changes under evaluation (A/B runs on the
                                        GPU box; default 0; no bit is assigned in this build). */
+#define CAGMRES_OPT_L2_PERSIST 19   /* 0 (default) = off; p in 1..100 = put the MPK SpMV's matrix
+                                       values (re-read by every step) in the persisting part of the
+                                       L2: the device-wide set-aside (cudaLimitPersistingL2CacheSize)
+                                       becomes p % of min(the device maximum, the values' bytes), and
+                                       every SpMV launch carries an access-policy window over them.
+                                       ENOTSUP if the device has no set-aside.  Same bits either way. */
 int cagmres_set_option(cagmres_t h, int opt, int64_t value);
 /* Current value of an option (e.g. the SpMV variant the create-time selection picked).
  * EINVAL for a null handle / pointer or an unknown option. */

@@ -155,13 +155,27 @@ class Solver:
         return C.c_char_p(bytes(buf.numpy()))
 
     # ------------------------------------------------------------------------------------
+    CUDA_STREAM_LEGACY = 1                       # cudaStreamLegacy: torch's default stream
+
     def use_torch_stream(self):
+        """Enqueue on torch's current stream, so the library's work is ordered after whatever the
+        caller queued on it (e.g. an asynchronous copy of b) — called before every device call.
+        torch reports its default (legacy) stream as handle 0, which the C ABI reads as "the
+        handle's own stream": pass cudaStreamLegacy for it instead.  In-process group ranks
+        never share the legacy stream (their collectives wait on each other's events): a rank
+        thread on the default stream keeps the handle's own stream."""
         import torch
-        s = torch.cuda.current_stream(self.device)
-        L.check(self._lib.cagmres_set_stream(self._h, C.c_void_p(s.cuda_stream)), "set_stream")
+        s = torch.cuda.current_stream(self.device).cuda_stream
+        if not s:
+            if getattr(self, "_group", None) is not None:
+                return
+            s = self.CUDA_STREAM_LEGACY
+        if s != getattr(self, "_bound_stream", None):
+            L.check(self._lib.cagmres_set_stream(self._h, C.c_void_p(s)), "set_stream")
+            self._bound_stream = s
 
     OPTIONS = {"mpk_wave": 1, "wave_chunk": 3, "wave_ctas": 4, "wave_lag": 5, "fuse": 6, "spmv": 7, "gram": 8,
-               "arnoldi": 9, "panel_tw": 10, "trsm": 11, "pdl": 12, "panel_pf": 13, "peer": 14, "graph": 15, "fold": 16, "serp": 17, "exp": 18}
+               "arnoldi": 9, "panel_tw": 10, "trsm": 11, "pdl": 12, "panel_pf": 13, "peer": 14, "graph": 15, "fold": 16, "serp": 17, "exp": 18, "l2_persist": 19}
 
     def set_option(self, opt, value):
         """opt: "mpk_wave", "wave_chunk", "wave_ctas", "wave_lag", "fuse", "spmv", "gram", "arnoldi" (CAGMRES_OPT_*)."""
@@ -213,6 +227,7 @@ class Solver:
 
     def mpk(self, q, sb, out=None):
         import torch
+        self.use_torch_stream()
         if out is None:
             out = torch.empty((sb + 1, self.n_loc), dtype=torch.float64, device=self.device).t()
         W, ldw = self._col_major(out, self.n_loc)
@@ -221,6 +236,7 @@ class Solver:
 
     def borth(self, Q, j, P, w):
         import torch
+        self.use_torch_stream()
         Cm = torch.zeros((w, max(j, 1)), dtype=torch.float64, device=self.device)  # j x w col-major
         qp, ldq = self._col_major(Q, self.n_loc)
         pp, ldp = self._col_major(P, self.n_loc)
@@ -230,6 +246,7 @@ class Solver:
 
     def tsqr(self, P, w, tsqr="cholqr", reorth=False, svqr_retry=False):
         import torch
+        self.use_torch_stream()
         R = torch.zeros((w, w), dtype=torch.float64, device=self.device)
         pp, ldp = self._col_major(P, self.n_loc)
         st = self._lib.cagmres_tsqr(self._h, C.c_void_p(pp), ldp, int(w), C.c_void_p(R.data_ptr()),
@@ -240,6 +257,7 @@ class Solver:
     def solve(self, b, x=None, tol=1e-8, maxit=200, timing=False, diag=False):
         """Solve on device tensors b, x (owned rows, float64); x updated in place."""
         import torch
+        self.use_torch_stream()
         if x is None:
             x = torch.zeros_like(b)
         hist = np.zeros(maxit + 1)

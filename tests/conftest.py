@@ -16,3 +16,21 @@ def pytest_configure(config):
 @pytest.fixture(scope="session")
 def golden_dir():
     return os.path.join(ROOT, "tests", "golden")
+
+
+@pytest.fixture(autouse=True)
+def _gpu_tests_on_a_side_stream(request):
+    """GPU tests run on a non-default torch stream, like bench.py: the library binds torch's
+    current stream (Solver.use_torch_stream), so its kernels are ordered with the test's own
+    torch ops and launched with programmatic dependent launch (not used on the legacy stream)."""
+    if request.node.get_closest_marker("gpu") is None:
+        yield
+        return
+    import torch
+    if not torch.cuda.is_available():
+        yield
+        return
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        yield
+    s.synchronize()

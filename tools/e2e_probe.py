@@ -24,6 +24,7 @@ cfg_name = sys.argv[1] if len(sys.argv) > 1 else "C3"
 K = int(sys.argv[2]) if len(sys.argv) > 2 else 5
 cfg = bench.CFG[cfg_name]
 torch.cuda.set_device(0)
+torch.cuda.set_stream(torch.cuda.Stream())     # an ordinary stream, as in bench.py (PDL on)
 A = cfg["build"]()
 S = Solver(A, cfg["s"], cfg["m"], basis=cfg["basis"], tsqr=cfg["tsqr"], reorth=cfg["reorth"])
 b_host = G.rhs(cfg["n"])

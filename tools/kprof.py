@@ -18,6 +18,7 @@ ap.add_argument("--config", default="C2")
 ap.add_argument("--mpk-only", action="store_true", help="three MPK blocks instead of a solve")
 args = ap.parse_args()
 torch.cuda.set_device(0)
+torch.cuda.set_stream(torch.cuda.Stream())     # an ordinary stream, as in bench.py (PDL on)
 if args.config == "C2":
     A, s, m = G.convection_diffusion(128, 3, 7), 10, 30
 else:
