@@ -27,6 +27,7 @@ def colmajor(M):
 
 def main():
     torch.cuda.set_device(0)
+    torch.cuda.set_stream(torch.cuda.Stream())     # ordinary stream, as bench.py (PDL on)
     A = G.banded()
     As = A.to_scipy()
     n, s = A.n, 10

@@ -99,6 +99,7 @@ def solve_margins():
 
 if __name__ == "__main__":
     torch.cuda.set_device(0)
+    torch.cuda.set_stream(torch.cuda.Stream())     # ordinary stream, as bench.py (PDL on)
     out = {"solve": solve_margins()}
     if not os.environ.get("MARGINS_ONLY"):
         out["mpk"] = mpk_margins()
