@@ -60,14 +60,42 @@ def peaks():
 
 
 class Clocks:
-    """nvidia-smi sampler running during the timed region."""
+    """SM clock / throttle-reason sampler running during the timed region: NVML from a thread
+    every 10 ms (starts at once, so even a short timed region gets samples); nvidia-smi -lms 100
+    as the fallback."""
+
+    NAMES = {"hw_slowdown": 0x8, "hw_thermal_slowdown": 0x40, "sw_thermal_slowdown": 0x20, "sw_power_cap": 0x4}
 
     def __init__(self, idx):
         self.idx = idx
         self.path = os.path.join("/tmp", f"clocks_{os.getpid()}.csv")
         self.p = None
+        self.th = None
+        self.samples = []
+
+    def _nvml_loop(self, nv, hnd):
+        while not self.stop.is_set():
+            try:
+                sm = nv.nvmlDeviceGetClockInfo(hnd, nv.NVML_CLOCK_SM)
+                mx = nv.nvmlDeviceGetMaxClockInfo(hnd, nv.NVML_CLOCK_SM)
+                rs = nv.nvmlDeviceGetCurrentClocksEventReasons(hnd)
+                self.samples.append((float(sm), float(mx), int(rs)))
+            except Exception:
+                pass
+            self.stop.wait(0.01)
 
     def __enter__(self):
+        import threading
+        try:
+            import pynvml as nv
+            nv.nvmlInit()
+            hnd = nv.nvmlDeviceGetHandleByIndex(self.idx)
+            self.stop = threading.Event()
+            self.th = threading.Thread(target=self._nvml_loop, args=(nv, hnd), daemon=True)
+            self.th.start()
+            return self
+        except Exception:
+            self.th = None
         try:
             self.f = open(self.path, "w")
             self.p = subprocess.Popen(
@@ -81,6 +109,9 @@ class Clocks:
         return self
 
     def __exit__(self, *a):
+        if self.th is not None:
+            self.stop.set()
+            self.th.join(timeout=5)
         if self.p is not None:
             self.p.terminate()
             try:
@@ -90,25 +121,34 @@ class Clocks:
             self.f.close()
 
     def summary(self):
-        if self.p is None or not os.path.exists(self.path):
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
         sm, mx, reasons = [], [], set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for line in open(self.path):
-            parts = [x.strip() for x in line.split(",")]
-            if len(parts) < 7:
-                continue
-            try:
-                sm.append(float(parts[0])); mx.append(float(parts[1]))
-            except ValueError:
-                continue
-            for nm, v in zip(names, parts[3:7]):
-                if v.lower().startswith("active"):
-                    reasons.add(nm)
+        if self.th is not None:
+            for a, b, r in self.samples:
+                sm.append(a); mx.append(b)
+                for nm, bit in self.NAMES.items():
+                    if r & bit:
+                        reasons.add(nm)
+            src = "nvml"
+        else:
+            if self.p is None or not os.path.exists(self.path):
+                return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+            names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+            for line in open(self.path):
+                parts = [x.strip() for x in line.split(",")]
+                if len(parts) < 7:
+                    continue
+                try:
+                    sm.append(float(parts[0])); mx.append(float(parts[1]))
+                except ValueError:
+                    continue
+                for nm, v in zip(names, parts[3:7]):
+                    if v.lower().startswith("active"):
+                        reasons.add(nm)
+            src = "nvidia-smi"
         if not sm:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
         return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": float(max(mx)), "reasons": sorted(reasons),
-                "samples": len(sm)}
+                "samples": len(sm), "source": src}
 
 
 def dist_env():

@@ -343,7 +343,7 @@ struct XtyWs { double* part = nullptr; size_t cap = 0; unsigned int* counter = n
 size_t xty_ws_doubles(const Dev& d, int jx, int w);
 int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const double* Y,
         int64_t ldy, int w, double* out, bool fin_chol, double* R, int* status,
-        const XtyWs& ws, cudaStream_t st, bool early_x = false);
+        const XtyWs& ws, cudaStream_t st);
 
 // Scalar-DFMA Gram G = P^T P (gram.cu; P 16-B aligned, ld even, w <= 12), same final
 // reduction / in-launch Cholesky contract as xty with X == Y.  Returns -1 if not applicable.

@@ -606,15 +606,14 @@ int halo(cagmres* h, double* vec, int depth) {
 
 // ---- building blocks ------------------------------------------------------------------
 // C = X^T Y summed over ranks (out ld ldo); optional R = chol(C) (CholQR Gram)
-// early: X is not written by the kernel in front of this one (BOrth pass 1 inside a cycle)
 int xty_global(cagmres* h, const double* X, int64_t ldx, int jx, const double* Y, int64_t ldy,
-               int w, double* out, bool chol, double* R, bool early = false) {
+               int w, double* out, bool chol, double* R) {
     if (h->nranks == 1) {
-        if (kern::xty(sdev(h), h->n_loc, X, ldx, jx, Y, ldy, w, out, chol, R, h->status, h->ws, h->stream, early))
+        if (kern::xty(sdev(h), h->n_loc, X, ldx, jx, Y, ldy, w, out, chol, R, h->status, h->ws, h->stream))
             return CAGMRES_EINVAL;
         return cudaGetLastError() == cudaSuccess ? CAGMRES_OK : CAGMRES_ECUDA;
     }
-    if (kern::xty(sdev(h), h->n_loc, X, ldx, jx, Y, ldy, w, out, false, nullptr, h->status, h->ws, h->stream, early))
+    if (kern::xty(sdev(h), h->n_loc, X, ldx, jx, Y, ldy, w, out, false, nullptr, h->status, h->ws, h->stream))
         return CAGMRES_EINVAL;
     if (chol && h->peer_ok && w <= 32) {
         // one-sided: the cross-rank sum of the Gram and its Cholesky in one launch reading the
@@ -761,14 +760,12 @@ int mpk_block(cagmres* h, int j, int sb, const std::vector<host::Step>& steps) {
 
 // BOrth of the panel columns P (n_loc x w, ld ldp) against Q (n_loc x j): CGS or MGS
 // (P:144).  C: device j x w, ld j.
-// early_q: Q is final before the kernel in front of the BOrth (inside a CA cycle; not for the
-// API call, where the caller's own kernels may have just written Q)
 int borth_panel(cagmres* h, const double* Q, int64_t ldq, int j, double* P, int64_t ldp, int w,
-                double* C, bool mgs, bool early_q = false) {
+                double* C, bool mgs) {
     if (j <= 0) return CAGMRES_OK;
     Scope sc(h, PH_BORTH);
     if (!mgs) {
-        TRY(xty_global(h, Q, ldq, j, P, ldp, w, C, false, nullptr, early_q));
+        TRY(xty_global(h, Q, ldq, j, P, ldp, w, C, false, nullptr));
         // C is jx x w with ld jx = j: xty writes ld jx
         kern::update(sdev(h), h->n_loc, Q, ldq, j, P, ldp, w, C, h->stream, true);   // after xty: early start
         h->bytes[PH_BORTH] += 8.0 * double(h->n_loc) * (2.0 * j + 3.0 * w);
@@ -988,7 +985,7 @@ int ca_cycle(cagmres* h, const std::vector<Block>& bl) {
                 if (fold) { h->fold_kind = 1; h->fold_pass = pass; }
                 continue;
             }
-            TRY(borth_panel(h, h->V, h->ldv, j, Pj + h->ldv, h->ldv, sb, C, mgs, true));
+            TRY(borth_panel(h, h->V, h->ldv, j, Pj + h->ldv, h->ldv, sb, C, mgs));
             const bool fold_tsqr = fold && (kind == CAGMRES_CHOLQR || kind == CAGMRES_SVQR);
             TRY(tsqr_panel(h, Pj, h->ldv, w, R, kind, 1, (h->orth & CAGMRES_SVQR_RETRY) != 0, fold_tsqr));
             if (fold_tsqr) { h->fold_kind = 1; h->fold_pass = pass; }

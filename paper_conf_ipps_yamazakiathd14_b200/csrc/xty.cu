@@ -41,7 +41,6 @@ struct XtyArgs {
     int* status;
     int pf = 0;                 // L2 prefetch ahead of the ring (Dev::panel_pf)
     int rev = 0;                // tile order (band_tile), from Dev::rev
-    int early_x = 0;            // X is not written by the preceding kernel: issue it before the PDL wait
 };
 
 // ---- CTA partial -> two-level fixed-order total (+ Cholesky) ---------------------------
@@ -171,6 +170,8 @@ constexpr int PIPE_S = 3;
 template <int MT, int NTN, bool SYM, int TW>
 __global__ void __launch_bounds__(NT, 1) k_xty_pipe(XtyArgs a) {
     extern __shared__ __align__(16) double smp[];
+    pdl_wait();
+    pdl_trigger();
     constexpr int SP = TW + 4;
     const int lane = threadIdx.x & 31, wp = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const int gid = lane >> 2, tig = lane & 3;
@@ -203,17 +204,6 @@ __global__ void __launch_bounds__(NT, 1) k_xty_pipe(XtyArgs a) {
         }
         ptx::cp_async_commit();
     };
-    // slot columns [c_lo, c_hi) of tile i only (one commit group)
-    auto issue_cols = [&](int64_t i, int stage, int c_lo, int c_hi) {
-        if (i < cnt) {
-            double* dst = ring + stage * stage_d + part2;
-            const int64_t r0 = band_tile(T, W, g, i, a.rev) * TW + part2;
-            int c = cfirst;
-            while (c < c_lo) c += CSTEP;
-            for (; c < c_hi; c += CSTEP) ptx::cp_async16(dst + c * SP, sCol[c] + r0);
-        }
-        ptx::cp_async_commit();
-    };
     // two accumulator sets, even / odd 4-row k-steps: twice the independent DMMA chains per warp
     // (ncu: the single set stalled on the DMMA dependency, "wait"); summed in a fixed order at the end
     double acc[MT][NTN][2], acc2[MT][NTN][2];
@@ -229,23 +219,8 @@ __global__ void __launch_bounds__(NT, 1) k_xty_pipe(XtyArgs a) {
 #pragma unroll
         for (int mt = 0; mt < MT; ++mt) xcol[mt] = (nx ? w : 0) + min(8 * mt + gid, nxc - 1);
     }
-    if (a.early_x && nx > 0) {
-        // BOrth pass 1 after the MPK: X = Q was final long before the kernel in front of this
-        // one (which only wrote the panel Y), so the first stages' X tiles are requested before
-        // griddepcontrol.wait and overlap that kernel's drain; Y follows after the wait.  Four
-        // prologue groups [X0 X1 Y0 Y1]: the loop's wait_group<S-1> still completes stage i in time.
 #pragma unroll
-        for (int s = 0; s < PIPE_S - 1; ++s) issue_cols(s, s, w, ncol);
-        pdl_wait();
-        pdl_trigger();
-#pragma unroll
-        for (int s = 0; s < PIPE_S - 1; ++s) issue_cols(s, s, 0, w);
-    } else {
-        pdl_wait();
-        pdl_trigger();
-#pragma unroll
-        for (int s = 0; s < PIPE_S - 1; ++s) issue(s, s);
-    }
+    for (int s = 0; s < PIPE_S - 1; ++s) issue(s, s);
     int stage = 0;
     for (int64_t i = 0; i < cnt; ++i) {
         issue(i + PIPE_S - 1, (stage + PIPE_S - 1) % PIPE_S);
@@ -442,7 +417,7 @@ int xty_pipe_launch(const Dev& d, Geo o, const XtyArgs& a, int ncol, const XtyWs
 
 int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const double* Y,
         int64_t ldy, int w, double* out, bool fin_chol, double* R, int* status,
-        const XtyWs& ws, cudaStream_t st, bool early_x) {
+        const XtyWs& ws, cudaStream_t st) {
     if (jx <= 0 || w <= 0 || w > 32 || n < 0) return -1;
     const bool same = (X == Y) && (ldx == ldy) && (jx == w);
     if (same && d.gram >= 1 && size_t(d.sms) * w * w * 2 <= ws.cap) {
@@ -451,8 +426,7 @@ int xty(const Dev& d, int64_t n, const double* X, int64_t ldx, int jx, const dou
     }
     Geo o = geometry(d, n, jx, w, same);
     if (size_t(o.gx) * o.gy * o.chunk * w * 2 > ws.cap || o.gy * TR_CNT > XTY_COUNTERS) return -1;
-    XtyArgs a{n, X, ldx, jx, Y, ldy, w, o.chunk, ws.part, out, ws.counter, fin_chol ? 1 : 0, R, status, d.panel_pf, d.rev,
-              (early_x && !(d.exp & 2)) ? 1 : 0};
+    XtyArgs a{n, X, ldx, jx, Y, ldy, w, o.chunk, ws.part, out, ws.counter, fin_chol ? 1 : 0, R, status, d.panel_pf, d.rev};
     const bool aligned = ((reinterpret_cast<uintptr_t>(X) | reinterpret_cast<uintptr_t>(Y)) % 16 == 0) &&
                          (ldx % 2 == 0) && (ldy % 2 == 0);
     if (aligned && n >= 32 * 64) {
