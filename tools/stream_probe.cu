@@ -70,6 +70,48 @@ __global__ void __launch_bounds__(256) k_read_dyn(const double2* __restrict__ p,
     if (acc == 1.2345) *sink = acc;
 }
 
+// Static band + dynamic tail: every warp reads its grid-stride share of the first `split` of the
+// buffer (the band order of the panel kernels), then takes 4 KB chunks of the rest from one of 8
+// atomic counters (its CTA's counter id = blockIdx % 8, region-interleaved) until all are done —
+// so SMs that finish their static share early absorb the stragglers' tail.
+__global__ void __launch_bounds__(256) k_read_tail(const double2* __restrict__ p, long n2, double* sink,
+                                                   unsigned long long* ctr, double split) {
+    const int lane = threadIdx.x & 31;
+    const long stride = long(gridDim.x) * blockDim.x;
+    const long ns = long(double(n2) * split) / stride * stride;      // statically assigned part
+    double acc = 0.0;
+    long i = long(blockIdx.x) * blockDim.x + threadIdx.x;
+    for (; i + 3 * stride < ns; i += 4 * stride) {
+        double2 v[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) v[u] = __ldcg(p + i + u * stride);
+#pragma unroll
+        for (int u = 0; u < 4; ++u) acc += v[u].x + v[u].y;
+    }
+    for (; i < ns; i += stride) acc += p[i].x + p[i].y;
+    constexpr int CH = 8;                                           // 8 x 16 B per lane = 4 KB per grab
+    const long per = 32L * CH;
+    const long rest = n2 - ns;
+    const int q = blockIdx.x & 7;                                   // 8 interleaved queues
+    const long nchunk = (rest + per - 1) / per;
+    for (;;) {
+        long c = 0;
+        if (lane == 0) c = long(atomicAdd(ctr + q, 1ull)) * 8 + q;
+        c = __shfl_sync(0xffffffffu, c, 0);
+        if (c >= nchunk) break;
+        const long c0 = ns + c * per;
+        double2 v[CH];
+#pragma unroll
+        for (int u = 0; u < CH; ++u) {
+            const long k = c0 + u * 32 + lane;
+            v[u] = k < n2 ? __ldcg(p + k) : make_double2(0.0, 0.0);
+        }
+#pragma unroll
+        for (int u = 0; u < CH; ++u) acc += v[u].x + v[u].y;
+    }
+    if (acc == 1.2345) *sink = acc;
+}
+
 // L2 eviction by READING another 512 MB: the timed kernel starts with clean lines (a write
 // flush would leave ~126 MB of dirty lines whose write-back the timed kernel would pay for)
 __global__ void k_flush(const double* f, long m, double* sink) {
@@ -90,7 +132,7 @@ int main() {
     cudaMalloc(&F, sizeof(double) * fm);
     cudaMalloc(&sink, 8);
     unsigned long long* ctr;
-    cudaMalloc(&ctr, 8);
+    cudaMalloc(&ctr, 64);
     cudaMemset(P, 0, maxb);
     cudaMemset(Q, 0, maxb);
     cudaMemset(F, 0, sizeof(double) * fm);
@@ -100,16 +142,17 @@ int main() {
     const long sizes_mb[] = {17, 64, 138, 185, 350, 520, 1024, 2048};
     for (long mb : sizes_mb) {
         const long n2 = (mb << 20) / 16;
-        for (int kind = 0; kind < 3; ++kind) {
+        for (int kind = 0; kind < 5; ++kind) {
             for (int cpsm : {4, 8}) {
                 float best = 1e9f;
                 for (int rep = 0; rep < 5; ++rep) {
                     k_flush<<<sms * 4, 512>>>(F, fm, sink);
-                    cudaMemsetAsync(ctr, 0, 8);
+                    cudaMemsetAsync(ctr, 0, 64);
                     cudaEventRecord(a);
                     if (kind == 0) k_read<8><<<sms * cpsm, 256>>>(P, n2, sink);
                     else if (kind == 1) k_copy<4><<<sms * cpsm, 256>>>(P, Q, n2 / 2);
-                    else k_read_dyn<8><<<sms * cpsm, 256>>>(P, n2, sink, ctr);
+                    else if (kind == 2) k_read_dyn<8><<<sms * cpsm, 256>>>(P, n2, sink, ctr);
+                    else k_read_tail<<<sms * cpsm, 256>>>(P, n2, sink, ctr, kind == 3 ? 0.75 : 0.9);
                     cudaEventRecord(b);
                     cudaEventSynchronize(b);
                     float t = 0.f;
@@ -117,7 +160,7 @@ int main() {
                     if (t < best) best = t;
                 }
                 const double bytes = kind == 0 ? double(mb << 20) : double(mb << 20);   // copy: mb/2 read + mb/2 written
-                printf("%-8s %5ld MB  ctas/SM %d  %9.1f us  %7.0f GB/s\n", kind == 0 ? "read" : (kind == 1 ? "copy" : "read-dyn"), mb, cpsm, best * 1e3,
+                printf("%-8s %5ld MB  ctas/SM %d  %9.1f us  %7.0f GB/s\n", kind == 0 ? "read" : (kind == 1 ? "copy" : (kind == 2 ? "read-dyn" : (kind == 3 ? "tail-25%" : "tail-10%"))), mb, cpsm, best * 1e3,
                        bytes / (best * 1e-3) / 1e9);
             }
         }
