@@ -227,8 +227,6 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
                                        first; 0 = every launch sweeps forward.  Row-wise kernels
                                        give identical results either way; the reductions (xTy, Gram,
                                        norms) sum in another fixed order (deterministic). */
-#define CAGMRES_OPT_EXPERIMENT 18   /* bit mask of kernel changes under evaluation (A/B runs on the
-                                       GPU box; default 0; no bit is assigned in this build). */
 #define CAGMRES_OPT_L2_PERSIST 19   /* 0 (default) = off; p in 1..100 = put the MPK SpMV's matrix
                                        values (re-read by every step) in the persisting part of the
                                        L2: the device-wide set-aside (cudaLimitPersistingL2CacheSize)

@@ -73,7 +73,6 @@ struct Dev {
     int rev = 0;                // direction of the next streaming launch (serpentine order, solver.cu)
     size_t apw_bytes = 0;       // CAGMRES_OPT_L2_PERSIST: window over the SpMV values (0 = off)
     float apw_hit = 0.f;
-    int exp = 0;                // CAGMRES_OPT_EXPERIMENT bits (A/B of kernel changes under evaluation)
 };
 
 // Tile order of the streaming kernels (DESIGN.md §6 "serpentine order").  Unit g of NU (a warp,

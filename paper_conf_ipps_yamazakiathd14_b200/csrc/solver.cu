@@ -1331,7 +1331,6 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
             return CAGMRES_OK;
         case CAGMRES_OPT_FOLD: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->fold = value != 0; return CAGMRES_OK;
         case CAGMRES_OPT_SERP: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->serp = value != 0; return CAGMRES_OK;
-        case CAGMRES_OPT_EXPERIMENT: h->dev.exp = int(value); return CAGMRES_OK;
         case CAGMRES_OPT_L2_PERSIST: {
             // the MPK SpMV's values in the persisting part of the L2: every step re-reads them
             if (value < 0 || value > 100) return CAGMRES_EINVAL;
@@ -1375,7 +1374,6 @@ int cagmres_get_option(cagmres_t h, int opt, int64_t* value) {
             return CAGMRES_OK;
         case CAGMRES_OPT_FOLD: *value = h->fold ? 1 : 0; return CAGMRES_OK;
         case CAGMRES_OPT_SERP: *value = h->serp ? 1 : 0; return CAGMRES_OK;
-        case CAGMRES_OPT_EXPERIMENT: *value = h->dev.exp; return CAGMRES_OK;
         case CAGMRES_OPT_L2_PERSIST: *value = h->dev.apw_bytes ? h->l2_persist : 0; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK: *value = h->wave_CH; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CTAS: *value = h->wave_ctas; return CAGMRES_OK;
