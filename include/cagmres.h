@@ -232,7 +232,9 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
                                        L2: the device-wide set-aside (cudaLimitPersistingL2CacheSize)
                                        becomes p % of min(the device maximum, the values' bytes), and
                                        every SpMV launch carries an access-policy window over them.
-                                       ENOTSUP if the device has no set-aside.  Same bits either way. */
+                                       ENOTSUP if the device has no set-aside.  Same bits either way.
+                                       Device-wide while set (released at destroy); measured slower
+                                       on C2 / C3 (the set-aside starves the panel kernels). */
 int cagmres_set_option(cagmres_t h, int opt, int64_t value);
 /* Current value of an option (e.g. the SpMV variant the create-time selection picked).
  * EINVAL for a null handle / pointer or an unknown option. */
