@@ -165,7 +165,9 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
  *                          window fits L2 ("reducing communication of MPK on a single
  *                          GPU"); 2 = force it whenever A is banded; 3 = every MPK block in
  *                          ONE persistent launch (DIA SpMV variants, one rank): the steps are
- *                          separated by grid barriers instead of kernel boundaries.  All
+ *                          separated by grid barriers instead of kernel boundaries (needs
+ *                          every CTA of the launch resident: do not run other kernels
+ *                          concurrently on the device; measured slower, off).  All
  *                          settings give the same bits.  EINVAL for other values.
  *   CAGMRES_OPT_SPMV     : SpMV kernel (default: the fastest on this matrix, timed once at create;
  *                          -1 re-runs that selection): 0 = one SELL-32 slice per warp; 5 = persistent
