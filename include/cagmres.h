@@ -229,14 +229,6 @@ int cagmres_set_stream(cagmres_t h, void* cuda_stream);
                                        first; 0 = every launch sweeps forward.  Row-wise kernels
                                        give identical results either way; the reductions (xTy, Gram,
                                        norms) sum in another fixed order (deterministic). */
-#define CAGMRES_OPT_L2_PERSIST 19   /* 0 (default) = off; p in 1..100 = put the MPK SpMV's matrix
-                                       values (re-read by every step) in the persisting part of the
-                                       L2: the device-wide set-aside (cudaLimitPersistingL2CacheSize)
-                                       becomes p % of min(the device maximum, the values' bytes), and
-                                       every SpMV launch carries an access-policy window over them.
-                                       ENOTSUP if the device has no set-aside.  Same bits either way.
-                                       Device-wide while set (released at destroy); measured slower
-                                       on C2 / C3 (the set-aside starves the panel kernels). */
 int cagmres_set_option(cagmres_t h, int opt, int64_t value);
 /* Current value of an option (e.g. the SpMV variant the create-time selection picked).
  * EINVAL for a null handle / pointer or an unknown option. */

@@ -34,32 +34,6 @@ inline void launch_pdl(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, 
     cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...);
 }
 
-// Same, plus an L2 access-policy window (persisting hits on [base, base + bytes) with probability
-// hit_ratio, streaming misses) for this launch only — the MPK SpMV's matrix values
-// (CAGMRES_OPT_L2_PERSIST); bytes == 0: plain launch_pdl.
-template <typename... KArgs, typename... Args>
-inline void launch_pdl_apw(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
-                           const void* base, size_t bytes, float hit_ratio, Args... args) {
-    if (bytes == 0) { launch_pdl(k, grid, block, smem, st, args...); return; }
-    cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = grid;
-    cfg.blockDim = block;
-    cfg.dynamicSmemBytes = smem;
-    cfg.stream = st;
-    cudaLaunchAttribute attr[2];
-    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    const bool legacy = st == nullptr || st == cudaStreamLegacy;
-    attr[0].val.programmaticStreamSerializationAllowed = (g_pdl && !legacy) ? 1 : 0;
-    attr[1].id = cudaLaunchAttributeAccessPolicyWindow;
-    attr[1].val.accessPolicyWindow.base_ptr = const_cast<void*>(base);
-    attr[1].val.accessPolicyWindow.num_bytes = bytes;
-    attr[1].val.accessPolicyWindow.hitRatio = hit_ratio;
-    attr[1].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-    attr[1].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-    cfg.attrs = attr;
-    cfg.numAttrs = 2;
-    cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...);
-}
 
 // Device properties used for grid sizing (filled once per handle).
 struct Dev {
@@ -71,8 +45,6 @@ struct Dev {
     int panel_tw16 = 1;
     int panel_pf = 1;           // panel rings: L2 prefetch PF_DIST tiles beyond the cp.async window
     int rev = 0;                // direction of the next streaming launch (serpentine order, solver.cu)
-    size_t apw_bytes = 0;       // CAGMRES_OPT_L2_PERSIST: window over the SpMV values (0 = off)
-    float apw_hit = 0.f;
 };
 
 // Tile order of the streaming kernels (DESIGN.md §6 "serpentine order").  Unit g of NU (a warp,

@@ -115,7 +115,6 @@ struct cagmres {
     // kernels) sweeps the rows opposite to the previous one (kern::band_tile), so it first reads
     // what its predecessor touched last, still in L2.  Reset at the start of every cycle.
     bool serp = true;
-    int l2_persist = 0;                    // CAGMRES_OPT_L2_PERSIST (percent of the max set-aside used)
     int* status = nullptr;
     double ms_setup = 0.0;                 // wall time of create
     // CUDA graph of one CA cycle (single rank, untimed solves): captured once per configuration
@@ -169,10 +168,6 @@ struct cagmres {
         cudaFree(d_done);
         for (int2* p : d_pairs) cudaFree(p);
         cudaFree(A.sptr); cudaFree(A.sinfo); cudaFree(A.dcol); cudaFree(A.val);
-        if (l2_persist) {                  // give the device-wide L2 set-aside back
-            cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, 0);
-            cudaCtxResetPersistingL2Cache();
-        }
         cudaFree(sweep_bar);
         cudaFree(V); cudaFree(xe); cudaFree(S); cudaFree(tab); cudaFree(gbuf); cudaFree(ybuf); cudaFree(caqr_ws); cudaFree(op_M);
         cudaFreeHost(h_tab); cudaFreeHost(h_y); cudaFreeHost(h_beta); cudaFreeHost(h_stat);
@@ -1331,22 +1326,6 @@ int cagmres_set_option(cagmres_t h, int opt, int64_t value) {
             return CAGMRES_OK;
         case CAGMRES_OPT_FOLD: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->fold = value != 0; return CAGMRES_OK;
         case CAGMRES_OPT_SERP: if (value < 0 || value > 1) return CAGMRES_EINVAL; h->serp = value != 0; return CAGMRES_OK;
-        case CAGMRES_OPT_L2_PERSIST: {
-            // the MPK SpMV's values in the persisting part of the L2: every step re-reads them
-            if (value < 0 || value > 100) return CAGMRES_EINVAL;
-            if (value == 0) { h->dev.apw_bytes = 0; h->dev.apw_hit = 0.f; return CAGMRES_OK; }
-            cudaDeviceProp pr{};
-            CU(cudaGetDeviceProperties(&pr, h->dev.device));
-            const size_t vbytes = sizeof(double) * size_t(h->A.nstored);
-            size_t setaside = std::min(size_t(pr.persistingL2CacheMaxSize), vbytes);
-            setaside = size_t(double(setaside) * double(value) / 100.0);
-            if (setaside == 0 || pr.accessPolicyMaxWindowSize <= 0) return CAGMRES_ENOTSUP;
-            CU(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, setaside));
-            h->dev.apw_bytes = std::min(vbytes, size_t(pr.accessPolicyMaxWindowSize));
-            h->dev.apw_hit = float(std::min(1.0, double(setaside) / double(h->dev.apw_bytes)));
-            h->l2_persist = int(value);
-            return CAGMRES_OK;
-        }
         case CAGMRES_OPT_WAVE_CHUNK:
             if (value < 256 || value % 256) return CAGMRES_EINVAL;
             h->wave_CH = int(value); wave_reset_pairs(h); return CAGMRES_OK;
@@ -1374,7 +1353,6 @@ int cagmres_get_option(cagmres_t h, int opt, int64_t* value) {
             return CAGMRES_OK;
         case CAGMRES_OPT_FOLD: *value = h->fold ? 1 : 0; return CAGMRES_OK;
         case CAGMRES_OPT_SERP: *value = h->serp ? 1 : 0; return CAGMRES_OK;
-        case CAGMRES_OPT_L2_PERSIST: *value = h->dev.apw_bytes ? h->l2_persist : 0; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CHUNK: *value = h->wave_CH; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_CTAS: *value = h->wave_ctas; return CAGMRES_OK;
         case CAGMRES_OPT_WAVE_LAG: *value = h->wave_lag; return CAGMRES_OK;

@@ -148,8 +148,7 @@ void go_dia(const Dev& d, const DiaArgs& a, cudaStream_t st) {
     int64_t g = int64_t(d.sms) * occ;
     const int64_t need = (nsl + DT_NT / 32 - 1) / (DT_NT / 32);
     if (g > need) g = need;
-    launch_pdl_apw(k_spmv_dia<MODE, WT, MINB, SX>, dim3(unsigned(g)), dim3(DT_NT), 0, st, a.val, d.apw_bytes,
-                   d.apw_hit, a);
+    launch_pdl(k_spmv_dia<MODE, WT, MINB, SX>, dim3(unsigned(g)), dim3(DT_NT), 0, st, a);
 }
 
 template <int WT, int MINB>

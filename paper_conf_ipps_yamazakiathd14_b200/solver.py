@@ -175,7 +175,7 @@ class Solver:
             self._bound_stream = s
 
     OPTIONS = {"mpk_wave": 1, "wave_chunk": 3, "wave_ctas": 4, "wave_lag": 5, "fuse": 6, "spmv": 7, "gram": 8,
-               "arnoldi": 9, "panel_tw": 10, "trsm": 11, "pdl": 12, "panel_pf": 13, "peer": 14, "graph": 15, "fold": 16, "serp": 17, "l2_persist": 19}
+               "arnoldi": 9, "panel_tw": 10, "trsm": 11, "pdl": 12, "panel_pf": 13, "peer": 14, "graph": 15, "fold": 16, "serp": 17}
 
     def set_option(self, opt, value):
         """opt: "mpk_wave", "wave_chunk", "wave_ctas", "wave_lag", "fuse", "spmv", "gram", "arnoldi" (CAGMRES_OPT_*)."""

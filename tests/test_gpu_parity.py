@@ -186,29 +186,6 @@ def test_mpk_sweep_bitwise_equals_stepwise(gen):
         assert np.array_equal(out[0][1].hist, out[1][1].hist) and torch.equal(out[0][0], out[1][0])
 
 
-def test_l2_persist_option_keeps_the_bits():
-    """CAGMRES_OPT_L2_PERSIST only changes where A's values are cached (an access-policy window on
-    every SpMV launch + the device's persisting L2 set-aside): MPK bases and solves are bitwise
-    those without it; the option reads back and is released with the handle."""
-    A = G.convection_diffusion(45, 3, 7)
-    q = dev(G.u(5, np.arange(A.n)))
-    b = dev(G.rhs(A.n))
-    out = []
-    for p in (100, 0):
-        S = Solver(A, s=10, m=30, basis="newton")
-        S.set_option("spmv", 16)
-        S.set_option("l2_persist", p)
-        assert S.get_option("l2_persist") == p
-        S.set_shifts(*SHIFTS)
-        W = S.mpk(q, 10)
-        S.clear_shifts()
-        x, st = S.solve(b, tol=1e-8, maxit=60)
-        out.append((W, x, st))
-        S.close()
-    assert torch.equal(out[0][0], out[1][0]) and torch.equal(out[0][1], out[1][1])
-    assert np.array_equal(out[0][2].hist, out[1][2].hist)
-
-
 @pytest.mark.parametrize("gen", ["cd27_ragged", "g3_small", "banded", "cd7_ragged"])
 def test_spmv_variants_bitwise(gen):
     """Every SpMV kernel variant (CAGMRES_OPT_SPMV: one or two SELL-32 slices per warp, load
