@@ -43,7 +43,8 @@ struct Dev {
     int arnoldi_ring = 1;       // first-cycle / GMRES Arnoldi passes: 1 = cp.async ring kernels
     int trsm_scalar = 1;        // CholQR/SVQR update: 1 = scalar DFMA ring (w <= 16), 0 = DMMA
     int panel_tw16 = 1;
-    int panel_pf = 1;           // panel rings: L2 prefetch PF_DIST tiles beyond the cp.async window
+    int panel_pf = 0;           // panel rings: L2 prefetch PF_DIST tiles beyond the cp.async window (off:
+                                // with the serpentine order it costs more L2 than it hides)
     int rev = 0;                // direction of the next streaming launch (serpentine order, solver.cu)
 };
 
